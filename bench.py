@@ -1,0 +1,367 @@
+"""bench.py — TCCG-48 GFLOP/s geomean (FP64) on B200 through libtc's C ABI.
+
+Contract:
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl libtc|reference] [--cases 1,2,..]
+One STEP = one pass of the hot path over the whole workload: all 48 TCCG contractions
+(SURVEY.md Appendix A extents, FP64, alpha = 1, beta = 0), inputs resident in HBM, one
+tc_execute each.  L2 is flushed (256 MiB memset) before every launch, outside the events.
+value = geomean over the 48 cases of 2*prod(N) / (median device time of that case) —
+the BASELINE.json metric.  N > 1 (torchrun): every case is C-slab sharded on its largest
+external index; A and B are broadcast from rank 0 over NCCL inside the timed
+region; time = max over ranks; scaling "strong".
+--impl reference: the CPU oracle (oracle/, the paper's plain nested loop) on this box's host
+cores, on a bounded sample of the same workload (rank 0 only).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import tcinputs  # noqa: E402
+
+METRIC = "TCCG-48 GFLOP/s geomean (FP64) at 1 GPU; % of FP64/tensor peak or HBM roofline"
+UNIT = "GFLOP/s"
+FP64_PEAK_TFLOPS = 37.16      # measured DMMA peak, profiles/r01_peaks.json (tools/peaks.cu)
+FP64_PEAK_DERIVED = 148 * 64 * 2 * 1.965e9 / 1e12   # 37.2: SMs x FMA/clk x 2 x max clock
+
+
+def geomean(xs):
+    return math.exp(sum(math.log(x) for x in xs) / len(xs))
+
+
+def parse_args():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="libtc", choices=["libtc", "reference"])
+    ap.add_argument("--cases", default="")
+    ap.add_argument("--cost", default="b200", choices=["b200", "paper"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of oracle work")
+    return ap.parse_args()
+
+
+def select_cases(spec):
+    cases = tcinputs.tccg48()
+    if spec:
+        ids = {int(x) for x in spec.split(",")}
+        cases = [c for c in cases if c.id in ids]
+    return cases
+
+
+# ---------------------------------------------------------------- oracle (CPU) timing
+def oracle_sample_rates(cases, budget_s, nthreads=0):
+    """Oracle GFLOP/s per case on a contiguous C range sized to ~budget/len(cases) s."""
+    import numpy as np
+    import oracle
+    per = budget_s / len(cases)
+    rates = {}
+    for c in cases:
+        ca, aa, ba = tcinputs.split_expr(c.expr)
+        ext = c.ext
+        nA, nB, nC = (tcinputs.numel(aa, ext), tcinputs.numel(ba, ext), tcinputs.numel(ca, ext))
+        K = 1
+        for x in aa:
+            if x not in ca:
+                K *= ext[x]
+        A = tcinputs.uniform_np(nA, 1000 + c.id)
+        B = tcinputs.uniform_np(nB, 2000 + c.id)
+        n = max(1, min(nC, 2048))
+        t0 = time.perf_counter()
+        oracle.contract(c.expr, c.extents, A, B, lo=0, hi=n, nthreads=nthreads)
+        dt = time.perf_counter() - t0
+        n2 = int(min(nC, max(n, n * per / max(dt, 1e-4))))
+        t0 = time.perf_counter()
+        oracle.contract(c.expr, c.extents, A, B, lo=0, hi=n2, nthreads=nthreads)
+        dt = time.perf_counter() - t0
+        rates[c.id] = (2.0 * K * n2 / dt / 1e9, n2, nC)
+    return rates
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import oracle
+    cases = select_cases(args.cases)
+    cores = len(os.sched_getaffinity(0))
+    per_step = max(2.0, 150.0 / max(1, args.steps + args.warmup))
+    for _ in range(args.warmup):
+        oracle_sample_rates(cases, per_step / 4)
+    t0 = time.perf_counter()
+    vals = []
+    for _ in range(args.steps):
+        r = oracle_sample_rates(cases, per_step)
+        vals.append(geomean([v[0] for v in r.values()]))
+    wall = time.perf_counter() - t0
+    v = geomean(vals)
+    line = {"impl": "reference", "metric": METRIC, "value": round(v, 4), "unit": UNIT,
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(wall / args.steps * 1e3, 1), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": "TCCG-48 suite (SURVEY App. A extents), FP64, alpha=1, beta=0",
+                       "cases": len(cases)},
+            "cpu_baseline": {"value": round(v, 4), "unit": UNIT, "cores": cores, "kind": "oracle",
+                             "threads": oracle.max_threads(),
+                             "sample": f"per case a contiguous range of C linear indices sized to "
+                                       f"~{per_step / len(cases):.2f}s of oracle work per step"},
+            "e2e": {"value": round(v, 4), "unit": UNIT, "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------- clocks
+class Clocks:
+    def __init__(self, path):
+        self.path = path
+        self.p = None
+
+    def __enter__(self):
+        try:
+            self.f = open(self.path, "w")
+            self.p = subprocess.Popen(
+                ["nvidia-smi", "--query-gpu=index,clocks.sm,clocks.max.sm,power.draw,"
+                 "clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+                 "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+                 "clocks_event_reasons.sw_power_cap", "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+        return self
+
+    def __exit__(self, *a):
+        if self.p:
+            self.p.terminate()
+            self.p.wait()
+            self.f.close()
+
+    def summary(self, dev=0):
+        try:
+            rows = [r.split(",") for r in open(self.path).read().strip().splitlines()]
+            rows = [[x.strip() for x in r] for r in rows if len(r) >= 9 and r[0].strip() == str(dev)]
+        except Exception:
+            return None
+        if not rows:
+            return None
+        sm = sorted(float(r[1]) for r in rows)
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i in range(4) if r[5 + i].lower() == "active"})
+        return {"sm_mhz": sm[len(sm) // 2], "sm_max_mhz": float(rows[0][2]), "reasons": reasons,
+                "samples": len(rows)}
+
+
+# ---------------------------------------------------------------- GPU run
+def run_libtc(args):
+    import torch
+    import torch.distributed as dist
+    from paper_conf_cgo_kimstkpprs19_b200 import binding as tc
+    from paper_conf_cgo_kimstkpprs19_b200 import dist as tcdist
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    cases = select_cases(args.cases)
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.current_stream()
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+
+    # plans + resident inputs (rank 0's inputs are the source of the broadcast at N > 1)
+    work = []
+    t_plan = 0.0
+    for c in cases:
+        t0 = time.perf_counter()
+        p = tc.plan(c.expr, c.extents, cost=args.cost)
+        if world > 1:
+            sh = tcdist.shard_plan(p, c.expr, c.extents, world, rank)
+        t_plan += time.perf_counter() - t0
+        A = tcinputs.uniform(p.numel("A"), 1000 + c.id, device=dev)
+        B = tcinputs.uniform(p.numel("B"), 2000 + c.id, device=dev)
+        if world == 1:
+            C = torch.empty(p.numel("C"), dtype=torch.float64, device=dev)
+            work.append((c, p, A, B, C, None))
+        else:
+            C = torch.empty(sh.c_numel, dtype=torch.float64, device=dev)
+            work.append((c, p, A, B, C, sh))
+
+    def one(i, record):
+        c, p, A, B, C, sh = work[i]
+        flush.zero_()
+        if world > 1:
+            dist.barrier()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        if sh is None:
+            p.execute(A, B, C)
+        else:
+            tcdist.broadcast_inputs(A, B, src=0)
+            sh.plan.execute(A, B, C)
+        e1.record(stream)
+        record.append((e0, e1))
+
+    for _ in range(args.warmup):
+        rec = []
+        for i in range(len(work)):
+            one(i, rec)
+    torch.cuda.synchronize()
+    times = [[] for _ in work]
+    clk_path = os.path.join(ROOT, "gpurun_out", f"bench_clocks_r{rank}.csv")
+    os.makedirs(os.path.dirname(clk_path), exist_ok=True)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with Clocks(clk_path) as clocks:
+        t_wall = time.perf_counter()
+        for _ in range(args.steps):
+            rec = []
+            for i in range(len(work)):
+                one(i, rec)
+            torch.cuda.synchronize()
+            for i, (e0, e1) in enumerate(rec):
+                times[i].append(e0.elapsed_time(e1))
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        t_wall = time.perf_counter() - t_wall
+    med = []
+    for ts in times:
+        s = sorted(ts)
+        med.append(s[len(s) // 2])
+    if world > 1:
+        t = torch.tensor(med, dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        med = t.tolist()
+    per_case = []
+    for (c, p, *_), ms in zip(work, med):
+        per_case.append({"id": c.id, "ms": round(ms, 5), "gflops": round(p.flops / ms / 1e6, 2),
+                         "variant": p.info()["variant"]})
+    value = geomean([r["gflops"] for r in per_case])
+    ms_step = sum(med)
+
+    # dominant kernel (largest share of the step) -> roofline
+    share = {}
+    for (c, p, *_), ms in zip(work, med):
+        v = p.info()["variant"]
+        f, t = share.get(v, (0.0, 0.0))
+        share[v] = (f + p.flops, t + ms)
+    dom = max(share, key=lambda v: share[v][1])
+    dflops, dms = share[dom]
+    achieved = dflops / (dms * 1e-3) / 1e12
+    nlaunch = sum(1 for (c, p, *_) in work if p.info()["variant"] == dom)
+    traffic = None
+    prof = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(prof):
+        try:
+            traffic = json.load(open(prof)).get(f"variant{dom}")
+        except Exception:
+            traffic = None
+    roof = {"bound": "tensor", "achieved": round(achieved, 3), "peak": FP64_PEAK_TFLOPS,
+            "unit": "TFLOP/s", "frac": round(achieved / FP64_PEAK_TFLOPS, 4), "traffic": traffic,
+            "kernel": f"tc_f64_dmma_kernel variant {dom}",
+            "peak_source": "measured FP64 DMMA peak (tools/peaks.cu, profiles/r01_peaks.json); "
+                           f"derived 148x64x2x1.965GHz = {FP64_PEAK_DERIVED:.2f}",
+            "launches_per_step": nlaunch,
+            "share_of_step": round(dms / ms_step, 4)}
+
+    # per-class roofline fraction: min(FP64 peak, I * HBM) per case
+    hbm = 6554.2e9
+    try:
+        hbm = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"] * 1e9
+    except Exception:
+        pass
+    fr = []
+    for (c, p, A, B, C, sh), ms in zip(work, med):
+        byts = 8.0 * (p.numel("A") + p.numel("B") + p.numel("C"))
+        attain = min(FP64_PEAK_TFLOPS * 1e12, p.flops / byts * hbm)
+        fr.append(p.flops / (ms * 1e-3) / attain)
+    clk = clocks.summary(local)
+
+    # end-to-end through tc_execute_host (pinned host buffers; copies inside the timing)
+    e2e = None
+    if not args.no_e2e and world == 1:
+        e2e_vals, h2d, d2h = [], 0, 0
+        maxA = max(w[1].numel("A") for w in work)
+        maxB = max(w[1].numel("B") for w in work)
+        maxC = max(w[1].numel("C") for w in work)
+        hA = torch.empty(maxA, dtype=torch.float64).pin_memory()
+        hB = torch.empty(maxB, dtype=torch.float64).pin_memory()
+        hC = torch.empty(maxC, dtype=torch.float64).pin_memory()
+        ws = torch.empty(max(w[1].workspace_bytes() for w in work) // 8 + 1, dtype=torch.float64,
+                         device=dev)
+        for (c, p, A, B, C, sh) in work:
+            hA[:A.numel()].copy_(A)
+            hB[:B.numel()].copy_(B)
+            ts = []
+            for r in range(2):
+                torch.cuda.synchronize()
+                t0 = time.perf_counter()
+                p.execute_host(hA, hB, hC, ws)
+                ts.append(time.perf_counter() - t0)
+            e2e_vals.append(p.flops / min(ts) / 1e9)
+            h2d += 8 * (A.numel() + B.numel())
+            d2h += 8 * p.numel("C")
+        e2e = {"value": round(geomean(e2e_vals), 3), "unit": UNIT, "h2d_bytes_per_step": h2d,
+               "d2h_bytes_per_step": d2h,
+               "how": "tc_execute_host per case: pinned host A,B -> device, kernel, C -> host, "
+                      "stream sync; wall clock, best of 2"}
+
+    cpu = None
+    if not args.no_cpu and rank == 0 and world == 1:
+        import oracle
+        rates = oracle_sample_rates(cases, args.cpu_budget)
+        cpu = {"value": round(geomean([v[0] for v in rates.values()]), 4), "unit": UNIT,
+               "cores": len(os.sched_getaffinity(0)), "threads": oracle.max_threads(),
+               "kind": "oracle",
+               "sample": f"per case a contiguous range of C linear indices sized to "
+                         f"~{args.cpu_budget / len(cases):.2f}s of oracle work "
+                         f"({sum(v[1] for v in rates.values())} of "
+                         f"{sum(v[2] for v in rates.values())} C elements)"}
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": round(value, 2), "unit": UNIT, "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_step, 4),
+                "higher_is_better": True, "scaling": "strong" if world > 1 else "weak",
+                "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+                "config": {"workload": "TCCG-48 suite (SURVEY App. A extents), FP64, alpha=1, beta=0",
+                           "cases": len(cases), "cost_model": args.cost,
+                           "l2": "flushed before every launch (256 MiB memset, outside events)",
+                           "timing": "CUDA events per launch on the launch stream; median of steps",
+                           "parallelism": f"C-slab shard x{world}" if world > 1 else "single GPU"},
+                "roofline": roof,
+                "roofline_geomean_frac": round(geomean(fr), 4),
+                "cpu_baseline": cpu, "e2e": e2e,
+                "gpu_launches": len(work) * args.steps,
+                "clocks": clk,
+                "plan_ms_total": round(t_plan * 1e3, 2),
+                "wall_s_timed": round(t_wall, 3),
+                "per_case": per_case}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def main():
+    args = parse_args()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_libtc(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,134 @@
+/*
+ * libtc.h — C ABI of libtc: direct (transpose-free) contraction of two dense tensors on
+ * NVIDIA B200 (sm_100a).
+ *
+ * The operation (Section II, eq. (1) and the sum below it):
+ *     C[a,b,c,d] = sum_{e,f} A[a,e,b,f] * B[d,f,c,e]
+ * generalised with the Einstein convention to any expression in which every index
+ * occurs in exactly two of the three tensors, and with the update
+ *     C = alpha * sum_int A * B + beta * C          (beta == 0: C is never read)
+ * (reading R3).  No transposed intermediate is ever created.
+ *
+ * Layout: every tensor is dense and the FIRST listed index of each
+ * tensor is its fastest varying index (stride 1): offset = sum_k i_k * prod_{j<k} N_j.
+ * As a row-major torch tensor the shape is the reversed index list.
+ *
+ * Functions are nothrow: no C++ exception crosses this boundary; every failure is a status
+ * code plus a thread-local detail string (tc_last_error).  The library never aborts.
+ */
+#ifndef LIBTC_H
+#define LIBTC_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct CUstream_st *tc_stream_t; /* == cudaStream_t; NULL = legacy default stream */
+
+typedef enum { TC_F64 = 0, TC_F32 = 1, TC_TF32 = 2, TC_BF16 = 3 } tc_dtype_t;
+
+typedef enum {
+  TC_SUCCESS = 0,
+  TC_ERR_INVALID_ARG = 1, /* NULL pointer/handle, C overlaps A or B, wrong device, bad opts */
+  TC_ERR_PARSE = 2,       /* malformed expression or extents string                          */
+  TC_ERR_INDEX = 3,       /* index in one tensor only or in all three, repeated in a tensor,
+                             extent missing / duplicated / naming an unknown index           */
+  TC_ERR_EXTENT = 4,      /* extent < 1, or an element count overflows int64                 */
+  TC_ERR_UNSUPPORTED = 5, /* rank > 8, > 16 distinct indices, extent > 2^31-1, dtype not built */
+  TC_ERR_NO_CONFIG = 6,   /* planner found no legal configuration (a bug)                    */
+  TC_ERR_CUDA = 7,        /* CUDA error at plan or launch (or no device); see tc_last_error  */
+  TC_ERR_ALLOC = 8        /* allocation of plan metadata failed                              */
+} tc_status_t;
+
+typedef struct tc_plan_s *tc_plan_t; /* opaque; immutable once created */
+
+/* Cost model used to rank configurations (Section IV-B). */
+typedef enum {
+  TC_COST_B200 = 0,  /* re-derived model: sectors, waves, padding, FP64 pipe, HBM */
+  TC_COST_PAPER = 1  /* Alg. 3 verbatim: 128-B transactions, V100 value sets  */
+} tc_cost_mode_t;
+
+/* Options for tc_plan_ex.  Zero-initialise, then set what you need. */
+typedef struct tc_plan_opts {
+  int cost_mode;     /* tc_cost_mode_t                                                       */
+  int host_only;     /* 1: plan without touching the GPU (no device tables; tc_execute fails) */
+  int variant;       /* -1 or 0: planner's choice; k>0: force kernel variant k-1 (tests)     */
+  /* forced per-index tiles (tests of Fig. 2/3-style configs): "a:16;b:4;e:1;f:16" or NULL.
+     Indices not listed keep the planner's choice only if force_tiles is NULL.               */
+  const char *force_tiles;
+  int no_fusion;     /* 1: do not merge adjacent indices (row a2)                            */
+  int reserved[8];
+} tc_plan_opts;
+
+/*
+ * Plan a contraction.
+ *   expr    : "abcd-aebf-dfce" (TCCG form C-A-B, one letter per index) or
+ *             "C[a,b,c,d] = A[a,e,b,f] * B[d,f,c,e]" (bracket form).
+ *   extents : "a:16;b:16;c:16;d:16;e:16;f:16", each index exactly once.
+ *   dtype   : A, B and C share it.  TC_F64 is the paper's precision (R20).
+ * On success *plan owns its host metadata and small device tables, allocated on the device
+ * that is current at the call (unless opts->host_only).  *plan is NULL on failure.
+ */
+tc_status_t tc_plan(tc_plan_t *plan, const char *expr, const char *extents, tc_dtype_t dtype);
+tc_status_t tc_plan_ex(tc_plan_t *plan, const char *expr, const char *extents, tc_dtype_t dtype,
+                       const tc_plan_opts *opts /* nullable */);
+
+/*
+ * C = alpha * sum_int A*B + beta * C on `stream` (asynchronous; no allocation, no sync).
+ * A, B, C are caller-owned DEVICE pointers on the plan's device, dense in the plan's layout
+ * (for a restricted plan: the parent tensors' base pointers unless TC_SLAB_* flags said
+ * otherwise).  Any cudaMalloc pointer works; 16-B aligned pointers enable the vectorised
+ * loads.  beta == 0 => C is only written (NaN in the old C does not propagate, R26).
+ * Errors: TC_ERR_INVALID_ARG (NULL, C overlapping A or B, wrong current device),
+ * TC_ERR_CUDA (launch error; asynchronous faults surface at the caller's next sync).
+ */
+tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void *C, double alpha,
+                       double beta, tc_stream_t stream);
+
+/*
+ * End-to-end call with HOST buffers (used for bench.py's "e2e" figure): copies A, B (and C
+ * when beta != 0) from host memory into the caller-provided device workspace, runs
+ * tc_execute, copies C back, and synchronises `stream`.  workspace must hold
+ * tc_plan_workspace_bytes(plan) bytes; host buffers should be pinned for full speed.
+ */
+size_t tc_plan_workspace_bytes(const tc_plan_t plan);
+tc_status_t tc_execute_host(const tc_plan_t plan, const void *A_host, const void *B_host,
+                            void *C_host, double alpha, double beta, void *workspace,
+                            size_t workspace_bytes, tc_stream_t stream);
+
+/* Flags of tc_plan_restrict: the operand passed to tc_execute is the compact slab itself. */
+#define TC_SLAB_A 1u
+#define TC_SLAB_B 2u
+#define TC_SLAB_C 4u
+
+/*
+ * Sub-plan over [begin, begin+len) of one index:
+ *   external index -> slab of C (multi-GPU C-slab sharding; no reduction needed);
+ *   internal index -> split-K partial sum (caller reduces the partial C's).
+ * Without flags the tensors keep the parent's strides and base pointers; with TC_SLAB_X the
+ * operand X is a dense tensor of its own with that index's extent = len.
+ */
+tc_status_t tc_plan_restrict(tc_plan_t *sub, const tc_plan_t parent, const char *index,
+                             int64_t begin, int64_t len, unsigned flags);
+
+/* JSON description of the plan (classes, fused indices, tiles, variant, predicted cost,
+   config-space statistics).  Writes at most cap bytes (NUL-terminated); *needed = full size. */
+tc_status_t tc_plan_info(const tc_plan_t plan, char *json, size_t cap, size_t *needed);
+
+double tc_plan_flops(const tc_plan_t plan);          /* 2 * prod(all extents) (R5)       */
+int64_t tc_plan_numel(const tc_plan_t plan, int t);  /* elements of 0=C, 1=A, 2=B        */
+void tc_plan_destroy(tc_plan_t plan);                /* NULL-safe                        */
+const char *tc_status_string(tc_status_t status);
+const char *tc_last_error(void);                     /* thread-local detail string       */
+const char *tc_version(void);
+
+/* Validation only (parse + classify), same rules and codes as tc_plan; no allocation. */
+tc_status_t tc_check(const char *expr, const char *extents);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* LIBTC_H */

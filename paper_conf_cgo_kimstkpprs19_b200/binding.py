@@ -1,0 +1,188 @@
+"""Thin ctypes binding of libtc (include/libtc.h) — argument marshalling only.
+
+Every step of the contraction runs in libtc.so's CUDA kernels; this module never computes
+anything itself and never falls back to another implementation: if libtc.so is missing or a
+call fails, it raises.  torch is used for device memory and streams only.
+
+Layout: the FIRST listed index of each tensor is stride-1, so a torch
+tensor for index list "aebf" has shape (N_f, N_b, N_e, N_a) (reversed) and is contiguous;
+``empty(plan, "A")`` allocates it.
+"""
+from __future__ import annotations
+
+import ctypes
+import json
+import os
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SO = os.path.join(_HERE, "libtc.so")
+
+STATUS = ["TC_SUCCESS", "TC_ERR_INVALID_ARG", "TC_ERR_PARSE", "TC_ERR_INDEX", "TC_ERR_EXTENT",
+          "TC_ERR_UNSUPPORTED", "TC_ERR_NO_CONFIG", "TC_ERR_CUDA", "TC_ERR_ALLOC"]
+DTYPES = {"f64": 0, "f32": 1, "tf32": 2, "bf16": 3}
+COST = {"b200": 0, "paper": 1}
+SLAB_A, SLAB_B, SLAB_C = 1, 2, 4
+
+
+class TcError(RuntimeError):
+    def __init__(self, status: int, detail: str):
+        super().__init__(f"{STATUS[status] if 0 <= status < len(STATUS) else status}: {detail}")
+        self.status = STATUS[status] if 0 <= status < len(STATUS) else str(status)
+        self.detail = detail
+
+
+class _Opts(ctypes.Structure):
+    _fields_ = [("cost_mode", ctypes.c_int), ("host_only", ctypes.c_int), ("variant", ctypes.c_int),
+                ("force_tiles", ctypes.c_char_p), ("no_fusion", ctypes.c_int),
+                ("reserved", ctypes.c_int * 8)]
+
+
+_lib = None
+
+
+def lib():
+    """Load libtc.so (built in-tree by build.py / __graft_entry__.build())."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(_SO):
+            raise ImportError(f"libtc.so not built ({_SO}); run __graft_entry__.build()")
+        L = ctypes.CDLL(_SO)
+        vp, cp, i64, dbl = ctypes.c_void_p, ctypes.c_char_p, ctypes.c_int64, ctypes.c_double
+        L.tc_plan_ex.argtypes = [ctypes.POINTER(vp), cp, cp, ctypes.c_int, ctypes.POINTER(_Opts)]
+        L.tc_plan_ex.restype = ctypes.c_int
+        L.tc_plan.argtypes = [ctypes.POINTER(vp), cp, cp, ctypes.c_int]
+        L.tc_plan.restype = ctypes.c_int
+        L.tc_execute.argtypes = [vp, vp, vp, vp, dbl, dbl, vp]
+        L.tc_execute.restype = ctypes.c_int
+        L.tc_execute_host.argtypes = [vp, vp, vp, vp, dbl, dbl, vp, ctypes.c_size_t, vp]
+        L.tc_execute_host.restype = ctypes.c_int
+        L.tc_plan_workspace_bytes.argtypes = [vp]
+        L.tc_plan_workspace_bytes.restype = ctypes.c_size_t
+        L.tc_plan_restrict.argtypes = [ctypes.POINTER(vp), vp, cp, i64, i64, ctypes.c_uint]
+        L.tc_plan_restrict.restype = ctypes.c_int
+        L.tc_plan_info.argtypes = [vp, ctypes.c_char_p, ctypes.c_size_t, ctypes.POINTER(ctypes.c_size_t)]
+        L.tc_plan_info.restype = ctypes.c_int
+        L.tc_plan_flops.argtypes = [vp]
+        L.tc_plan_flops.restype = dbl
+        L.tc_plan_numel.argtypes = [vp, ctypes.c_int]
+        L.tc_plan_numel.restype = i64
+        L.tc_plan_destroy.argtypes = [vp]
+        L.tc_plan_destroy.restype = None
+        L.tc_status_string.argtypes = [ctypes.c_int]
+        L.tc_status_string.restype = cp
+        L.tc_last_error.restype = cp
+        L.tc_version.restype = cp
+        L.tc_check.argtypes = [cp, cp]
+        L.tc_check.restype = ctypes.c_int
+        _lib = L
+    return _lib
+
+
+def _raise(st: int):
+    if st != 0:
+        raise TcError(st, lib().tc_last_error().decode())
+
+
+def check(expr: str, extents: str) -> str:
+    """Parse + validate only; returns the status name."""
+    return STATUS[lib().tc_check(expr.encode(), extents.encode())]
+
+
+def version() -> str:
+    return lib().tc_version().decode()
+
+
+def _stream_ptr(stream):
+    if stream is None:
+        import torch
+        if torch.cuda.is_available():
+            return ctypes.c_void_p(torch.cuda.current_stream().cuda_stream)
+        return ctypes.c_void_p(0)
+    if isinstance(stream, int):
+        return ctypes.c_void_p(stream)
+    return ctypes.c_void_p(stream.cuda_stream)
+
+
+class Plan:
+    """A libtc plan (tc_plan_t).  Immutable; execute() may be called any number of times."""
+
+    def __init__(self, handle: ctypes.c_void_p, expr: str, extents: str, dtype: str):
+        self._h = handle
+        self.expr, self.extents, self.dtype = expr, extents, dtype
+        self._info = None
+
+    def __del__(self):
+        h = getattr(self, "_h", None)
+        if h and _lib is not None:
+            _lib.tc_plan_destroy(h)
+            self._h = None
+
+    @property
+    def handle(self):
+        return self._h
+
+    def info(self) -> dict:
+        if self._info is None:
+            need = ctypes.c_size_t(0)
+            _raise(lib().tc_plan_info(self._h, None, 0, ctypes.byref(need)))
+            buf = ctypes.create_string_buffer(need.value)
+            _raise(lib().tc_plan_info(self._h, buf, need.value, ctypes.byref(need)))
+            self._info = json.loads(buf.value.decode())
+        return self._info
+
+    @property
+    def flops(self) -> float:
+        return lib().tc_plan_flops(self._h)
+
+    def numel(self, which: str) -> int:
+        return int(lib().tc_plan_numel(self._h, "CAB".index(which)))
+
+    def workspace_bytes(self) -> int:
+        return int(lib().tc_plan_workspace_bytes(self._h))
+
+    def restrict(self, index: str, begin: int, length: int, flags: int = 0) -> "Plan":
+        h = ctypes.c_void_p()
+        _raise(lib().tc_plan_restrict(ctypes.byref(h), self._h, index.encode(), int(begin),
+                                      int(length), int(flags)))
+        return Plan(h, self.expr, f"{self.extents}|{index}[{begin}:{begin + length}]", self.dtype)
+
+    def execute_ptr(self, A: int, B: int, C: int, alpha=1.0, beta=0.0, stream=None):
+        _raise(lib().tc_execute(self._h, ctypes.c_void_p(A), ctypes.c_void_p(B), ctypes.c_void_p(C),
+                                float(alpha), float(beta), _stream_ptr(stream)))
+
+    def execute(self, A, B, C, alpha=1.0, beta=0.0, stream=None):
+        """C = alpha * sum A*B + beta * C on torch CUDA tensors (current stream)."""
+        for name, t, w in (("A", A, "A"), ("B", B, "B"), ("C", C, "C")):
+            if not t.is_cuda or not t.is_contiguous():
+                raise TcError(1, f"{name} must be a contiguous CUDA tensor")
+        self.execute_ptr(A.data_ptr(), B.data_ptr(), C.data_ptr(), alpha, beta, stream)
+        return C
+
+    def execute_host(self, A, B, C, workspace, alpha=1.0, beta=0.0, stream=None):
+        """End-to-end: host (pinned) A, B, C; device workspace of workspace_bytes()."""
+        _raise(lib().tc_execute_host(self._h, ctypes.c_void_p(A.data_ptr()), ctypes.c_void_p(B.data_ptr()),
+                                     ctypes.c_void_p(C.data_ptr()), float(alpha), float(beta),
+                                     ctypes.c_void_p(workspace.data_ptr()),
+                                     ctypes.c_size_t(workspace.numel() * workspace.element_size()),
+                                     _stream_ptr(stream)))
+        return C
+
+
+def plan(expr: str, extents: str, dtype: str = "f64", cost: str = "b200", host_only: bool = False,
+         variant: int | None = None, force_tiles: str | None = None, fusion: bool = True) -> Plan:
+    o = _Opts()
+    o.cost_mode = COST[cost]
+    o.host_only = int(host_only)
+    o.variant = 0 if variant is None else int(variant) + 1
+    o.force_tiles = force_tiles.encode() if force_tiles else None
+    o.no_fusion = int(not fusion)
+    h = ctypes.c_void_p()
+    _raise(lib().tc_plan_ex(ctypes.byref(h), expr.encode(), extents.encode(), DTYPES[dtype], ctypes.byref(o)))
+    p = Plan(h, expr, extents, dtype)
+    p._opts = o  # keep force_tiles bytes alive for the call's duration
+    return p
+
+
+def shape_of(indices: str, extents: dict) -> tuple:
+    """torch shape of a tensor with the given index list (reversed: first index fastest)."""
+    return tuple(extents[c] for c in reversed(indices))

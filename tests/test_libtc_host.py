@@ -1,0 +1,136 @@
+"""CPU tests of libtc's host side: the C-ABI library loads and exports every symbol of
+include/libtc.h; parser / classifier against the shared rules table; fusion; planner
+invariants and statistics (host_only plans: no GPU needed)."""
+import ctypes
+import json
+import os
+import re
+
+import pytest
+
+import tcinputs
+from paper_conf_cgo_kimstkpprs19_b200 import binding as tc
+from paper_conf_cgo_kimstkpprs19_b200 import build
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _built():
+    build.build()
+
+
+def test_exports_every_header_symbol():
+    hdr = open(os.path.join(ROOT, "include", "libtc.h")).read()
+    names = set(re.findall(r"\b(tc_[a-z_]+)\s*\(", hdr))
+    assert len(names) >= 14
+    L = ctypes.CDLL(build.SO)
+    for n in sorted(names):
+        assert hasattr(L, n), n
+
+
+def test_validation_rules_golden():
+    rules = json.load(open(os.path.join(ROOT, "tests", "golden", "validation_rules.json")))["rules"]
+    for expr, extents, want in rules:
+        assert tc.check(expr, extents) == want, (expr, extents)
+
+
+def test_classification_eq1_and_bracket_form():
+    a = tc.plan("abcd-aebf-dfce", tcinputs.EQ1_EXTENTS, host_only=True).info()
+    b = tc.plan("C[a,b,c,d] = A[a,e,b,f] * B[d,f,c,e]", tcinputs.EQ1_EXTENTS, host_only=True).info()
+    cls = {x["name"]: x["cls"] for x in a["indices"]}
+    assert cls == {"a": "extA", "b": "extA", "c": "extB", "d": "extB", "e": "int", "f": "int"}
+    assert a["X"] == "A"          # C's FVI a lives in A
+    for k in ("indices", "m", "n", "k", "variant", "Mt", "Nt", "Kt", "nctas", "nsteps"):
+        assert a[k] == b[k], k
+
+
+def test_fusion_row_a2():
+    i = tc.plan("abcd-ea-ebcd", "a:72;b:72;c:72;d:72;e:72", host_only=True).info()
+    assert sorted(x["name"] for x in i["indices"]) == ["a", "b*c*d", "e"]
+    i = tc.plan("abcd-abef-efcd", ";".join(f"{c}:8" for c in "abcdef"), host_only=True).info()
+    assert sorted(x["name"] for x in i["indices"]) == ["a*b", "c*d", "e*f"]   # a pure GEMM
+    i = tc.plan("abcd-aebf-dfce", "a:1;b:5;c:6;d:7;e:2;f:3", host_only=True).info()
+    assert "a" not in [x["name"] for x in i["indices"]]                        # extent 1 dropped
+    i = tc.plan("abcd-ea-ebcd", "a:72;b:72;c:72;d:72;e:72", host_only=True, fusion=False).info()
+    assert len(i["indices"]) == 5
+
+
+@pytest.mark.parametrize("cost", ["b200", "paper"])
+def test_planner_invariants_tccg(cost):
+    for case in [tcinputs.eq1()] + tcinputs.tccg48():
+        i = tc.plan(case.expr, case.extents, host_only=True, cost=cost).info()
+        assert i["Mt"] <= i["BM"] and i["Nt"] <= i["BN"] and i["Kt"] <= i["BK"]
+        for x in i["indices"]:
+            assert 1 <= x["tile"] <= x["n"]
+        assert i["flops_padded"] >= i["flops"] * (1 - 1e-12)
+        assert i["stats"]["plan_ms"] < 200
+        # every index is on exactly one side (an index maps to one dimension)
+        names = i["m"] + i["n"] + i["k"]
+        assert sorted(names) == sorted(x["name"] for x in i["indices"])
+
+
+def test_paper_mode_eq1_config_space():
+    # SURVEY 8(a) worked fixture: eq. (1) at N = 16 with the V100 value sets of P:L176:
+    # TB_x {a:4|8|16} x REG_x {b:2|4|6|8} x TB_y {d:4|8|16} x REG_y {c:2|4|6|8}
+    # x TB_k {e:4|8|16 or f:4|8|16} = 3*4*3*4*6 = 864 raw configurations.
+    i = tc.plan("abcd-aebf-dfce", tcinputs.EQ1_EXTENTS, host_only=True, cost="paper").info()
+    assert i["stats"]["raw"] == 864
+    assert i["stats"]["pruned"] + i["stats"]["ranked"] == 864
+    assert i["stats"]["pruned"] > 0
+    assert i["paper_mapping"].startswith("TB_x=[a:")
+
+
+def test_forced_fig3_config():
+    # Fig. 3: N = 16, T_a = 16, T_e = 1, T_b = 4, T_f = 16, T_d = 4.
+    i = tc.plan("abcd-aebf-dfce", tcinputs.EQ1_EXTENTS, host_only=True,
+                force_tiles="a:16;e:1;b:4;f:16;d:4;c:1").info()
+    t = {x["name"]: x["tile"] for x in i["indices"]}
+    assert t == {"a": 16, "b": 4, "c": 1, "d": 4, "e": 1, "f": 16}
+    assert i["Mt"] == 64 and i["Nt"] == 4 and i["Kt"] == 16
+    assert i["nctas"] == 1 * 4 * 16 * 4 and i["nsteps"] == 16
+
+
+def test_forced_fig2_config():
+    # Fig. 2: T_a = T_b = T_c = T_d = 2 -> 16 C elements per thread block.
+    i = tc.plan("abcd-aebf-dfce", "a:2;b:2;c:2;d:2;e:2;f:2", host_only=True,
+                force_tiles="a:2;b:2;c:2;d:2;e:2;f:2").info()
+    assert i["Mt"] * i["Nt"] == 16 and i["nctas"] == 1
+
+
+def test_restrict_offsets_and_extents():
+    p = tc.plan("abcdef-gdab-efgc", "a:8;b:4;c:4;d:8;e:4;f:6;g:8", host_only=True, fusion=False)
+    s = p.restrict("f", 2, 3)
+    i = s.info()
+    assert {x["name"]: x["n"] for x in i["indices"]}["f"] == 3
+    # f is C's slowest index: C base = 2 * stride_C(f) = 2 * 8*4*4*8*4
+    assert i["tensors"]["C"]["base"] == 2 * 8 * 4 * 4 * 8 * 4
+    assert i["tensors"]["B"]["base"] == 2 * 4      # B = efgc: stride(f) = N_e
+    s2 = p.restrict("f", 2, 3, tc.SLAB_C)
+    assert s2.info()["tensors"]["C"]["base"] == 0
+    k = p.restrict("g", 0, 4)                      # split-K slab of the internal index
+    assert {x["name"]: x["n"] for x in k.info()["indices"]}["g"] == 4
+    with pytest.raises(tc.TcError):
+        p.restrict("f", 5, 3)
+    with pytest.raises(tc.TcError):
+        p.restrict("z", 0, 1)
+
+
+def test_plan_is_deterministic():
+    a = tc.plan("abcd-aebf-fdec", ";".join(f"{c}:72" for c in "abcdef"), host_only=True).info()
+    b = tc.plan("abcd-aebf-fdec", ";".join(f"{c}:72" for c in "abcdef"), host_only=True).info()
+    a["stats"].pop("plan_ms"); b["stats"].pop("plan_ms")
+    assert a == b
+
+
+def test_errors_are_status_codes():
+    with pytest.raises(tc.TcError) as e:
+        tc.plan("abcd-aebf-dfc", "a:2;b:2;c:2;d:2;e:2;f:2", host_only=True)
+    assert e.value.status == "TC_ERR_INDEX" and "exactly two" in e.value.detail
+    with pytest.raises(tc.TcError) as e:
+        tc.plan("ab-ac-cb", "a:2;b:2;c:2", dtype="bf16", host_only=True)
+    assert e.value.status == "TC_ERR_UNSUPPORTED"
+    p = tc.plan("ab-ac-cb", "a:2;b:2;c:2", host_only=True)
+    with pytest.raises(tc.TcError) as e:
+        p.execute_ptr(16, 32, 64)
+    assert e.value.status == "TC_ERR_CUDA"          # host_only plans cannot execute
