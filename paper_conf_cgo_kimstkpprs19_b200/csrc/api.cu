@@ -6,8 +6,6 @@
 #include <cmath>
 #include <cstdio>
 #include <cstring>
-#include <map>
-#include <memory>
 #include <new>
 #include <sstream>
 #include <string>
@@ -18,6 +16,7 @@
 #include "kernel_f64.cuh"
 #include "kparams.hpp"
 #include "planner.hpp"
+#include "tiles.hpp"
 
 using namespace tc;
 
@@ -36,29 +35,28 @@ struct KernelEntry {
   size_t smem;
 };
 
-template <int BM, int BN, int BK, int WM, int WN, int ST>
+template <int BM, int BN, int BK, int WM, int WN, int ST, int MINB>
 KernelEntry entry() {
   using K = F64Kernel<BM, BN, BK, WM, WN, ST>;
-  return {(const void *)&tc_f64_dmma_kernel<BM, BN, BK, WM, WN, ST>, K::THREADS, K::smem_bytes()};
+  return {(const void *)&tc_f64_dmma_kernel<BM, BN, BK, WM, WN, ST, MINB>, K::THREADS, K::smem_bytes()};
 }
 
 const std::vector<KernelEntry> &kernels() {
-  // must match planner.cpp variants() one-to-one
+  // one-to-one with tiles.cpp variants(): BM, BN, BK, WM, WN, stages, CTAs/SM
   static const std::vector<KernelEntry> k = {
-      entry<128, 128, 16, 64, 32, 4>(),
-      entry<128, 64, 16, 64, 32, 3>(),
-      entry<64, 128, 16, 32, 64, 3>(),
-      entry<64, 64, 16, 32, 32, 4>(),
-      entry<128, 128, 8, 64, 32, 4>(),
-      entry<64, 64, 8, 32, 32, 4>(),
+      entry<128, 128, 16, 64, 32, 4, 1>(),  // 0
+      entry<128, 64, 16, 64, 32, 3, 2>(),   // 1
+      entry<64, 128, 16, 32, 64, 3, 2>(),   // 2
+      entry<64, 64, 16, 32, 32, 4, 2>(),    // 3
+      entry<128, 128, 8, 64, 32, 4, 1>(),   // 4
+      entry<64, 64, 8, 32, 32, 4, 3>(),     // 5
+      entry<128, 32, 16, 32, 32, 4, 2>(),   // 6
+      entry<32, 128, 16, 32, 32, 4, 2>(),   // 7
+      entry<128, 32, 8, 32, 32, 4, 3>(),    // 8
+      entry<32, 128, 8, 32, 32, 4, 3>(),    // 9
   };
   return k;
 }
-
-struct DevTables {
-  void *buf = nullptr;
-  size_t bytes = 0;
-};
 
 }  // namespace
 
@@ -67,26 +65,25 @@ struct tc_plan_s {
   Contraction c;           // normalised (dropped extent-1 indices, fused runs)
   int dtype = 0;
   int device = -1;
+  int sms = 148;
   bool host_only = false;
   Config cfg;
   PlanStats stats;
   tc_plan_opts opts{};
   std::string force_tiles;
-  // host copies of the tables
-  std::vector<int64_t> stepX, stepY;
-  std::vector<uint64_t> kmask;
-  std::vector<uint32_t> slotX1, slotY1, slotX2, slotY2;
-  bool vecX_ok = false, vecY_ok = false;
-  KParams kp{};            // device pointers filled in; X/Y/C/alpha/beta set per call
-  DevTables dev;
-  // device pointers into dev.buf
-  const uint32_t *d_slotX1 = nullptr, *d_slotY1 = nullptr, *d_slotX2 = nullptr, *d_slotY2 = nullptr;
+  TileTables tt;
+  SlotTable slotX1, slotY1, slotX2, slotY2;
+  KParams kp{};            // device pointers filled in; X/Y/C/alpha/beta/slots set per call
+  void *dev = nullptr;     // one device buffer with every table
+  size_t dev_bytes = 0;
+  const int64_t *d_relX1 = nullptr, *d_relY1 = nullptr, *d_relX2 = nullptr, *d_relY2 = nullptr;
+  const uint32_t *d_packX1 = nullptr, *d_packY1 = nullptr, *d_packX2 = nullptr, *d_packY2 = nullptr;
   ~tc_plan_s() {
-    if (dev.buf) {
+    if (dev) {
       int cur = -1;
       cudaGetDevice(&cur);
       if (cur != device) cudaSetDevice(device);
-      cudaFree(dev.buf);
+      cudaFree(dev);
       if (cur != device && cur >= 0) cudaSetDevice(cur);
     }
   }
@@ -94,203 +91,102 @@ struct tc_plan_s {
 
 namespace {
 
-int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
-
-// Load slots of operand t (X or Y) in the operand's OWN memory order, packed
-// (mn << 8) | k.  vec = 2: the operand's FVI is stepped by 2 (16-B cp.async).
-std::vector<uint32_t> build_slots(const Contraction &c, const Config &cfg, int t, int vec,
-                                  const std::vector<int> &side) {
-  std::vector<uint32_t> out;
-  const auto &v = c.t[t];
-  const int r = (int)v.idx.size();
-  std::vector<int> T(r), mul(r), isk(r);
-  // multipliers of each index in the compute-order multi-index (side digits / k digits)
-  for (int p = 0; p < r; p++) {
-    const int id = v.idx[p];
-    T[p] = cfg.T[id];
-    isk[p] = c.ix[id].cls == INTL;
-    const auto &lst = isk[p] ? cfg.kdig : side;
-    int m = 1;
-    for (int q : lst) {
-      if (q == id) break;
-      m *= cfg.T[q];
-    }
-    mul[p] = m;
-  }
-  std::vector<int> d(r, 0);
-  for (;;) {
-    int mn = 0, k = 0;
-    for (int p = 0; p < r; p++) (isk[p] ? k : mn) += d[p] * mul[p];
-    out.push_back(((uint32_t)mn << 8) | (uint32_t)k);
-    int p = 0;
-    for (; p < r; p++) {
-      d[p] += (p == 0 ? vec : 1);
-      if (d[p] < T[p]) break;
-      d[p] = 0;
-    }
-    if (p == r) break;
-  }
-  return out;
-}
-
-// Can operand t use 16-B vectors?  Its FVI must be the leading digit of its smem-contiguous
-// dimension, with even tile and extent, stride 1, and every other stride / base even.
-bool vec_ok(const Contraction &c, const Config &cfg, int t, const std::vector<int> &side) {
-  const auto &v = c.t[t];
-  if (v.idx.empty() || v.stride[0] != 1) return false;
-  const int f = v.idx[0];
-  const bool isk = c.ix[f].cls == INTL;
-  const auto &lst = isk ? cfg.kdig : side;
-  if (lst.empty() || lst[0] != f) return false;
-  if (cfg.T[f] % 2 || c.ix[f].n % 2) return false;
-  for (size_t p = 1; p < v.stride.size(); p++) if (v.stride[p] % 2) return false;
-  return v.base % 2 == 0;
-}
-
-Status build_tables(tc_plan_s *P, std::string &err) {
+void build_host_tables(tc_plan_s *P) {
   const Contraction &c = P->c;
   const Config &cfg = P->cfg;
-  const Variant &var = variants()[cfg.variant];
+  const Variant &v = variants()[cfg.variant];
+  P->tt = build_tile_tables(c, cfg, v);
+  P->slotX1 = build_slots(c, cfg, cfg.X, 1, cfg.xKmajor, v.BM, v.BK);
+  P->slotY1 = build_slots(c, cfg, cfg.Y, 1, cfg.yKmajor, v.BN, v.BK);
+  if (cfg.vecX == 2) P->slotX2 = build_slots(c, cfg, cfg.X, 2, cfg.xKmajor, v.BM, v.BK);
+  if (cfg.vecY == 2) P->slotY2 = build_slots(c, cfg, cfg.Y, 2, cfg.yKmajor, v.BN, v.BK);
   KParams &kp = P->kp;
   std::memset(&kp, 0, sizeof(kp));
-  const int X = cfg.X, Y = cfg.Y;
-  kp.baseX = c.t[X].base;
-  kp.baseY = c.t[Y].base;
-  kp.baseC = c.t[0].base;
-  auto side = [&](SideDesc &sd, const std::vector<int> &dig, int op) {
-    sd.nd = (int)dig.size();
-    sd.tiles = 1;
-    for (int i = 0; i < sd.nd; i++) {
-      const int id = dig[i];
-      sd.T[i] = cfg.T[id];
-      sd.N[i] = c.ix[id].n;
-      sd.ntile[i] = cdiv(c.ix[id].n, cfg.T[id]);
-      sd.sOp[i] = c.stride_of(op, id);
-      sd.sC[i] = c.stride_of(0, id);
-      sd.tiles *= sd.ntile[i];
-    }
-  };
-  if ((int)cfg.mdig.size() > kMaxDigits || (int)cfg.ndig.size() > kMaxDigits) {
-    err = "too many digits";
-    return ST_UNSUPPORTED;
-  }
-  side(kp.m, cfg.mdig, X);
-  side(kp.n, cfg.ndig, Y);
-  kp.nctas = kp.m.tiles * kp.n.tiles;
+  kp.mtiles = (int)cfg.mtiles;
+  kp.ntiles = (int)cfg.ntiles;
+  kp.ntotal = (int)cfg.nctas;
   kp.group_m = 8;
-  // k side
-  const int nk = (int)cfg.kdig.size();
-  std::vector<int64_t> kt(nk), kn(nk);
-  int64_t steps = 1;
-  for (int i = 0; i < nk; i++) {
-    kn[i] = c.ix[cfg.kdig[i]].n;
-    kt[i] = cfg.T[cfg.kdig[i]];
-    steps *= cdiv(kn[i], kt[i]);
-  }
-  if (steps > (1LL << 30)) { err = "too many k steps"; return ST_UNSUPPORTED; }
-  kp.nsteps = (int)steps;
-  for (int k = 0; k < 64; k++) { kp.relKX[k] = 0; kp.relKY[k] = 0; }
-  const int Kt = (int)cfg.Kt;
-  for (int k = 0; k < Kt && k < 64; k++) {
-    int q = k;
-    for (int i = 0; i < nk; i++) {
-      const int d = q % (int)kt[i];
-      q /= (int)kt[i];
-      kp.relKX[k] += d * c.stride_of(X, cfg.kdig[i]);
-      kp.relKY[k] += d * c.stride_of(Y, cfg.kdig[i]);
-    }
-  }
-  P->stepX.resize(steps);
-  P->stepY.resize(steps);
-  P->kmask.resize(steps);
-  std::vector<int64_t> cd(nk, 0);
-  for (int64_t s = 0; s < steps; s++) {
-    int64_t bx = 0, by = 0;
-    for (int i = 0; i < nk; i++) {
-      bx += cd[i] * kt[i] * c.stride_of(X, cfg.kdig[i]);
-      by += cd[i] * kt[i] * c.stride_of(Y, cfg.kdig[i]);
-    }
-    uint64_t mask = 0;
-    for (int k = 0; k < Kt; k++) {
-      int q = k;
-      bool ok = true;
-      for (int i = 0; i < nk; i++) {
-        const int d = q % (int)kt[i];
-        q /= (int)kt[i];
-        ok &= cd[i] * kt[i] + d < kn[i];
-      }
-      if (ok) mask |= 1ull << k;
-    }
-    P->stepX[s] = bx;
-    P->stepY[s] = by;
-    P->kmask[s] = mask;
-    for (int i = 0; i < nk; i++) {
-      if (++cd[i] < cdiv(kn[i], kt[i])) break;
-      cd[i] = 0;
-    }
-  }
-  // smem layouts: k-contiguous iff the operand's FVI is internal
-  kp.xKmajor = !c.t[X].idx.empty() && c.ix[c.t[X].idx[0]].cls == INTL;
-  kp.yKmajor = !c.t[Y].idx.empty() && c.ix[c.t[Y].idx[0]].cls == INTL;
-  P->slotX1 = build_slots(c, cfg, X, 1, cfg.mdig);
-  P->slotY1 = build_slots(c, cfg, Y, 1, cfg.ndig);
-  P->vecX_ok = vec_ok(c, cfg, X, cfg.mdig);
-  P->vecY_ok = vec_ok(c, cfg, Y, cfg.ndig);
-  if (P->vecX_ok) P->slotX2 = build_slots(c, cfg, X, 2, cfg.mdig);
-  if (P->vecY_ok) P->slotY2 = build_slots(c, cfg, Y, 2, cfg.ndig);
-  (void)var;
-  return ST_OK;
+  kp.Mt = (int)cfg.Mt;
+  kp.Nt = (int)cfg.Nt;
+  kp.fullM = P->tt.fullM;
+  kp.fullN = P->tt.fullN;
+  kp.nsteps = (int)cfg.nsteps;
+  kp.xKmajor = cfg.xKmajor;
+  kp.yKmajor = cfg.yKmajor;
 }
 
 Status upload(tc_plan_s *P, std::string &err) {
-  // one device buffer: stepX | stepY | kmask | slotX1 | slotY1 | slotX2 | slotY2
-  size_t off[8];
+  struct Part { const void *src; size_t bytes; size_t off; };
+  std::vector<Part> parts;
   size_t o = 0;
-  auto al = [](size_t x) { return (x + 255) & ~(size_t)255; };
-  off[0] = o; o = al(o + 8 * P->stepX.size());
-  off[1] = o; o = al(o + 8 * P->stepY.size());
-  off[2] = o; o = al(o + 8 * P->kmask.size());
-  off[3] = o; o = al(o + 4 * P->slotX1.size());
-  off[4] = o; o = al(o + 4 * P->slotY1.size());
-  off[5] = o; o = al(o + 4 * P->slotX2.size());
-  off[6] = o; o = al(o + 4 * P->slotY2.size());
-  off[7] = o;
-  std::vector<char> h(o, 0);
-  std::memcpy(h.data() + off[0], P->stepX.data(), 8 * P->stepX.size());
-  std::memcpy(h.data() + off[1], P->stepY.data(), 8 * P->stepY.size());
-  std::memcpy(h.data() + off[2], P->kmask.data(), 8 * P->kmask.size());
-  std::memcpy(h.data() + off[3], P->slotX1.data(), 4 * P->slotX1.size());
-  std::memcpy(h.data() + off[4], P->slotY1.data(), 4 * P->slotY1.size());
-  if (!P->slotX2.empty()) std::memcpy(h.data() + off[5], P->slotX2.data(), 4 * P->slotX2.size());
-  if (!P->slotY2.empty()) std::memcpy(h.data() + off[6], P->slotY2.data(), 4 * P->slotY2.size());
-  cudaError_t e = cudaMalloc(&P->dev.buf, o);
+  auto add = [&](const void *src, size_t bytes) {
+    parts.push_back({src, bytes, o});
+    o = (o + bytes + 255) & ~(size_t)255;
+    return parts.size() - 1;
+  };
+  const TileTables &tt = P->tt;
+  size_t iM = add(tt.tileM.data(), sizeof(TileInfo) * tt.tileM.size());
+  size_t iN = add(tt.tileN.data(), sizeof(TileInfo) * tt.tileN.size());
+  size_t iRm = add(tt.relCm.data(), 8 * tt.relCm.size());
+  size_t iRn = add(tt.relCn.data(), 8 * tt.relCn.size());
+  size_t iDm = add(tt.digM.data(), 8 * tt.digM.size());
+  size_t iDn = add(tt.digN.data(), 8 * tt.digN.size());
+  size_t iSx = add(tt.stepX.data(), 8 * tt.stepX.size());
+  size_t iSy = add(tt.stepY.data(), 8 * tt.stepY.size());
+  size_t iK = add(tt.kmask.data(), 8 * tt.kmask.size());
+  size_t iX1 = add(P->slotX1.rel.data(), 8 * P->slotX1.rel.size());
+  size_t iX1p = add(P->slotX1.pack.data(), 4 * P->slotX1.pack.size());
+  size_t iY1 = add(P->slotY1.rel.data(), 8 * P->slotY1.rel.size());
+  size_t iY1p = add(P->slotY1.pack.data(), 4 * P->slotY1.pack.size());
+  size_t iX2 = add(P->slotX2.rel.data(), 8 * P->slotX2.rel.size());
+  size_t iX2p = add(P->slotX2.pack.data(), 4 * P->slotX2.pack.size());
+  size_t iY2 = add(P->slotY2.rel.data(), 8 * P->slotY2.rel.size());
+  size_t iY2p = add(P->slotY2.pack.data(), 4 * P->slotY2.pack.size());
+  std::vector<char> h(o + 256, 0);
+  for (auto &p : parts) if (p.bytes) std::memcpy(h.data() + p.off, p.src, p.bytes);
+  cudaError_t e = cudaMalloc(&P->dev, h.size());
   if (e != cudaSuccess) { err = std::string("cudaMalloc: ") + cudaGetErrorString(e); return ST_ALLOC; }
-  P->dev.bytes = o;
-  e = cudaMemcpy(P->dev.buf, h.data(), o, cudaMemcpyHostToDevice);
+  P->dev_bytes = h.size();
+  e = cudaMemcpy(P->dev, h.data(), h.size(), cudaMemcpyHostToDevice);
   if (e != cudaSuccess) { err = std::string("cudaMemcpy: ") + cudaGetErrorString(e); return ST_CUDA; }
-  char *b = (char *)P->dev.buf;
-  P->kp.stepX = (const int64_t *)(b + off[0]);
-  P->kp.stepY = (const int64_t *)(b + off[1]);
-  P->kp.kmask = (const uint64_t *)(b + off[2]);
-  P->d_slotX1 = (const uint32_t *)(b + off[3]);
-  P->d_slotY1 = (const uint32_t *)(b + off[4]);
-  P->d_slotX2 = (const uint32_t *)(b + off[5]);
-  P->d_slotY2 = (const uint32_t *)(b + off[6]);
+  char *b = (char *)P->dev;
+  KParams &kp = P->kp;
+  kp.tileM = (const TileInfo *)(b + parts[iM].off);
+  kp.tileN = (const TileInfo *)(b + parts[iN].off);
+  kp.relCm = (const int64_t *)(b + parts[iRm].off);
+  kp.relCn = (const int64_t *)(b + parts[iRn].off);
+  kp.digM = (const uint64_t *)(b + parts[iDm].off);
+  kp.digN = (const uint64_t *)(b + parts[iDn].off);
+  kp.stepX = (const int64_t *)(b + parts[iSx].off);
+  kp.stepY = (const int64_t *)(b + parts[iSy].off);
+  kp.kmask = (const uint64_t *)(b + parts[iK].off);
+  P->d_relX1 = (const int64_t *)(b + parts[iX1].off);
+  P->d_packX1 = (const uint32_t *)(b + parts[iX1p].off);
+  P->d_relY1 = (const int64_t *)(b + parts[iY1].off);
+  P->d_packY1 = (const uint32_t *)(b + parts[iY1p].off);
+  P->d_relX2 = (const int64_t *)(b + parts[iX2].off);
+  P->d_packX2 = (const uint32_t *)(b + parts[iX2p].off);
+  P->d_relY2 = (const int64_t *)(b + parts[iY2].off);
+  P->d_packY2 = (const uint32_t *)(b + parts[iY2p].off);
   const KernelEntry &ke = kernels()[P->cfg.variant];
   e = cudaFuncSetAttribute(ke.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ke.smem);
   if (e != cudaSuccess) { err = std::string("cudaFuncSetAttribute: ") + cudaGetErrorString(e); return ST_CUDA; }
+  int occ = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ke.fn, ke.threads, ke.smem);
+  if (e != cudaSuccess || occ < 1) { err = "kernel variant cannot be resident"; return ST_CUDA; }
+  cudaDeviceGetAttribute(&P->sms, cudaDevAttrMultiProcessorCount, P->device);
+  P->sms *= std::min(occ, variants()[P->cfg.variant].occ);
   return ST_OK;
 }
 
 bool parse_force(const char *s, ForcedTiles &ft) {
   ft.on = s != nullptr;
   if (!s) return true;
-  std::string str(s);
-  std::stringstream ss(str);
+  std::stringstream ss{std::string(s)};
   std::string item;
   while (std::getline(ss, item, ';')) {
-    auto p = item.find(':');
     if (item.find_first_not_of(" \t") == std::string::npos) continue;
+    auto p = item.find(':');
     if (p == std::string::npos) return false;
     std::string k = item.substr(0, p);
     k.erase(0, k.find_first_not_of(" \t"));
@@ -306,21 +202,16 @@ bool parse_force(const char *s, ForcedTiles &ft) {
 
 tc_status_t finish_plan(tc_plan_s *P, tc_plan_t *out) {
   std::string err;
-  P->c = P->parsed;
-  normalize(P->c, !P->opts.no_fusion);
   ForcedTiles ft;
   if (!parse_force(P->opts.force_tiles, ft)) { delete P; return fail(ST_INVALID_ARG, "malformed force_tiles"); }
-  if (ft.on && !P->opts.no_fusion) {
-    // forced tiles name the original indices: plan without fusion so names survive
-    P->c = P->parsed;
-    normalize(P->c, false);
-  }
-  int fv = P->opts.variant > 0 ? P->opts.variant - 1 : -1;
+  // forced tiles name the original indices: plan without fusion so the names survive
+  P->c = P->parsed;
+  normalize(P->c, !P->opts.no_fusion && !ft.on);
+  const int fv = P->opts.variant > 0 ? P->opts.variant - 1 : -1;
   if (fv >= (int)variants().size()) { delete P; return fail(ST_INVALID_ARG, "variant out of range"); }
   Status s = choose(P->c, P->opts.cost_mode, fv, ft, P->cfg, P->stats, err);
   if (s != ST_OK) { delete P; return fail(s, err); }
-  s = build_tables(P, err);
-  if (s != ST_OK) { delete P; return fail(s, err); }
+  build_host_tables(P);
   if (!P->host_only) {
     if (cudaGetDevice(&P->device) != cudaSuccess) {
       cudaGetLastError();
@@ -343,7 +234,7 @@ bool overlaps(const void *a, size_t na, const void *b, size_t nb) {
 
 extern "C" {
 
-const char *tc_version(void) { return "libtc 0.1 (sm_100a, FP64 DMMA)"; }
+const char *tc_version(void) { return "libtc 0.2 (sm_100a, FP64 DMMA, persistent)"; }
 
 const char *tc_status_string(tc_status_t s) {
   switch (s) {
@@ -458,35 +349,35 @@ tc_status_t tc_plan_restrict(tc_plan_t *sub, const tc_plan_t parent, const char 
 tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void *C, double alpha,
                        double beta, tc_stream_t stream) {
   if (!plan || !A || !B || !C) return fail(ST_INVALID_ARG, "NULL plan or tensor pointer");
-  if (plan->host_only || !plan->dev.buf) return fail(ST_CUDA, "plan was made host_only");
-  const Contraction &c = plan->c;
-  const size_t es = 8;
-  const size_t nA = (size_t)plan->parsed.span(1) * es, nB = (size_t)plan->parsed.span(2) * es,
-               nC = (size_t)plan->parsed.span(0) * es;
+  if (plan->host_only || !plan->dev) return fail(ST_CUDA, "plan was made host_only");
+  const size_t nA = (size_t)plan->parsed.span(1) * 8, nB = (size_t)plan->parsed.span(2) * 8,
+               nC = (size_t)plan->parsed.span(0) * 8;
   if (overlaps(C, nC, A, nA) || overlaps(C, nC, B, nB)) return fail(ST_INVALID_ARG, "C overlaps A or B");
   int cur = -1;
   if (cudaGetDevice(&cur) != cudaSuccess || cur != plan->device)
     return fail(ST_INVALID_ARG, "current device differs from the plan's device");
   KParams kp = plan->kp;
-  const int X = plan->cfg.X;
-  kp.X = X == 1 ? A : B;
-  kp.Y = X == 1 ? B : A;
+  const Config &cfg = plan->cfg;
+  kp.X = cfg.X == 1 ? A : B;
+  kp.Y = cfg.X == 1 ? B : A;
   kp.C = C;
   kp.alpha = alpha;
   kp.beta = beta;
-  const bool ax = ((uintptr_t)kp.X % 16) == 0, ay = ((uintptr_t)kp.Y % 16) == 0;
-  const bool vx = plan->vecX_ok && ax, vy = plan->vecY_ok && ay;
-  kp.slotX = vx ? plan->d_slotX2 : plan->d_slotX1;
-  kp.nslotX = (int)(vx ? plan->slotX2.size() : plan->slotX1.size());
+  // 16-B vectors need 16-B aligned operands; otherwise the scalar slot tables run
+  const bool vx = cfg.vecX == 2 && ((uintptr_t)kp.X % 16) == 0;
+  const bool vy = cfg.vecY == 2 && ((uintptr_t)kp.Y % 16) == 0;
+  kp.relX = vx ? plan->d_relX2 : plan->d_relX1;
+  kp.packX = vx ? plan->d_packX2 : plan->d_packX1;
+  kp.nslotX = (int)(vx ? plan->slotX2.pack.size() : plan->slotX1.pack.size());
   kp.vecX = vx ? 2 : 1;
-  kp.slotY = vy ? plan->d_slotY2 : plan->d_slotY1;
-  kp.nslotY = (int)(vy ? plan->slotY2.size() : plan->slotY1.size());
+  kp.relY = vy ? plan->d_relY2 : plan->d_relY1;
+  kp.packY = vy ? plan->d_packY2 : plan->d_packY1;
+  kp.nslotY = (int)(vy ? plan->slotY2.pack.size() : plan->slotY1.pack.size());
   kp.vecY = vy ? 2 : 1;
-  (void)c;
-  const KernelEntry &ke = kernels()[plan->cfg.variant];
+  const KernelEntry &ke = kernels()[cfg.variant];
+  const int grid = (int)std::min<int64_t>(cfg.nctas, plan->sms);
   void *args[] = {&kp};
-  cudaError_t e = cudaLaunchKernel(ke.fn, dim3((unsigned)kp.nctas), dim3(ke.threads), args, ke.smem,
-                                   (cudaStream_t)stream);
+  cudaError_t e = cudaLaunchKernel(ke.fn, dim3(grid), dim3(ke.threads), args, ke.smem, (cudaStream_t)stream);
   if (e != cudaSuccess) return fail(ST_CUDA, std::string("launch: ") + cudaGetErrorString(e));
   return TC_SUCCESS;
 }
@@ -548,12 +439,14 @@ tc_status_t tc_plan_info(const tc_plan_t plan, char *json, size_t cap, size_t *n
       o << "],\"base\":" << c.t[t].base << "}";
     }
     o << "},\"m\":" << names(g.mdig) << ",\"n\":" << names(g.ndig) << ",\"k\":" << names(g.kdig);
+    o << ",\"morder\":" << g.morder << ",\"korder\":" << g.korder;
     o << ",\"variant\":" << g.variant << ",\"BM\":" << v.BM << ",\"BN\":" << v.BN << ",\"BK\":" << v.BK
       << ",\"threads\":" << v.threads << ",\"stages\":" << v.stages << ",\"occ\":" << v.occ;
     o << ",\"Mt\":" << g.Mt << ",\"Nt\":" << g.Nt << ",\"Kt\":" << g.Kt << ",\"nctas\":" << g.nctas
-      << ",\"nsteps\":" << g.nsteps;
-    o << ",\"vecX\":" << (plan->vecX_ok ? 2 : 1) << ",\"vecY\":" << (plan->vecY_ok ? 2 : 1)
-      << ",\"xKmajor\":" << plan->kp.xKmajor << ",\"yKmajor\":" << plan->kp.yKmajor;
+      << ",\"mtiles\":" << g.mtiles << ",\"ntiles\":" << g.ntiles << ",\"nsteps\":" << g.nsteps
+      << ",\"grid\":" << std::min<int64_t>(g.nctas, plan->sms);
+    o << ",\"vecX\":" << g.vecX << ",\"vecY\":" << g.vecY << ",\"xKmajor\":" << g.xKmajor
+      << ",\"yKmajor\":" << g.yKmajor << ",\"wfX\":" << g.wfX << ",\"wfY\":" << g.wfY;
     char buf[512];
     std::snprintf(buf, sizeof buf,
                   ",\"t_pred_ms\":%.6g,\"t_comp_ms\":%.6g,\"t_mem_ms\":%.6g,\"t_l2_ms\":%.6g,"

@@ -5,35 +5,18 @@
 #include <algorithm>
 #include <chrono>
 #include <cmath>
+#include <map>
 #include <set>
-#include <sstream>
 
 namespace tc {
 
 // ---------------------------------------------------------------- hardware constants
-// B200, measured in profiles/r01_peaks.json (DMMA 37.1 TFLOP/s = 148 SM x 64 FMA/clk x
-// 2 x 1.965 GHz; HBM read 7.36 TB/s, write 6.7 TB/s, copy 6.55 TB/s MEASURED_PEAKS).
+// B200, measured (profiles/r01_peaks.json): DMMA 37.1 TFLOP/s = 148 SMs x 64 FMA/clk x 2 x
+// 1.965 GHz; HBM read 7.36 TB/s, f64 write 6.7 TB/s, copy 6.55 TB/s (MEASURED_PEAKS.json).
 static constexpr double kSMs = 148, kFmaPerClk = 64, kClk = 1.965e9;
-static constexpr double kHbm = 6.5e12, kL2Bw = 10.0e12, kL2Bytes = 126.0e6;
+static constexpr double kHbm = 6.5e12, kL2Bw = 12.0e12, kL2Bytes = 126.0e6;
 static constexpr double kLaunch = 3.0e-6;
-
-const std::vector<Variant> &variants() {
-  // BM, BN, BK, WM, WN, stages, threads, CTAs/SM (from ptxas registers and smem)
-  static const std::vector<Variant> v = {
-      {128, 128, 16, 64, 32, 4, 256, 1},
-      {128, 64, 16, 64, 32, 3, 128, 2},
-      {64, 128, 16, 32, 64, 3, 128, 2},
-      {64, 64, 16, 32, 32, 4, 128, 2},
-      {128, 128, 8, 64, 32, 4, 256, 1},
-      {64, 64, 8, 32, 32, 4, 128, 3},
-  };
-  return v;
-}
-
-int x_tensor(const Contraction &c) {
-  if (c.t[0].idx.empty()) return 1;
-  return c.pos_in(1, c.t[0].idx[0]) >= 0 ? 1 : 2;
-}
+static constexpr double kStepOverhead = 60;   // cycles per k-step: barrier + bookkeeping
 
 static int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
@@ -57,46 +40,66 @@ static double sector_eff(int64_t run) {
   return b / (std::ceil(b / 32.0) * 32.0);
 }
 
+// Simulated cp.async wavefronts of operand t, memoised on everything the slot table depends
+// on (the operand's tiles, digit orders, layout, vector width, tile shape).
+static double operand_wavefronts(const Contraction &c, const Config &cfg, int t, int vec, bool kmaj,
+                                 int BMN, int BK, WfCache *cache) {
+  std::vector<int64_t> key{t, vec, kmaj, BMN, BK, cfg.morder, cfg.korder};
+  for (int id : c.t[t].idx) key.push_back(cfg.T[id]);
+  for (int id : cfg.kdig) key.push_back(cfg.T[id]);
+  if (cache) {
+    auto it = cache->find(key);
+    if (it != cache->end()) return it->second;
+  }
+  const double wf = slot_wavefronts(build_slots(c, cfg, t, vec, kmaj, BMN, BK), vec);
+  if (cache) (*cache)[key] = wf;
+  return wf;
+}
+
 // ---------------------------------------------------------------- B200 cost model
-double model_time(const Contraction &c, const Config &cfg, const Variant &v, double *comp,
-                  double *mem, double *l2, double *dram) {
-  const auto &T = cfg.T;
-  int64_t mt = 1, nt = 1, steps = 1;
-  for (int id : cfg.mdig) mt *= cdiv(c.ix[id].n, T[id]);
-  for (int id : cfg.ndig) nt *= cdiv(c.ix[id].n, T[id]);
-  for (int id : cfg.kdig) steps *= cdiv(c.ix[id].n, T[id]);
-  const double nctas = (double)mt * nt;
-  // FP64 pipe time of the PADDED work, quantised to waves of 148 * occ CTAs
+double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *cache) {
+  finish_counts(c, cfg);
+  const double nctas = (double)cfg.nctas, steps = (double)cfg.nsteps;
+  // per CTA-step pipe cycles on one SM: FP64 (DMMA) and shared memory
+  const double dmma = (double)v.BM * v.BN * v.BK / kFmaPerClk;
+  cfg.vecX = vec_possible(c, cfg, cfg.X) ? 2 : 1;
+  cfg.vecY = vec_possible(c, cfg, cfg.Y) ? 2 : 1;
+  cfg.wfX = operand_wavefronts(c, cfg, cfg.X, cfg.vecX, cfg.xKmajor, v.BM, v.BK, cache);
+  cfg.wfY = operand_wavefronts(c, cfg, cfg.Y, cfg.vecY, cfg.yKmajor, v.BN, v.BK, cache);
+  const int MI = v.WM / 8, NJ = v.WN / 8, warps = v.threads / 32;
+  const double lds = (double)warps * (v.BK / 4) * (MI + NJ) * 2;
+  const double step = std::max(dmma, cfg.wfX + cfg.wfY + lds) + kStepOverhead;
+  const double epi = (double)warps * MI * NJ * 2 * 8 / 4;     // store issue per tile
+  // persistent CTAs: grid = 148 * occ, tiles round-robin
   const double slots = kSMs * v.occ;
-  const double waves = std::ceil(nctas / slots);
-  const double fma_cta = (double)steps * v.BM * v.BN * v.BK;
-  const double t_comp = waves * v.occ * fma_cta / (kFmaPerClk * kClk);
-  // sector efficiencies of each tensor's tile along its own memory order
-  const double eX = sector_eff(contiguous_run(c, cfg.X, T));
-  const double eY = sector_eff(contiguous_run(c, cfg.Y, T));
-  const double eC = sector_eff(contiguous_run(c, 0, T));
-  // L2 -> SM traffic: every CTA streams its X and Y slabs
-  const double Mt = (double)cfg.Mt, Nt = (double)cfg.Nt, Kt = (double)cfg.Kt;
-  const double l2b = nctas * steps * 8.0 * (Mt * Kt / eX + Kt * Nt / eY);
-  const double t_l2 = l2b / kL2Bw;
-  // DRAM: inputs once if they stay in L2, otherwise re-read per tile row / column
+  const double tiles_per_cta = std::ceil(nctas / slots);
+  const double cyc_sm = tiles_per_cta * v.occ * (steps * step + epi);
+  cfg.t_comp = cyc_sm / kClk;
+  // memory: sector efficiencies of each tensor's tile along its own memory order
+  const double eX = sector_eff(contiguous_run(c, cfg.X, cfg.T));
+  const double eY = sector_eff(contiguous_run(c, cfg.Y, cfg.T));
+  const double eC = sector_eff(contiguous_run(c, 0, cfg.T));
+  // store-instruction efficiency: 8 consecutive rows of a DMMA fragment are contiguous in C
+  // iff m's first digit is C's FVI
+  double eS = 0.25;
+  if (c.t[0].idx.empty()) eS = 1;
+  else if (!cfg.mdig.empty() && cfg.mdig[0] == c.t[0].idx[0])
+    eS = sector_eff(std::min<int64_t>(8, cfg.T[cfg.mdig[0]]));
   const double bx = 8.0 * c.numel(cfg.X), by = 8.0 * c.numel(cfg.Y), bc = 8.0 * c.numel(0);
   double rx = 1, ry = 1;
   if (bx + by > 0.5 * kL2Bytes) {
     const double f = (bx + by) / kL2Bytes;
-    rx = std::min((double)nt, 1.0 + f);
-    ry = std::min((double)mt, 1.0 + f);
+    rx = std::min((double)cfg.ntiles, 1.0 + f);
+    ry = std::min((double)cfg.mtiles, 1.0 + f);
   }
-  const double d = bx * rx / eX + by * ry / eY + bc / eC;
-  const double t_mem = d / kHbm;
-  // with one CTA per SM the C store of a tile is not overlapped by MMA work
-  const double t_store = (bc / eC) / kHbm / std::max(1, v.occ);
-  double t = std::max({t_comp + t_store, t_mem, t_l2}) + kLaunch;
-  if (comp) *comp = t_comp;
-  if (mem) *mem = t_mem;
-  if (l2) *l2 = t_l2;
-  if (dram) *dram = d;
-  return t;
+  cfg.dram_bytes = bx * rx / eX + by * ry / eY + bc / eC;
+  cfg.t_mem = cfg.dram_bytes / kHbm;
+  const double l2b = nctas * steps * 8.0 * ((double)cfg.Mt * cfg.Kt / eX + (double)cfg.Kt * cfg.Nt / eY) +
+                     bc / eS;
+  cfg.t_l2 = l2b / kL2Bw;
+  cfg.flops_pad = 2.0 * nctas * steps * v.BM * v.BN * v.BK;
+  cfg.t_pred = std::max({cfg.t_comp, cfg.t_mem, cfg.t_l2}) + kLaunch;
+  return cfg.t_pred;
 }
 
 // ---------------------------------------------------------------- Alg. 3 (paper mode)
@@ -142,9 +145,9 @@ int64_t pow2_le(int64_t x) {
   return p;
 }
 
-// Crossing-tile candidates when index of extent n overshoots the target: P:L218 uses
-// floor(target/prev) (R12); we add the largest divisor of n and the largest power of two
-// not above it, which avoid partial tiles / keep vector alignment.
+// Crossing-tile candidates when an index of extent n overshoots the target: P:L218 uses
+// floor(target/prev) (R12); the B200 mode adds the largest divisor of n and the largest
+// power of two not above it (no partial tiles / vector alignment).
 std::vector<int64_t> crossing(int64_t n, int64_t cap, bool paper) {
   std::vector<int64_t> v{std::max<int64_t>(1, cap)};
   if (!paper) {
@@ -191,13 +194,13 @@ std::vector<std::vector<int>> rotations(const std::vector<int> &lst) {
     v.insert(v.end(), lst.begin(), lst.begin() + s);
     r.push_back(v);
   }
-  if (r.empty()) r.push_back({});
+  if (r.empty()) r.push_back(std::vector<int>());
   return r;
 }
 
-// Two-level enumeration (TB then REG) for one side of the B200 kernel:
-// the first index of each rotation gets a first-level tile from the power-of-two targets,
-// the rest are filled greedily up to the side's total target S.
+// Two-level enumeration (TB then REG) for one side of the B200 kernel: the
+// first index of each rotation gets a first-level tile from the power-of-two targets, the
+// rest are filled greedily up to the side's total target S.
 std::vector<Tiling> enum_side(const Contraction &c, const std::vector<int> &order, int fixed_first,
                               int64_t S) {
   std::set<Tiling> uniq;
@@ -214,24 +217,18 @@ std::vector<Tiling> enum_side(const Contraction &c, const std::vector<int> &orde
     rots = rotations(order);
   }
   for (auto &seq : rots) {
-    if (seq.empty()) { uniq.insert(Tiling{}); continue; }
+    if (seq.empty()) { uniq.insert(Tiling()); continue; }
     const int first = seq[0];
     const int64_t n0 = c.ix[first].n;
     std::set<int64_t> t0s;
-    for (int64_t s1 = 1; s1 <= S; s1 *= 2) {
+    for (int64_t s1 = 1; s1 <= S; s1 *= 2)
       for (int64_t t : crossing(n0, s1, false)) t0s.insert(std::min(t, n0));
-    }
     t0s.insert(std::min(n0, S));
     for (int64_t t0 : t0s) {
       Tiling cur{{first, (int)t0}};
       std::vector<Tiling> res;
-      if (t0 < n0) {
-        res.push_back(cur);  // first index alone (others tile 1)
-        // plus filling the rest on top (TB then REG)
-        greedy(c, seq, 1, t0, S, cur, false, res);
-      } else {
-        greedy(c, seq, 1, t0, S, cur, false, res);
-      }
+      if (t0 < n0) res.push_back(cur);  // first index alone (the others on the grid)
+      greedy(c, seq, 1, t0, S, cur, false, res);
       for (auto &x : res) uniq.insert(x);
     }
   }
@@ -254,65 +251,55 @@ std::string tiling_str(const Contraction &c, const Tiling &t) {
   return "[" + s + "]";
 }
 
-}  // namespace
-
-// Compute-order digit lists (kparams.hpp): m = C's indices in X, n = C's indices in Y (both
-// in C order, so C's FVI leads m); k = internals with an input's FVI first.
-static void digit_orders(const Contraction &c, Config &cfg) {
-  cfg.X = x_tensor(c);
-  cfg.Y = 3 - cfg.X;
-  cfg.mdig.clear(); cfg.ndig.clear(); cfg.kdig.clear();
-  for (int id : c.t[0].idx) (c.pos_in(cfg.X, id) >= 0 ? cfg.mdig : cfg.ndig).push_back(id);
-  int first = -1;
-  const auto &xv = c.t[cfg.X].idx, &yv = c.t[cfg.Y].idx;
-  if (!xv.empty() && c.ix[xv[0]].cls == INTL) first = xv[0];
-  else if (!yv.empty() && c.ix[yv[0]].cls == INTL) first = yv[0];
-  if (first >= 0) cfg.kdig.push_back(first);
-  for (int id : xv)
-    if (c.ix[id].cls == INTL && id != first) cfg.kdig.push_back(id);
-}
-
-static void finish(const Contraction &c, Config &cfg) {
-  cfg.Mt = cfg.Nt = cfg.Kt = 1;
-  cfg.nctas = 1;
-  cfg.nsteps = 1;
-  for (int id : cfg.mdig) { cfg.Mt *= cfg.T[id]; cfg.nctas *= cdiv(c.ix[id].n, cfg.T[id]); }
-  for (int id : cfg.ndig) { cfg.Nt *= cfg.T[id]; cfg.nctas *= cdiv(c.ix[id].n, cfg.T[id]); }
-  for (int id : cfg.kdig) { cfg.Kt *= cfg.T[id]; cfg.nsteps *= cdiv(c.ix[id].n, cfg.T[id]); }
-}
-
-static bool better(const Config &a, const Config &b) {
-  // deterministic: cost, then more CTAs, then larger tile, then variant id
+bool better(const Config &a, const Config &b) {
+  // deterministic: cost, then more CTAs, then larger tile, then variant / order ids
   if (a.t_pred != b.t_pred) return a.t_pred < b.t_pred;
   if (a.nctas != b.nctas) return a.nctas > b.nctas;
   if (a.Mt * a.Nt != b.Mt * b.Nt) return a.Mt * a.Nt > b.Mt * b.Nt;
-  return a.variant < b.variant;
+  if (a.variant != b.variant) return a.variant < b.variant;
+  if (a.morder != b.morder) return a.morder < b.morder;
+  return a.korder < b.korder;
 }
 
-static void evaluate(const Contraction &c, Config &cfg, int vi) {
-  cfg.variant = vi;
-  finish(c, cfg);
-  cfg.t_pred = model_time(c, cfg, variants()[vi], &cfg.t_comp, &cfg.t_mem, &cfg.t_l2, &cfg.dram_bytes);
-  const auto &v = variants()[vi];
-  cfg.flops_pad = 2.0 * (double)cfg.nctas * cfg.nsteps * v.BM * v.BN * v.BK;
+bool fits(const Config &cfg, const Variant &v) {
+  return cfg.Mt <= v.BM && cfg.Nt <= v.BN && cfg.Kt <= v.BK && cfg.nctas < (1LL << 31) &&
+         cfg.mtiles < (1LL << 24) && cfg.ntiles < (1LL << 24) && cfg.nsteps < (1LL << 24);
 }
 
-static bool fits(const Config &cfg, const Variant &v) {
-  return cfg.Mt <= v.BM && cfg.Nt <= v.BN && cfg.Kt <= v.BK && cfg.nctas < (1LL << 31);
+// The distinct (morder, korder) digit-order options of a contraction.
+std::vector<Config> order_options(const Contraction &c) {
+  std::vector<Config> out;
+  for (int mo = 0; mo < 2; mo++)
+    for (int ko = 0; ko < 2; ko++) {
+      Config cfg;
+      cfg.morder = mo;
+      cfg.korder = ko;
+      digit_orders(c, cfg);
+      bool dup = false;
+      for (auto &o : out) dup |= o.mdig == cfg.mdig && o.kdig == cfg.kdig;
+      if (!dup) out.push_back(cfg);
+    }
+  return out;
 }
+
+}  // namespace
 
 // ---------------------------------------------------------------- B200 mode
 static Status choose_b200(const Contraction &c, int forced_variant, Config &best, PlanStats &st) {
+  WfCache cache;
   Config base;
   digit_orders(c, base);
   base.T.assign(c.ix.size(), 1);
-  // the X side's externals in X's order (Alg. 2 walks the input's index list)
+  // Alg. 2 walks each input's index list; C's FVI is mapped first on the X side
   std::vector<int> mx, ny, kx;
   for (int id : c.t[base.X].idx) if (c.ix[id].cls != INTL) mx.push_back(id);
   for (int id : c.t[base.Y].idx) if (c.ix[id].cls != INTL) ny.push_back(id);
-  kx = base.kdig;
-  const int c0 = base.mdig.empty() ? -1 : base.mdig[0];
-  const int kfirst = base.kdig.empty() ? -1 : base.kdig[0];
+  for (int id : c.t[base.X].idx) if (c.ix[id].cls == INTL) kx.push_back(id);
+  const int c0 = c.t[0].idx.empty() ? -1 : c.t[0].idx[0];
+  int kfirst = -1;
+  if (!c.t[base.X].idx.empty() && c.ix[c.t[base.X].idx[0]].cls == INTL) kfirst = c.t[base.X].idx[0];
+  else if (!c.t[base.Y].idx.empty() && c.ix[c.t[base.Y].idx[0]].cls == INTL) kfirst = c.t[base.Y].idx[0];
+  const auto orders = order_options(c);
   bool found = false;
   for (int vi = 0; vi < (int)variants().size(); vi++) {
     if (forced_variant >= 0 && vi != forced_variant) continue;
@@ -320,37 +307,47 @@ static Status choose_b200(const Contraction &c, int forced_variant, Config &best
     auto ms = enum_side(c, mx, c0, v.BM);
     auto ns = enum_side(c, ny, -1, v.BN);
     auto ks = enum_side(c, kx, kfirst, v.BK);
-    // keep the k tilings with the least padding (ties: longer runs), top 4
+    // keep the k tilings with the least padding, top 3
     std::vector<std::pair<double, Tiling>> kr;
     for (auto &k : ks) {
       if (tprod(k) > v.BK) continue;
       std::vector<int> T(c.ix.size(), 1);
       apply_tiling(k, T);
       double steps = 1, need = 1;
-      for (int id : base.kdig) { steps *= (double)cdiv(c.ix[id].n, T[id]); need *= (double)c.ix[id].n; }
-      double pad = steps * v.BK / need;
-      kr.push_back({pad, k});
+      for (int id : kx) { steps *= (double)cdiv(c.ix[id].n, T[id]); need *= (double)c.ix[id].n; }
+      kr.push_back({steps * v.BK / need, k});
     }
-    std::sort(kr.begin(), kr.end(), [](auto &a, auto &b) { return a.first < b.first; });
-    if (kr.size() > 4) kr.resize(4);
-    st.raw += (int64_t)ms.size() * ns.size() * ks.size();
-    for (auto &m : ms) {
-      if (tprod(m) > v.BM) { st.pruned += (int64_t)ns.size() * ks.size(); continue; }
-      for (auto &n : ns) {
-        if (tprod(n) > v.BN) { st.pruned += (int64_t)ks.size(); continue; }
-        for (auto &k : kr) {
-          Config cfg = base;
-          apply_tiling(m, cfg.T);
-          apply_tiling(n, cfg.T);
-          apply_tiling(k.second, cfg.T);
-          finish(c, cfg);
-          if (!fits(cfg, v)) { st.pruned++; continue; }
-          evaluate(c, cfg, vi);
-          st.ranked++;
-          if (!found || better(cfg, best)) { best = cfg; found = true; }
-        }
-      }
-    }
+    std::stable_sort(kr.begin(), kr.end(), [](auto &a, auto &b) { return a.first < b.first; });
+    if (kr.size() > 3) kr.resize(3);
+    // drop m / n tilings that fill less than half of what the fullest one fills
+    auto fill = [](std::vector<Tiling> &v, int64_t S) {
+      int64_t mx = 0;
+      for (auto &t : v) if (tprod(t) <= S) mx = std::max(mx, tprod(t));
+      std::vector<Tiling> o;
+      for (auto &t : v) if (tprod(t) <= S && 2 * tprod(t) >= mx) o.push_back(t);
+      return o;
+    };
+    const size_t raw_m = ms.size(), raw_n = ns.size();
+    ms = fill(ms, v.BM);
+    ns = fill(ns, v.BN);
+    st.raw += (int64_t)raw_m * raw_n * ks.size() * orders.size();
+    st.pruned += (int64_t)(raw_m * raw_n * ks.size() - ms.size() * ns.size() * kr.size()) * orders.size();
+    for (auto &m : ms)
+      for (auto &n : ns)
+        for (auto &k : kr)
+          for (const auto &o : orders) {
+            Config cfg = o;
+            cfg.T.assign(c.ix.size(), 1);
+            apply_tiling(m, cfg.T);
+            apply_tiling(n, cfg.T);
+            apply_tiling(k.second, cfg.T);
+            finish_counts(c, cfg);
+            if (!fits(cfg, v)) { st.pruned++; continue; }
+            cfg.variant = vi;
+            model_time(c, cfg, v, &cache);
+            st.ranked++;
+            if (!found || better(cfg, best)) { best = cfg; found = true; }
+          }
   }
   return found ? ST_OK : ST_NO_CONFIG;
 }
@@ -360,11 +357,12 @@ static Status choose_b200(const Contraction &c, int forced_variant, Config &best
 // greedy (floor crossing tile, R12); product; prune by P:L172 (smem, registers) and
 // P:L174 (FVI on a thread dimension, #TBs above one wave); rank by Alg. 3.
 static Status choose_paper(const Contraction &c, int forced_variant, Config &best, PlanStats &st) {
+  WfCache cache;
   Config base;
   digit_orders(c, base);
   base.T.assign(c.ix.size(), 1);
   const int X = base.X, Y = base.Y;
-  const int c0 = base.mdig.empty() ? -1 : base.mdig[0];
+  const int c0 = c.t[0].idx.empty() ? -1 : c.t[0].idx[0];
   std::vector<int> xe, ye, ki;
   for (int id : c.t[X].idx) if (c.ix[id].cls != INTL) xe.push_back(id);
   for (int id : c.t[Y].idx) if (c.ix[id].cls != INTL) ye.push_back(id);
@@ -389,7 +387,7 @@ static Status choose_paper(const Contraction &c, int forced_variant, Config &bes
       }
       for (auto &seq : seqs) {
         std::vector<Tiling> tbs;
-        greedy(c, seq, 0, 1, S, {}, true, tbs);
+        greedy(c, seq, 0, 1, S, Tiling(), true, tbs);
         for (auto &tb : tbs) {
           if (fvi_rule >= 0) {
             bool has = false;
@@ -403,14 +401,13 @@ static Status choose_paper(const Contraction &c, int forced_variant, Config &bes
             if (!used) left.push_back(id);
           }
           bool any = false;
-          for (int64_t R : REGS) {
+          for (int64_t R : REGS)
             for (auto &rs : rotations(left)) {
               std::vector<Tiling> regs;
-              greedy(c, rs, 0, 1, R, {}, true, regs);
+              greedy(c, rs, 0, 1, R, Tiling(), true, regs);
               for (auto &rg : regs) { uniq.insert({tb, rg}); any = true; }
             }
-          }
-          if (!any) uniq.insert({tb, {}});
+          if (!any) uniq.insert({tb, Tiling()});
         }
       }
     }
@@ -422,13 +419,12 @@ static Status choose_paper(const Contraction &c, int forced_variant, Config &bes
   auto px = enum_tb_reg(xe, c0, -1);
   auto py = enum_tb_reg(ye, -1, yfvi);
   std::set<Tiling> kset;
-  int kfvi = -1;
-  if (!c.t[X].idx.empty() && c.ix[c.t[X].idx[0]].cls == INTL) kfvi = c.t[X].idx[0];
-  int kfvi2 = (!c.t[Y].idx.empty() && c.ix[c.t[Y].idx[0]].cls == INTL) ? c.t[Y].idx[0] : -1;
+  const int kfvi = (!c.t[X].idx.empty() && c.ix[c.t[X].idx[0]].cls == INTL) ? c.t[X].idx[0] : -1;
+  const int kfvi2 = (!c.t[Y].idx.empty() && c.ix[c.t[Y].idx[0]].cls == INTL) ? c.t[Y].idx[0] : -1;
   for (int64_t S : TBS)
     for (auto &seq : rotations(ki)) {
       std::vector<Tiling> r;
-      greedy(c, seq, 0, 1, S, {}, true, r);
+      greedy(c, seq, 0, 1, S, Tiling(), true, r);
       for (auto &t : r) {
         bool ok = true;
         for (int f : {kfvi, kfvi2}) {
@@ -440,7 +436,7 @@ static Status choose_paper(const Contraction &c, int forced_variant, Config &bes
         if (ok) kset.insert(t);
       }
     }
-  if (kset.empty()) kset.insert(Tiling{});
+  if (kset.empty()) kset.insert(Tiling());
   st.raw = (int64_t)px.size() * py.size() * kset.size();
   bool found = false;
   for (auto &x : px)
@@ -450,7 +446,7 @@ static Status choose_paper(const Contraction &c, int forced_variant, Config &bes
         apply_tiling(x.tb, cfg.T); apply_tiling(x.reg, cfg.T);
         apply_tiling(y.tb, cfg.T); apply_tiling(y.reg, cfg.T);
         apply_tiling(k, cfg.T);
-        finish(c, cfg);
+        finish_counts(c, cfg);
         const double TBx = (double)tprod(x.tb), REGx = (double)tprod(x.reg);
         const double TBy = (double)tprod(y.tb), REGy = (double)tprod(y.reg);
         const double TBk = (double)tprod(k);
@@ -467,21 +463,20 @@ static Status choose_paper(const Contraction &c, int forced_variant, Config &bes
             if (forced_variant >= 0 && vi != forced_variant) continue;
             if (!fits(cfg, variants()[vi])) continue;
             Config t = cfg;
-            evaluate(c, t, vi);
+            t.variant = vi;
+            model_time(c, t, variants()[vi], &cache);
             if (vi_best < 0 || better(t, fit)) { fit = t; vi_best = vi; }
           }
         }
         if (!ok || vi_best < 0) { st.pruned++; continue; }
-        fit.paper_cost = paper_alg3_cost(c, fit, [&] { std::vector<int> v; for (auto &q : x.tb) v.push_back(q.first); return v; }(),
-                                         [&] { std::vector<int> v; for (auto &q : x.reg) v.push_back(q.first); return v; }(),
-                                         [&] { std::vector<int> v; for (auto &q : y.tb) v.push_back(q.first); return v; }(),
-                                         [&] { std::vector<int> v; for (auto &q : y.reg) v.push_back(q.first); return v; }());
+        auto ids = [](const Tiling &t) { std::vector<int> v; for (auto &q : t) v.push_back(q.first); return v; };
+        fit.paper_cost = paper_alg3_cost(c, fit, ids(x.tb), ids(x.reg), ids(y.tb), ids(y.reg));
         fit.paper_mapping = "TB_x=" + tiling_str(c, x.tb) + " REG_x=" + tiling_str(c, x.reg) +
                             " TB_y=" + tiling_str(c, y.tb) + " REG_y=" + tiling_str(c, y.reg) +
                             " TB_k=" + tiling_str(c, k);
         st.ranked++;
-        bool win = !found || fit.paper_cost < best.paper_cost ||
-                   (fit.paper_cost == best.paper_cost && better(fit, best));
+        const bool win = !found || fit.paper_cost < best.paper_cost ||
+                         (fit.paper_cost == best.paper_cost && better(fit, best));
         if (win) { best = fit; found = true; }
       }
   return found ? ST_OK : ST_NO_CONFIG;
@@ -490,21 +485,25 @@ static Status choose_paper(const Contraction &c, int forced_variant, Config &bes
 // ---------------------------------------------------------------- forced tiles
 static Status choose_forced(const Contraction &c, const ForcedTiles &ft, int forced_variant,
                             Config &best, std::string &err) {
-  Config cfg;
-  digit_orders(c, cfg);
-  cfg.T.assign(c.ix.size(), 1);
-  for (size_t id = 0; id < c.ix.size(); id++) {
-    auto it = ft.tile.find(c.ix[id].name);
-    if (it != ft.tile.end()) cfg.T[id] = (int)std::max<int64_t>(1, std::min<int64_t>(it->second, c.ix[id].n));
-  }
-  finish(c, cfg);
+  WfCache cache;
   bool found = false;
-  for (int vi = 0; vi < (int)variants().size(); vi++) {
-    if (forced_variant >= 0 && vi != forced_variant) continue;
-    if (!fits(cfg, variants()[vi])) continue;
-    Config t = cfg;
-    evaluate(c, t, vi);
-    if (!found || better(t, best)) { best = t; found = true; }
+  for (const auto &o : order_options(c)) {
+    Config cfg = o;
+    cfg.T.assign(c.ix.size(), 1);
+    for (size_t id = 0; id < c.ix.size(); id++) {
+      auto it = ft.tile.find(c.ix[id].name);
+      if (it != ft.tile.end())
+        cfg.T[id] = (int)std::max<int64_t>(1, std::min<int64_t>(it->second, c.ix[id].n));
+    }
+    finish_counts(c, cfg);
+    for (int vi = 0; vi < (int)variants().size(); vi++) {
+      if (forced_variant >= 0 && vi != forced_variant) continue;
+      if (!fits(cfg, variants()[vi])) continue;
+      Config t = cfg;
+      t.variant = vi;
+      model_time(c, t, variants()[vi], &cache);
+      if (!found || better(t, best)) { best = t; found = true; }
+    }
   }
   if (!found) { err = "forced tiles fit no compiled kernel variant"; return ST_NO_CONFIG; }
   return ST_OK;

@@ -1,0 +1,244 @@
+// tiles.cpp — see tiles.hpp.
+#include "tiles.hpp"
+
+#include <algorithm>
+#include <set>
+
+namespace tc {
+
+const std::vector<Variant> &variants() {
+  // BM, BN, BK, WM, WN, stages, threads, CTAs/SM (= __launch_bounds__ min blocks; smem and
+  // registers checked with ptxas -v).  Must match api.cu's kernel table.
+  static const std::vector<Variant> v = {
+      {128, 128, 16, 64, 32, 4, 256, 1},  // 0
+      {128, 64, 16, 64, 32, 3, 128, 2},   // 1
+      {64, 128, 16, 32, 64, 3, 128, 2},   // 2
+      {64, 64, 16, 32, 32, 4, 128, 2},    // 3
+      {128, 128, 8, 64, 32, 4, 256, 1},   // 4
+      {64, 64, 8, 32, 32, 4, 128, 3},     // 5
+      {128, 32, 16, 32, 32, 4, 128, 2},   // 6
+      {32, 128, 16, 32, 32, 4, 128, 2},   // 7
+      {128, 32, 8, 32, 32, 4, 128, 3},    // 8
+      {32, 128, 8, 32, 32, 4, 128, 3},    // 9
+  };
+  return v;
+}
+
+static int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+void digit_orders(const Contraction &c, Config &cfg) {
+  cfg.X = c.t[0].idx.empty() ? 1 : (c.pos_in(1, c.t[0].idx[0]) >= 0 ? 1 : 2);
+  cfg.Y = 3 - cfg.X;
+  cfg.mdig.clear();
+  cfg.ndig.clear();
+  cfg.kdig.clear();
+  const auto &xv = c.t[cfg.X].idx, &yv = c.t[cfg.Y].idx;
+  // m: C order puts C's FVI first (coalesced C rows); X order follows X's memory
+  // (coalesced, vectorisable X loads)
+  if (cfg.morder == 0) {
+    for (int id : c.t[0].idx) if (c.pos_in(cfg.X, id) >= 0) cfg.mdig.push_back(id);
+  } else {
+    for (int id : xv) if (c.ix[id].cls != INTL) cfg.mdig.push_back(id);
+  }
+  // n: Y's memory order (C's FVI is never on the n side)
+  for (int id : yv) if (c.ix[id].cls != INTL) cfg.ndig.push_back(id);
+  // k: X's or Y's order of the internal indices
+  for (int id : (cfg.korder == 0 ? xv : yv)) if (c.ix[id].cls == INTL) cfg.kdig.push_back(id);
+  // smem layout: k-contiguous iff the operand's FVI is internal
+  cfg.xKmajor = !xv.empty() && c.ix[xv[0]].cls == INTL;
+  cfg.yKmajor = !yv.empty() && c.ix[yv[0]].cls == INTL;
+}
+
+void finish_counts(const Contraction &c, Config &cfg) {
+  cfg.Mt = cfg.Nt = cfg.Kt = 1;
+  cfg.mtiles = cfg.ntiles = cfg.nsteps = 1;
+  for (int id : cfg.mdig) { cfg.Mt *= cfg.T[id]; cfg.mtiles *= cdiv(c.ix[id].n, cfg.T[id]); }
+  for (int id : cfg.ndig) { cfg.Nt *= cfg.T[id]; cfg.ntiles *= cdiv(c.ix[id].n, cfg.T[id]); }
+  for (int id : cfg.kdig) { cfg.Kt *= cfg.T[id]; cfg.nsteps *= cdiv(c.ix[id].n, cfg.T[id]); }
+  cfg.nctas = cfg.mtiles * cfg.ntiles;
+}
+
+bool vec_possible(const Contraction &c, const Config &cfg, int t) {
+  // the operand's FVI leads its smem-contiguous dimension; even tile and extent; stride 1;
+  // every other stride and the base even (so every pair is 16-B aligned)
+  const auto &v = c.t[t];
+  if (v.idx.empty() || v.stride[0] != 1) return false;
+  const int f = v.idx[0];
+  const bool isk = c.ix[f].cls == INTL;
+  const bool kmaj = t == cfg.X ? cfg.xKmajor : cfg.yKmajor;
+  if (isk != kmaj) return false;
+  const auto &lst = isk ? cfg.kdig : (t == cfg.X ? cfg.mdig : cfg.ndig);
+  if (lst.empty() || lst[0] != f) return false;
+  if (cfg.T[f] % 2 || c.ix[f].n % 2) return false;
+  for (size_t p = 1; p < v.stride.size(); p++) if (v.stride[p] % 2) return false;
+  return v.base % 2 == 0;
+}
+
+SlotTable build_slots(const Contraction &c, const Config &cfg, int t, int vec, bool kmajor,
+                      int BMN, int BK) {
+  SlotTable out;
+  const auto &v = c.t[t];
+  const auto &side = t == cfg.X ? cfg.mdig : cfg.ndig;
+  const int r = (int)v.idx.size();
+  std::vector<int> T(r), mul(r), isk(r);
+  std::vector<int64_t> st(r);
+  for (int p = 0; p < r; p++) {
+    const int id = v.idx[p];
+    T[p] = cfg.T[id];
+    isk[p] = c.ix[id].cls == INTL;
+    st[p] = v.stride[p];
+    const auto &lst = isk[p] ? cfg.kdig : side;
+    int m = 1;
+    for (int q : lst) {
+      if (q == id) break;
+      m *= cfg.T[q];
+    }
+    mul[p] = m;
+  }
+  std::vector<int> d(r, 0);
+  for (;;) {
+    int mn = 0, k = 0;
+    int64_t rel = 0;
+    for (int p = 0; p < r; p++) {
+      (isk[p] ? k : mn) += d[p] * mul[p];
+      rel += d[p] * st[p];
+    }
+    out.rel.push_back(rel);
+    out.pack.push_back((uint32_t)smem_off(kmajor, mn, k, BMN, BK) | ((uint32_t)k << 13) |
+                       ((uint32_t)mn << 19));
+    int p = 0;
+    for (; p < r; p++) {
+      d[p] += (p == 0 ? vec : 1);
+      if (d[p] < T[p]) break;
+      d[p] = 0;
+    }
+    if (p == r) break;
+  }
+  return out;
+}
+
+double slot_wavefronts(const SlotTable &s, int vec) {
+  const size_t n = s.pack.size();
+  double total = 0;
+  for (size_t b = 0; b < n; b += 32) {
+    const size_t e = std::min(n, b + 32);
+    int cnt[32] = {0};
+    std::set<uint32_t> words[32];
+    for (size_t i = b; i < e; i++) {
+      const uint32_t off = s.pack[i] & 8191;           // in doubles
+      for (int w = 0; w < 2 * vec; w++) {
+        const uint32_t word = off * 2 + w;             // 32-bit words
+        words[word & 31].insert(word);
+      }
+    }
+    int wf = 0;
+    for (int k = 0; k < 32; k++) wf = std::max(wf, (int)words[k].size());
+    const int minwf = (int)((e - b) * 8 * vec + 127) / 128;
+    total += std::max(wf, minwf);
+    (void)cnt;
+  }
+  return total;
+}
+
+static uint64_t pack_bytes(const std::vector<int> &vals) {
+  uint64_t r = 0;
+  for (size_t i = 0; i < vals.size(); i++) r |= (uint64_t)(vals[i] & 0x7F) << (8 * i);
+  return r;
+}
+
+TileTables build_tile_tables(const Contraction &c, const Config &cfg, const Variant &v) {
+  TileTables tt;
+  const int X = cfg.X, Y = cfg.Y;
+  auto side = [&](const std::vector<int> &dig, int op, int64_t opbase, int64_t cbase,
+                  std::vector<TileInfo> &tiles, std::vector<int64_t> &relC,
+                  std::vector<uint64_t> &digp, uint64_t &full, int BMN) {
+    const int nd = (int)dig.size();
+    std::vector<int64_t> nt(nd);
+    int64_t ntot = 1;
+    std::vector<int> fl(nd);
+    for (int i = 0; i < nd; i++) {
+      nt[i] = cdiv(c.ix[dig[i]].n, cfg.T[dig[i]]);
+      ntot *= nt[i];
+      fl[i] = cfg.T[dig[i]] - 1;
+    }
+    full = pack_bytes(fl);
+    tiles.resize(ntot);
+    std::vector<int64_t> cd(nd, 0);
+    for (int64_t t = 0; t < ntot; t++) {
+      TileInfo ti{opbase, cbase, 0};
+      std::vector<int> lim(nd);
+      for (int i = 0; i < nd; i++) {
+        const int id = dig[i];
+        const int64_t o = cd[i] * cfg.T[id];
+        ti.op += o * c.stride_of(op, id);
+        ti.c += o * c.stride_of(0, id);
+        lim[i] = (int)std::min<int64_t>(cfg.T[id], c.ix[id].n - o) - 1;
+      }
+      ti.lim = pack_bytes(lim);
+      tiles[t] = ti;
+      for (int i = 0; i < nd; i++) {
+        if (++cd[i] < nt[i]) break;
+        cd[i] = 0;
+      }
+    }
+    relC.assign(BMN, 0);
+    digp.assign(BMN, ~0ull);
+    int64_t tot = 1;
+    for (int id : dig) tot *= cfg.T[id];
+    for (int64_t r = 0; r < tot && r < BMN; r++) {
+      int64_t q = r, off = 0;
+      std::vector<int> dd(nd);
+      for (int i = 0; i < nd; i++) {
+        dd[i] = (int)(q % cfg.T[dig[i]]);
+        q /= cfg.T[dig[i]];
+        off += dd[i] * c.stride_of(0, dig[i]);
+      }
+      relC[r] = off;
+      digp[r] = pack_bytes(dd);
+    }
+  };
+  side(cfg.mdig, X, c.t[X].base, c.t[0].base, tt.tileM, tt.relCm, tt.digM, tt.fullM, v.BM);
+  side(cfg.ndig, Y, c.t[Y].base, 0, tt.tileN, tt.relCn, tt.digN, tt.fullN, v.BN);
+  // k steps
+  const int nk = (int)cfg.kdig.size();
+  std::vector<int64_t> kt(nk), kn(nk);
+  int64_t steps = 1;
+  for (int i = 0; i < nk; i++) {
+    kn[i] = c.ix[cfg.kdig[i]].n;
+    kt[i] = cfg.T[cfg.kdig[i]];
+    steps *= cdiv(kn[i], kt[i]);
+  }
+  tt.stepX.resize(steps);
+  tt.stepY.resize(steps);
+  tt.kmask.resize(steps);
+  std::vector<int64_t> cd(nk, 0);
+  const int Kt = (int)cfg.Kt;
+  for (int64_t s = 0; s < steps; s++) {
+    int64_t bx = 0, by = 0;
+    for (int i = 0; i < nk; i++) {
+      bx += cd[i] * kt[i] * c.stride_of(X, cfg.kdig[i]);
+      by += cd[i] * kt[i] * c.stride_of(Y, cfg.kdig[i]);
+    }
+    uint64_t mask = 0;
+    for (int k = 0; k < Kt; k++) {
+      int q = k;
+      bool ok = true;
+      for (int i = 0; i < nk; i++) {
+        const int d = q % (int)kt[i];
+        q /= (int)kt[i];
+        ok &= cd[i] * kt[i] + d < kn[i];
+      }
+      if (ok) mask |= 1ull << k;
+    }
+    tt.stepX[s] = bx;
+    tt.stepY[s] = by;
+    tt.kmask[s] = mask;
+    for (int i = 0; i < nk; i++) {
+      if (++cd[i] < cdiv(kn[i], kt[i])) break;
+      cd[i] = 0;
+    }
+  }
+  return tt;
+}
+
+}  // namespace tc

@@ -1,0 +1,70 @@
+// tiles.hpp — digit orders, load-slot tables, shared-memory bank simulation and tile tables
+// (SURVEY 8(a) rows a3/a4).  Shared by the planner (for the cost model) and the launcher
+// (for the device tables), so the model scores exactly what the kernel will execute.
+#pragma once
+#include <cstdint>
+#include <vector>
+
+#include "contraction.hpp"
+#include "kparams.hpp"
+
+namespace tc {
+
+// Compiled kernel shapes (kernel_f64.cuh template instances, api.cu kernel table).
+struct Variant {
+  int BM, BN, BK, WM, WN, stages, threads, occ;
+};
+const std::vector<Variant> &variants();
+
+// Smem pitches (must match SmemLayout in kernel_f64.cuh): 4 (mod 16) doubles.
+inline int smem_off(bool kmajor, int mn, int k, int BMN, int BK) {
+  return kmajor ? mn * (BK + 4) + k : k * (BMN + 4) + mn;
+}
+
+struct Config {
+  int variant = -1;
+  int X = 1, Y = 2;                  // tensor ids (1 = A, 2 = B) on the M / N side
+  int morder = 0;                    // 0: m digits in C order (C's FVI first); 1: X order
+  int korder = 0;                    // 0: k digits in X order; 1: in Y order
+  std::vector<int> mdig, ndig, kdig; // index ids, compute order
+  std::vector<int> T;                // tile per index id (size = nidx)
+  bool xKmajor = false, yKmajor = false;
+  int vecX = 1, vecY = 1;            // vector width the plan allows (aligned pointers)
+  int64_t Mt = 1, Nt = 1, Kt = 1, mtiles = 1, ntiles = 1, nctas = 1, nsteps = 1;
+  // model outputs
+  double t_pred = 0, t_comp = 0, t_mem = 0, t_l2 = 0, dram_bytes = 0, flops_pad = 0;
+  double wfX = 0, wfY = 0;           // LDGSTS smem wavefronts per stage (simulated)
+  double paper_cost = 0;             // Alg. 3 transactions (paper mode)
+  std::string paper_mapping;         // Table II lists (paper mode)
+};
+
+// Digit lists for the given order options (X = input holding C's FVI).
+void digit_orders(const Contraction &c, Config &cfg);
+// Tile counts / extents from cfg.T.
+void finish_counts(const Contraction &c, Config &cfg);
+// Can operand t use 16-B vectors with this config?
+bool vec_possible(const Contraction &c, const Config &cfg, int t);
+
+struct SlotTable {
+  std::vector<int64_t> rel;    // element offset inside (tile, step)
+  std::vector<uint32_t> pack;  // smem offset | k << 13 | mn << 19
+};
+// Slots of operand t (X or Y) in the operand's own memory order.
+SlotTable build_slots(const Contraction &c, const Config &cfg, int t, int vec, bool kmajor,
+                      int BMN, int BK);
+// Shared-memory wavefronts of the cp.async writes of one stage (32 consecutive slots per
+// warp instruction; a bank serves one 32-bit word per wavefront).
+double slot_wavefronts(const SlotTable &s, int vec);
+
+// Device-side tables for one configuration.
+struct TileTables {
+  std::vector<TileInfo> tileM, tileN;
+  std::vector<int64_t> relCm, relCn;
+  std::vector<uint64_t> digM, digN;
+  uint64_t fullM = 0, fullN = 0;
+  std::vector<int64_t> stepX, stepY;
+  std::vector<uint64_t> kmask;
+};
+TileTables build_tile_tables(const Contraction &c, const Config &cfg, const Variant &v);
+
+}  // namespace tc

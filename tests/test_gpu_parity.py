@@ -10,6 +10,7 @@ import oracle
 import tcinputs
 from paper_conf_cgo_kimstkpprs19_b200 import binding as tc
 from paper_conf_cgo_kimstkpprs19_b200 import build
+from paper_conf_cgo_kimstkpprs19_b200.csrc_variants import NUM_VARIANTS
 from tests.layouts import PRIME_EXT, layouts_one_contraction, layouts_two_contractions
 
 pytestmark = pytest.mark.gpu
@@ -93,7 +94,7 @@ def test_alpha_beta_and_nan_c():
     check_case(e, ext, seed=5, integer=True, alpha=1.0, beta=0.0)
 
 
-@pytest.mark.parametrize("variant", range(6))
+@pytest.mark.parametrize("variant", range(NUM_VARIANTS))
 def test_every_kernel_variant(variant):
     check_case("abcdef-gdab-efgc", "a:9;b:6;c:7;d:10;e:5;f:6;g:11", seed=variant, integer=True,
                variant=variant)
