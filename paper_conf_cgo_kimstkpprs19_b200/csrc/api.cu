@@ -13,7 +13,7 @@
 
 #include "../../include/libtc.h"
 #include "contraction.hpp"
-#include "kernel_f64.cuh"
+#include "kernel_table.cuh"
 #include "kparams.hpp"
 #include "planner.hpp"
 #include "tiles.hpp"
@@ -35,27 +35,16 @@ struct KernelEntry {
   size_t smem;
 };
 
-template <int BM, int BN, int BK, int WM, int WN, int ST, int MINB>
-KernelEntry entry() {
-  using K = F64Kernel<BM, BN, BK, WM, WN, ST>;
-  return {(const void *)&tc_f64_dmma_kernel<BM, BN, BK, WM, WN, ST, MINB>, K::THREADS, K::smem_bytes()};
-}
-
-const std::vector<KernelEntry> &kernels() {
-  // one-to-one with tiles.cpp variants(): BM, BN, BK, WM, WN, stages, CTAs/SM
-  static const std::vector<KernelEntry> k = {
-      entry<128, 128, 16, 64, 32, 4, 1>(),  // 0
-      entry<128, 64, 16, 64, 32, 3, 2>(),   // 1
-      entry<64, 128, 16, 32, 64, 3, 2>(),   // 2
-      entry<64, 64, 16, 32, 32, 4, 2>(),    // 3
-      entry<128, 128, 8, 64, 32, 4, 1>(),   // 4
-      entry<64, 64, 8, 32, 32, 4, 3>(),     // 5
-      entry<128, 32, 16, 32, 32, 4, 2>(),   // 6
-      entry<32, 128, 16, 32, 32, 4, 2>(),   // 7
-      entry<128, 32, 8, 32, 32, 4, 3>(),    // 8
-      entry<32, 128, 8, 32, 32, 4, 3>(),    // 9
-  };
-  return k;
+// The instance for the plan's variant and smem layouts (kernel_table.cuh).
+KernelEntry kernel_for(const Config &cfg) {
+  const Variant &v = variants()[cfg.variant];
+  const void *fn = cfg.xKmajor ? (cfg.yKmajor ? kernel_ptr_11(cfg.variant) : kernel_ptr_10(cfg.variant))
+                               : (cfg.yKmajor ? kernel_ptr_01(cfg.variant) : kernel_ptr_00(cfg.variant));
+  // must equal F64Kernel<...>::smem_bytes()
+  const size_t PM = v.BM + 4, PN = v.BN + 4, PK = v.BK + 4;
+  const size_t XS = std::max(v.BM * PK, v.BK * PM), YS = std::max(v.BN * PK, v.BK * PN);
+  const size_t smem = 8 * (size_t)v.stages * (XS + YS) + 16 * (size_t)v.stages + 8 * (size_t)(v.BM + v.BN);
+  return {fn, v.threads(), smem};
 }
 
 }  // namespace
@@ -106,13 +95,12 @@ void build_host_tables(tc_plan_s *P) {
   kp.ntiles = (int)cfg.ntiles;
   kp.ntotal = (int)cfg.nctas;
   kp.group_m = 8;
-  kp.Mt = (int)cfg.Mt;
-  kp.Nt = (int)cfg.Nt;
-  kp.fullM = P->tt.fullM;
-  kp.fullN = P->tt.fullN;
   kp.nsteps = (int)cfg.nsteps;
-  kp.xKmajor = cfg.xKmajor;
-  kp.yKmajor = cfg.yKmajor;
+  for (int w = 0; w < kMaskWords; w++) {
+    kp.fullM[w] = P->tt.tileM[0].mask[w];   // the origin tile is always interior (T <= N)
+    kp.fullN[w] = P->tt.tileN[0].mask[w];
+  }
+  kp.fullK = cfg.Kt >= 64 ? ~0ull : ((1ull << cfg.Kt) - 1);
 }
 
 Status upload(tc_plan_s *P, std::string &err) {
@@ -129,8 +117,6 @@ Status upload(tc_plan_s *P, std::string &err) {
   size_t iN = add(tt.tileN.data(), sizeof(TileInfo) * tt.tileN.size());
   size_t iRm = add(tt.relCm.data(), 8 * tt.relCm.size());
   size_t iRn = add(tt.relCn.data(), 8 * tt.relCn.size());
-  size_t iDm = add(tt.digM.data(), 8 * tt.digM.size());
-  size_t iDn = add(tt.digN.data(), 8 * tt.digN.size());
   size_t iSx = add(tt.stepX.data(), 8 * tt.stepX.size());
   size_t iSy = add(tt.stepY.data(), 8 * tt.stepY.size());
   size_t iK = add(tt.kmask.data(), 8 * tt.kmask.size());
@@ -155,8 +141,6 @@ Status upload(tc_plan_s *P, std::string &err) {
   kp.tileN = (const TileInfo *)(b + parts[iN].off);
   kp.relCm = (const int64_t *)(b + parts[iRm].off);
   kp.relCn = (const int64_t *)(b + parts[iRn].off);
-  kp.digM = (const uint64_t *)(b + parts[iDm].off);
-  kp.digN = (const uint64_t *)(b + parts[iDn].off);
   kp.stepX = (const int64_t *)(b + parts[iSx].off);
   kp.stepY = (const int64_t *)(b + parts[iSy].off);
   kp.kmask = (const uint64_t *)(b + parts[iK].off);
@@ -168,7 +152,7 @@ Status upload(tc_plan_s *P, std::string &err) {
   P->d_packX2 = (const uint32_t *)(b + parts[iX2p].off);
   P->d_relY2 = (const int64_t *)(b + parts[iY2].off);
   P->d_packY2 = (const uint32_t *)(b + parts[iY2p].off);
-  const KernelEntry &ke = kernels()[P->cfg.variant];
+  const KernelEntry ke = kernel_for(P->cfg);
   e = cudaFuncSetAttribute(ke.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ke.smem);
   if (e != cudaSuccess) { err = std::string("cudaFuncSetAttribute: ") + cudaGetErrorString(e); return ST_CUDA; }
   int occ = 0;
@@ -374,7 +358,7 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
   kp.packY = vy ? plan->d_packY2 : plan->d_packY1;
   kp.nslotY = (int)(vy ? plan->slotY2.pack.size() : plan->slotY1.pack.size());
   kp.vecY = vy ? 2 : 1;
-  const KernelEntry &ke = kernels()[cfg.variant];
+  const KernelEntry ke = kernel_for(cfg);
   const int grid = (int)std::min<int64_t>(cfg.nctas, plan->sms);
   void *args[] = {&kp};
   cudaError_t e = cudaLaunchKernel(ke.fn, dim3(grid), dim3(ke.threads), args, ke.smem, (cudaStream_t)stream);
@@ -441,7 +425,7 @@ tc_status_t tc_plan_info(const tc_plan_t plan, char *json, size_t cap, size_t *n
     o << "},\"m\":" << names(g.mdig) << ",\"n\":" << names(g.ndig) << ",\"k\":" << names(g.kdig);
     o << ",\"morder\":" << g.morder << ",\"korder\":" << g.korder;
     o << ",\"variant\":" << g.variant << ",\"BM\":" << v.BM << ",\"BN\":" << v.BN << ",\"BK\":" << v.BK
-      << ",\"threads\":" << v.threads << ",\"stages\":" << v.stages << ",\"occ\":" << v.occ;
+      << ",\"threads\":" << v.threads() << ",\"stages\":" << v.stages << ",\"occ\":" << v.occ;
     o << ",\"Mt\":" << g.Mt << ",\"Nt\":" << g.Nt << ",\"Kt\":" << g.Kt << ",\"nctas\":" << g.nctas
       << ",\"mtiles\":" << g.mtiles << ",\"ntiles\":" << g.ntiles << ",\"nsteps\":" << g.nsteps
       << ",\"grid\":" << std::min<int64_t>(g.nctas, plan->sms);

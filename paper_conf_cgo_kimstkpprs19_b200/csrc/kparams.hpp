@@ -5,23 +5,23 @@
 // n over the externals of Y, k over the internal indices.  Each is a multi-index whose
 // digits carry their own tile size T_i (a CTA owns a hyper-rectangle prod T_i of
 // C; the grid has prod ceil(N_i / T_i) tiles).  Addresses are separable:
-//   addr_X(tile, step, m, k) = tileX[mt] + stepX[s] + rel_slot(m, k)
+//   addr_X(tile, step, slot) = tileM[mt].op + stepX[s] + relX[slot]
 //   addr_C(tile, m, n)       = tileM[mt].c + tileN[nt].c + relCm[m] + relCn[n]
 // so one compiled kernel serves every index permutation; only tile shapes are templates.
-// Bounds ("correct for any problem size"): each tile carries its per-digit limits
-// packed one byte per digit (lim-1, 7 bits) and every tile-local row / column its packed
-// digits; "in range" is one SWAR compare.
+// Bounds ("correct for any problem size"): every tile carries a bitmask of its
+// in-range tile-local rows (m) / columns (n); every k-step a bitmask of in-range k.
 #pragma once
 #include <cstdint>
 
 namespace tc {
 
 constexpr int kMaxDigits = 8;
+constexpr int kMaskWords = 2;   // BM, BN <= 128 -> two 64-bit words per tile
 
 struct TileInfo {           // one m-tile (or n-tile)
   int64_t op;               // element offset of the tile origin in X (or Y), incl. base
-  int64_t c;                // element offset of the tile origin in C (m: incl. C's base)
-  uint64_t lim;             // byte d = min(T_d, N_d - origin_d) - 1
+  int64_t c;                // element offset of the tile origin in C (m side incl. C's base)
+  uint64_t mask[kMaskWords];// bit r: tile-local row (column) r lies inside the tensor
 };
 
 struct KParams {
@@ -31,15 +31,12 @@ struct KParams {
   double alpha, beta;
   int mtiles, ntiles, ntotal;   // tiles per side, total tiles
   int group_m;              // CTA rasterisation: m-tiles per group (L2 locality)
-  int Mt, Nt;               // tile extents (<= BM, BN)
   const TileInfo *tileM;    // [mtiles]
   const TileInfo *tileN;    // [ntiles]
-  uint64_t fullM, fullN;    // lim of a full (interior) tile
-  // tile-local row / column tables [BM] / [BN]
-  const int64_t *relCm;     // offset in C of tile-local m
-  const uint64_t *digM;     // packed digits of tile-local m
-  const int64_t *relCn;
-  const uint64_t *digN;
+  uint64_t fullM[kMaskWords], fullN[kMaskWords];  // masks of an interior tile
+  uint64_t fullK;           // k mask of a step with every tile-local k in range
+  const int64_t *relCm;     // [BM] offset in C of tile-local m
+  const int64_t *relCn;     // [BN]
   // k side: steps in mixed radix over the internal tile grid
   int nsteps;
   const int64_t *stepX;     // [nsteps] element offset of step s's origin in X
@@ -53,19 +50,6 @@ struct KParams {
   const uint32_t *packY;
   int nslotX, nslotY;
   int vecX, vecY;           // 1 or 2 elements per slot (16-B cp.async when 2)
-  int xKmajor, yKmajor;     // smem layout: 1 = k contiguous, 0 = m (n) contiguous
 };
-
-#ifdef __CUDACC__
-#define TC_HD __host__ __device__
-#else
-#define TC_HD
-#endif
-
-// byte-wise a_d <= b_d for 8 packed 7-bit values
-TC_HD inline bool swar_le(uint64_t a, uint64_t b) {
-  const uint64_t H = 0x8080808080808080ull;
-  return (((b | H) - a) & H) == H;
-}
 
 }  // namespace tc

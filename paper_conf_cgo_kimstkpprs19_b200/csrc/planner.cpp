@@ -16,7 +16,7 @@ namespace tc {
 static constexpr double kSMs = 148, kFmaPerClk = 64, kClk = 1.965e9;
 static constexpr double kHbm = 6.5e12, kL2Bw = 12.0e12, kL2Bytes = 126.0e6;
 static constexpr double kLaunch = 3.0e-6;
-static constexpr double kStepOverhead = 60;   // cycles per k-step: barrier + bookkeeping
+static constexpr double kStepOverhead = 40;   // cycles per k-step: mbarrier hand-off
 
 static int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
@@ -66,10 +66,13 @@ double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *
   cfg.vecY = vec_possible(c, cfg, cfg.Y) ? 2 : 1;
   cfg.wfX = operand_wavefronts(c, cfg, cfg.X, cfg.vecX, cfg.xKmajor, v.BM, v.BK, cache);
   cfg.wfY = operand_wavefronts(c, cfg, cfg.Y, cfg.vecY, cfg.yKmajor, v.BN, v.BK, cache);
-  const int MI = v.WM / 8, NJ = v.WN / 8, warps = v.threads / 32;
+  const int MI = v.WM / 8, NJ = v.WN / 8, warps = v.cwarps();
   const double lds = (double)warps * (v.BK / 4) * (MI + NJ) * 2;
-  const double step = std::max(dmma, cfg.wfX + cfg.wfY + lds) + kStepOverhead;
-  const double epi = (double)warps * MI * NJ * 2 * 8 / 4;     // store issue per tile
+  // producer warps: one LDGSTS warp-instruction per 32 slots, ~8 LSU cycles each
+  const double nslots = (double)cfg.Mt * cfg.Kt / cfg.vecX + (double)cfg.Kt * cfg.Nt / cfg.vecY;
+  const double ldgsts = std::ceil(nslots / 32.0) * 8.0;
+  const double step = std::max({dmma, cfg.wfX + cfg.wfY + lds, ldgsts}) + kStepOverhead;
+  const double epi = (double)warps * MI * NJ * 2 * 6 / 4;     // store issue per tile
   // persistent CTAs: grid = 148 * occ, tiles round-robin
   const double slots = kSMs * v.occ;
   const double tiles_per_cta = std::ceil(nctas / slots);
@@ -344,6 +347,13 @@ static Status choose_b200(const Contraction &c, int forced_variant, Config &best
             finish_counts(c, cfg);
             if (!fits(cfg, v)) { st.pruned++; continue; }
             cfg.variant = vi;
+            // bound: the FP64-pipe time of the padded work alone (no smem / memory terms)
+            if (found) {
+              const double tiles = std::ceil((double)cfg.nctas / (kSMs * v.occ));
+              const double lb = tiles * v.occ * (double)cfg.nsteps * v.BM * v.BN * v.BK /
+                                kFmaPerClk / kClk + kLaunch;
+              if (lb > best.t_pred) { st.pruned++; continue; }
+            }
             model_time(c, cfg, v, &cache);
             st.ranked++;
             if (!found || better(cfg, best)) { best = cfg; found = true; }

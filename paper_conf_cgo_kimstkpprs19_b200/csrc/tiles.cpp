@@ -7,19 +7,20 @@
 namespace tc {
 
 const std::vector<Variant> &variants() {
-  // BM, BN, BK, WM, WN, stages, threads, CTAs/SM (= __launch_bounds__ min blocks; smem and
-  // registers checked with ptxas -v).  Must match api.cu's kernel table.
+  // BM, BN, BK, WM, WN, stages, producer warps, CTAs/SM (= __launch_bounds__ min blocks;
+  // smem and registers checked with ptxas -v).  Must match kernels_*.cu.
   static const std::vector<Variant> v = {
-      {128, 128, 16, 64, 32, 4, 256, 1},  // 0
-      {128, 64, 16, 64, 32, 3, 128, 2},   // 1
-      {64, 128, 16, 32, 64, 3, 128, 2},   // 2
-      {64, 64, 16, 32, 32, 4, 128, 2},    // 3
-      {128, 128, 8, 64, 32, 4, 256, 1},   // 4
-      {64, 64, 8, 32, 32, 4, 128, 3},     // 5
-      {128, 32, 16, 32, 32, 4, 128, 2},   // 6
-      {32, 128, 16, 32, 32, 4, 128, 2},   // 7
-      {128, 32, 8, 32, 32, 4, 128, 3},    // 8
-      {32, 128, 8, 32, 32, 4, 128, 3},    // 9
+      {128, 64, 16, 32, 32, 3, 4, 1},   // 0
+      {64, 128, 16, 32, 32, 3, 4, 1},   // 1
+      {64, 64, 16, 32, 32, 4, 4, 2},    // 2
+      {64, 64, 24, 32, 32, 3, 4, 2},    // 3
+      {128, 64, 24, 32, 32, 3, 4, 1},   // 4
+      {64, 128, 24, 32, 32, 3, 4, 1},   // 5
+      {128, 32, 16, 32, 32, 4, 4, 2},   // 6
+      {32, 128, 16, 32, 32, 4, 4, 2},   // 7
+      {128, 32, 24, 32, 32, 3, 4, 2},   // 8
+      {32, 128, 24, 32, 32, 3, 4, 2},   // 9
+      {64, 64, 8, 32, 32, 4, 4, 2},     // 10
   };
   return v;
 }
@@ -140,65 +141,67 @@ double slot_wavefronts(const SlotTable &s, int vec) {
   return total;
 }
 
-static uint64_t pack_bytes(const std::vector<int> &vals) {
-  uint64_t r = 0;
-  for (size_t i = 0; i < vals.size(); i++) r |= (uint64_t)(vals[i] & 0x7F) << (8 * i);
-  return r;
-}
 
 TileTables build_tile_tables(const Contraction &c, const Config &cfg, const Variant &v) {
   TileTables tt;
   const int X = cfg.X, Y = cfg.Y;
   auto side = [&](const std::vector<int> &dig, int op, int64_t opbase, int64_t cbase,
-                  std::vector<TileInfo> &tiles, std::vector<int64_t> &relC,
-                  std::vector<uint64_t> &digp, uint64_t &full, int BMN) {
+                  std::vector<TileInfo> &tiles, std::vector<int64_t> &relC, int BMN) {
     const int nd = (int)dig.size();
     std::vector<int64_t> nt(nd);
     int64_t ntot = 1;
-    std::vector<int> fl(nd);
     for (int i = 0; i < nd; i++) {
       nt[i] = cdiv(c.ix[dig[i]].n, cfg.T[dig[i]]);
       ntot *= nt[i];
-      fl[i] = cfg.T[dig[i]] - 1;
     }
-    full = pack_bytes(fl);
+    // tile-local digits and C offsets of every row (column) of the tile
+    int64_t tot = 1;
+    for (int id : dig) tot *= cfg.T[id];
+    relC.assign(BMN, 0);
+    std::vector<std::vector<int>> rd(std::min<int64_t>(tot, BMN), std::vector<int>(nd));
+    for (int64_t r = 0; r < tot && r < BMN; r++) {
+      int64_t q = r, off = 0;
+      for (int i = 0; i < nd; i++) {
+        rd[r][i] = (int)(q % cfg.T[dig[i]]);
+        q /= cfg.T[dig[i]];
+        off += rd[r][i] * c.stride_of(0, dig[i]);
+      }
+      relC[r] = off;
+    }
     tiles.resize(ntot);
     std::vector<int64_t> cd(nd, 0);
+    std::vector<int64_t> lim(nd);
     for (int64_t t = 0; t < ntot; t++) {
-      TileInfo ti{opbase, cbase, 0};
-      std::vector<int> lim(nd);
+      TileInfo ti{opbase, cbase, {0, 0}};
       for (int i = 0; i < nd; i++) {
         const int id = dig[i];
         const int64_t o = cd[i] * cfg.T[id];
         ti.op += o * c.stride_of(op, id);
         ti.c += o * c.stride_of(0, id);
-        lim[i] = (int)std::min<int64_t>(cfg.T[id], c.ix[id].n - o) - 1;
+        lim[i] = std::min<int64_t>(cfg.T[id], c.ix[id].n - o);
       }
-      ti.lim = pack_bytes(lim);
+      bool full = true;
+      for (int i = 0; i < nd; i++) full &= lim[i] == cfg.T[dig[i]];
+      if (full && t > 0) {
+        // interior tile: same rows as tile 0 (the origin tile is always interior, T <= N)
+        ti.mask[0] = tiles[0].mask[0];
+        ti.mask[1] = tiles[0].mask[1];
+      } else {
+        for (size_t r = 0; r < rd.size(); r++) {
+          bool ok = true;
+          for (int i = 0; i < nd; i++) ok &= rd[r][i] < lim[i];
+          if (ok) ti.mask[r >> 6] |= 1ull << (r & 63);
+        }
+      }
       tiles[t] = ti;
       for (int i = 0; i < nd; i++) {
         if (++cd[i] < nt[i]) break;
         cd[i] = 0;
       }
     }
-    relC.assign(BMN, 0);
-    digp.assign(BMN, ~0ull);
-    int64_t tot = 1;
-    for (int id : dig) tot *= cfg.T[id];
-    for (int64_t r = 0; r < tot && r < BMN; r++) {
-      int64_t q = r, off = 0;
-      std::vector<int> dd(nd);
-      for (int i = 0; i < nd; i++) {
-        dd[i] = (int)(q % cfg.T[dig[i]]);
-        q /= cfg.T[dig[i]];
-        off += dd[i] * c.stride_of(0, dig[i]);
-      }
-      relC[r] = off;
-      digp[r] = pack_bytes(dd);
-    }
   };
-  side(cfg.mdig, X, c.t[X].base, c.t[0].base, tt.tileM, tt.relCm, tt.digM, tt.fullM, v.BM);
-  side(cfg.ndig, Y, c.t[Y].base, 0, tt.tileN, tt.relCn, tt.digN, tt.fullN, v.BN);
+  side(cfg.mdig, X, c.t[X].base, c.t[0].base, tt.tileM, tt.relCm, v.BM);
+  side(cfg.ndig, Y, c.t[Y].base, 0, tt.tileN, tt.relCn, v.BN);
   // k steps
   const int nk = (int)cfg.kdig.size();
   std::vector<int64_t> kt(nk), kn(nk);

@@ -12,7 +12,9 @@ namespace tc {
 
 // Compiled kernel shapes (kernel_f64.cuh template instances, api.cu kernel table).
 struct Variant {
-  int BM, BN, BK, WM, WN, stages, threads, occ;
+  int BM, BN, BK, WM, WN, stages, pw, occ;   // pw = producer warps
+  int threads() const { return ((BM / WM) * (BN / WN) + pw) * 32; }
+  int cwarps() const { return (BM / WM) * (BN / WN); }
 };
 const std::vector<Variant> &variants();
 
@@ -60,8 +62,6 @@ double slot_wavefronts(const SlotTable &s, int vec);
 struct TileTables {
   std::vector<TileInfo> tileM, tileN;
   std::vector<int64_t> relCm, relCn;
-  std::vector<uint64_t> digM, digN;
-  uint64_t fullM = 0, fullN = 0;
   std::vector<int64_t> stepX, stepY;
   std::vector<uint64_t> kmask;
 };

@@ -1,2 +1,2 @@
 """Number of compiled FP64 kernel variants (tiles.cpp variants(), api.cu kernels())."""
-NUM_VARIANTS = 10
+NUM_VARIANTS = 11

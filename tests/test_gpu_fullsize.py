@@ -1,0 +1,70 @@
+"""Full-size parity: every TCCG-48 contraction at the benchmark extents,
+in the exact launch configuration bench.py times (same plan, same seeded device inputs),
+checked against the CPU oracle on sampled outputs (random + first + last elements), and
+against the rank-1 closed form on EVERY output element for a subset.  Needs a B200."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import tcinputs
+from paper_conf_cgo_kimstkpprs19_b200 import binding as tc
+from paper_conf_cgo_kimstkpprs19_b200 import build
+
+pytestmark = pytest.mark.gpu
+TAU64 = 1e-12
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _dev():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    build.build()
+    torch.cuda.set_device(0)
+
+
+@pytest.mark.parametrize("case", tcinputs.tccg48(), ids=lambda c: f"tccg{c.id}")
+def test_tccg_full_size_sampled(case):
+    p = tc.plan(case.expr, case.extents)
+    A = tcinputs.uniform(p.numel("A"), 1000 + case.id, device="cuda")
+    B = tcinputs.uniform(p.numel("B"), 2000 + case.id, device="cuda")
+    C = torch.full((p.numel("C"),), float("nan"), dtype=torch.float64, device="cuda")
+    p.execute(A, B, C)
+    torch.cuda.synchronize()
+    n = C.numel()
+    rng = np.random.default_rng(case.id)
+    idx = np.unique(np.concatenate([rng.integers(0, n, 1500), np.arange(min(n, 256)),
+                                    np.arange(max(0, n - 256), n)]))
+    got = C[torch.as_tensor(idx, device="cuda")].cpu().numpy()
+    want, S = oracle.sample(case.expr, case.extents, A.cpu().numpy(), B.cpu().numpy(), idx,
+                            with_scale=True)
+    bad = np.flatnonzero(~(np.abs(got - want) <= TAU64 * S))
+    assert bad.size == 0, (case.id, idx[bad[:5]], got[bad[:5]], want[bad[:5]])
+    assert torch.isfinite(C).all()          # every element was written
+
+
+@pytest.mark.parametrize("cid", [1, 6, 9, 12, 13, 16, 18, 31, 40, 48])
+def test_tccg_full_size_rank1_every_element(cid):
+    # A = prod u_i[idx_i], B = prod v_i[idx_i] => C[x] = prod_ext(u or v) * prod_int <u_j, v_j>
+    case = [c for c in tcinputs.tccg48() if c.id == cid][0]
+    c, a, b = tcinputs.split_expr(case.expr)
+    ext = case.ext
+    u = tcinputs.outer_factors(a, ext, 100 + cid)
+    v = tcinputs.outer_factors(b, ext, 200 + cid)
+    p = tc.plan(case.expr, case.extents)
+    A = torch.as_tensor(tcinputs.outer_tensor(a, u), device="cuda")
+    B = torch.as_tensor(tcinputs.outer_tensor(b, v), device="cuda")
+    C = torch.full((p.numel("C"),), float("nan"), dtype=torch.float64, device="cuda")
+    p.execute(A, B, C)
+    torch.cuda.synchronize()
+    fac = {x: (u[x] if x in a else v[x]) for x in c}
+    want = tcinputs.outer_tensor(c, fac)
+    scale = 1.0
+    for j in a:
+        if j not in c:
+            scale *= float(np.dot(u[j], v[j]))
+    want *= scale
+    got = C.cpu().numpy()
+    # S[x] = sum |A B| = want (all factors positive); tau * S plus the closed form's own
+    # rounding (a product of <= 8 factors: 8 ulp)
+    assert np.all(np.abs(got - want) <= (TAU64 + 16 * 2.2e-16) * np.abs(want))
