@@ -42,7 +42,7 @@ KernelEntry kernel_for(const Config &cfg) {
                                : (cfg.yKmajor ? kernel_ptr_01(cfg.variant) : kernel_ptr_00(cfg.variant));
   // must equal F64Kernel<...>::smem_bytes()
   const size_t PM = v.BM + 4, PN = v.BN + 4, PK = v.BK + 4;
-  const size_t XS = std::max(v.BM * PK, v.BK * PM), YS = std::max(v.BN * PK, v.BK * PN);
+  const size_t XS = std::max(v.BM * PK, v.BK * PM) + 2, YS = std::max(v.BN * PK, v.BK * PN) + 2;
   const size_t smem = 8 * (size_t)v.stages * (XS + YS) + 16 * (size_t)v.stages + 8 * (size_t)(v.BM + v.BN);
   return {fn, v.threads(), smem};
 }
