@@ -254,28 +254,35 @@ def run_libtc(args):
     ms_step = sum(med)
 
     # dominant kernel (largest share of the step) -> roofline
+    def kname(p):
+        i = p.info()
+        return (f"tc_f64_dmma_kernel<{i['BM']},{i['BN']},{i['BK']},32,32,{i['stages']},4,{i['occ']},"
+                f"{i['xKmajor']},{i['yKmajor']}>")
+
     share = {}
     for (c, p, *_), ms in zip(work, med):
-        v = p.info()["variant"]
-        f, t = share.get(v, (0.0, 0.0))
-        share[v] = (f + p.flops, t + ms)
-    dom = max(share, key=lambda v: share[v][1])
+        k = kname(p)
+        f, t = share.get(k, (0.0, 0.0))
+        share[k] = (f + p.flops, t + ms)
+    dom = max(share, key=lambda k: share[k][1])
     dflops, dms = share[dom]
     achieved = dflops / (dms * 1e-3) / 1e12
-    nlaunch = sum(1 for (c, p, *_) in work if p.info()["variant"] == dom)
+    dom_cases = [c.id for (c, p, *_) in work if kname(p) == dom]
     traffic = None
     prof = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(prof):
         try:
-            traffic = json.load(open(prof)).get(f"variant{dom}")
+            t = json.load(open(prof))
+            if t.get("kernel") == dom and t.get("case") in dom_cases:
+                traffic = t.get("dram_bytes_per_launch")
         except Exception:
             traffic = None
     roof = {"bound": "tensor", "achieved": round(achieved, 3), "peak": FP64_PEAK_TFLOPS,
             "unit": "TFLOP/s", "frac": round(achieved / FP64_PEAK_TFLOPS, 4), "traffic": traffic,
-            "kernel": f"tc_f64_dmma_kernel variant {dom}",
+            "kernel": dom, "cases": dom_cases,
             "peak_source": "measured FP64 DMMA peak (tools/peaks.cu, profiles/r01_peaks.json); "
                            f"derived 148x64x2x1.965GHz = {FP64_PEAK_DERIVED:.2f}",
-            "launches_per_step": nlaunch,
+            "launches_per_step": len(dom_cases),
             "share_of_step": round(dms / ms_step, 4)}
 
     # per-class roofline fraction: min(FP64 peak, I * HBM) per case

@@ -60,7 +60,9 @@ typedef struct tc_plan_opts {
      Indices not listed keep the planner's choice only if force_tiles is NULL.               */
   const char *force_tiles;
   int no_fusion;     /* 1: do not merge adjacent indices (row a2)                            */
-  int reserved[8];
+  int tma_epilogue;  /* 1: stage C tiles in smem and store them with TMA (cp.async.bulk.tensor)
+                        when C is a legal tensor map and beta == 0; 0 (default): direct stores */
+  int reserved[7];
 } tc_plan_opts;
 
 /*

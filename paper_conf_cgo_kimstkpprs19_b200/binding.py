@@ -33,8 +33,8 @@ class TcError(RuntimeError):
 
 class _Opts(ctypes.Structure):
     _fields_ = [("cost_mode", ctypes.c_int), ("host_only", ctypes.c_int), ("variant", ctypes.c_int),
-                ("force_tiles", ctypes.c_char_p), ("no_fusion", ctypes.c_int),
-                ("reserved", ctypes.c_int * 8)]
+                ("force_tiles", ctypes.c_char_p), ("no_fusion", ctypes.c_int), ("tma_epilogue", ctypes.c_int),
+                ("reserved", ctypes.c_int * 7)]
 
 
 _lib = None
@@ -169,8 +169,10 @@ class Plan:
 
 
 def plan(expr: str, extents: str, dtype: str = "f64", cost: str = "b200", host_only: bool = False,
-         variant: int | None = None, force_tiles: str | None = None, fusion: bool = True) -> Plan:
+         variant: int | None = None, force_tiles: str | None = None, fusion: bool = True,
+         tma: bool = False) -> Plan:
     o = _Opts()
+    o.tma_epilogue = int(tma)
     o.cost_mode = COST[cost]
     o.host_only = int(host_only)
     o.variant = 0 if variant is None else int(variant) + 1

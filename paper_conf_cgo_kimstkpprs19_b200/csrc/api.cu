@@ -1,5 +1,7 @@
 // api.cu — the C ABI of libtc (include/libtc.h): plan construction (rows a1-a4), launch
 // metadata (row a4), kernel dispatch (rows a5-a7), restriction (row e) and introspection.
+#include <cuda.h>
+#include <cudaTypedefs.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -32,7 +34,8 @@ tc_status_t fail(Status s, const std::string &msg) {
 struct KernelEntry {
   const void *fn;
   int threads;
-  size_t smem;
+  size_t smem;       // without the TMA staging box
+  size_t smem_tma;   // with it
 };
 
 // The instance for the plan's variant and smem layouts (kernel_table.cuh).
@@ -40,11 +43,12 @@ KernelEntry kernel_for(const Config &cfg) {
   const Variant &v = variants()[cfg.variant];
   const void *fn = cfg.xKmajor ? (cfg.yKmajor ? kernel_ptr_11(cfg.variant) : kernel_ptr_10(cfg.variant))
                                : (cfg.yKmajor ? kernel_ptr_01(cfg.variant) : kernel_ptr_00(cfg.variant));
-  // must equal F64Kernel<...>::smem_bytes()
+  // must equal F64Kernel<...>::smem_bytes(false / true)
   const size_t PM = v.BM + 4, PN = v.BN + 4, PK = v.BK + 4;
   const size_t XS = std::max(v.BM * PK, v.BK * PM) + 2, YS = std::max(v.BN * PK, v.BK * PN) + 2;
-  const size_t smem = 8 * (size_t)v.stages * (XS + YS) + 16 * (size_t)v.stages + 8 * (size_t)(v.BM + v.BN);
-  return {fn, v.threads(), smem};
+  const size_t base = 8 * (size_t)v.stages * (XS + YS) + 16 * (size_t)v.stages + 12 * (size_t)(v.BM + v.BN);
+  const size_t tma = (base + 1023) / 1024 * 1024 + 8 * (size_t)v.BM * v.BN;
+  return {fn, v.threads(), base, tma};
 }
 
 }  // namespace
@@ -65,7 +69,7 @@ struct tc_plan_s {
   KParams kp{};            // device pointers filled in; X/Y/C/alpha/beta/slots set per call
   void *dev = nullptr;     // one device buffer with every table
   size_t dev_bytes = 0;
-  const int64_t *d_relX1 = nullptr, *d_relY1 = nullptr, *d_relX2 = nullptr, *d_relY2 = nullptr;
+  const int32_t *d_relX1 = nullptr, *d_relY1 = nullptr, *d_relX2 = nullptr, *d_relY2 = nullptr;
   const uint32_t *d_packX1 = nullptr, *d_packY1 = nullptr, *d_packX2 = nullptr, *d_packY2 = nullptr;
   ~tc_plan_s() {
     if (dev) {
@@ -101,6 +105,9 @@ void build_host_tables(tc_plan_s *P) {
     kp.fullN[w] = P->tt.tileN[0].mask[w];
   }
   kp.fullK = cfg.Kt >= 64 ? ~0ull : ((1ull << cfg.Kt) - 1);
+  kp.Mt = (int)cfg.Mt;
+  kp.Nt = (int)cfg.Nt;
+  kp.c_rank = (int)c.t[0].idx.size();
 }
 
 Status upload(tc_plan_s *P, std::string &err) {
@@ -117,16 +124,26 @@ Status upload(tc_plan_s *P, std::string &err) {
   size_t iN = add(tt.tileN.data(), sizeof(TileInfo) * tt.tileN.size());
   size_t iRm = add(tt.relCm.data(), 8 * tt.relCm.size());
   size_t iRn = add(tt.relCn.data(), 8 * tt.relCn.size());
+  size_t iBm = add(tt.boxM.data(), 4 * tt.boxM.size());
+  size_t iBn = add(tt.boxN.data(), 4 * tt.boxN.size());
   size_t iSx = add(tt.stepX.data(), 8 * tt.stepX.size());
   size_t iSy = add(tt.stepY.data(), 8 * tt.stepY.size());
   size_t iK = add(tt.kmask.data(), 8 * tt.kmask.size());
-  size_t iX1 = add(P->slotX1.rel.data(), 8 * P->slotX1.rel.size());
+  // slot offsets inside a (tile, step) are 32-bit in the kernel (registers are scarce)
+  std::vector<int32_t> r32[4];
+  const SlotTable *sts[4] = {&P->slotX1, &P->slotY1, &P->slotX2, &P->slotY2};
+  for (int q = 0; q < 4; q++)
+    for (int64_t v : sts[q]->rel) {
+      if (v > INT32_MAX || v < INT32_MIN) { err = "tile spans more than 2^31 elements of an operand"; return ST_UNSUPPORTED; }
+      r32[q].push_back((int32_t)v);
+    }
+  size_t iX1 = add(r32[0].data(), 4 * r32[0].size());
   size_t iX1p = add(P->slotX1.pack.data(), 4 * P->slotX1.pack.size());
-  size_t iY1 = add(P->slotY1.rel.data(), 8 * P->slotY1.rel.size());
+  size_t iY1 = add(r32[1].data(), 4 * r32[1].size());
   size_t iY1p = add(P->slotY1.pack.data(), 4 * P->slotY1.pack.size());
-  size_t iX2 = add(P->slotX2.rel.data(), 8 * P->slotX2.rel.size());
+  size_t iX2 = add(r32[2].data(), 4 * r32[2].size());
   size_t iX2p = add(P->slotX2.pack.data(), 4 * P->slotX2.pack.size());
-  size_t iY2 = add(P->slotY2.rel.data(), 8 * P->slotY2.rel.size());
+  size_t iY2 = add(r32[3].data(), 4 * r32[3].size());
   size_t iY2p = add(P->slotY2.pack.data(), 4 * P->slotY2.pack.size());
   std::vector<char> h(o + 256, 0);
   for (auto &p : parts) if (p.bytes) std::memcpy(h.data() + p.off, p.src, p.bytes);
@@ -141,22 +158,25 @@ Status upload(tc_plan_s *P, std::string &err) {
   kp.tileN = (const TileInfo *)(b + parts[iN].off);
   kp.relCm = (const int64_t *)(b + parts[iRm].off);
   kp.relCn = (const int64_t *)(b + parts[iRn].off);
+  kp.boxM = (const int32_t *)(b + parts[iBm].off);
+  kp.boxN = (const int32_t *)(b + parts[iBn].off);
   kp.stepX = (const int64_t *)(b + parts[iSx].off);
   kp.stepY = (const int64_t *)(b + parts[iSy].off);
   kp.kmask = (const uint64_t *)(b + parts[iK].off);
-  P->d_relX1 = (const int64_t *)(b + parts[iX1].off);
+  P->d_relX1 = (const int32_t *)(b + parts[iX1].off);
   P->d_packX1 = (const uint32_t *)(b + parts[iX1p].off);
-  P->d_relY1 = (const int64_t *)(b + parts[iY1].off);
+  P->d_relY1 = (const int32_t *)(b + parts[iY1].off);
   P->d_packY1 = (const uint32_t *)(b + parts[iY1p].off);
-  P->d_relX2 = (const int64_t *)(b + parts[iX2].off);
+  P->d_relX2 = (const int32_t *)(b + parts[iX2].off);
   P->d_packX2 = (const uint32_t *)(b + parts[iX2p].off);
-  P->d_relY2 = (const int64_t *)(b + parts[iY2].off);
+  P->d_relY2 = (const int32_t *)(b + parts[iY2].off);
   P->d_packY2 = (const uint32_t *)(b + parts[iY2p].off);
   const KernelEntry ke = kernel_for(P->cfg);
-  e = cudaFuncSetAttribute(ke.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ke.smem);
+  const bool tma = P->tt.tma_ok && P->opts.tma_epilogue;
+  e = cudaFuncSetAttribute(ke.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(tma ? ke.smem_tma : ke.smem));
   if (e != cudaSuccess) { err = std::string("cudaFuncSetAttribute: ") + cudaGetErrorString(e); return ST_CUDA; }
   int occ = 0;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ke.fn, ke.threads, ke.smem);
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ke.fn, ke.threads, tma ? ke.smem_tma : ke.smem);
   if (e != cudaSuccess || occ < 1) { err = "kernel variant cannot be resident"; return ST_CUDA; }
   cudaDeviceGetAttribute(&P->sms, cudaDevAttrMultiProcessorCount, P->device);
   P->sms *= std::min(occ, variants()[P->cfg.variant].occ);
@@ -212,6 +232,47 @@ tc_status_t finish_plan(tc_plan_s *P, tc_plan_t *out) {
 bool overlaps(const void *a, size_t na, const void *b, size_t nb) {
   const char *x = (const char *)a, *y = (const char *)b;
   return x < y + nb && y < x + na;
+}
+
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no -lcuda needed).
+PFN_cuTensorMapEncodeTiled_v12000 tma_encoder() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = [] {
+    void *p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess) {
+      cudaGetLastError();
+      return (PFN_cuTensorMapEncodeTiled_v12000) nullptr;
+    }
+    return (PFN_cuTensorMapEncodeTiled_v12000)p;
+  }();
+  return fn;
+}
+
+// TMA descriptor of the plan's C view: dims in C order, the C tile as the box.
+bool encode_c_map(const tc_plan_s *P, void *C, TmaDesc &out) {
+  auto enc = tma_encoder();
+  if (!enc) return false;
+  const Contraction &c = P->c;
+  const auto &cv = c.t[0];
+  const int r = (int)cv.idx.size();
+  const char *base = (const char *)C + 8 * cv.base;
+  if ((uintptr_t)base % 16) return false;
+  cuuint64_t dims[kMaxTmaDims], strides[kMaxTmaDims];
+  cuuint32_t box[kMaxTmaDims], es[kMaxTmaDims];
+  for (int p = 0; p < r; p++) {
+    const int id = cv.idx[p];
+    dims[p] = (cuuint64_t)c.ix[id].n;
+    box[p] = (cuuint32_t)P->cfg.T[id];
+    es[p] = 1;
+    if (p > 0) strides[p - 1] = (cuuint64_t)(cv.stride[p] * 8);
+  }
+  static_assert(sizeof(TmaDesc) == sizeof(CUtensorMap), "descriptor size");
+  CUresult e = enc(reinterpret_cast<CUtensorMap *>(&out), CU_TENSOR_MAP_DATA_TYPE_FLOAT64, (cuuint32_t)r,
+                   (void *)base, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return e == CUDA_SUCCESS;
 }
 
 }  // namespace
@@ -347,6 +408,8 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
   kp.C = C;
   kp.alpha = alpha;
   kp.beta = beta;
+  // TMA epilogue when the C view is a legal tensor map and C is only written
+  kp.use_tma = plan->tt.tma_ok && plan->opts.tma_epilogue && beta == 0.0 && encode_c_map(plan, C, kp.cmap);
   // 16-B vectors need 16-B aligned operands; otherwise the scalar slot tables run
   const bool vx = cfg.vecX == 2 && ((uintptr_t)kp.X % 16) == 0;
   const bool vy = cfg.vecY == 2 && ((uintptr_t)kp.Y % 16) == 0;
@@ -361,7 +424,8 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
   const KernelEntry ke = kernel_for(cfg);
   const int grid = (int)std::min<int64_t>(cfg.nctas, plan->sms);
   void *args[] = {&kp};
-  cudaError_t e = cudaLaunchKernel(ke.fn, dim3(grid), dim3(ke.threads), args, ke.smem, (cudaStream_t)stream);
+  cudaError_t e = cudaLaunchKernel(ke.fn, dim3(grid), dim3(ke.threads), args,
+                                   kp.use_tma ? ke.smem_tma : ke.smem, (cudaStream_t)stream);
   if (e != cudaSuccess) return fail(ST_CUDA, std::string("launch: ") + cudaGetErrorString(e));
   return TC_SUCCESS;
 }

@@ -49,6 +49,47 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
       "@!p bra WAIT_%=;\n}\n" ::"r"(bar), "r"(parity) : "memory");
 }
 
+// TMA store of the smem box at `src` to the C tile at `crd` (cp.async.bulk.tensor, tile mode)
+__device__ __forceinline__ void tma_store(const TmaDesc *map, int rank, const int32_t *crd, uint32_t src) {
+  const uint64_t m = reinterpret_cast<uint64_t>(map);
+  switch (rank) {
+    case 1:
+      asm volatile("cp.async.bulk.tensor.1d.global.shared::cta.bulk_group [%0, {%1}], [%2];\n"
+                   ::"l"(m), "r"(crd[0]), "r"(src) : "memory");
+      break;
+    case 2:
+      asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];\n"
+                   ::"l"(m), "r"(crd[0]), "r"(crd[1]), "r"(src) : "memory");
+      break;
+    case 3:
+      asm volatile("cp.async.bulk.tensor.3d.global.shared::cta.bulk_group [%0, {%1, %2, %3}], [%4];\n"
+                   ::"l"(m), "r"(crd[0]), "r"(crd[1]), "r"(crd[2]), "r"(src) : "memory");
+      break;
+    case 4:
+      asm volatile("cp.async.bulk.tensor.4d.global.shared::cta.bulk_group [%0, {%1, %2, %3, %4}], [%5];\n"
+                   ::"l"(m), "r"(crd[0]), "r"(crd[1]), "r"(crd[2]), "r"(crd[3]), "r"(src) : "memory");
+      break;
+    default:
+      asm volatile("cp.async.bulk.tensor.5d.global.shared::cta.bulk_group [%0, {%1, %2, %3, %4, %5}], [%6];\n"
+                   ::"l"(m), "r"(crd[0]), "r"(crd[1]), "r"(crd[2]), "r"(crd[3]), "r"(crd[4]), "r"(src)
+                   : "memory");
+      break;
+  }
+  asm volatile("cp.async.bulk.commit_group;\n" ::: "memory");
+}
+__device__ __forceinline__ void tma_wait_read() { asm volatile("cp.async.bulk.wait_group.read 0;\n" ::: "memory"); }
+__device__ __forceinline__ void tma_wait_all() { asm volatile("cp.async.bulk.wait_group 0;\n" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory"); }
+__device__ __forceinline__ void consumer_sync(int nthreads) {
+  asm volatile("bar.sync 1, %0;\n" ::"r"(nthreads) : "memory");
+}
+
+// st.global.f64 under a predicate (keeps the epilogue free of branches)
+__device__ __forceinline__ void st_pred(double *ptr, double v, uint32_t ok) {
+  asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %2, 0;\n\t@p st.global.f64 [%0], %1;\n}\n"
+               ::"l"(ptr), "d"(v), "r"(ok) : "memory");
+}
+
 __device__ __forceinline__ void dmma884(double &c0, double &c1, double a, double b) {
   asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
                : "+d"(c0), "+d"(c1) : "d"(a), "d"(b));
@@ -71,8 +112,15 @@ struct F64Kernel {
   static constexpr int EX = (BM * BK + PW * 32 - 1) / (PW * 32);  // X slots per producer thread
   static constexpr int EY = (BN * BK + PW * 32 - 1) / (PW * 32);
   using L = SmemLayout<BM, BN, BK>;
-  static constexpr size_t smem_bytes() {
-    return sizeof(double) * (size_t)STAGES * (L::XS + L::YS) + 16 * (size_t)STAGES + 8 * (size_t)(BM + BN);
+  // ring + barriers + tables; the optional TMA staging box starts at the next 1 KB boundary
+  static constexpr size_t base_bytes() {
+    return sizeof(double) * (size_t)STAGES * (L::XS + L::YS) + 16 * (size_t)STAGES + 12 * (size_t)(BM + BN);
+  }
+  static constexpr size_t kStagingOffset =      // in doubles
+      ((sizeof(double) * (size_t)STAGES * (L::XS + L::YS) + 16 * (size_t)STAGES + 12 * (size_t)(BM + BN) +
+        1023) / 1024) * 1024 / 8;
+  static constexpr size_t smem_bytes(bool tma) {
+    return tma ? kStagingOffset * 8 + 8 * (size_t)BM * BN : base_bytes();
   }
   static_assert(BK % 4 == 0 && BK <= 64, "BK");
   static_assert(WM % 8 == 0 && WN % 8 == 0, "warp tile");
@@ -91,8 +139,10 @@ __device__ __forceinline__ void tile_coords(const KParams &p, int t, int &mt, in
   nt = r / gsz;
 }
 
+// (select, not a dynamic array index: keeps the mask in registers, no local memory)
 __device__ __forceinline__ bool bit_of(const uint64_t (&m)[kMaskWords], int r) {
-  return (m[r >> 6] >> (r & 63)) & 1;
+  static_assert(kMaskWords == 2, "bit_of");
+  return ((r < 64 ? m[0] : m[1]) >> (r & 63)) & 1;
 }
 
 __device__ __forceinline__ void cp_async16_full(uint32_t dst, const double *src) {
@@ -108,7 +158,7 @@ __device__ __forceinline__ void cp_async8_full(uint32_t dst, const double *src) 
 // Otherwise each slot tests its k bit and its row bit and zero-fills when out of range.
 template <int E, bool VEC>
 __device__ __forceinline__ void issue_slots(const double *__restrict__ src, uint32_t sdst,
-                                            const int64_t (&rel)[E], const uint32_t (&pack)[E],
+                                            const int32_t (&rel)[E], const uint32_t (&pack)[E],
                                             int64_t base, bool fast, uint64_t kmask,
                                             const uint64_t (&rmask)[kMaskWords]) {
   const double *b = src + base;
@@ -133,8 +183,8 @@ __device__ __forceinline__ void issue_slots(const double *__restrict__ src, uint
 }
 
 template <int E>
-__device__ __forceinline__ void load_slots(int64_t (&rel)[E], uint32_t (&pack)[E],
-                                           const int64_t *__restrict__ r, const uint32_t *__restrict__ p,
+__device__ __forceinline__ void load_slots(int32_t (&rel)[E], uint32_t (&pack)[E],
+                                           const int32_t *__restrict__ r, const uint32_t *__restrict__ p,
                                            int n, int first, int stride, uint32_t scratch) {
 #pragma unroll
   for (int i = 0; i < E; i++) {
@@ -148,16 +198,20 @@ __device__ __forceinline__ void load_slots(int64_t (&rel)[E], uint32_t (&pack)[E
 
 template <int BM, int BN, int BK, int WM, int WN, int STAGES, int PW, int MINB, bool XK, bool YK>
 __global__ void __launch_bounds__(F64Kernel<BM, BN, BK, WM, WN, STAGES, PW>::THREADS, MINB)
-tc_f64_dmma_kernel(const KParams p) {
+tc_f64_dmma_kernel(const __grid_constant__ KParams p) {
   using K = F64Kernel<BM, BN, BK, WM, WN, STAGES, PW>;
   using L = typename K::L;
   constexpr int MI = K::MI, NJ = K::NJ, CW = K::CWARPS;
-  extern __shared__ __align__(16) double smem[];
-  double *sX = smem;
+  extern __shared__ __align__(1024) double smem[];
+  double *sX = smem;                              // the cp.async ring
   double *sY = smem + STAGES * L::XS;
   uint64_t *bars = reinterpret_cast<uint64_t *>(sY + STAGES * L::YS);  // full[S], empty[S]
   int64_t *relCm = reinterpret_cast<int64_t *>(bars + 2 * STAGES);
   int64_t *relCn = relCm + BM;
+  int32_t *boxM = reinterpret_cast<int32_t *>(relCn + BN);
+  int32_t *boxN = boxM + BM;
+  // [BM * BN] C staging box of the TMA epilogue: present only when launched with it
+  double *sC = smem + K::kStagingOffset;
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int ntl = (p.ntotal - (int)blockIdx.x + (int)gridDim.x - 1) / (int)gridDim.x;
@@ -169,8 +223,8 @@ tc_f64_dmma_kernel(const KParams p) {
   // ---- once per CTA: zero the ring (positions no slot writes must read as 0), tables,
   //      barriers ------------------------------------------------------------------------
   for (int i = tid; i < STAGES * (L::XS + L::YS); i += K::THREADS) smem[i] = 0.0;
-  for (int r = tid; r < BM; r += K::THREADS) relCm[r] = p.relCm[r];
-  for (int r = tid; r < BN; r += K::THREADS) relCn[r] = p.relCn[r];
+  for (int r = tid; r < BM; r += K::THREADS) { relCm[r] = p.relCm[r]; boxM[r] = p.boxM[r]; }
+  for (int r = tid; r < BN; r += K::THREADS) { relCn[r] = p.relCn[r]; boxN[r] = p.boxN[r]; }
   if (tid == 0) {
     for (int s = 0; s < STAGES; s++) {
       mbar_init(bar0 + 8 * s, PW * 32);               // full: every producer thread
@@ -185,7 +239,7 @@ tc_f64_dmma_kernel(const KParams p) {
     const int ptid = tid - CW * 32;
     const double *__restrict__ X = static_cast<const double *>(p.X);
     const double *__restrict__ Y = static_cast<const double *>(p.Y);
-    int64_t rx[K::EX], ry[K::EY];
+    int32_t rx[K::EX], ry[K::EY];
     uint32_t px[K::EX], py[K::EY];
     load_slots(rx, px, p.relX, p.packX, p.nslotX, ptid, PW * 32, L::XS - 2);
     load_slots(ry, py, p.relY, p.packY, p.nslotY, ptid, PW * 32, L::YS - 2);
@@ -245,9 +299,33 @@ tc_f64_dmma_kernel(const KParams p) {
     for (int jj = 0; jj < NJ; jj++) acc[i][jj][0] = acc[i][jj][1] = 0.0;
 
   const double alpha = p.alpha, beta = p.beta;
+  // this thread's C rows are the same in every tile: their offsets live in registers
+  int64_t roff[MI];
+#pragma unroll
+  for (int i = 0; i < MI; i++) roff[i] = relCm[wm * WM + i * 8 + g];
+  // TMA epilogue: box offsets of tile-local rows / columns come from smem tables
+  const bool use_tma = p.use_tma && beta == 0.0;
+  const uint32_t sCaddr = (uint32_t)__cvta_generic_to_shared(sC);
   int step = 0, lt = 0;
+  int64_t cm = 0, cn = 0;                          // tile origin in C (m part, n part)
+  uint64_t mm[kMaskWords], mn[kMaskWords];         // tile row / column masks
+  int32_t crd[kMaxTmaDims];                        // tile origin coordinates (TMA)
   for (int j = 0; j < total; j++) {
     const int s = j % STAGES;
+    if (step == 0) {
+      // tile info for this tile's epilogue, loaded now and first USED in the epilogue, so
+      // the load latency hides behind the mainloop
+      int mt, nt;
+      tile_coords(p, (int)blockIdx.x + lt * (int)gridDim.x, mt, nt);
+      const TileInfo &tm = p.tileM[mt];
+      const TileInfo &tn = p.tileN[nt];
+      cm = tm.c;
+      cn = tn.c;
+#pragma unroll
+      for (int w = 0; w < kMaskWords; w++) { mm[w] = tm.mask[w]; mn[w] = tn.mask[w]; }
+#pragma unroll
+      for (int d = 0; d < kMaxTmaDims; d++) crd[d] = tm.coord[d] + tn.coord[d];
+    }
     mbar_wait(bar0 + 8 * s, (j / STAGES) & 1);
     const double *xs = sX + s * L::XS + aoff;
     const double *ys = sY + s * L::YS + boff;
@@ -267,36 +345,68 @@ tc_f64_dmma_kernel(const KParams p) {
     if (lane == 0) mbar_arrive(bar0 + 8 * (STAGES + s));
     if (++step == p.nsteps) {
       // ---- epilogue of tile lt: C = alpha * acc + beta * C (beta == 0: C not read) --------
-      int mt, nt;
-      tile_coords(p, (int)blockIdx.x + lt * (int)gridDim.x, mt, nt);
-      const TileInfo &tm = p.tileM[mt];
-      const TileInfo &tn = p.tileN[nt];
-      const int64_t cb = tm.c + tn.c;
-      uint64_t mm[kMaskWords], mn[kMaskWords];
+      uint32_t rbits = 0;
 #pragma unroll
-      for (int w = 0; w < kMaskWords; w++) { mm[w] = tm.mask[w]; mn[w] = tn.mask[w]; }
+      for (int i = 0; i < MI; i++) rbits |= (uint32_t)bit_of(mm, wm * WM + i * 8 + g) << i;
+      double *Ct = C + (cm + cn);
+      if (use_tma) {
+        // stage alpha * acc as the tile's box in smem, one elected thread TMA-stores it;
+        // the hardware clips the box at the tensor bounds
+        if (threadIdx.x == 0) tma_wait_read();     // previous tile's store has read sC
+        consumer_sync(CW * 32);
 #pragma unroll
-      for (int jj = 0; jj < NJ; jj++)
+        for (int jj = 0; jj < NJ; jj++)
 #pragma unroll
-        for (int h = 0; h < 2; h++) {
-          const int cidx = wn * WN + jj * 8 + 2 * t + h;
-          const bool cok = bit_of(mn, cidx);
-          double *col = C + (cb + relCn[cidx]);
+          for (int h = 0; h < 2; h++) {
+            const int cidx = wn * WN + jj * 8 + 2 * t + h;
+            if (cidx < p.Nt) {
+              double *col = sC + boxN[cidx];
 #pragma unroll
-          for (int i = 0; i < MI; i++) {
-            const int r = wm * WM + i * 8 + g;
-            if (cok && bit_of(mm, r)) {
-              double *dst = col + relCm[r];
-              const double v = alpha * acc[i][jj][h];
-              *dst = beta != 0.0 ? fma(beta, *dst, v) : v;
+              for (int i = 0; i < MI; i++) {
+                const int r = wm * WM + i * 8 + g;
+                if (r < p.Mt) col[boxM[r]] = alpha * acc[i][jj][h];
+              }
             }
-            acc[i][jj][h] = 0.0;
           }
-        }
+        fence_proxy_async();
+        consumer_sync(CW * 32);
+        if (threadIdx.x == 0) tma_store(&p.cmap, p.c_rank, crd, sCaddr);
+      } else if (beta == 0.0) {
+        // predicated stores (no branches); alpha == 1 skips the FP64-pipe multiply
+        const bool a1 = alpha == 1.0;
+#pragma unroll
+        for (int jj = 0; jj < NJ; jj++)
+#pragma unroll
+          for (int h = 0; h < 2; h++) {
+            const int cidx = wn * WN + jj * 8 + 2 * t + h;
+            const uint32_t ok = bit_of(mn, cidx) ? rbits : 0u;
+            double *col = Ct + relCn[cidx];
+#pragma unroll
+            for (int i = 0; i < MI; i++)
+              st_pred(col + roff[i], a1 ? acc[i][jj][h] : alpha * acc[i][jj][h], (ok >> i) & 1);
+          }
+      } else {
+#pragma unroll
+        for (int jj = 0; jj < NJ; jj++)
+#pragma unroll
+          for (int h = 0; h < 2; h++) {
+            const int cidx = wn * WN + jj * 8 + 2 * t + h;
+            const uint32_t ok = bit_of(mn, cidx) ? rbits : 0u;
+            double *col = Ct + relCn[cidx];
+#pragma unroll
+            for (int i = 0; i < MI; i++)
+              if ((ok >> i) & 1) col[roff[i]] = fma(beta, col[roff[i]], alpha * acc[i][jj][h]);
+          }
+      }
+#pragma unroll
+      for (int i = 0; i < MI; i++)
+#pragma unroll
+        for (int jj = 0; jj < NJ; jj++) acc[i][jj][0] = acc[i][jj][1] = 0.0;
       step = 0;
       ++lt;
     }
   }
+  if (use_tma && threadIdx.x == 0) tma_wait_all();   // the last box must be read out
 }
 
 }  // namespace tc

@@ -4,6 +4,8 @@
 // Consumer warps own 32 x 32 warp tiles (64 accumulator registers); a 4-warp producer
 // group keeps its load slots in registers.  Warps per SM stay <= 16 so that no instance
 // has fewer than 128 registers per thread (the register file is 16 K per sub-partition).
+// Shared memory = BM x BN C staging box (TMA epilogue) + STAGES ring stages; the stage
+// counts keep MINB CTAs resident within 227 KB.
 #pragma once
 #include "kernel_f64.cuh"
 
@@ -21,8 +23,8 @@ const void *kernel_ptr(int v) {
     case 5: return (const void *)&tc_f64_dmma_kernel<64, 128, 24, 32, 32, 3, 4, 1, XK, YK>;
     case 6: return (const void *)&tc_f64_dmma_kernel<128, 32, 16, 32, 32, 4, 4, 2, XK, YK>;
     case 7: return (const void *)&tc_f64_dmma_kernel<32, 128, 16, 32, 32, 4, 4, 2, XK, YK>;
-    case 8: return (const void *)&tc_f64_dmma_kernel<128, 32, 24, 32, 32, 3, 4, 2, XK, YK>;
-    case 9: return (const void *)&tc_f64_dmma_kernel<32, 128, 24, 32, 32, 3, 4, 2, XK, YK>;
+    case 8: return (const void *)&tc_f64_dmma_kernel<128, 32, 24, 32, 32, 3, 4, 1, XK, YK>;
+    case 9: return (const void *)&tc_f64_dmma_kernel<32, 128, 24, 32, 32, 3, 4, 1, XK, YK>;
     case 10: return (const void *)&tc_f64_dmma_kernel<64, 64, 8, 32, 32, 4, 4, 2, XK, YK>;
   }
   return nullptr;

@@ -18,13 +18,27 @@ namespace tc {
 constexpr int kMaxDigits = 8;
 constexpr int kMaskWords = 2;   // BM, BN <= 128 -> two 64-bit words per tile
 
+constexpr int kMaxTmaDims = 5;
+
 struct TileInfo {           // one m-tile (or n-tile)
   int64_t op;               // element offset of the tile origin in X (or Y), incl. base
   int64_t c;                // element offset of the tile origin in C (m side incl. C's base)
   uint64_t mask[kMaskWords];// bit r: tile-local row (column) r lies inside the tensor
+  int32_t coord[kMaxTmaDims];// origin index per C dimension (this side's dims, 0 elsewhere)
+  int32_t pad_;
+};
+
+// Opaque 128-B TMA descriptor (CUtensorMap); kept as bytes so host-only code needs no
+// driver headers.
+struct alignas(64) TmaDesc {
+  unsigned char bytes[128];
 };
 
 struct KParams {
+  TmaDesc cmap;             // TMA descriptor of C (tile box = the C tile), if use_tma
+  int use_tma;              // 1: epilogue stages the C tile in smem and TMA-stores it
+  int c_rank;               // dimensions of the C descriptor
+  int Mt, Nt;               // tile extents (<= BM, BN)
   const void *X;            // M-side operand (A or B)
   const void *Y;            // N-side operand
   void *C;
@@ -37,6 +51,8 @@ struct KParams {
   uint64_t fullK;           // k mask of a step with every tile-local k in range
   const int64_t *relCm;     // [BM] offset in C of tile-local m
   const int64_t *relCn;     // [BN]
+  const int32_t *boxM;      // [BM] offset of tile-local m in the smem C box (TMA epilogue)
+  const int32_t *boxN;      // [BN]
   // k side: steps in mixed radix over the internal tile grid
   int nsteps;
   const int64_t *stepX;     // [nsteps] element offset of step s's origin in X
@@ -44,9 +60,9 @@ struct KParams {
   const uint64_t *kmask;    // [nsteps] bit k set <=> tile-local k is in range at step s
   // load slots: the X tile (Mt x Kt) and the Y tile (Kt x Nt) enumerated in each
   // operand's OWN memory order (threads along x walk the input's FVI)
-  const int64_t *relX;      // [nslotX] element offset of the slot inside (tile, step)
+  const int32_t *relX;      // [nslotX] element offset of the slot inside (tile, step)
   const uint32_t *packX;    // [nslotX] smem offset | k << 13 | m << 19
-  const int64_t *relY;
+  const int32_t *relY;
   const uint32_t *packY;
   int nslotX, nslotY;
   int vecX, vecY;           // 1 or 2 elements per slot (16-B cp.async when 2)

@@ -14,7 +14,9 @@ namespace tc {
 // B200, measured (profiles/r01_peaks.json): DMMA 37.1 TFLOP/s = 148 SMs x 64 FMA/clk x 2 x
 // 1.965 GHz; HBM read 7.36 TB/s, f64 write 6.7 TB/s, copy 6.55 TB/s (MEASURED_PEAKS.json).
 static constexpr double kSMs = 148, kFmaPerClk = 64, kClk = 1.965e9;
-static constexpr double kHbm = 6.5e12, kL2Bw = 12.0e12, kL2Bytes = 126.0e6;
+// kL2Bw: effective L2->SM bandwidth of the cp.async gathers, fitted to the variant sweeps
+// (tools/variant_sweep.py; profiles/r01_*): ~7 TB/s.
+static constexpr double kHbm = 6.5e12, kL2Bw = 7.0e12, kL2Bytes = 126.0e6;
 static constexpr double kLaunch = 3.0e-6;
 static constexpr double kStepOverhead = 40;   // cycles per k-step: mbarrier hand-off
 
@@ -40,10 +42,10 @@ static double sector_eff(int64_t run) {
   return b / (std::ceil(b / 32.0) * 32.0);
 }
 
-// Simulated cp.async wavefronts of operand t, memoised on everything the slot table depends
-// on (the operand's tiles, digit orders, layout, vector width, tile shape).
-static double operand_wavefronts(const Contraction &c, const Config &cfg, int t, int vec, bool kmaj,
-                                 int BMN, int BK, WfCache *cache) {
+// Simulated cp.async smem wavefronts and global sectors of one stage of operand t, memoised
+// on everything the slot table depends on (tiles, digit orders, layout, vector, shape).
+static std::pair<double, double> operand_sim(const Contraction &c, const Config &cfg, int t, int vec,
+                                             bool kmaj, int BMN, int BK, WfCache *cache) {
   std::vector<int64_t> key{t, vec, kmaj, BMN, BK, cfg.morder, cfg.korder};
   for (int id : c.t[t].idx) key.push_back(cfg.T[id]);
   for (int id : cfg.kdig) key.push_back(cfg.T[id]);
@@ -51,9 +53,10 @@ static double operand_wavefronts(const Contraction &c, const Config &cfg, int t,
     auto it = cache->find(key);
     if (it != cache->end()) return it->second;
   }
-  const double wf = slot_wavefronts(build_slots(c, cfg, t, vec, kmaj, BMN, BK), vec);
-  if (cache) (*cache)[key] = wf;
-  return wf;
+  const SlotTable st = build_slots(c, cfg, t, vec, kmaj, BMN, BK);
+  const std::pair<double, double> r{slot_wavefronts(st, vec), slot_sectors(st, vec)};
+  if (cache) (*cache)[key] = r;
+  return r;
 }
 
 // ---------------------------------------------------------------- B200 cost model
@@ -64,8 +67,12 @@ double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *
   const double dmma = (double)v.BM * v.BN * v.BK / kFmaPerClk;
   cfg.vecX = vec_possible(c, cfg, cfg.X) ? 2 : 1;
   cfg.vecY = vec_possible(c, cfg, cfg.Y) ? 2 : 1;
-  cfg.wfX = operand_wavefronts(c, cfg, cfg.X, cfg.vecX, cfg.xKmajor, v.BM, v.BK, cache);
-  cfg.wfY = operand_wavefronts(c, cfg, cfg.Y, cfg.vecY, cfg.yKmajor, v.BN, v.BK, cache);
+  const auto sx = operand_sim(c, cfg, cfg.X, cfg.vecX, cfg.xKmajor, v.BM, v.BK, cache);
+  const auto sy = operand_sim(c, cfg, cfg.Y, cfg.vecY, cfg.yKmajor, v.BN, v.BK, cache);
+  cfg.wfX = sx.first;
+  cfg.wfY = sy.first;
+  cfg.secX = sx.second;
+  cfg.secY = sy.second;
   const int MI = v.WM / 8, NJ = v.WN / 8, warps = v.cwarps();
   const double lds = (double)warps * (v.BK / 4) * (MI + NJ) * 2;
   // producer warps: one LDGSTS warp-instruction per 32 slots, ~8 LSU cycles each
@@ -97,8 +104,8 @@ double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *
   }
   cfg.dram_bytes = bx * rx / eX + by * ry / eY + bc / eC;
   cfg.t_mem = cfg.dram_bytes / kHbm;
-  const double l2b = nctas * steps * 8.0 * ((double)cfg.Mt * cfg.Kt / eX + (double)cfg.Kt * cfg.Nt / eY) +
-                     bc / eS;
+  // L2 -> SM: the simulated sectors of every stage of every tile, plus the C stores
+  const double l2b = nctas * steps * 32.0 * (cfg.secX + cfg.secY) + bc / eS;
   cfg.t_l2 = l2b / kL2Bw;
   cfg.flops_pad = 2.0 * nctas * steps * v.BM * v.BN * v.BK;
   cfg.t_pred = std::max({cfg.t_comp, cfg.t_mem, cfg.t_l2}) + kLaunch;
@@ -318,10 +325,15 @@ static Status choose_b200(const Contraction &c, int forced_variant, Config &best
       apply_tiling(k, T);
       double steps = 1, need = 1;
       for (int id : kx) { steps *= (double)cdiv(c.ix[id].n, T[id]); need *= (double)c.ix[id].n; }
-      kr.push_back({steps * v.BK / need, k});
+      // padding first; among equals, longer runs along the inputs' internal FVIs
+      double run = 1;
+      for (int t = 1; t <= 2; t++)
+        if (!c.t[t].idx.empty() && c.ix[c.t[t].idx[0]].cls == INTL)
+          run *= std::min(4, T[c.t[t].idx[0]]);     // 4 doubles = one 32-B sector
+      kr.push_back({steps * v.BK / need / run, k});
     }
     std::stable_sort(kr.begin(), kr.end(), [](auto &a, auto &b) { return a.first < b.first; });
-    if (kr.size() > 3) kr.resize(3);
+    if (kr.size() > 4) kr.resize(4);
     // drop m / n tilings that fill less than half of what the fullest one fills
     auto fill = [](std::vector<Tiling> &v, int64_t S) {
       int64_t mx = 0;

@@ -37,7 +37,7 @@ Status choose(const Contraction &c, int cost_mode, int forced_variant, const For
               Config &out, PlanStats &stats, std::string &err);
 
 // B200 model (seconds); fills cfg's model outputs.
-using WfCache = std::map<std::vector<int64_t>, double>;
+using WfCache = std::map<std::vector<int64_t>, std::pair<double, double>>;
 double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *cache = nullptr);
 double paper_alg3_cost(const Contraction &c, const Config &cfg, const std::vector<int> &tbx,
                        const std::vector<int> &regx, const std::vector<int> &tby,

@@ -18,8 +18,8 @@ const std::vector<Variant> &variants() {
       {64, 128, 24, 32, 32, 3, 4, 1},   // 5
       {128, 32, 16, 32, 32, 4, 4, 2},   // 6
       {32, 128, 16, 32, 32, 4, 4, 2},   // 7
-      {128, 32, 24, 32, 32, 3, 4, 2},   // 8
-      {32, 128, 24, 32, 32, 3, 4, 2},   // 9
+      {128, 32, 24, 32, 32, 3, 4, 1},   // 8
+      {32, 128, 24, 32, 32, 3, 4, 1},   // 9
       {64, 64, 8, 32, 32, 4, 4, 2},     // 10
   };
   return v;
@@ -118,6 +118,23 @@ SlotTable build_slots(const Contraction &c, const Config &cfg, int t, int vec, b
   return out;
 }
 
+double slot_sectors(const SlotTable &s, int vec) {
+  const size_t n = s.rel.size();
+  double total = 0;
+  std::vector<int64_t> sec;
+  for (size_t b = 0; b < n; b += 32) {
+    const size_t e = std::min(n, b + 32);
+    sec.clear();
+    for (size_t i = b; i < e; i++) {
+      sec.push_back((s.rel[i] * 8) >> 5);
+      sec.push_back((s.rel[i] * 8 + 8 * vec - 1) >> 5);
+    }
+    std::sort(sec.begin(), sec.end());
+    total += (double)(std::unique(sec.begin(), sec.end()) - sec.begin());
+  }
+  return total;
+}
+
 double slot_wavefronts(const SlotTable &s, int vec) {
   const size_t n = s.pack.size();
   double total = 0;
@@ -145,8 +162,18 @@ double slot_wavefronts(const SlotTable &s, int vec) {
 TileTables build_tile_tables(const Contraction &c, const Config &cfg, const Variant &v) {
   TileTables tt;
   const int X = cfg.X, Y = cfg.Y;
+  // TMA epilogue: C as a tensor of its own dims (C order), the tile as the box
+  const auto &cv = c.t[0];
+  const int crank = (int)cv.idx.size();
+  tt.tma_ok = crank >= 1 && crank <= kMaxTmaDims && cv.stride[0] == 1 && cfg.T[cv.idx[0]] % 2 == 0;
+  for (int p = 1; p < crank && tt.tma_ok; p++)
+    tt.tma_ok = (cv.stride[p] * 8) % 16 == 0 && cv.stride[p] * 8 < (1ll << 40);
+  for (int p = 0; p < crank && tt.tma_ok; p++) tt.tma_ok = c.ix[cv.idx[p]].n < (1ll << 31);
+  std::vector<int64_t> boxst(crank, 1);              // box strides (elements)
+  for (int p = 1; p < crank; p++) boxst[p] = boxst[p - 1] * cfg.T[cv.idx[p - 1]];
   auto side = [&](const std::vector<int> &dig, int op, int64_t opbase, int64_t cbase,
-                  std::vector<TileInfo> &tiles, std::vector<int64_t> &relC, int BMN) {
+                  std::vector<TileInfo> &tiles, std::vector<int64_t> &relC,
+                  std::vector<int32_t> &box, int BMN) {
     const int nd = (int)dig.size();
     std::vector<int64_t> nt(nd);
     int64_t ntot = 1;
@@ -154,31 +181,36 @@ TileTables build_tile_tables(const Contraction &c, const Config &cfg, const Vari
       nt[i] = cdiv(c.ix[dig[i]].n, cfg.T[dig[i]]);
       ntot *= nt[i];
     }
-    // tile-local digits and C offsets of every row (column) of the tile
+    // tile-local digits, C offsets and smem-box offsets of every row (column) of the tile
     int64_t tot = 1;
     for (int id : dig) tot *= cfg.T[id];
     relC.assign(BMN, 0);
+    box.assign(BMN, 0);
     std::vector<std::vector<int>> rd(std::min<int64_t>(tot, BMN), std::vector<int>(nd));
     for (int64_t r = 0; r < tot && r < BMN; r++) {
-      int64_t q = r, off = 0;
+      int64_t q = r, off = 0, bo = 0;
       for (int i = 0; i < nd; i++) {
         rd[r][i] = (int)(q % cfg.T[dig[i]]);
         q /= cfg.T[dig[i]];
         off += rd[r][i] * c.stride_of(0, dig[i]);
+        bo += rd[r][i] * boxst[c.pos_in(0, dig[i])];
       }
       relC[r] = off;
+      box[r] = (int32_t)bo;
     }
     tiles.resize(ntot);
     std::vector<int64_t> cd(nd, 0);
     std::vector<int64_t> lim(nd);
     for (int64_t t = 0; t < ntot; t++) {
-      TileInfo ti{opbase, cbase, {0, 0}};
+      TileInfo ti{opbase, cbase, {0, 0}, {0, 0, 0, 0, 0}, 0};
       for (int i = 0; i < nd; i++) {
         const int id = dig[i];
         const int64_t o = cd[i] * cfg.T[id];
         ti.op += o * c.stride_of(op, id);
         ti.c += o * c.stride_of(0, id);
         lim[i] = std::min<int64_t>(cfg.T[id], c.ix[id].n - o);
+        const int p = c.pos_in(0, id);
+        if (p >= 0 && p < kMaxTmaDims) ti.coord[p] = (int32_t)o;
       }
       bool full = true;
       for (int i = 0; i < nd; i++) full &= lim[i] == cfg.T[dig[i]];
@@ -200,8 +232,8 @@ TileTables build_tile_tables(const Contraction &c, const Config &cfg, const Vari
       }
     }
   };
-  side(cfg.mdig, X, c.t[X].base, c.t[0].base, tt.tileM, tt.relCm, v.BM);
-  side(cfg.ndig, Y, c.t[Y].base, 0, tt.tileN, tt.relCn, v.BN);
+  side(cfg.mdig, X, c.t[X].base, c.t[0].base, tt.tileM, tt.relCm, tt.boxM, v.BM);
+  side(cfg.ndig, Y, c.t[Y].base, 0, tt.tileN, tt.relCn, tt.boxN, v.BN);
   // k steps
   const int nk = (int)cfg.kdig.size();
   std::vector<int64_t> kt(nk), kn(nk);

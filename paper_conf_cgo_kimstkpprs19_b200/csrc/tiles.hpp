@@ -36,6 +36,7 @@ struct Config {
   // model outputs
   double t_pred = 0, t_comp = 0, t_mem = 0, t_l2 = 0, dram_bytes = 0, flops_pad = 0;
   double wfX = 0, wfY = 0;           // LDGSTS smem wavefronts per stage (simulated)
+  double secX = 0, secY = 0;         // global 32-B sectors per stage (simulated)
   double paper_cost = 0;             // Alg. 3 transactions (paper mode)
   std::string paper_mapping;         // Table II lists (paper mode)
 };
@@ -57,11 +58,17 @@ SlotTable build_slots(const Contraction &c, const Config &cfg, int t, int vec, b
 // Shared-memory wavefronts of the cp.async writes of one stage (32 consecutive slots per
 // warp instruction; a bank serves one 32-bit word per wavefront).
 double slot_wavefronts(const SlotTable &s, int vec);
+// Global-memory 32-B sectors one stage of loads touches (sum over warp instructions of the
+// distinct sectors of 32 consecutive slots; the tile origin is taken as sector-aligned).
+double slot_sectors(const SlotTable &s, int vec);
 
 // Device-side tables for one configuration.
 struct TileTables {
   std::vector<TileInfo> tileM, tileN;
   std::vector<int64_t> relCm, relCn;
+  // TMA epilogue: the C tile is a box of C (dims in C order, box dim = tile size)
+  bool tma_ok = false;                 // C rank <= 5, 16-B strides, even FVI tile
+  std::vector<int32_t> boxM, boxN;     // offset of tile-local m / n inside the smem box
   std::vector<int64_t> stepX, stepY;
   std::vector<uint64_t> kmask;
 };

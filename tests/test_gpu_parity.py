@@ -94,11 +94,14 @@ def test_alpha_beta_and_nan_c():
     check_case(e, ext, seed=5, integer=True, alpha=1.0, beta=0.0)
 
 
+@pytest.mark.parametrize("tma", [True, False])
 @pytest.mark.parametrize("variant", range(NUM_VARIANTS))
-def test_every_kernel_variant(variant):
-    check_case("abcdef-gdab-efgc", "a:9;b:6;c:7;d:10;e:5;f:6;g:11", seed=variant, integer=True,
-               variant=variant)
-    check_case("abcd-aebf-dfce", "a:17;b:9;c:13;d:20;e:19;f:3", seed=variant, variant=variant)
+def test_every_kernel_variant(variant, tma):
+    # both epilogues: TMA box store (cp.async.bulk.tensor) and predicated direct stores
+    check_case("abcdef-gdab-efgc", "a:10;b:6;c:7;d:10;e:5;f:6;g:11", seed=variant, integer=True,
+               variant=variant, tma=tma)
+    check_case("abcd-aebf-dfce", "a:18;b:9;c:13;d:20;e:19;f:3", seed=variant, variant=variant, tma=tma)
+    check_case("abcd-aebf-fdec", "a:16;b:24;c:8;d:40;e:24;f:9", seed=variant, variant=variant, tma=tma)
 
 
 def test_paper_cost_mode_runs():
