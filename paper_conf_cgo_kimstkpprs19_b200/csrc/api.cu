@@ -41,6 +41,12 @@ struct KernelEntry {
 // The instance for the plan's variant and smem layouts (kernel_table.cuh).
 KernelEntry kernel_for(const Config &cfg) {
   const Variant &v = variants()[cfg.variant];
+  if (v.kind == KIND_BF16_UMMA) {
+    size_t smem = 0;
+    int threads = 0;
+    const void *fn = kernel_ptr_bf16(cfg.variant, cfg.xKmajor, cfg.yKmajor, &smem, &threads);
+    return {fn, threads, smem, smem};
+  }
   const void *fn = cfg.xKmajor ? (cfg.yKmajor ? kernel_ptr_11(cfg.variant) : kernel_ptr_10(cfg.variant))
                                : (cfg.yKmajor ? kernel_ptr_01(cfg.variant) : kernel_ptr_00(cfg.variant));
   // must equal F64Kernel<...>::smem_bytes(false / true)
@@ -65,7 +71,7 @@ struct tc_plan_s {
   tc_plan_opts opts{};
   std::string force_tiles;
   TileTables tt;
-  SlotTable slotX1, slotY1, slotX2, slotY2;
+  SlotTable slotX1, slotY1, slotX2, slotY2;   // scalar and cfg.vecX / cfg.vecY wide slots
   KParams kp{};            // device pointers filled in; X/Y/C/alpha/beta/slots set per call
   void *dev = nullptr;     // one device buffer with every table
   size_t dev_bytes = 0;
@@ -91,8 +97,8 @@ void build_host_tables(tc_plan_s *P) {
   P->tt = build_tile_tables(c, cfg, v);
   P->slotX1 = build_slots(c, cfg, cfg.X, 1, cfg.xKmajor, v.BM, v.BK);
   P->slotY1 = build_slots(c, cfg, cfg.Y, 1, cfg.yKmajor, v.BN, v.BK);
-  if (cfg.vecX == 2) P->slotX2 = build_slots(c, cfg, cfg.X, 2, cfg.xKmajor, v.BM, v.BK);
-  if (cfg.vecY == 2) P->slotY2 = build_slots(c, cfg, cfg.Y, 2, cfg.yKmajor, v.BN, v.BK);
+  if (cfg.vecX > 1) P->slotX2 = build_slots(c, cfg, cfg.X, cfg.vecX, cfg.xKmajor, v.BM, v.BK);
+  if (cfg.vecY > 1) P->slotY2 = build_slots(c, cfg, cfg.Y, cfg.vecY, cfg.yKmajor, v.BN, v.BK);
   KParams &kp = P->kp;
   std::memset(&kp, 0, sizeof(kp));
   kp.mtiles = (int)cfg.mtiles;
@@ -172,7 +178,7 @@ Status upload(tc_plan_s *P, std::string &err) {
   P->d_relY2 = (const int32_t *)(b + parts[iY2].off);
   P->d_packY2 = (const uint32_t *)(b + parts[iY2p].off);
   const KernelEntry ke = kernel_for(P->cfg);
-  const bool tma = P->tt.tma_ok && P->opts.tma_epilogue;
+  const bool tma = P->tt.tma_ok && P->opts.tma_epilogue && P->cfg.kind == KIND_F64_DMMA;
   e = cudaFuncSetAttribute(ke.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(tma ? ke.smem_tma : ke.smem));
   if (e != cudaSuccess) { err = std::string("cudaFuncSetAttribute: ") + cudaGetErrorString(e); return ST_CUDA; }
   int occ = 0;
@@ -213,7 +219,9 @@ tc_status_t finish_plan(tc_plan_s *P, tc_plan_t *out) {
   normalize(P->c, !P->opts.no_fusion && !ft.on);
   const int fv = P->opts.variant > 0 ? P->opts.variant - 1 : -1;
   if (fv >= (int)variants().size()) { delete P; return fail(ST_INVALID_ARG, "variant out of range"); }
-  Status s = choose(P->c, P->opts.cost_mode, fv, ft, P->cfg, P->stats, err);
+  const int kind = P->dtype == TC_BF16 ? KIND_BF16_UMMA : KIND_F64_DMMA;
+  if (fv >= 0 && variants()[fv].kind != kind) { delete P; return fail(ST_INVALID_ARG, "variant is not built for this dtype"); }
+  Status s = choose(P->c, kind, P->opts.cost_mode, fv, ft, P->cfg, P->stats, err);
   if (s != ST_OK) { delete P; return fail(s, err); }
   build_host_tables(P);
   if (!P->host_only) {
@@ -228,6 +236,8 @@ tc_status_t finish_plan(tc_plan_s *P, tc_plan_t *out) {
   *out = P;
   return TC_SUCCESS;
 }
+
+size_t elem_bytes(const tc_plan_s *P) { return P->dtype == TC_BF16 ? 2 : 8; }
 
 bool overlaps(const void *a, size_t na, const void *b, size_t nb) {
   const char *x = (const char *)a, *y = (const char *)b;
@@ -279,7 +289,7 @@ bool encode_c_map(const tc_plan_s *P, void *C, TmaDesc &out) {
 
 extern "C" {
 
-const char *tc_version(void) { return "libtc 0.2 (sm_100a, FP64 DMMA, persistent)"; }
+const char *tc_version(void) { return "libtc 0.3 (sm_100a, FP64 DMMA + BF16 tcgen05, persistent)"; }
 
 const char *tc_status_string(tc_status_t s) {
   switch (s) {
@@ -325,7 +335,8 @@ tc_status_t tc_plan_ex(tc_plan_t *plan, const char *expr, const char *extents, t
     std::string err;
     Status s = parse(expr, extents, P->parsed, err);
     if (s != ST_OK) { delete P; return fail(s, err); }
-    if (dtype != TC_F64) { delete P; return fail(ST_UNSUPPORTED, "only TC_F64 is built in this version"); }
+    if (dtype != TC_F64 && dtype != TC_BF16)
+      { delete P; return fail(ST_UNSUPPORTED, "only TC_F64 and TC_BF16 are built in this version"); }
     if (opts && (opts->cost_mode < 0 || opts->cost_mode > 1)) { delete P; return fail(ST_INVALID_ARG, "cost_mode"); }
     P->dtype = dtype;
     return finish_plan(P, plan);
@@ -395,8 +406,9 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
                        double beta, tc_stream_t stream) {
   if (!plan || !A || !B || !C) return fail(ST_INVALID_ARG, "NULL plan or tensor pointer");
   if (plan->host_only || !plan->dev) return fail(ST_CUDA, "plan was made host_only");
-  const size_t nA = (size_t)plan->parsed.span(1) * 8, nB = (size_t)plan->parsed.span(2) * 8,
-               nC = (size_t)plan->parsed.span(0) * 8;
+  const size_t es = elem_bytes(plan);
+  const size_t nA = (size_t)plan->parsed.span(1) * es, nB = (size_t)plan->parsed.span(2) * es,
+               nC = (size_t)plan->parsed.span(0) * es;
   if (overlaps(C, nC, A, nA) || overlaps(C, nC, B, nB)) return fail(ST_INVALID_ARG, "C overlaps A or B");
   int cur = -1;
   if (cudaGetDevice(&cur) != cudaSuccess || cur != plan->device)
@@ -409,18 +421,19 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
   kp.alpha = alpha;
   kp.beta = beta;
   // TMA epilogue when the C view is a legal tensor map and C is only written
-  kp.use_tma = plan->tt.tma_ok && plan->opts.tma_epilogue && beta == 0.0 && encode_c_map(plan, C, kp.cmap);
-  // 16-B vectors need 16-B aligned operands; otherwise the scalar slot tables run
-  const bool vx = cfg.vecX == 2 && ((uintptr_t)kp.X % 16) == 0;
-  const bool vy = cfg.vecY == 2 && ((uintptr_t)kp.Y % 16) == 0;
+  kp.use_tma = plan->tt.tma_ok && plan->opts.tma_epilogue && cfg.kind == KIND_F64_DMMA && beta == 0.0 &&
+               encode_c_map(plan, C, kp.cmap);
+  // vector slots need operands aligned to the vector; otherwise the scalar slot tables run
+  const bool vx = cfg.vecX > 1 && ((uintptr_t)kp.X % (es * cfg.vecX)) == 0;
+  const bool vy = cfg.vecY > 1 && ((uintptr_t)kp.Y % (es * cfg.vecY)) == 0;
   kp.relX = vx ? plan->d_relX2 : plan->d_relX1;
   kp.packX = vx ? plan->d_packX2 : plan->d_packX1;
   kp.nslotX = (int)(vx ? plan->slotX2.pack.size() : plan->slotX1.pack.size());
-  kp.vecX = vx ? 2 : 1;
+  kp.vecX = vx ? cfg.vecX : 1;
   kp.relY = vy ? plan->d_relY2 : plan->d_relY1;
   kp.packY = vy ? plan->d_packY2 : plan->d_packY1;
   kp.nslotY = (int)(vy ? plan->slotY2.pack.size() : plan->slotY1.pack.size());
-  kp.vecY = vy ? 2 : 1;
+  kp.vecY = vy ? cfg.vecY : 1;
   const KernelEntry ke = kernel_for(cfg);
   const int grid = (int)std::min<int64_t>(cfg.nctas, plan->sms);
   void *args[] = {&kp};
@@ -434,7 +447,8 @@ size_t tc_plan_workspace_bytes(const tc_plan_t plan) {
   if (!plan) return 0;
   auto al = [](size_t x) { return (x + 255) & ~(size_t)255; };
   const Contraction &c = plan->parsed;
-  return al(8 * c.parent_numel[1]) + al(8 * c.parent_numel[2]) + al(8 * c.parent_numel[0]);
+  const size_t es = elem_bytes(plan);
+  return al(es * c.parent_numel[1]) + al(es * c.parent_numel[2]) + al(es * c.parent_numel[0]);
 }
 
 tc_status_t tc_execute_host(const tc_plan_t plan, const void *A_host, const void *B_host, void *C_host,
@@ -444,7 +458,8 @@ tc_status_t tc_execute_host(const tc_plan_t plan, const void *A_host, const void
   if (workspace_bytes < tc_plan_workspace_bytes(plan)) return fail(ST_INVALID_ARG, "workspace too small");
   auto al = [](size_t x) { return (x + 255) & ~(size_t)255; };
   const Contraction &c = plan->parsed;
-  const size_t bA = 8 * c.parent_numel[1], bB = 8 * c.parent_numel[2], bC = 8 * c.parent_numel[0];
+  const size_t es = elem_bytes(plan);
+  const size_t bA = es * c.parent_numel[1], bB = es * c.parent_numel[2], bC = es * c.parent_numel[0];
   char *w = (char *)workspace;
   void *dA = w, *dB = w + al(bA), *dC = w + al(bA) + al(bB);
   cudaStream_t s = (cudaStream_t)stream;
@@ -472,7 +487,7 @@ tc_status_t tc_plan_info(const tc_plan_t plan, char *json, size_t cap, size_t *n
       for (size_t i = 0; i < l.size(); i++) s += (i ? ",\"" : "\"") + c.ix[l[i]].name + "\"";
       return s + "]";
     };
-    o << "{\"dtype\":\"f64\",\"X\":\"" << (g.X == 1 ? "A" : "B") << "\"";
+    o << "{\"dtype\":\"" << (g.kind == KIND_BF16_UMMA ? "bf16" : "f64") << "\",\"X\":\"" << (g.X == 1 ? "A" : "B") << "\"";
     o << ",\"indices\":[";
     for (size_t i = 0; i < c.ix.size(); i++) {
       const char *cls = c.ix[i].cls == EXT_A ? "extA" : c.ix[i].cls == EXT_B ? "extB" : "int";

@@ -35,5 +35,7 @@ const void *kernel_ptr_00(int v);
 const void *kernel_ptr_01(int v);
 const void *kernel_ptr_10(int v);
 const void *kernel_ptr_11(int v);
+// defined in kernels_bf16.cu (BF16 tcgen05 variants; smem bytes and block size out)
+const void *kernel_ptr_bf16(int v, bool xk, bool yk, size_t *smem, int *threads);
 
 }  // namespace tc

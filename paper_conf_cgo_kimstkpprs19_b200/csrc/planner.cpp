@@ -21,6 +21,10 @@ static constexpr double kLaunch = 3.0e-6;
 static constexpr double kStepOverhead = 40;   // cycles per k-step: mbarrier hand-off
 
 static int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+// multiply-adds per clock per SM of the kernel family's MMA pipe: DMMA 64 (measured), BF16
+// tcgen05 4096 (2.25 PFLOP/s dense nominal at 1.86 GHz; MEASURED_PEAKS.json has cuBLAS's
+// sustained figure)
+static double fma_per_clk(int kind) { return kind == KIND_BF16_UMMA ? 4096.0 : kFmaPerClk; }
 
 int64_t contiguous_run(const Contraction &c, int t, const std::vector<int> &T) {
   // cal_Cont: elements contiguous in memory within the tile hyper-rectangle
@@ -37,8 +41,8 @@ int64_t contiguous_run(const Contraction &c, int t, const std::vector<int> &T) {
 }
 
 // Fraction of 32-B sector bytes that are useful for a run of `run` doubles.
-static double sector_eff(int64_t run) {
-  double b = 8.0 * run;
+static double sector_eff(int64_t run, double es = 8.0) {
+  double b = es * run;
   return b / (std::ceil(b / 32.0) * 32.0);
 }
 
@@ -46,7 +50,7 @@ static double sector_eff(int64_t run) {
 // on everything the slot table depends on (tiles, digit orders, layout, vector, shape).
 static std::pair<double, double> operand_sim(const Contraction &c, const Config &cfg, int t, int vec,
                                              bool kmaj, int BMN, int BK, WfCache *cache) {
-  std::vector<int64_t> key{t, vec, kmaj, BMN, BK, cfg.morder, cfg.korder};
+  std::vector<int64_t> key{t, vec, kmaj, BMN, BK, cfg.morder, cfg.korder, cfg.kind};
   for (int id : c.t[t].idx) key.push_back(cfg.T[id]);
   for (int id : cfg.kdig) key.push_back(cfg.T[id]);
   if (cache) {
@@ -54,7 +58,8 @@ static std::pair<double, double> operand_sim(const Contraction &c, const Config 
     if (it != cache->end()) return it->second;
   }
   const SlotTable st = build_slots(c, cfg, t, vec, kmaj, BMN, BK);
-  const std::pair<double, double> r{slot_wavefronts(st, vec), slot_sectors(st, vec)};
+  const int es = cfg.kind == KIND_BF16_UMMA ? 2 : 8;
+  const std::pair<double, double> r{slot_wavefronts(st, vec, es, cfg.kind), slot_sectors(st, vec, es)};
   if (cache) (*cache)[key] = r;
   return r;
 }
@@ -64,9 +69,11 @@ double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *
   finish_counts(c, cfg);
   const double nctas = (double)cfg.nctas, steps = (double)cfg.nsteps;
   // per CTA-step pipe cycles on one SM: FP64 (DMMA) and shared memory
-  const double dmma = (double)v.BM * v.BN * v.BK / kFmaPerClk;
-  cfg.vecX = vec_possible(c, cfg, cfg.X) ? 2 : 1;
-  cfg.vecY = vec_possible(c, cfg, cfg.Y) ? 2 : 1;
+  const double dmma = (double)v.BM * v.BN * v.BK / fma_per_clk(v.kind);
+  const bool umma = v.kind == KIND_BF16_UMMA;
+  const int maxv = cfg.kind == KIND_BF16_UMMA ? 8 : 2;   // 16 B per cp.async
+  cfg.vecX = vec_width(c, cfg, cfg.X, maxv);
+  cfg.vecY = vec_width(c, cfg, cfg.Y, maxv);
   const auto sx = operand_sim(c, cfg, cfg.X, cfg.vecX, cfg.xKmajor, v.BM, v.BK, cache);
   const auto sy = operand_sim(c, cfg, cfg.Y, cfg.vecY, cfg.yKmajor, v.BN, v.BK, cache);
   cfg.wfX = sx.first;
@@ -74,28 +81,35 @@ double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *
   cfg.secX = sx.second;
   cfg.secY = sy.second;
   const int MI = v.WM / 8, NJ = v.WN / 8, warps = v.cwarps();
-  const double lds = (double)warps * (v.BK / 4) * (MI + NJ) * 2;
+  // FP64: consumer-warp fragment loads; UMMA reads its operands from smem descriptors
+  const double lds = umma ? 0.0 : (double)warps * (v.BK / 4) * (MI + NJ) * 2;
   // producer warps: one LDGSTS warp-instruction per 32 slots, ~8 LSU cycles each
   const double nslots = (double)cfg.Mt * cfg.Kt / cfg.vecX + (double)cfg.Kt * cfg.Nt / cfg.vecY;
   const double ldgsts = std::ceil(nslots / 32.0) * 8.0;
   const double step = std::max({dmma, cfg.wfX + cfg.wfY + lds, ldgsts}) + kStepOverhead;
-  const double epi = (double)warps * MI * NJ * 2 * 6 / 4;     // store issue per tile
+  // store issue per tile; UMMA: 4 warps x BN column stores, overlapped with the next
+  // tile's MMAs by the double-buffered TMEM accumulator
+  const double epi = umma ? 0.0 : (double)warps * MI * NJ * 2 * 6 / 4;
+  const double epi_umma = umma ? (double)v.BN * 4 * 4 : 0.0;
   // persistent CTAs: grid = 148 * occ, tiles round-robin
   const double slots = kSMs * v.occ;
   const double tiles_per_cta = std::ceil(nctas / slots);
-  const double cyc_sm = tiles_per_cta * v.occ * (steps * step + epi);
+  const double cyc_sm = tiles_per_cta * v.occ * std::max(steps * step + epi, epi_umma);
   cfg.t_comp = cyc_sm / kClk;
   // memory: sector efficiencies of each tensor's tile along its own memory order
-  const double eX = sector_eff(contiguous_run(c, cfg.X, cfg.T));
-  const double eY = sector_eff(contiguous_run(c, cfg.Y, cfg.T));
-  const double eC = sector_eff(contiguous_run(c, 0, cfg.T));
+  const double es = v.esize();
+  const double eX = sector_eff(contiguous_run(c, cfg.X, cfg.T), es);
+  const double eY = sector_eff(contiguous_run(c, cfg.Y, cfg.T), es);
+  const double eC = sector_eff(contiguous_run(c, 0, cfg.T), es);
   // store-instruction efficiency: 8 consecutive rows of a DMMA fragment are contiguous in C
   // iff m's first digit is C's FVI
-  double eS = 0.25;
+  // (UMMA: a warp stores 32 rows of one column)
+  const int64_t srun = umma ? 32 : 8;
+  double eS = es / 32.0;
   if (c.t[0].idx.empty()) eS = 1;
   else if (!cfg.mdig.empty() && cfg.mdig[0] == c.t[0].idx[0])
-    eS = sector_eff(std::min<int64_t>(8, cfg.T[cfg.mdig[0]]));
-  const double bx = 8.0 * c.numel(cfg.X), by = 8.0 * c.numel(cfg.Y), bc = 8.0 * c.numel(0);
+    eS = sector_eff(std::min<int64_t>(srun, cfg.T[cfg.mdig[0]]), es);
+  const double bx = es * c.numel(cfg.X), by = es * c.numel(cfg.Y), bc = es * c.numel(0);
   double rx = 1, ry = 1;
   if (bx + by > 0.5 * kL2Bytes) {
     const double f = (bx + by) / kL2Bytes;
@@ -277,13 +291,14 @@ bool fits(const Config &cfg, const Variant &v) {
 }
 
 // The distinct (morder, korder) digit-order options of a contraction.
-std::vector<Config> order_options(const Contraction &c) {
+std::vector<Config> order_options(const Contraction &c, int kind) {
   std::vector<Config> out;
   for (int mo = 0; mo < 2; mo++)
     for (int ko = 0; ko < 2; ko++) {
       Config cfg;
       cfg.morder = mo;
       cfg.korder = ko;
+      cfg.kind = kind;
       digit_orders(c, cfg);
       bool dup = false;
       for (auto &o : out) dup |= o.mdig == cfg.mdig && o.kdig == cfg.kdig;
@@ -295,9 +310,10 @@ std::vector<Config> order_options(const Contraction &c) {
 }  // namespace
 
 // ---------------------------------------------------------------- B200 mode
-static Status choose_b200(const Contraction &c, int forced_variant, Config &best, PlanStats &st) {
+static Status choose_b200(const Contraction &c, int kind, int forced_variant, Config &best, PlanStats &st) {
   WfCache cache;
   Config base;
+  base.kind = kind;
   digit_orders(c, base);
   base.T.assign(c.ix.size(), 1);
   // Alg. 2 walks each input's index list; C's FVI is mapped first on the X side
@@ -309,10 +325,11 @@ static Status choose_b200(const Contraction &c, int forced_variant, Config &best
   int kfirst = -1;
   if (!c.t[base.X].idx.empty() && c.ix[c.t[base.X].idx[0]].cls == INTL) kfirst = c.t[base.X].idx[0];
   else if (!c.t[base.Y].idx.empty() && c.ix[c.t[base.Y].idx[0]].cls == INTL) kfirst = c.t[base.Y].idx[0];
-  const auto orders = order_options(c);
+  const auto orders = order_options(c, kind);
   bool found = false;
   for (int vi = 0; vi < (int)variants().size(); vi++) {
     if (forced_variant >= 0 && vi != forced_variant) continue;
+    if (variants()[vi].kind != kind) continue;
     const auto &v = variants()[vi];
     auto ms = enum_side(c, mx, c0, v.BM);
     auto ns = enum_side(c, ny, -1, v.BN);
@@ -329,7 +346,7 @@ static Status choose_b200(const Contraction &c, int forced_variant, Config &best
       double run = 1;
       for (int t = 1; t <= 2; t++)
         if (!c.t[t].idx.empty() && c.ix[c.t[t].idx[0]].cls == INTL)
-          run *= std::min(4, T[c.t[t].idx[0]]);     // 4 doubles = one 32-B sector
+          run *= std::min(32 / v.esize(), T[c.t[t].idx[0]]);   // one 32-B sector
       kr.push_back({steps * v.BK / need / run, k});
     }
     std::stable_sort(kr.begin(), kr.end(), [](auto &a, auto &b) { return a.first < b.first; });
@@ -363,7 +380,7 @@ static Status choose_b200(const Contraction &c, int forced_variant, Config &best
             if (found) {
               const double tiles = std::ceil((double)cfg.nctas / (kSMs * v.occ));
               const double lb = tiles * v.occ * (double)cfg.nsteps * v.BM * v.BN * v.BK /
-                                kFmaPerClk / kClk + kLaunch;
+                                fma_per_clk(v.kind) / kClk + kLaunch;
               if (lb > best.t_pred) { st.pruned++; continue; }
             }
             model_time(c, cfg, v, &cache);
@@ -378,9 +395,10 @@ static Status choose_b200(const Contraction &c, int forced_variant, Config &best
 // enum_X_TB / enum_X_REG / Y / TB_k with the V100 value sets of P:L176 and Alg. 2's
 // greedy (floor crossing tile, R12); product; prune by P:L172 (smem, registers) and
 // P:L174 (FVI on a thread dimension, #TBs above one wave); rank by Alg. 3.
-static Status choose_paper(const Contraction &c, int forced_variant, Config &best, PlanStats &st) {
+static Status choose_paper(const Contraction &c, int kind, int forced_variant, Config &best, PlanStats &st) {
   WfCache cache;
   Config base;
+  base.kind = kind;
   digit_orders(c, base);
   base.T.assign(c.ix.size(), 1);
   const int X = base.X, Y = base.Y;
@@ -473,7 +491,7 @@ static Status choose_paper(const Contraction &c, int forced_variant, Config &bes
         const double TBy = (double)tprod(y.tb), REGy = (double)tprod(y.reg);
         const double TBk = (double)tprod(k);
         // P:L172 hardware constraints (V100: 48 KB smem per block, 255 registers/thread)
-        const double smem = 8.0 * (TBx * TBk * REGx + TBy * TBk * REGy);
+        const double smem = (kind == KIND_BF16_UMMA ? 2.0 : 8.0) * (TBx * TBk * REGx + TBy * TBk * REGy);
         bool ok = smem <= 48 * 1024 && REGx * REGy <= 64 && TBx * TBy <= 1024;
         // enough thread blocks (R16: at least one wave of the running GPU)
         ok &= (double)cfg.nctas >= kSMs;
@@ -483,6 +501,7 @@ static Status choose_paper(const Contraction &c, int forced_variant, Config &bes
         if (ok) {
           for (int vi = 0; vi < (int)variants().size(); vi++) {
             if (forced_variant >= 0 && vi != forced_variant) continue;
+            if (variants()[vi].kind != kind) continue;
             if (!fits(cfg, variants()[vi])) continue;
             Config t = cfg;
             t.variant = vi;
@@ -505,11 +524,11 @@ static Status choose_paper(const Contraction &c, int forced_variant, Config &bes
 }
 
 // ---------------------------------------------------------------- forced tiles
-static Status choose_forced(const Contraction &c, const ForcedTiles &ft, int forced_variant,
+static Status choose_forced(const Contraction &c, int kind, const ForcedTiles &ft, int forced_variant,
                             Config &best, std::string &err) {
   WfCache cache;
   bool found = false;
-  for (const auto &o : order_options(c)) {
+  for (const auto &o : order_options(c, kind)) {
     Config cfg = o;
     cfg.T.assign(c.ix.size(), 1);
     for (size_t id = 0; id < c.ix.size(); id++) {
@@ -520,6 +539,7 @@ static Status choose_forced(const Contraction &c, const ForcedTiles &ft, int for
     finish_counts(c, cfg);
     for (int vi = 0; vi < (int)variants().size(); vi++) {
       if (forced_variant >= 0 && vi != forced_variant) continue;
+      if (variants()[vi].kind != kind) continue;
       if (!fits(cfg, variants()[vi])) continue;
       Config t = cfg;
       t.variant = vi;
@@ -531,20 +551,20 @@ static Status choose_forced(const Contraction &c, const ForcedTiles &ft, int for
   return ST_OK;
 }
 
-Status choose(const Contraction &c, int cost_mode, int forced_variant, const ForcedTiles &ft,
+Status choose(const Contraction &c, int kind, int cost_mode, int forced_variant, const ForcedTiles &ft,
               Config &out, PlanStats &stats, std::string &err) {
   auto t0 = std::chrono::steady_clock::now();
   stats = PlanStats();
   stats.cost_mode = cost_mode;
   Status s;
-  if (ft.on) s = choose_forced(c, ft, forced_variant, out, err);
-  else if (cost_mode == 1) s = choose_paper(c, forced_variant, out, stats);
-  else s = choose_b200(c, forced_variant, out, stats);
+  if (ft.on) s = choose_forced(c, kind, ft, forced_variant, out, err);
+  else if (cost_mode == 1) s = choose_paper(c, kind, forced_variant, out, stats);
+  else s = choose_b200(c, kind, forced_variant, out, stats);
   if (s == ST_NO_CONFIG && !ft.on && cost_mode == 1) {
     // the paper's value sets can leave nothing after pruning (tiny problems): fall back to
     // the B200 enumeration so that every legal contraction gets a plan (R13)
     PlanStats st2;
-    s = choose_b200(c, forced_variant, out, st2);
+    s = choose_b200(c, kind, forced_variant, out, st2);
     stats.ranked += st2.ranked;
   }
   if (s != ST_OK && err.empty()) err = "no legal configuration";

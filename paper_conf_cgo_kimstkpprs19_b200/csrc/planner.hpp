@@ -33,7 +33,7 @@ struct ForcedTiles {
 };
 
 // Choose a configuration.  forced_variant < 0: planner's choice.
-Status choose(const Contraction &c, int cost_mode, int forced_variant, const ForcedTiles &ft,
+Status choose(const Contraction &c, int kind, int cost_mode, int forced_variant, const ForcedTiles &ft,
               Config &out, PlanStats &stats, std::string &err);
 
 // B200 model (seconds); fills cfg's model outputs.

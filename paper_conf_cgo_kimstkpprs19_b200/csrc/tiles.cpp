@@ -21,6 +21,9 @@ const std::vector<Variant> &variants() {
       {128, 32, 24, 32, 32, 3, 4, 1},   // 8
       {32, 128, 24, 32, 32, 3, 4, 1},   // 9
       {64, 64, 8, 32, 32, 4, 4, 2},     // 10
+      // BF16 x BF16 -> FP32 on tcgen05 (kernel_bf16.cuh): BM = 128 (UMMA M), BK = 64
+      {128, 64, 64, 32, 32, 6, 4, 1, KIND_BF16_UMMA},    // 11
+      {128, 128, 64, 32, 32, 5, 4, 1, KIND_BF16_UMMA},   // 12
   };
   return v;
 }
@@ -59,21 +62,26 @@ void finish_counts(const Contraction &c, Config &cfg) {
   cfg.nctas = cfg.mtiles * cfg.ntiles;
 }
 
-bool vec_possible(const Contraction &c, const Config &cfg, int t) {
-  // the operand's FVI leads its smem-contiguous dimension; even tile and extent; stride 1;
-  // every other stride and the base even (so every pair is 16-B aligned)
+int vec_width(const Contraction &c, const Config &cfg, int t, int maxv) {
+  // the operand's FVI leads its smem-contiguous dimension; tile, extent, every other stride
+  // and the base divisible by the width (every vector aligned to its size)
   const auto &v = c.t[t];
-  if (v.idx.empty() || v.stride[0] != 1) return false;
+  if (v.idx.empty() || v.stride[0] != 1) return 1;
   const int f = v.idx[0];
   const bool isk = c.ix[f].cls == INTL;
   const bool kmaj = t == cfg.X ? cfg.xKmajor : cfg.yKmajor;
-  if (isk != kmaj) return false;
+  if (isk != kmaj) return 1;
   const auto &lst = isk ? cfg.kdig : (t == cfg.X ? cfg.mdig : cfg.ndig);
-  if (lst.empty() || lst[0] != f) return false;
-  if (cfg.T[f] % 2 || c.ix[f].n % 2) return false;
-  for (size_t p = 1; p < v.stride.size(); p++) if (v.stride[p] % 2) return false;
-  return v.base % 2 == 0;
+  if (lst.empty() || lst[0] != f) return 1;
+  for (int w = maxv; w >= 2; w /= 2) {
+    bool ok = cfg.T[f] % w == 0 && c.ix[f].n % w == 0 && v.base % w == 0;
+    for (size_t p = 1; p < v.stride.size(); p++) ok &= v.stride[p] % w == 0;
+    if (ok) return w;
+  }
+  return 1;
 }
+
+bool vec_possible(const Contraction &c, const Config &cfg, int t) { return vec_width(c, cfg, t, 2) == 2; }
 
 SlotTable build_slots(const Contraction &c, const Config &cfg, int t, int vec, bool kmajor,
                       int BMN, int BK) {
@@ -96,6 +104,8 @@ SlotTable build_slots(const Contraction &c, const Config &cfg, int t, int vec, b
     }
     mul[p] = m;
   }
+  // packed slot: smem offset (elements) | k | row; FP64: 13 | 6 | 13 bits, BF16: 14 | 6 | 12
+  const int kshift = cfg.kind == KIND_BF16_UMMA ? 14 : 13, mshift = cfg.kind == KIND_BF16_UMMA ? 20 : 19;
   std::vector<int> d(r, 0);
   for (;;) {
     int mn = 0, k = 0;
@@ -105,8 +115,8 @@ SlotTable build_slots(const Contraction &c, const Config &cfg, int t, int vec, b
       rel += d[p] * st[p];
     }
     out.rel.push_back(rel);
-    out.pack.push_back((uint32_t)smem_off(kmajor, mn, k, BMN, BK) | ((uint32_t)k << 13) |
-                       ((uint32_t)mn << 19));
+    out.pack.push_back((uint32_t)smem_off(cfg.kind, kmajor, mn, k, BMN, BK) | ((uint32_t)k << kshift) |
+                       ((uint32_t)mn << mshift));
     int p = 0;
     for (; p < r; p++) {
       d[p] += (p == 0 ? vec : 1);
@@ -118,7 +128,7 @@ SlotTable build_slots(const Contraction &c, const Config &cfg, int t, int vec, b
   return out;
 }
 
-double slot_sectors(const SlotTable &s, int vec) {
+double slot_sectors(const SlotTable &s, int vec, int esize) {
   const size_t n = s.rel.size();
   double total = 0;
   std::vector<int64_t> sec;
@@ -126,8 +136,8 @@ double slot_sectors(const SlotTable &s, int vec) {
     const size_t e = std::min(n, b + 32);
     sec.clear();
     for (size_t i = b; i < e; i++) {
-      sec.push_back((s.rel[i] * 8) >> 5);
-      sec.push_back((s.rel[i] * 8 + 8 * vec - 1) >> 5);
+      sec.push_back((s.rel[i] * esize) >> 5);
+      sec.push_back((s.rel[i] * esize + esize * vec - 1) >> 5);
     }
     std::sort(sec.begin(), sec.end());
     total += (double)(std::unique(sec.begin(), sec.end()) - sec.begin());
@@ -135,29 +145,23 @@ double slot_sectors(const SlotTable &s, int vec) {
   return total;
 }
 
-double slot_wavefronts(const SlotTable &s, int vec) {
+double slot_wavefronts(const SlotTable &s, int vec, int esize, int kind) {
   const size_t n = s.pack.size();
   double total = 0;
   for (size_t b = 0; b < n; b += 32) {
     const size_t e = std::min(n, b + 32);
-    int cnt[32] = {0};
     std::set<uint32_t> words[32];
     for (size_t i = b; i < e; i++) {
-      const uint32_t off = s.pack[i] & 8191;           // in doubles
-      for (int w = 0; w < 2 * vec; w++) {
-        const uint32_t word = off * 2 + w;             // 32-bit words
-        words[word & 31].insert(word);
-      }
+      const uint32_t byte0 = slot_off(s.pack[i], kind) * (uint32_t)esize;
+      for (uint32_t w = byte0 / 4; w < (byte0 + (uint32_t)(esize * vec) + 3) / 4; w++) words[w & 31].insert(w);
     }
     int wf = 0;
     for (int k = 0; k < 32; k++) wf = std::max(wf, (int)words[k].size());
-    const int minwf = (int)((e - b) * 8 * vec + 127) / 128;
+    const int minwf = (int)(((e - b) * esize * vec + 127) / 128);
     total += std::max(wf, minwf);
-    (void)cnt;
   }
   return total;
 }
-
 
 TileTables build_tile_tables(const Contraction &c, const Config &cfg, const Variant &v) {
   TileTables tt;

@@ -11,20 +11,31 @@
 namespace tc {
 
 // Compiled kernel shapes (kernel_f64.cuh template instances, api.cu kernel table).
+enum Kind { KIND_F64_DMMA = 0, KIND_BF16_UMMA = 1 };
+
 struct Variant {
   int BM, BN, BK, WM, WN, stages, pw, occ;   // pw = producer warps
-  int threads() const { return ((BM / WM) * (BN / WN) + pw) * 32; }
-  int cwarps() const { return (BM / WM) * (BN / WN); }
+  int kind = KIND_F64_DMMA;
+  int threads() const { return kind == KIND_BF16_UMMA ? 13 * 32 : ((BM / WM) * (BN / WN) + pw) * 32; }
+  int cwarps() const { return kind == KIND_BF16_UMMA ? 8 : (BM / WM) * (BN / WN); }
+  int esize() const { return kind == KIND_BF16_UMMA ? 2 : 8; }
 };
 const std::vector<Variant> &variants();
 
-// Smem pitches (must match SmemLayout in kernel_f64.cuh): 4 (mod 16) doubles.
-inline int smem_off(bool kmajor, int mn, int k, int BMN, int BK) {
+// Smem offset (in elements) of element (row mn, k) of one operand stage.
+//  FP64 (kernel_f64.cuh SmemLayout): pitch 4 (mod 16) doubles, k- or mn-contiguous.
+//  BF16 (kernel_bf16.cuh): UMMA canonical no-swizzle layout of 8 x 16-B core matrices;
+//  K-major: core (mn/8, k/8) at (mn/8)*BK*8 + (k/8)*64, MN-major: at (mn/8)*64 + (k/8)*BMN*8.
+inline int smem_off(int kind, bool kmajor, int mn, int k, int BMN, int BK) {
+  if (kind == KIND_BF16_UMMA)
+    return kmajor ? (mn / 8) * (BK * 8) + (k / 8) * 64 + (mn % 8) * 8 + (k % 8)
+                  : (mn / 8) * 64 + (k / 8) * (BMN * 8) + (k % 8) * 8 + (mn % 8);
   return kmajor ? mn * (BK + 4) + k : k * (BMN + 4) + mn;
 }
 
 struct Config {
   int variant = -1;
+  int kind = KIND_F64_DMMA;          // which kernel family (from the dtype)
   int X = 1, Y = 2;                  // tensor ids (1 = A, 2 = B) on the M / N side
   int morder = 0;                    // 0: m digits in C order (C's FVI first); 1: X order
   int korder = 0;                    // 0: k digits in X order; 1: in Y order
@@ -47,6 +58,8 @@ void digit_orders(const Contraction &c, Config &cfg);
 void finish_counts(const Contraction &c, Config &cfg);
 // Can operand t use 16-B vectors with this config?
 bool vec_possible(const Contraction &c, const Config &cfg, int t);
+// Largest elements-per-slot vector (<= maxv, power of two) the operand's layout allows.
+int vec_width(const Contraction &c, const Config &cfg, int t, int maxv);
 
 struct SlotTable {
   std::vector<int64_t> rel;    // element offset inside (tile, step)
@@ -57,10 +70,12 @@ SlotTable build_slots(const Contraction &c, const Config &cfg, int t, int vec, b
                       int BMN, int BK);
 // Shared-memory wavefronts of the cp.async writes of one stage (32 consecutive slots per
 // warp instruction; a bank serves one 32-bit word per wavefront).
-double slot_wavefronts(const SlotTable &s, int vec);
+double slot_wavefronts(const SlotTable &s, int vec, int esize = 8, int kind = KIND_F64_DMMA);
 // Global-memory 32-B sectors one stage of loads touches (sum over warp instructions of the
 // distinct sectors of 32 consecutive slots; the tile origin is taken as sector-aligned).
-double slot_sectors(const SlotTable &s, int vec);
+double slot_sectors(const SlotTable &s, int vec, int esize = 8);
+// Smem offset field of a packed slot (13 bits for FP64, 14 bits for BF16).
+inline uint32_t slot_off(uint32_t pack, int kind) { return kind == KIND_BF16_UMMA ? (pack & 0x3FFF) : (pack & 8191); }
 
 // Device-side tables for one configuration.
 struct TileTables {

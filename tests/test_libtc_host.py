@@ -11,6 +11,7 @@ import pytest
 import tcinputs
 from paper_conf_cgo_kimstkpprs19_b200 import binding as tc
 from paper_conf_cgo_kimstkpprs19_b200 import build
+from paper_conf_cgo_kimstkpprs19_b200.csrc_variants import BF16_VARIANTS
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
@@ -56,10 +57,14 @@ def test_fusion_row_a2():
     assert len(i["indices"]) == 5
 
 
+@pytest.mark.parametrize("dtype", ["f64", "bf16"])
 @pytest.mark.parametrize("cost", ["b200", "paper"])
-def test_planner_invariants_tccg(cost):
+def test_planner_invariants_tccg(cost, dtype):
     for case in [tcinputs.eq1()] + tcinputs.tccg48():
-        i = tc.plan(case.expr, case.extents, host_only=True, cost=cost).info()
+        i = tc.plan(case.expr, case.extents, host_only=True, cost=cost, dtype=dtype).info()
+        assert i["dtype"] == dtype
+        assert (i["variant"] in BF16_VARIANTS) == (dtype == "bf16")
+        assert i["vecX"] <= (8 if dtype == "bf16" else 2) and i["vecY"] <= (8 if dtype == "bf16" else 2)
         assert i["Mt"] <= i["BM"] and i["Nt"] <= i["BN"] and i["Kt"] <= i["BK"]
         for x in i["indices"]:
             assert 1 <= x["tile"] <= x["n"]
@@ -128,8 +133,11 @@ def test_errors_are_status_codes():
         tc.plan("abcd-aebf-dfc", "a:2;b:2;c:2;d:2;e:2;f:2", host_only=True)
     assert e.value.status == "TC_ERR_INDEX" and "exactly two" in e.value.detail
     with pytest.raises(tc.TcError) as e:
-        tc.plan("ab-ac-cb", "a:2;b:2;c:2", dtype="bf16", host_only=True)
+        tc.plan("ab-ac-cb", "a:2;b:2;c:2", dtype="f32", host_only=True)
     assert e.value.status == "TC_ERR_UNSUPPORTED"
+    with pytest.raises(tc.TcError) as e:              # an FP64 variant for a BF16 plan
+        tc.plan("ab-ac-cb", "a:2;b:2;c:2", dtype="bf16", host_only=True, variant=0)
+    assert e.value.status == "TC_ERR_INVALID_ARG"
     p = tc.plan("ab-ac-cb", "a:2;b:2;c:2", host_only=True)
     with pytest.raises(tc.TcError) as e:
         p.execute_ptr(16, 32, 64)

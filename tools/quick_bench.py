@@ -12,6 +12,8 @@ from paper_conf_cgo_kimstkpprs19_b200 import binding as tc  # noqa: E402
 
 def main():
     cost = sys.argv[1] if len(sys.argv) > 1 else "b200"
+    dtype = os.environ.get("TC_DTYPE", "f64")
+    tdt = torch.bfloat16 if dtype == "bf16" else torch.float64
     ids = [int(x) for x in sys.argv[2].split(",")] if len(sys.argv) > 2 else None
     torch.cuda.set_device(0)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
@@ -19,11 +21,11 @@ def main():
     for case in tcinputs.tccg48():
         if ids and case.id not in ids:
             continue
-        p = tc.plan(case.expr, case.extents, cost=cost)
+        p = tc.plan(case.expr, case.extents, cost=cost, dtype=dtype)
         info = p.info()
-        A = tcinputs.uniform(p.numel("A"), 1000 + case.id, device="cuda")
-        B = tcinputs.uniform(p.numel("B"), 2000 + case.id, device="cuda")
-        C = torch.empty(p.numel("C"), dtype=torch.float64, device="cuda")
+        A = tcinputs.uniform(p.numel("A"), 1000 + case.id, device="cuda").to(tdt)
+        B = tcinputs.uniform(p.numel("B"), 2000 + case.id, device="cuda").to(tdt)
+        C = torch.empty(p.numel("C"), dtype=tdt, device="cuda")
         for _ in range(3):
             p.execute(A, B, C)
         ts = []
@@ -39,6 +41,7 @@ def main():
         ms = ts[len(ts) // 2]
         gf = p.flops / ms / 1e6
         r = {"id": case.id, "expr": case.expr, "ms": round(ms, 4), "gflops": round(gf, 1),
+             "vec": [info["vecX"], info["vecY"]], "kmaj": [info["xKmajor"], info["yKmajor"]],
              "pred_ms": round(info["t_pred_ms"], 4), "variant": info["variant"],
              "Mt": info["Mt"], "Nt": info["Nt"], "Kt": info["Kt"],
              "tiles": {x["name"]: x["tile"] for x in info["indices"]}}

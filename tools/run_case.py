@@ -14,10 +14,12 @@ reps = int(sys.argv[2]) if len(sys.argv) > 2 else 3
 cost = sys.argv[3] if len(sys.argv) > 3 else "b200"
 variant = int(sys.argv[4]) if len(sys.argv) > 4 else None
 case = [c for c in tcinputs.tccg48() if c.id == cid][0] if cid > 0 else tcinputs.eq1()
-p = tc.plan(case.expr, case.extents, cost=cost, variant=variant)
-A = tcinputs.uniform(p.numel("A"), 1000 + cid, device="cuda")
-B = tcinputs.uniform(p.numel("B"), 2000 + cid, device="cuda")
-C = torch.empty(p.numel("C"), dtype=torch.float64, device="cuda")
+dtype = os.environ.get("TC_DTYPE", "f64")
+tdt = torch.bfloat16 if dtype == "bf16" else torch.float64
+p = tc.plan(case.expr, case.extents, cost=cost, variant=variant, dtype=dtype)
+A = tcinputs.uniform(p.numel("A"), 1000 + cid, device="cuda").to(tdt)
+B = tcinputs.uniform(p.numel("B"), 2000 + cid, device="cuda").to(tdt)
+C = torch.empty(p.numel("C"), dtype=tdt, device="cuda")
 for _ in range(reps):
     p.execute(A, B, C)
 torch.cuda.synchronize()
