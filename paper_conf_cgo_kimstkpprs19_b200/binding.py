@@ -170,8 +170,9 @@ class Plan:
 
 def plan(expr: str, extents: str, dtype: str = "f64", cost: str = "b200", host_only: bool = False,
          variant: int | None = None, force_tiles: str | None = None, fusion: bool = True,
-         tma: bool = False) -> Plan:
+         tma: bool = False, dbg: int = 0) -> Plan:
     o = _Opts()
+    o.reserved[0] = int(dbg)
     o.tma_epilogue = int(tma)
     o.cost_mode = COST[cost]
     o.host_only = int(host_only)

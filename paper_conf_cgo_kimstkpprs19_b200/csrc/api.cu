@@ -72,6 +72,7 @@ struct tc_plan_s {
   std::string force_tiles;
   TileTables tt;
   SlotTable slotX1, slotY1, slotX2, slotY2;   // scalar and cfg.vecX / cfg.vecY wide slots
+  int cvec = 1;            // c_vec_width of the plan (BF16 staged epilogue when 8)
   KParams kp{};            // device pointers filled in; X/Y/C/alpha/beta/slots set per call
   void *dev = nullptr;     // one device buffer with every table
   size_t dev_bytes = 0;
@@ -99,6 +100,7 @@ void build_host_tables(tc_plan_s *P) {
   P->slotY1 = build_slots(c, cfg, cfg.Y, 1, cfg.yKmajor, v.BN, v.BK);
   if (cfg.vecX > 1) P->slotX2 = build_slots(c, cfg, cfg.X, cfg.vecX, cfg.xKmajor, v.BM, v.BK);
   if (cfg.vecY > 1) P->slotY2 = build_slots(c, cfg, cfg.Y, cfg.vecY, cfg.yKmajor, v.BN, v.BK);
+  P->cvec = cfg.kind == KIND_BF16_UMMA ? c_vec_width(c, cfg, 8) : 1;
   KParams &kp = P->kp;
   std::memset(&kp, 0, sizeof(kp));
   kp.mtiles = (int)cfg.mtiles;
@@ -111,6 +113,12 @@ void build_host_tables(tc_plan_s *P) {
     kp.fullN[w] = P->tt.tileN[0].mask[w];
   }
   kp.fullK = cfg.Kt >= 64 ? ~0ull : ((1ull << cfg.Kt) - 1);
+  kp.kcnt0 = P->tt.kcnt0;
+  kp.kdX0 = P->tt.kdX0;
+  kp.kdY0 = P->tt.kdY0;
+  kp.ktail0 = P->tt.ktail0;
+  kp.kbase = P->tt.kbase;
+  kp.nouter = (int)P->tt.kouter.size();
   kp.Mt = (int)cfg.Mt;
   kp.Nt = (int)cfg.Nt;
   kp.c_rank = (int)c.t[0].idx.size();
@@ -132,9 +140,7 @@ Status upload(tc_plan_s *P, std::string &err) {
   size_t iRn = add(tt.relCn.data(), 8 * tt.relCn.size());
   size_t iBm = add(tt.boxM.data(), 4 * tt.boxM.size());
   size_t iBn = add(tt.boxN.data(), 4 * tt.boxN.size());
-  size_t iSx = add(tt.stepX.data(), 8 * tt.stepX.size());
-  size_t iSy = add(tt.stepY.data(), 8 * tt.stepY.size());
-  size_t iK = add(tt.kmask.data(), 8 * tt.kmask.size());
+  size_t iKo = add(tt.kouter.data(), sizeof(KOuter) * tt.kouter.size());
   // slot offsets inside a (tile, step) are 32-bit in the kernel (registers are scarce)
   std::vector<int32_t> r32[4];
   const SlotTable *sts[4] = {&P->slotX1, &P->slotY1, &P->slotX2, &P->slotY2};
@@ -166,9 +172,7 @@ Status upload(tc_plan_s *P, std::string &err) {
   kp.relCn = (const int64_t *)(b + parts[iRn].off);
   kp.boxM = (const int32_t *)(b + parts[iBm].off);
   kp.boxN = (const int32_t *)(b + parts[iBn].off);
-  kp.stepX = (const int64_t *)(b + parts[iSx].off);
-  kp.stepY = (const int64_t *)(b + parts[iSy].off);
-  kp.kmask = (const uint64_t *)(b + parts[iK].off);
+  kp.kouter = (const KOuter *)(b + parts[iKo].off);
   P->d_relX1 = (const int32_t *)(b + parts[iX1].off);
   P->d_packX1 = (const uint32_t *)(b + parts[iX1p].off);
   P->d_relY1 = (const int32_t *)(b + parts[iY1].off);
@@ -434,6 +438,8 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
   kp.packY = vy ? plan->d_packY2 : plan->d_packY1;
   kp.nslotY = (int)(vy ? plan->slotY2.pack.size() : plan->slotY1.pack.size());
   kp.vecY = vy ? cfg.vecY : 1;
+  kp.dbg = plan->opts.reserved[0];
+  kp.vecC = plan->cvec == 8 && ((uintptr_t)C % 16) == 0 ? 8 : 1;
   const KernelEntry ke = kernel_for(cfg);
   const int grid = (int)std::min<int64_t>(cfg.nctas, plan->sms);
   void *args[] = {&kp};
@@ -508,7 +514,7 @@ tc_status_t tc_plan_info(const tc_plan_t plan, char *json, size_t cap, size_t *n
     o << ",\"Mt\":" << g.Mt << ",\"Nt\":" << g.Nt << ",\"Kt\":" << g.Kt << ",\"nctas\":" << g.nctas
       << ",\"mtiles\":" << g.mtiles << ",\"ntiles\":" << g.ntiles << ",\"nsteps\":" << g.nsteps
       << ",\"grid\":" << std::min<int64_t>(g.nctas, plan->sms);
-    o << ",\"vecX\":" << g.vecX << ",\"vecY\":" << g.vecY << ",\"xKmajor\":" << g.xKmajor
+    o << ",\"vecX\":" << g.vecX << ",\"vecY\":" << g.vecY << ",\"vecC\":" << plan->cvec << ",\"xKmajor\":" << g.xKmajor
       << ",\"yKmajor\":" << g.yKmajor << ",\"wfX\":" << g.wfX << ",\"wfY\":" << g.wfY;
     char buf[512];
     std::snprintf(buf, sizeof buf,

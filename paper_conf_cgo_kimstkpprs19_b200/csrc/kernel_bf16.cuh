@@ -67,40 +67,70 @@ __device__ __forceinline__ void cp_async8v_full(uint32_t dst, const void *src) {
 // one operand; `cnt` of the E entries are real.  Interior tile and full k-step: no bounds
 // work; otherwise each slot tests its k bit and its row bit and zero-fills.
 template <int E>
-__device__ __forceinline__ void bf16_load_slots(int32_t (&rel)[E], uint32_t (&pack)[E], const int32_t *__restrict__ r,
+__device__ __forceinline__ void bf16_load_slots(int32_t (&rel)[E], uint32_t (&soff)[E], const int32_t *__restrict__ r,
                                                 const uint32_t *__restrict__ pk, int n, int first, int stride) {
 #pragma unroll
   for (int i = 0; i < E; i++) {
     const int q = first + i * stride;
     rel[i] = q < n ? __ldg(r + q) : 0;
-    pack[i] = q < n ? __ldg(pk + q) : 0u;
+    soff[i] = q < n ? 2u * (__ldg(pk + q) & 0x3FFF) : 0u;   // smem byte offset in the stage
   }
 }
 
-template <int E, int VB>
+// One operand, one (tile, step): this thread's `cnt` cached 16-B slots.  Interior tile and
+// full k-step (fast): straight copies.  Otherwise each slot re-reads its packed (k, row) from
+// the slot table, tests the step's k mask and the tile's row mask and zero-fills.
+template <int E>
 __device__ __forceinline__ void bf16_issue(const __nv_bfloat16 *__restrict__ src, uint32_t sdst,
-                                           const int32_t (&rel)[E], const uint32_t (&pack)[E], int cnt,
-                                           int64_t base, bool fast, uint64_t kmask, const uint64_t (&rmask)[kMaskWords]) {
+                                           const int32_t (&rel)[E], const uint32_t (&soff)[E], int cnt,
+                                           int64_t base, bool fast, uint64_t kmask, const uint64_t (&rmask)[kMaskWords],
+                                           const uint32_t *__restrict__ pack, int first, int stride) {
   const __nv_bfloat16 *b = src + base;
   if (fast) {
 #pragma unroll
-    for (int i = 0; i < E; i++) {
-      if (i < cnt) {
-        const uint32_t d = sdst + 2u * (pack[i] & 0x3FFF);
-        if (VB == 16) cp_async16v_full(d, b + rel[i]);
-        else cp_async8v_full(d, b + rel[i]);
-      }
-    }
+    for (int i = 0; i < E; i++)
+      if (i < cnt) cp_async16v_full(sdst + soff[i], b + rel[i]);
   } else {
 #pragma unroll
     for (int i = 0; i < E; i++) {
       if (i < cnt) {
-        const uint32_t pk = pack[i];
+        const uint32_t pk = __ldg(pack + first + i * stride);
         const int k = (pk >> 14) & 63, m = pk >> 20;
         const bool ok = ((kmask >> k) & 1) && bit_of(rmask, m);
-        const uint32_t d = sdst + 2u * (pk & 0x3FFF);
-        if (VB == 16) cp_async16v(d, ok ? b + rel[i] : src, ok ? 16 : 0);
-        else cp_async8v(d, ok ? b + rel[i] : src, ok ? 8 : 0);
+        cp_async16v(sdst + soff[i], ok ? b + rel[i] : src, ok ? 16 : 0);
+      }
+    }
+  }
+}
+
+// Generic producer path (any vector width, slot tables read from global memory): every slot
+// tests its k bit and its row bit and zero-fills when out of range.
+template <int PW>
+__device__ __forceinline__ void bf16_issue_generic_t(const KParams &p, const __nv_bfloat16 *__restrict__ X,
+                                                     const __nv_bfloat16 *__restrict__ Y, int pt, uint32_t dx,
+                                                     uint32_t dy, int64_t bx, int64_t by, uint64_t km,
+                                                     const uint64_t (&mm)[kMaskWords],
+                                                     const uint64_t (&mn)[kMaskWords]) {
+  for (int side = 0; side < 2; side++) {
+    const __nv_bfloat16 *src = side ? Y : X;
+    const int32_t *rel = side ? p.relY : p.relX;
+    const uint32_t *pack = side ? p.packY : p.packX;
+    const int n = side ? p.nslotY : p.nslotX, vec = side ? p.vecY : p.vecX;
+    const int64_t base = side ? by : bx;
+    const uint32_t dst0 = side ? dy : dx;
+    const uint64_t *rm = side ? mn : mm;
+    for (int q = pt; q < n; q += PW * 32) {
+      const uint32_t pk = __ldg(pack + q);
+      const int k = (pk >> 14) & 63, m = pk >> 20;
+      const bool ok = ((km >> k) & 1) && ((((m < 64) ? rm[0] : rm[1]) >> (m & 63)) & 1);
+      const __nv_bfloat16 *g = ok ? src + (base + __ldg(rel + q)) : src;
+      const uint32_t d = dst0 + 2u * (pk & 0x3FFF);
+      if (vec == 8) cp_async16v(d, g, ok ? 16 : 0);
+      else if (vec == 4) cp_async8v(d, g, ok ? 8 : 0);
+      else if (vec == 2) cp_async4(d, g, ok ? 4 : 0);
+      else {   // single elements: plain load / store (cp.async has no 2-byte form)
+        const unsigned short v = ok ? *reinterpret_cast<const unsigned short *>(g) : (unsigned short)0;
+        asm volatile("st.shared.u16 [%0], %1;\n" ::"r"(d), "h"(v) : "memory");
       }
     }
   }
@@ -126,11 +156,12 @@ __device__ __forceinline__ void tc05_ld(uint32_t taddr, uint32_t (&v)[W]) {
   }
 }
 
-// UMMA shared-memory descriptor, no swizzle (SM100 layout: start>>4 [0,14), LBO>>4
-// [16,30), SBO>>4 [32,46), version 1 [46,48), layout type 0 [61,64)).
+// UMMA shared-memory descriptor, 128-B swizzle (SM100 layout: start>>4 [0,14), LBO>>4
+// [16,30), SBO>>4 [32,46), version 1 [46,48), base offset 0 [49,52), layout type
+// SWIZZLE_128B = 2 [61,64)).
 __device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
   return (uint64_t)((saddr >> 4) & 0x3FFF) | ((uint64_t)((lbo >> 4) & 0x3FFF) << 16) |
-         ((uint64_t)((sbo >> 4) & 0x3FFF) << 32) | (1ull << 46);
+         ((uint64_t)((sbo >> 4) & 0x3FFF) << 32) | (1ull << 46) | (2ull << 61);
 }
 
 template <int BN, int STAGES>
@@ -138,10 +169,12 @@ struct Bf16Kernel {
   static constexpr int BM = 128, BK = 64;            // one UMMA M = 128, four K = 16 per stage
   static constexpr int EW = 8, PW = 4;               // epilogue warps, producer warps
   static constexpr int THREADS = (EW + PW + 1) * 32; // + one MMA warp
-  static constexpr int XS = BM * BK + 8, YS = BN * BK + 8;   // elements per stage (+16-B scratch)
-  static constexpr int TMEM_COLS = 2 * BN;           // double-buffered FP32 accumulator
+  static constexpr int XS = BM * BK, YS = BN * BK;   // elements per stage (1 KB multiples)
+  static constexpr int NBUF = 512 / BN;              // FP32 accumulators in flight (all of TMEM)
+  static constexpr int TMEM_COLS = NBUF * BN;
   static constexpr size_t smem_bytes() {
-    return 2 * (size_t)STAGES * (XS + YS) + 8 * (2 * STAGES + 4) + 16 + 8 * (size_t)(BM + BN);
+    return 1024 + 2 * (size_t)STAGES * (XS + YS) + 8 * (2 * STAGES + 2 * NBUF) + 16 + 8 * (size_t)(BM + BN) +
+           4 * (size_t)EW * 32 * 32;   // + per-epilogue-warp FP32 staging (32 x 32)
   }
   // register-cached slots per producer thread (16-B vectors)
   static constexpr int EX = BM * BK / 8 / (PW * 32), EY = BN * BK / 8 / (PW * 32);
@@ -160,20 +193,25 @@ __global__ void __launch_bounds__(Bf16Kernel<BN, STAGES>::THREADS, 1)
 tc_bf16_umma_kernel(const __grid_constant__ KParams p) {
   using K = Bf16Kernel<BN, STAGES>;
   constexpr int BM = K::BM, BK = K::BK;
-  extern __shared__ __align__(1024) unsigned char smem_raw[];
+  extern __shared__ __align__(1024) unsigned char smem_dyn[];
+  // the 128-B swizzle atoms (8 rows x 128 B) must sit on 1 KB boundaries
+  unsigned char *smem_raw =
+      smem_dyn + ((1024u - ((uint32_t)__cvta_generic_to_shared(smem_dyn) & 1023u)) & 1023u);
   __nv_bfloat16 *sX = reinterpret_cast<__nv_bfloat16 *>(smem_raw);
   __nv_bfloat16 *sY = sX + STAGES * K::XS;
   uint64_t *bars = reinterpret_cast<uint64_t *>(sY + STAGES * K::YS);  // full, empty, tfull[2], tempty[2]
-  uint32_t *tmem_holder = reinterpret_cast<uint32_t *>(bars + 2 * STAGES + 4);
+  uint32_t *tmem_holder = reinterpret_cast<uint32_t *>(bars + 2 * STAGES + 2 * K::NBUF);
   int64_t *relCm = reinterpret_cast<int64_t *>(tmem_holder + 4);
   int64_t *relCn = relCm + BM;
+  float *stage = reinterpret_cast<float *>(relCn + BN);   // [EW][32 columns][32 rows]
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int ntl = (p.ntotal - (int)blockIdx.x + (int)gridDim.x - 1) / (int)gridDim.x;
   const int total = max(ntl, 0) * p.nsteps;
   const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(smem_raw);
   const uint32_t bar0 = (uint32_t)__cvta_generic_to_shared(bars);
-  const uint32_t FULL = bar0, EMPTY = bar0 + 8 * STAGES, TFULL = bar0 + 16 * STAGES, TEMPTY = TFULL + 16;
+  const uint32_t FULL = bar0, EMPTY = bar0 + 8 * STAGES, TFULL = bar0 + 16 * STAGES,
+                 TEMPTY = TFULL + 8 * K::NBUF;
 
   // ---- once per CTA ------------------------------------------------------------------------
   for (int i = tid; i < STAGES * (K::XS + K::YS) / 8; i += K::THREADS)
@@ -185,7 +223,7 @@ tc_bf16_umma_kernel(const __grid_constant__ KParams p) {
       mbar_init(FULL + 8 * s, K::PW * 32);   // producer threads (cp.async arrivals)
       mbar_init(EMPTY + 8 * s, 1);           // tcgen05.commit of the MMA thread
     }
-    for (int b = 0; b < 2; b++) {
+    for (int b = 0; b < K::NBUF; b++) {
       mbar_init(TFULL + 8 * b, 1);           // tcgen05.commit after a tile's last MMA
       mbar_init(TEMPTY + 8 * b, K::EW);      // one arrive per epilogue warp
     }
@@ -207,10 +245,6 @@ tc_bf16_umma_kernel(const __grid_constant__ KParams p) {
     const int pt = tid - K::EW * 32;
     const __nv_bfloat16 *__restrict__ X = static_cast<const __nv_bfloat16 *>(p.X);
     const __nv_bfloat16 *__restrict__ Y = static_cast<const __nv_bfloat16 *>(p.Y);
-    int step = 0, lt = 0;
-    int64_t ox = 0, oy = 0;
-    uint64_t mm[kMaskWords], mn[kMaskWords];
-    bool fm = true, fn = true;
     // fast path: both operands in 16-B vectors, slots cached in registers
     const bool cached = p.vecX == 8 && p.vecY == 8 && p.nslotX <= K::EX * K::PW * 32 &&
                         p.nslotY <= K::EY * K::PW * 32;
@@ -223,90 +257,77 @@ tc_bf16_umma_kernel(const __grid_constant__ KParams p) {
       cx = (p.nslotX - pt + K::PW * 32 - 1) / (K::PW * 32);
       cy = (p.nslotY - pt + K::PW * 32 - 1) / (K::PW * 32);
     }
+    // next tile's origins / masks fetched during the current tile's last stage; k steps by
+    // the register odometer
+    ProdTile cur;
+    if (ntl > 0) cur.fetch(p, (int)blockIdx.x);
+    KStep ks;
+    ks.reset(p);
+    int step = 0, lt = 0;
     for (int j = 0; j < total; j++) {
       const int s = j % STAGES;
       if (j >= STAGES) mbar_wait(EMPTY + 8 * s, ((j / STAGES) & 1) ^ 1);
-      if (step == 0) {
-        int mt, nt;
-        tile_coords(p, (int)blockIdx.x + lt * (int)gridDim.x, mt, nt);
-        ox = p.tileM[mt].op;
-        oy = p.tileN[nt].op;
-#pragma unroll
-        for (int w = 0; w < kMaskWords; w++) { mm[w] = p.tileM[mt].mask[w]; mn[w] = p.tileN[nt].mask[w]; }
-        fm = fn = true;
-#pragma unroll
-        for (int w = 0; w < kMaskWords; w++) { fm &= mm[w] == p.fullM[w]; fn &= mn[w] == p.fullN[w]; }
-      }
-      const uint64_t km = __ldg(p.kmask + step);
+      if (step + 1 == p.nsteps && lt + 1 < ntl) ProdTile::prefetch(p, (int)blockIdx.x + (lt + 1) * (int)gridDim.x);
+      const uint64_t km = ks.mask(p);
       const bool fk = km == p.fullK;
-      const int64_t bx = ox + __ldg(p.stepX + step), by = oy + __ldg(p.stepY + step);
+      const bool fm = cur.fm, fn = cur.fn;
+      const uint64_t(&mm)[kMaskWords] = cur.mm;
+      const uint64_t(&mn)[kMaskWords] = cur.mn;
+      const int64_t bx = cur.ox + ks.sx(), by = cur.oy + ks.sy();
       const uint32_t dx = sbase + 2u * (uint32_t)(s * K::XS);
       const uint32_t dy = sbase + 2u * (uint32_t)(STAGES * K::XS + s * K::YS);
-      if (cached) {
-        bf16_issue<K::EX, 16>(X, dx, rx, px, cx, bx, fm && fk, km, mm);
-        bf16_issue<K::EY, 16>(Y, dy, ry, py, cy, by, fn && fk, km, mn);
+      if (p.dbg & 8) {
+        mbar_arrive(FULL + 8 * s);
+      } else if (cached) {
+        bf16_issue<K::EX>(X, dx, rx, px, cx, bx, fm && fk, km, mm, p.packX, pt, K::PW * 32);
+        bf16_issue<K::EY>(Y, dy, ry, py, cy, by, fn && fk, km, mn, p.packY, pt, K::PW * 32);
         mbar_arrive_cp_async(FULL + 8 * s);
-        if (++step == p.nsteps) { step = 0; ++lt; }
-        continue;
-      }
-      for (int side = 0; side < 2; side++) {
-        const __nv_bfloat16 *src = side ? Y : X;
-        const int32_t *rel = side ? p.relY : p.relX;
-        const uint32_t *pack = side ? p.packY : p.packX;
-        const int n = side ? p.nslotY : p.nslotX, vec = side ? p.vecY : p.vecX;
-        const int64_t base = side ? by : bx;
-        const uint32_t dst0 = side ? dy : dx;
-        const uint64_t *rm = side ? mn : mm;
-        for (int q = pt; q < n; q += K::PW * 32) {
-          const uint32_t pk = __ldg(pack + q);
-          const int k = (pk >> 14) & 63, m = pk >> 20;
-          const bool ok = ((km >> k) & 1) && ((((m < 64) ? rm[0] : rm[1]) >> (m & 63)) & 1);
-          const __nv_bfloat16 *g = ok ? src + (base + __ldg(rel + q)) : src;
-          const uint32_t d = dst0 + 2u * (pk & 0x3FFF);
-          if (vec == 8) cp_async16v(d, g, ok ? 16 : 0);
-          else if (vec == 4) cp_async8v(d, g, ok ? 8 : 0);
-          else if (vec == 2) cp_async4(d, g, ok ? 4 : 0);
-          else {   // single elements: plain load / store (cp.async has no 2-byte form)
-            const unsigned short v = ok ? *reinterpret_cast<const unsigned short *>(g) : (unsigned short)0;
-            asm volatile("st.shared.u16 [%0], %1;\n" ::"r"(d), "h"(v) : "memory");
-          }
+      } else {
+        bf16_issue_generic_t<K::PW>(p, X, Y, pt, dx, dy, bx, by, km, mm, mn);
+        if (p.vecX == 1 || p.vecY == 1) {
+          // plain stores are published by a release arrive once this thread's copies landed
+          asm volatile("cp.async.wait_all;\n" ::: "memory");
+          mbar_arrive(FULL + 8 * s);
+        } else {
+          mbar_arrive_cp_async(FULL + 8 * s);
         }
       }
-      if (p.vecX == 1 || p.vecY == 1) {
-        // plain stores are published by a release arrive once this thread's copies landed
-        asm volatile("cp.async.wait_all;\n" ::: "memory");
-        mbar_arrive(FULL + 8 * s);
-      } else {
-        mbar_arrive_cp_async(FULL + 8 * s);
+      ks.advance(p);
+      if (++step == p.nsteps) {
+        step = 0;
+        if (++lt < ntl) cur.fetch(p, (int)blockIdx.x + lt * (int)gridDim.x);
       }
-      if (++step == p.nsteps) { step = 0; ++lt; }
     }
   } else if (warp == K::EW + K::PW) {
     // ======================= MMA issuer ===================================================
     constexpr uint32_t IDESC = umma_idesc_bf16(BN, !XK, !YK);
     // canonical no-swizzle layouts (bytes): K-major LBO = 128 (k groups), SBO = 1024 (8-row
     // groups); MN-major SBO = 128 (8-row groups), LBO = rows/8 * 128 (k groups)
-    constexpr uint32_t A_LBO = XK ? 128 : (BM / 8) * 128, A_SBO = XK ? (BK / 8) * 128 : 128;
-    constexpr uint32_t B_LBO = YK ? 128 : (BN / 8) * 128, B_SBO = YK ? (BK / 8) * 128 : 128;
-    constexpr uint32_t A_KSTEP = XK ? 256 : 2 * A_LBO, B_KSTEP = YK ? 256 : 2 * B_LBO;  // per K = 16
+    // 128-B swizzled layouts (tiles.hpp smem_off): K-major = 8-row x 128-B atoms stacked
+    // along M/N (SBO = 1 KB; K = 16 advances the start by 32 B inside the atom); MN-major =
+    // 64-element x 8-k atoms, MN atoms at LBO = 1 KB, 8-k groups at SBO = BMN/64 KB
+    constexpr uint32_t A_LBO = XK ? 16 : 1024, A_SBO = XK ? 1024 : (BM / 64) * 1024;
+    constexpr uint32_t B_LBO = YK ? 16 : 1024, B_SBO = YK ? 1024 : (BN / 64) * 1024;
+    constexpr uint32_t A_KSTEP = XK ? 32 : 2 * A_SBO, B_KSTEP = YK ? 32 : 2 * B_SBO;  // per K = 16
     int step = 0, lt = 0;
     for (int j = 0; j < total; j++) {
       const int s = j % STAGES;
-      const int buf = lt & 1;
-      if (step == 0 && lt >= 2) mbar_wait(TEMPTY + 8 * buf, ((lt >> 1) & 1) ^ 1);
+      const int buf = lt % K::NBUF;
+      if (step == 0 && lt >= K::NBUF) mbar_wait(TEMPTY + 8 * buf, ((lt / K::NBUF) & 1) ^ 1);
       mbar_wait(FULL + 8 * s, (j / STAGES) & 1);
       // the stage was written through the generic proxy (cp.async / st.shared); the MMA
       // reads it through the async proxy
-      asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
+      if (!(p.dbg & 16)) asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
       tc05_fence_after();
       if (lane == 0) {
         const uint32_t ax = sbase + 2u * (uint32_t)(s * K::XS);
         const uint32_t by = sbase + 2u * (uint32_t)(STAGES * K::XS + s * K::YS);
 #pragma unroll
         for (int kk = 0; kk < BK / 16; kk++)
-          tc05_mma_bf16(tmem + (uint32_t)(buf * BN), umma_desc(ax + kk * A_KSTEP, A_LBO, A_SBO),
+          if (!(p.dbg & 2)) tc05_mma_bf16(tmem + (uint32_t)(buf * BN), umma_desc(ax + kk * A_KSTEP, A_LBO, A_SBO),
                         umma_desc(by + kk * B_KSTEP, B_LBO, B_SBO), IDESC, (step > 0 || kk > 0) ? 1u : 0u);
-        tc05_commit(EMPTY + 8 * s);                      // smem stage free once MMAs read it
+        if (p.dbg & 64) mbar_arrive(EMPTY + 8 * s);
+        else tc05_commit(EMPTY + 8 * s);                      // smem stage free once MMAs read it
         if (step + 1 == p.nsteps) tc05_commit(TFULL + 8 * buf);   // accumulator ready
       }
       __syncwarp();
@@ -322,25 +343,90 @@ tc_bf16_umma_kernel(const __grid_constant__ KParams p) {
     const int row = quarter * 32 + lane;               // TMEM lane = tile row m
     const int64_t roff = relCm[row];
     constexpr int HC = BN / 2;                          // columns per warp
-    for (int lt = 0; lt < ntl; lt++) {
-      const int buf = lt & 1;
+    // staged path: lane drains row group g (8 C-contiguous rows) of columns lane/4 + 8i
+    float *stg = stage + warp * 32 * 32;
+    const int g = lane & 3;
+    const int grow = quarter * 32 + g * 8;
+    const int64_t goff = relCm[grow];
+    // tile info is fetched one tile ahead: its load latency hides behind the current tile
+    int64_t ncoff = 0;
+    uint64_t nrm0 = 0, nrm1 = 0, ncm0 = 0, ncm1 = 0;
+    auto fetch = [&](int t) {
       int mt, nt;
-      tile_coords(p, (int)blockIdx.x + lt * (int)gridDim.x, mt, nt);
-      const TileInfo &tm = p.tileM[mt];
-      const TileInfo &tn = p.tileN[nt];
-      const bool rok = ((row < 64 ? tm.mask[0] : tm.mask[1]) >> (row & 63)) & 1;
-      __nv_bfloat16 *Crow = C + (tm.c + tn.c + roff);
-      const uint64_t cm0 = tn.mask[0], cm1 = tn.mask[1];
+      tile_coords(p, (int)blockIdx.x + t * (int)gridDim.x, mt, nt);
+      ncoff = p.tileM[mt].c + p.tileN[nt].c;
+      nrm0 = p.tileM[mt].mask[0];
+      nrm1 = p.tileM[mt].mask[1];
+      ncm0 = p.tileN[nt].mask[0];
+      ncm1 = p.tileN[nt].mask[1];
+    };
+    if (ntl > 0) fetch(0);
+    for (int lt = 0; lt < ntl; lt++) {
+      const int buf = lt % K::NBUF;
+      const int64_t coff = ncoff;
+      const uint64_t rm0 = nrm0, rm1 = nrm1, cm0 = ncm0, cm1 = ncm1;
+      if (lt + 1 < ntl) fetch(lt + 1);
+      const bool rok = ((row < 64 ? rm0 : rm1) >> (row & 63)) & 1;
+      __nv_bfloat16 *Crow = C + (coff + roff);
       const bool cfull = cm0 == p.fullN[0] && cm1 == p.fullN[1];
-      mbar_wait(TFULL + 8 * buf, (lt >> 1) & 1);
+      const bool gok = ((grow < 64 ? rm0 : rm1) >> (grow & 63)) & 1;
+      __nv_bfloat16 *Cg = C + (coff + goff);
+      if (p.dbg & 256) mbar_wait(TFULL + 8 * buf, (lt / K::NBUF) & 1);
+      else mbar_wait_sleep(TFULL + 8 * buf, (lt / K::NBUF) & 1);
       tc05_fence_after();
 #pragma unroll
       for (int c0 = 0; c0 < HC; c0 += 32 > HC ? HC : 32) {
         constexpr int W = 32 > HC ? HC : 32;
         if (half * HC + c0 >= p.Nt) break;             // columns past the tile's Nt: padding
+        if (p.dbg & 4) break;
         uint32_t v[W];
         tc05_ld<W>(tmem + ((uint32_t)(quarter * 32) << 16) + (uint32_t)(buf * BN + half * HC + c0), v);
-        if (rok) {
+        if (p.vecC == 8) {
+          // FP32 accumulators to smem as [column][row], then one 16-B store per 8 rows
+          // (C's FVI leads m with an 8-multiple tile: 8 tile rows are 8 C-contiguous elements)
+#pragma unroll
+          for (int q = 0; q < W; q++) stg[q * 32 + lane] = __uint_as_float(v[q]);
+          __syncwarp();
+          // all smem reads first (independent), then the stores
+          float4 d[W / 8][2];
+          int64_t rc[W / 8];
+          bool ok[W / 8];
+#pragma unroll
+          for (int i = 0; i < W / 8; i++) {
+            const int cc = (lane >> 2) + 8 * i;
+            const int c = half * HC + c0 + cc;
+            ok[i] = gok && c < p.Nt && (((c < 64 ? cm0 : cm1) >> (c & 63)) & 1);
+            rc[i] = relCn[c];
+            d[i][0] = *reinterpret_cast<const float4 *>(stg + cc * 32 + g * 8);
+            d[i][1] = *reinterpret_cast<const float4 *>(stg + cc * 32 + g * 8 + 4);
+          }
+#pragma unroll
+          for (int i = 0; i < W / 8; i++) {
+            if (ok[i]) {
+              float r[8] = {alpha * d[i][0].x, alpha * d[i][0].y, alpha * d[i][0].z, alpha * d[i][0].w,
+                            alpha * d[i][1].x, alpha * d[i][1].y, alpha * d[i][1].z, alpha * d[i][1].w};
+              uint4 *dst = reinterpret_cast<uint4 *>(Cg + rc[i]);
+              if (beta != 0.0f) {
+                const uint4 o = *dst;
+                const uint32_t ow[4] = {o.x, o.y, o.z, o.w};
+#pragma unroll
+                for (int j = 0; j < 4; j++) {
+                  r[2 * j] = fmaf(beta, __uint_as_float(ow[j] << 16), r[2 * j]);
+                  r[2 * j + 1] = fmaf(beta, __uint_as_float(ow[j] & 0xFFFF0000u), r[2 * j + 1]);
+                }
+              }
+              uint32_t w[4];
+#pragma unroll
+              for (int j = 0; j < 4; j++) {
+                const __nv_bfloat162 b2 = __floats2bfloat162_rn(r[2 * j], r[2 * j + 1]);
+                w[j] = *reinterpret_cast<const uint32_t *>(&b2);
+              }
+              if (!(p.dbg & 1)) *dst = make_uint4(w[0], w[1], w[2], w[3]);
+              else if (w[0] == 12345u) *dst = make_uint4(w[0], w[1], w[2], w[3]);
+            }
+          }
+          __syncwarp();
+        } else if (rok) {
           if (cfull && beta == 0.0f) {
 #pragma unroll
             for (int q = 0; q < W; q++)

@@ -49,6 +49,22 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
       "@!p bra WAIT_%=;\n}\n" ::"r"(bar), "r"(parity) : "memory");
 }
 
+// Wait with back-off: for warps that wait long (e.g. the epilogue during a long k loop), so
+// that their polling does not steal issue slots and barrier-unit bandwidth from the warps
+// on the critical path.
+__device__ __forceinline__ void mbar_wait_sleep(uint32_t bar, uint32_t parity) {
+  uint32_t done;
+  for (;;) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n}\n"
+        : "=r"(done) : "r"(bar), "r"(parity) : "memory");
+    if (done) return;
+    __nanosleep(256);
+  }
+}
+
 // TMA store of the smem box at `src` to the C tile at `crd` (cp.async.bulk.tensor, tile mode)
 __device__ __forceinline__ void tma_store(const TmaDesc *map, int rank, const int32_t *crd, uint32_t src) {
   const uint64_t m = reinterpret_cast<uint64_t>(map);
@@ -138,6 +154,75 @@ __device__ __forceinline__ void tile_coords(const KParams &p, int t, int &mt, in
   mt = first + r % gsz;
   nt = r / gsz;
 }
+
+__device__ __forceinline__ void prefetch_l1(const void *ptr) {
+  asm volatile("prefetch.global.L1 [%0];\n" ::"l"(ptr));
+}
+
+// Walk over the k-tile grid (P:L126 mixed radix): origin offsets of the current step in X and
+// Y and its k mask.  The inner moving digit steps in registers; a carry into the outer
+// digits reads the next entry of p.kouter (prefetched into L1 at the previous carry).
+struct KStep {
+  int c0, o;
+  int64_t s0x, s0y;          // inner digit's offsets
+  KOuter cur;                // outer digits' current combination
+  __device__ __forceinline__ void reset(const KParams &p) {
+    c0 = 0;
+    o = 0;
+    s0x = s0y = 0;
+    cur = p.kouter[0];
+    if (p.nouter > 1) prefetch_l1(p.kouter + 1);
+  }
+  __device__ __forceinline__ int64_t sx() const { return cur.x + s0x; }
+  __device__ __forceinline__ int64_t sy() const { return cur.y + s0y; }
+  __device__ __forceinline__ uint64_t mask(const KParams &p) const {
+    return (c0 == p.kcnt0 - 1 ? p.ktail0 : p.kbase) & cur.mask;
+  }
+  __device__ __forceinline__ void advance(const KParams &p) {
+    if (++c0 < p.kcnt0) {
+      s0x += p.kdX0;
+      s0y += p.kdY0;
+      return;
+    }
+    c0 = 0;
+    s0x = s0y = 0;
+    if (p.nouter > 1) {
+      o = o + 1 == p.nouter ? 0 : o + 1;
+      cur = p.kouter[o];
+      prefetch_l1(p.kouter + (o + 1 == p.nouter ? 0 : o + 1));
+    }
+  }
+};
+
+// A producer's view of one CTA tile: operand origins and row masks.
+struct ProdTile {
+  int64_t ox, oy;
+  uint64_t mm[kMaskWords], mn[kMaskWords];
+  bool fm, fn;   // interior on the m / n side
+  // pull tile t's two TileInfo records into L1 (read by fetch at the tile's first step)
+  static __device__ __forceinline__ void prefetch(const KParams &p, int t) {
+    int mt, nt;
+    tile_coords(p, t, mt, nt);
+    prefetch_l1(p.tileM + mt);
+    prefetch_l1(p.tileN + nt);
+  }
+  __device__ __forceinline__ void fetch(const KParams &p, int t) {
+    int mt, nt;
+    tile_coords(p, t, mt, nt);
+    const TileInfo &tm = p.tileM[mt];
+    const TileInfo &tn = p.tileN[nt];
+    ox = tm.op;
+    oy = tn.op;
+    fm = fn = true;
+#pragma unroll
+    for (int w = 0; w < kMaskWords; w++) {
+      mm[w] = tm.mask[w];
+      mn[w] = tn.mask[w];
+      fm &= mm[w] == p.fullM[w];
+      fn &= mn[w] == p.fullN[w];
+    }
+  }
+};
 
 // (select, not a dynamic array index: keeps the mask in registers, no local memory)
 __device__ __forceinline__ bool bit_of(const uint64_t (&m)[kMaskWords], int r) {
@@ -245,31 +330,23 @@ tc_f64_dmma_kernel(const __grid_constant__ KParams p) {
     load_slots(ry, py, p.relY, p.packY, p.nslotY, ptid, PW * 32, L::YS - 2);
     const bool vx = p.vecX == 2, vy = p.vecY == 2;
     int step = 0, lt = 0;
-    int64_t ox = 0, oy = 0;
-    bool fm = true, fn = true;
-    uint64_t mm[kMaskWords], mn[kMaskWords];
+    // the next tile's operand origins and masks are fetched while the current tile's last
+    // stage is issued (their load latency hides behind it)
+    ProdTile cur;
+    cur.fetch(p, (int)blockIdx.x);
+    KStep ks;
+    ks.reset(p);
     for (int j = 0; j < total; j++) {
       const int s = j % STAGES;
       if (j >= STAGES) mbar_wait(bar0 + 8 * (STAGES + s), ((j / STAGES) & 1) ^ 1);
-      if (step == 0) {
-        int mt, nt;
-        tile_coords(p, (int)blockIdx.x + lt * (int)gridDim.x, mt, nt);
-        const TileInfo &tm = p.tileM[mt];
-        const TileInfo &tn = p.tileN[nt];
-        ox = tm.op;
-        oy = tn.op;
-        fm = fn = true;
-#pragma unroll
-        for (int w = 0; w < kMaskWords; w++) {
-          mm[w] = tm.mask[w];
-          mn[w] = tn.mask[w];
-          fm &= mm[w] == p.fullM[w];
-          fn &= mn[w] == p.fullN[w];
-        }
-      }
-      const uint64_t km = __ldg(p.kmask + step);
+      if (step + 1 == p.nsteps && lt + 1 < ntl) ProdTile::prefetch(p, (int)blockIdx.x + (lt + 1) * (int)gridDim.x);
+      const int64_t ox = cur.ox, oy = cur.oy;
+      const bool fm = cur.fm, fn = cur.fn;
+      const uint64_t(&mm)[kMaskWords] = cur.mm;
+      const uint64_t(&mn)[kMaskWords] = cur.mn;
+      const uint64_t km = ks.mask(p);
       const bool fk = km == p.fullK;
-      const int64_t bx = ox + __ldg(p.stepX + step), by = oy + __ldg(p.stepY + step);
+      const int64_t bx = ox + ks.sx(), by = oy + ks.sy();
       const uint32_t dx = sbase + 8u * (uint32_t)(s * L::XS);
       const uint32_t dy = sbase + 8u * (uint32_t)(STAGES * L::XS + s * L::YS);
       if (vx) issue_slots<K::EX, true>(X, dx, rx, px, bx, fm && fk, km, mm);
@@ -277,7 +354,11 @@ tc_f64_dmma_kernel(const __grid_constant__ KParams p) {
       if (vy) issue_slots<K::EY, true>(Y, dy, ry, py, by, fn && fk, km, mn);
       else issue_slots<K::EY, false>(Y, dy, ry, py, by, fn && fk, km, mn);
       mbar_arrive_cp_async(bar0 + 8 * s);
-      if (++step == p.nsteps) { step = 0; ++lt; }
+      ks.advance(p);
+      if (++step == p.nsteps) {
+        step = 0;
+        if (++lt < ntl) cur.fetch(p, (int)blockIdx.x + lt * (int)gridDim.x);
+      }
     }
     return;
   }

@@ -28,6 +28,11 @@ struct TileInfo {           // one m-tile (or n-tile)
   int32_t pad_;
 };
 
+struct KOuter {            // one combination of the outer moving k digits
+  int64_t x, y;
+  uint64_t mask;
+};
+
 // Opaque 128-B TMA descriptor (CUtensorMap); kept as bytes so host-only code needs no
 // driver headers.
 struct alignas(64) TmaDesc {
@@ -53,11 +58,17 @@ struct KParams {
   const int64_t *relCn;     // [BN]
   const int32_t *boxM;      // [BM] offset of tile-local m in the smem C box (TMA epilogue)
   const int32_t *boxN;      // [BN]
-  // k side: steps in mixed radix over the internal tile grid
+  // k side: steps in mixed radix over the internal tile grid (kdig order, first digit
+  // fastest).  Digits whose tile covers the extent never move (their mask is folded into
+  // kbase); the first moving digit is stepped in registers, the others (rare carries) come
+  // from a small table, prefetched one carry ahead (KStep, kernel_f64.cuh).
   int nsteps;
-  const int64_t *stepX;     // [nsteps] element offset of step s's origin in X
-  const int64_t *stepY;     // [nsteps]
-  const uint64_t *kmask;    // [nsteps] bit k set <=> tile-local k is in range at step s
+  int kcnt0;                // tiles of the inner moving digit (1: none)
+  int64_t kdX0, kdY0;       // offset in X / Y of one inner tile step
+  uint64_t ktail0;          // k-mask factor while the inner digit is at its last tile
+  uint64_t kbase;           // k mask of the fixed digits (all in-range bits otherwise)
+  int nouter;               // combinations of the outer moving digits
+  const KOuter *kouter;     // [nouter] their X / Y offsets and k-mask factor
   // load slots: the X tile (Mt x Kt) and the Y tile (Kt x Nt) enumerated in each
   // operand's OWN memory order (threads along x walk the input's FVI)
   const int32_t *relX;      // [nslotX] element offset of the slot inside (tile, step)
@@ -65,7 +76,10 @@ struct KParams {
   const int32_t *relY;
   const uint32_t *packY;
   int nslotX, nslotY;
-  int vecX, vecY;           // 1 or 2 elements per slot (16-B cp.async when 2)
+  int vecX, vecY;           // elements per slot (16-B cp.async at 2 FP64 / 8 BF16)
+  int dbg;                  // TEMPORARY experiment knob
+  int vecC;                 // BF16: 8 => tile rows come in aligned C-contiguous runs of 8
+                            // (staged epilogue with 16-B stores); 1 => per-element stores
 };
 
 }  // namespace tc

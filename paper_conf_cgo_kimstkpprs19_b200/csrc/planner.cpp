@@ -91,16 +91,28 @@ double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *
   // tile's MMAs by the double-buffered TMEM accumulator
   const double epi = umma ? 0.0 : (double)warps * MI * NJ * 2 * 6 / 4;
   const double epi_umma = umma ? (double)v.BN * 4 * 4 : 0.0;
-  // persistent CTAs: grid = 148 * occ, tiles round-robin
-  const double slots = kSMs * v.occ;
-  const double tiles_per_cta = std::ceil(nctas / slots);
-  const double cyc_sm = tiles_per_cta * v.occ * std::max(steps * step + epi, epi_umma);
-  cfg.t_comp = cyc_sm / kClk;
   // memory: sector efficiencies of each tensor's tile along its own memory order
   const double es = v.esize();
   const double eX = sector_eff(contiguous_run(c, cfg.X, cfg.T), es);
   const double eY = sector_eff(contiguous_run(c, cfg.Y, cfg.T), es);
   const double eC = sector_eff(contiguous_run(c, 0, cfg.T), es);
+  // the C tile leaves at the SM's share of the HBM write bandwidth (profiles/r01_*: the 6D
+  // CCSD(T) cases); FP64: not overlapped with the same CTA's mainloop (the consumer warps
+  // store), only with the other resident CTAs'; UMMA: overlapped through the TMEM buffers
+  const double c_tile = (double)cfg.Mt * cfg.Nt * es / eC / (kHbm / kSMs / kClk);
+  const double t_main = steps * step;
+  double t_tile;
+  if (umma) {
+    t_tile = std::max({t_main, epi_umma, c_tile});
+  } else {
+    const double t_epi = std::max(epi, c_tile);
+    t_tile = std::max(t_main, t_epi) + std::min(t_main, t_epi) / v.occ;
+  }
+  // persistent CTAs: grid = 148 * occ, tiles round-robin; t_tile is per tile per SM
+  const double slots = kSMs * v.occ;
+  const double tiles_per_sm = std::ceil(nctas / slots) * v.occ;
+  const double cyc_sm = tiles_per_sm * t_tile;
+  cfg.t_comp = cyc_sm / kClk;
   // store-instruction efficiency: 8 consecutive rows of a DMMA fragment are contiguous in C
   // iff m's first digit is C's FVI
   // (UMMA: a warp stores 32 rows of one column)

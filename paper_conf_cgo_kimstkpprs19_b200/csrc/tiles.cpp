@@ -81,6 +81,18 @@ int vec_width(const Contraction &c, const Config &cfg, int t, int maxv) {
   return 1;
 }
 
+int c_vec_width(const Contraction &c, const Config &cfg, int maxv) {
+  const auto &v = c.t[0];
+  if (v.idx.empty() || v.stride[0] != 1 || cfg.mdig.empty() || cfg.mdig[0] != v.idx[0]) return 1;
+  const int f = v.idx[0];
+  for (int w = maxv; w >= 2; w /= 2) {
+    bool ok = cfg.T[f] % w == 0 && c.ix[f].n % w == 0 && v.base % w == 0;
+    for (size_t p = 1; p < v.stride.size(); p++) ok &= v.stride[p] % w == 0;
+    if (ok) return w;
+  }
+  return 1;
+}
+
 bool vec_possible(const Contraction &c, const Config &cfg, int t) { return vec_width(c, cfg, t, 2) == 2; }
 
 SlotTable build_slots(const Contraction &c, const Config &cfg, int t, int vec, bool kmajor,
@@ -241,41 +253,61 @@ TileTables build_tile_tables(const Contraction &c, const Config &cfg, const Vari
   // k steps
   const int nk = (int)cfg.kdig.size();
   std::vector<int64_t> kt(nk), kn(nk);
-  int64_t steps = 1;
   for (int i = 0; i < nk; i++) {
     kn[i] = c.ix[cfg.kdig[i]].n;
     kt[i] = cfg.T[cfg.kdig[i]];
-    steps *= cdiv(kn[i], kt[i]);
   }
-  tt.stepX.resize(steps);
-  tt.stepY.resize(steps);
-  tt.kmask.resize(steps);
-  std::vector<int64_t> cd(nk, 0);
   const int Kt = (int)cfg.Kt;
-  for (int64_t s = 0; s < steps; s++) {
-    int64_t bx = 0, by = 0;
-    for (int i = 0; i < nk; i++) {
-      bx += cd[i] * kt[i] * c.stride_of(X, cfg.kdig[i]);
-      by += cd[i] * kt[i] * c.stride_of(Y, cfg.kdig[i]);
+  const uint64_t full = Kt >= 64 ? ~0ull : ((1ull << Kt) - 1);
+  // per digit: tile count, offset per tile step and the k-mask factor at its last tile
+  std::vector<int64_t> cnt(nk), dx(nk), dy(nk);
+  std::vector<uint64_t> tail(nk);
+  int64_t inner = 1;                      // product of the tiles of the faster k digits
+  for (int i = 0; i < nk; i++) {
+    cnt[i] = cdiv(kn[i], kt[i]);
+    const int64_t rem = kn[i] - (cnt[i] - 1) * kt[i];
+    dx[i] = kt[i] * c.stride_of(X, cfg.kdig[i]);
+    dy[i] = kt[i] * c.stride_of(Y, cfg.kdig[i]);
+    uint64_t m = 0;
+    for (int k = 0; k < Kt; k++)
+      if ((k / inner) % kt[i] < rem) m |= 1ull << k;
+    tail[i] = m & full;
+    inner *= kt[i];
+  }
+  tt.kbase = full;
+  std::vector<int> moving;
+  for (int i = 0; i < nk; i++) {
+    if (cnt[i] == 1) tt.kbase &= tail[i];   // fixed digit: its (partial) range always applies
+    else moving.push_back(i);
+  }
+  tt.kcnt0 = 1;
+  tt.ktail0 = tt.kbase;
+  size_t first_outer = 0;
+  if (!moving.empty()) {
+    const int i = moving[0];
+    tt.kcnt0 = (int)cnt[i];
+    tt.kdX0 = dx[i];
+    tt.kdY0 = dy[i];
+    tt.ktail0 = tt.kbase & tail[i];
+    first_outer = 1;
+  }
+  // outer moving digits: every combination, first outer digit fastest
+  std::vector<int64_t> od(moving.size(), 0);
+  for (;;) {
+    KOuter e{0, 0, ~0ull};
+    for (size_t q = first_outer; q < moving.size(); q++) {
+      const int i = moving[q];
+      e.x += od[q] * dx[i];
+      e.y += od[q] * dy[i];
+      if (od[q] == cnt[i] - 1) e.mask &= tail[i];
     }
-    uint64_t mask = 0;
-    for (int k = 0; k < Kt; k++) {
-      int q = k;
-      bool ok = true;
-      for (int i = 0; i < nk; i++) {
-        const int d = q % (int)kt[i];
-        q /= (int)kt[i];
-        ok &= cd[i] * kt[i] + d < kn[i];
-      }
-      if (ok) mask |= 1ull << k;
+    tt.kouter.push_back(e);
+    size_t q = first_outer;
+    for (; q < moving.size(); q++) {
+      if (++od[q] < cnt[moving[q]]) break;
+      od[q] = 0;
     }
-    tt.stepX[s] = bx;
-    tt.stepY[s] = by;
-    tt.kmask[s] = mask;
-    for (int i = 0; i < nk; i++) {
-      if (++cd[i] < cdiv(kn[i], kt[i])) break;
-      cd[i] = 0;
-    }
+    if (q == moving.size()) break;
   }
   return tt;
 }

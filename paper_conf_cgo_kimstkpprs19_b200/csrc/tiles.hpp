@@ -24,12 +24,23 @@ const std::vector<Variant> &variants();
 
 // Smem offset (in elements) of element (row mn, k) of one operand stage.
 //  FP64 (kernel_f64.cuh SmemLayout): pitch 4 (mod 16) doubles, k- or mn-contiguous.
-//  BF16 (kernel_bf16.cuh): UMMA canonical no-swizzle layout of 8 x 16-B core matrices;
-//  K-major: core (mn/8, k/8) at (mn/8)*BK*8 + (k/8)*64, MN-major: at (mn/8)*64 + (k/8)*BMN*8.
+//  BF16 (kernel_bf16.cuh): UMMA 128-B swizzled layouts (stage base 1 KB aligned); the 16-B
+//  chunk index inside a 128-B row is XORed with the row's index inside its 8-row atom.
+//  K-major (BK = 64 = one 128-B row): row mn at (mn/8) KB + (mn%8) 128 B, k along the row.
+//  MN-major: atom (mn/64, k/8) at ((k/8) (BMN/64) + mn/64) KB, row k%8, mn%64 along the row.
 inline int smem_off(int kind, bool kmajor, int mn, int k, int BMN, int BK) {
-  if (kind == KIND_BF16_UMMA)
-    return kmajor ? (mn / 8) * (BK * 8) + (k / 8) * 64 + (mn % 8) * 8 + (k % 8)
-                  : (mn / 8) * 64 + (k / 8) * (BMN * 8) + (k % 8) * 8 + (mn % 8);
+  if (kind == KIND_BF16_UMMA) {
+    int byte;
+    if (kmajor) {
+      const int r = mn % 8;
+      byte = (mn / 8) * 1024 + r * 128 + ((((k * 2) >> 4) ^ r) << 4) + (k * 2 & 15);
+    } else {
+      const int r = k % 8, e = mn % 64;
+      byte = ((k / 8) * (BMN / 64) + mn / 64) * 1024 + r * 128 + ((((e * 2) >> 4) ^ r) << 4) + (e * 2 & 15);
+    }
+    (void)BK;
+    return byte / 2;
+  }
   return kmajor ? mn * (BK + 4) + k : k * (BMN + 4) + mn;
 }
 
@@ -60,6 +71,10 @@ void finish_counts(const Contraction &c, Config &cfg);
 bool vec_possible(const Contraction &c, const Config &cfg, int t);
 // Largest elements-per-slot vector (<= maxv, power of two) the operand's layout allows.
 int vec_width(const Contraction &c, const Config &cfg, int t, int maxv);
+// Largest w <= maxv (power of two) such that tile rows come in runs of w consecutive,
+// w-aligned C elements: C's FVI is the first m digit, its tile, its extent, C's base and
+// every other C stride are multiples of w.
+int c_vec_width(const Contraction &c, const Config &cfg, int maxv);
 
 struct SlotTable {
   std::vector<int64_t> rel;    // element offset inside (tile, step)
@@ -84,8 +99,11 @@ struct TileTables {
   // TMA epilogue: the C tile is a box of C (dims in C order, box dim = tile size)
   bool tma_ok = false;                 // C rank <= 5, 16-B strides, even FVI tile
   std::vector<int32_t> boxM, boxN;     // offset of tile-local m / n inside the smem box
-  std::vector<int64_t> stepX, stepY;
-  std::vector<uint64_t> kmask;
+  // k walk (KParams::kcnt0 ...): inner moving digit, fixed-digit mask, outer table
+  int kcnt0 = 1;
+  int64_t kdX0 = 0, kdY0 = 0;
+  uint64_t ktail0 = 0, kbase = 0;
+  std::vector<KOuter> kouter;
 };
 TileTables build_tile_tables(const Contraction &c, const Config &cfg, const Variant &v);
 

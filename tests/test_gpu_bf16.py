@@ -48,7 +48,8 @@ def _klen(expr, extents):
     return k
 
 
-def check_bf16(expr, extents, seed=0, integer=False, alpha=1.0, beta=0.0, misalign=0, **plan_kw):
+def check_bf16(expr, extents, seed=0, integer=False, alpha=1.0, beta=0.0, misalign=0, cmisalign=0,
+               **plan_kw):
     p = tc.plan(expr, extents, dtype="bf16", **plan_kw)
     assert p.info()["dtype"] == "bf16"
     nA, nB, nC = p.numel("A"), p.numel("B"), p.numel("C")
@@ -56,11 +57,12 @@ def check_bf16(expr, extents, seed=0, integer=False, alpha=1.0, beta=0.0, misali
     A, B = tcinputs.bf16_bits(gen(nA, 1000 + seed)), tcinputs.bf16_bits(gen(nB, 2000 + seed))
     C0 = tcinputs.bf16_bits(gen(nC, 3000 + seed)) if beta != 0 else None
     dA, dB = _dev_bf16(A, misalign), _dev_bf16(B, misalign)
-    dC = (_dev_bf16(C0) if C0 is not None
-          else torch.full((nC,), float("nan"), dtype=torch.bfloat16, device="cuda"))
-    p.execute_ptr(dA.data_ptr() + 2 * misalign, dB.data_ptr() + 2 * misalign, dC.data_ptr(), alpha, beta)
+    dC = (_dev_bf16(C0, cmisalign) if C0 is not None
+          else torch.full((nC + cmisalign,), float("nan"), dtype=torch.bfloat16, device="cuda"))
+    p.execute_ptr(dA.data_ptr() + 2 * misalign, dB.data_ptr() + 2 * misalign, dC.data_ptr() + 2 * cmisalign,
+                  alpha, beta)
     torch.cuda.synchronize()
-    got = dC.cpu().view(torch.int16).numpy().view(np.uint16)
+    got = dC[cmisalign:].cpu().view(torch.int16).numpy().view(np.uint16)
     if integer:
         want = oracle.contract(expr, extents, A, B, C=C0, alpha=alpha, beta=beta, dtype="bf16")
         assert np.array_equal(got, want), (expr, extents, np.flatnonzero(got != want)[:10])
@@ -107,6 +109,15 @@ def test_bf16_alpha_beta():
     e, ext = "abcd-aebf-dfce", "a:9;b:10;c:11;d:12;e:5;f:7"
     check_bf16(e, ext, seed=3, integer=True, alpha=2.0, beta=1.0)
     check_bf16(e, ext, seed=4, alpha=0.5, beta=-1.25)
+    # staged 16-B epilogue (C's FVI leads m in multiples of 8), with and without beta
+    e, ext = "abcdef-gdab-efgc", "a:16;b:6;c:7;d:10;e:5;f:6;g:11"
+    assert tc.plan(e, ext, dtype="bf16", host_only=True).info()["vecC"] == 8
+    check_bf16(e, ext, seed=5, integer=True, alpha=2.0, beta=1.0)
+    check_bf16(e, ext, seed=6, alpha=0.5, beta=-1.25)
+    check_bf16(e, ext, seed=7, integer=True)
+    # C only 2-B aligned: the per-element epilogue runs
+    check_bf16(e, ext, seed=8, integer=True, alpha=2.0, beta=1.0, cmisalign=1)
+    check_bf16(e, ext, seed=9, integer=True, cmisalign=3)
 
 
 def test_bf16_unaligned_pointers_and_tails():
