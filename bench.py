@@ -122,42 +122,75 @@ def run_reference(args):
 
 # ---------------------------------------------------------------- clocks
 class Clocks:
+    """nvidia-smi sampler (B200_PROFILING.md clocks line).  Started BEFORE the warm-up (the
+    tool needs ~1 s to start); each line is stamped on arrival and only the lines that arrive
+    inside [mark_start, mark_end] (the timed region) are summarised."""
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
     def __init__(self, path):
         self.path = path
         self.p = None
+        self.rows = []          # (time, fields)
+        self.t0 = self.t1 = None
 
     def __enter__(self):
+        import threading
         try:
-            self.f = open(self.path, "w")
-            self.p = subprocess.Popen(
-                ["nvidia-smi", "--query-gpu=index,clocks.sm,clocks.max.sm,power.draw,"
-                 "clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
-                 "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
-                 "clocks_event_reasons.sw_power_cap", "--format=csv,noheader,nounits", "-lms", "100"],
-                stdout=self.f, stderr=subprocess.DEVNULL)
+            self.p = subprocess.Popen(["nvidia-smi", "--query-gpu=" + self.FIELDS,
+                                       "--format=csv,noheader,nounits", "-lms", "50"],
+                                      stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
         except Exception:
             self.p = None
+            return self
+
+        def reader():
+            for line in self.p.stdout:
+                self.rows.append((time.perf_counter(), line.strip()))
+        self.th = threading.Thread(target=reader, daemon=True)
+        self.th.start()
+        t = time.perf_counter()
+        while not self.rows and time.perf_counter() - t < 15 and self.p.poll() is None:
+            time.sleep(0.05)
         return self
+
+    def mark_start(self):
+        self.t0 = time.perf_counter()
+
+    def mark_end(self):
+        self.t1 = time.perf_counter()
+        if self.p:
+            time.sleep(0.06)
 
     def __exit__(self, *a):
         if self.p:
             self.p.terminate()
             self.p.wait()
-            self.f.close()
+            self.th.join(timeout=2)
+        try:
+            with open(self.path, "w") as f:
+                for t, line in self.rows:
+                    inside = self.t0 is not None and self.t0 <= t <= (self.t1 or t)
+                    f.write(f"{t:.3f},{int(inside)},{line}\n")
+        except Exception:
+            pass
 
     def summary(self, dev=0):
-        try:
-            rows = [r.split(",") for r in open(self.path).read().strip().splitlines()]
-            rows = [[x.strip() for x in r] for r in rows if len(r) >= 9 and r[0].strip() == str(dev)]
-        except Exception:
-            return None
+        rows = []
+        for t, line in self.rows:
+            if self.t0 is None or not (self.t0 <= t <= (self.t1 or t)):
+                continue
+            r = [x.strip() for x in line.split(",")]
+            if len(r) >= 9 and r[0] == str(dev):
+                rows.append(r)
         if not rows:
             return None
         sm = sorted(float(r[1]) for r in rows)
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         reasons = sorted({names[i] for r in rows for i in range(4) if r[5 + i].lower() == "active"})
         return {"sm_mhz": sm[len(sm) // 2], "sm_max_mhz": float(rows[0][2]), "reasons": reasons,
-                "samples": len(rows)}
+                "samples": len(rows), "power_w_max": max(float(r[3]) for r in rows)}
 
 
 # ---------------------------------------------------------------- GPU run
@@ -214,18 +247,19 @@ def run_libtc(args):
         e1.record(stream)
         record.append((e0, e1))
 
-    for _ in range(args.warmup):
-        rec = []
-        for i in range(len(work)):
-            one(i, rec)
-    torch.cuda.synchronize()
-    times = [[] for _ in work]
     clk_path = os.path.join(ROOT, "gpurun_out", f"bench_clocks_r{rank}.csv")
     os.makedirs(os.path.dirname(clk_path), exist_ok=True)
-    if world > 1:
-        dist.barrier()
-    torch.cuda.synchronize()
+    times = [[] for _ in work]
     with Clocks(clk_path) as clocks:
+        for _ in range(args.warmup):
+            rec = []
+            for i in range(len(work)):
+                one(i, rec)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        clocks.mark_start()
         t_wall = time.perf_counter()
         for _ in range(args.steps):
             rec = []
@@ -238,6 +272,7 @@ def run_libtc(args):
             dist.barrier()
         torch.cuda.synchronize()
         t_wall = time.perf_counter() - t_wall
+        clocks.mark_end()
     med = []
     for ts in times:
         s = sorted(ts)
