@@ -101,6 +101,20 @@ tc_status_t tc_execute_host(const tc_plan_t plan, const void *A_host, const void
                             void *C_host, double alpha, double beta, void *workspace,
                             size_t workspace_bytes, tc_stream_t stream);
 
+/*
+ * Measured tuning (the paper's "auto-tuned across a selected set",
+ * P:L346-348): the cost model ranks the kernel variants by the predicted time of their best
+ * configuration; the best configurations of the top `topk` variants are each launched
+ * 1 + `reps` times on `stream` with the caller's A, B, C (alpha = 1, beta = 0: C's contents
+ * are OVERWRITTEN) and the fastest (minimum over reps) becomes *tuned, a new plan with the same
+ * contraction, layout, device and options as `plan` (which stays valid and unchanged).
+ * Synchronises `stream`.  tc_plan_info(*tuned) lists the candidates' times ("tuned").
+ * Errors: TC_ERR_INVALID_ARG (NULL, topk < 1, reps < 1), TC_ERR_CUDA (host_only plan, launch
+ * failure), as tc_execute for the pointers.  *tuned is NULL on failure.
+ */
+tc_status_t tc_plan_tuned(tc_plan_t *tuned, const tc_plan_t plan, const void *A, const void *B,
+                          void *C, int topk, int reps, tc_stream_t stream);
+
 /* Flags of tc_plan_restrict: the operand passed to tc_execute is the compact slab itself. */
 #define TC_SLAB_A 1u
 #define TC_SLAB_B 2u

@@ -9,7 +9,7 @@ CSRC = os.path.join(HERE, "csrc")
 SO = os.path.join(HERE, "libtc.so")
 SOURCES = ["api.cu", "contraction.cpp", "planner.cpp", "tiles.cpp", "kernels_00.cu", "kernels_01.cu",
            "kernels_10.cu", "kernels_11.cu", "kernels_bf16.cu"]
-HEADERS = ["contraction.hpp", "planner.hpp", "kparams.hpp", "kernel_f64.cuh", "tiles.hpp",
+HEADERS = ["contraction.hpp", "planner.hpp", "kparams.hpp", "kernel_f64.cuh", "tiles.hpp", "variants.def",
            "kernel_table.cuh", "kernel_bf16.cuh"]
 NVCC_FLAGS = ["-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo",
               "-Xcompiler", "-fPIC", "-shared"]
@@ -25,10 +25,30 @@ def _stale() -> bool:
 
 
 def build(force: bool = False, verbose: bool = False) -> str:
+    """Compile every translation unit in parallel (the kernel tables are split across TUs),
+    then link libtc.so."""
     if force or _stale():
+        from concurrent.futures import ThreadPoolExecutor
         nvcc = os.path.join(os.environ.get("CUDA_HOME", "/usr/local/cuda"), "bin", "nvcc")
-        cmd = [nvcc] + NVCC_FLAGS + (["-Xptxas", "-v"] if verbose else []) + SOURCES + ["-o", SO]
-        subprocess.check_call(cmd, cwd=CSRC)
+        objdir = os.path.join(HERE, "build")
+        os.makedirs(objdir, exist_ok=True)
+        cflags = [f for f in NVCC_FLAGS if f != "-shared"]
+
+        def one(src):
+            obj = os.path.join(objdir, os.path.splitext(src)[0] + ".o")
+            cmd = [nvcc] + cflags + (["-Xptxas", "-v"] if verbose else []) + ["-c", src, "-o", obj]
+            r = subprocess.run(cmd, cwd=CSRC, capture_output=True, text=True)
+            if r.returncode != 0:
+                raise RuntimeError(f"nvcc failed on {src}:\n{r.stderr}")
+            if verbose:
+                print(r.stderr)
+            return obj
+
+        with ThreadPoolExecutor(max_workers=max(1, min(len(SOURCES), os.cpu_count() or 1))) as ex:
+            objs = list(ex.map(one, SOURCES))
+        subprocess.check_call([nvcc, "-shared", "-gencode", "arch=compute_100a,code=sm_100a"] + objs +
+                              ["-o", SO + ".tmp"])
+        os.replace(SO + ".tmp", SO)
     return SO
 
 

@@ -47,14 +47,9 @@ KernelEntry kernel_for(const Config &cfg) {
     const void *fn = kernel_ptr_bf16(cfg.variant, cfg.xKmajor, cfg.yKmajor, &smem, &threads);
     return {fn, threads, smem, smem};
   }
-  const void *fn = cfg.xKmajor ? (cfg.yKmajor ? kernel_ptr_11(cfg.variant) : kernel_ptr_10(cfg.variant))
-                               : (cfg.yKmajor ? kernel_ptr_01(cfg.variant) : kernel_ptr_00(cfg.variant));
-  // must equal F64Kernel<...>::smem_bytes(false / true)
-  const size_t PM = v.BM + 4, PN = v.BN + 4, PK = v.BK + 4;
-  const size_t XS = std::max(v.BM * PK, v.BK * PM) + 2, YS = std::max(v.BN * PK, v.BK * PN) + 2;
-  const size_t base = 8 * (size_t)v.stages * (XS + YS) + 16 * (size_t)v.stages + 12 * (size_t)(v.BM + v.BN);
-  const size_t tma = (base + 1023) / 1024 * 1024 + 8 * (size_t)v.BM * v.BN;
-  return {fn, v.threads(), base, tma};
+  const F64Instance k = cfg.xKmajor ? (cfg.yKmajor ? f64_instance_11(cfg.variant) : f64_instance_10(cfg.variant))
+                                    : (cfg.yKmajor ? f64_instance_01(cfg.variant) : f64_instance_00(cfg.variant));
+  return {k.fn, k.threads, k.smem, k.smem_tma};
 }
 
 }  // namespace
@@ -72,7 +67,8 @@ struct tc_plan_s {
   std::string force_tiles;
   TileTables tt;
   SlotTable slotX1, slotY1, slotX2, slotY2;   // scalar and cfg.vecX / cfg.vecY wide slots
-  int cvec = 1;            // c_vec_width of the plan (BF16 staged epilogue when 8)
+  int cvec = 1;            // c_vec_width of the plan (16-B C stores when > 1)
+  std::vector<std::pair<int, double>> tuned;   // tc_plan_tuned: (variant, measured ms) per candidate
   KParams kp{};            // device pointers filled in; X/Y/C/alpha/beta/slots set per call
   void *dev = nullptr;     // one device buffer with every table
   size_t dev_bytes = 0;
@@ -100,7 +96,7 @@ void build_host_tables(tc_plan_s *P) {
   P->slotY1 = build_slots(c, cfg, cfg.Y, 1, cfg.yKmajor, v.BN, v.BK);
   if (cfg.vecX > 1) P->slotX2 = build_slots(c, cfg, cfg.X, cfg.vecX, cfg.xKmajor, v.BM, v.BK);
   if (cfg.vecY > 1) P->slotY2 = build_slots(c, cfg, cfg.Y, cfg.vecY, cfg.yKmajor, v.BN, v.BK);
-  P->cvec = cfg.kind == KIND_BF16_UMMA ? c_vec_width(c, cfg, 8) : 1;
+  P->cvec = cfg.kind == KIND_BF16_UMMA ? c_vec_width(c, cfg, 8) : (v.stg ? c_vec_width(c, cfg, 2) : 1);
   KParams &kp = P->kp;
   std::memset(&kp, 0, sizeof(kp));
   kp.mtiles = (int)cfg.mtiles;
@@ -182,7 +178,8 @@ Status upload(tc_plan_s *P, std::string &err) {
   P->d_relY2 = (const int32_t *)(b + parts[iY2].off);
   P->d_packY2 = (const uint32_t *)(b + parts[iY2p].off);
   const KernelEntry ke = kernel_for(P->cfg);
-  const bool tma = P->tt.tma_ok && P->opts.tma_epilogue && P->cfg.kind == KIND_F64_DMMA;
+  const bool tma = P->tt.tma_ok && P->opts.tma_epilogue && P->cfg.kind == KIND_F64_DMMA &&
+                   !variants()[P->cfg.variant].stg;
   e = cudaFuncSetAttribute(ke.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(tma ? ke.smem_tma : ke.smem));
   if (e != cudaSuccess) { err = std::string("cudaFuncSetAttribute: ") + cudaGetErrorString(e); return ST_CUDA; }
   int occ = 0;
@@ -364,6 +361,70 @@ int64_t tc_plan_numel(const tc_plan_t plan, int t) {
   return plan->parsed.numel(t);
 }
 
+tc_status_t tc_plan_tuned(tc_plan_t *tuned, const tc_plan_t plan, const void *A, const void *B, void *C,
+                          int topk, int reps, tc_stream_t stream) {
+  if (!tuned || !plan || !A || !B || !C) return fail(ST_INVALID_ARG, "NULL argument");
+  *tuned = nullptr;
+  if (plan->host_only || !plan->dev) return fail(ST_CUDA, "plan was made host_only");
+  if (topk < 1 || reps < 1) return fail(ST_INVALID_ARG, "topk and reps must be >= 1");
+  try {
+    // candidates: the best configuration of each of the top-k variants by predicted time
+    std::vector<int> cand;
+    for (auto &pv : plan->stats.per_variant)
+      if ((int)cand.size() < topk) cand.push_back(pv.first);
+    if (cand.empty()) cand.push_back(plan->cfg.variant);
+    cudaEvent_t e0, e1;
+    if (cudaEventCreate(&e0) != cudaSuccess || cudaEventCreate(&e1) != cudaSuccess)
+      return fail(ST_CUDA, "cudaEventCreate");
+    tc_plan_t best = nullptr;
+    float best_ms = 0;
+    std::vector<std::pair<int, double>> log;
+    tc_status_t rc = TC_SUCCESS;
+    for (int v : cand) {
+      tc_plan_s *P = new tc_plan_s();
+      P->opts = plan->opts;
+      P->force_tiles = plan->force_tiles;
+      P->opts.force_tiles = plan->opts.force_tiles ? P->force_tiles.c_str() : nullptr;
+      P->opts.variant = v + 1;
+      P->dtype = plan->dtype;
+      P->parsed = plan->parsed;
+      tc_plan_t cp = nullptr;
+      rc = finish_plan(P, &cp);
+      if (rc != TC_SUCCESS) break;
+      cp->stats.per_variant = plan->stats.per_variant;
+      // one warm-up, then the minimum over reps single launches (C is overwritten)
+      rc = tc_execute(cp, A, B, C, 1.0, 0.0, stream);
+      float ms = 1e30f;
+      for (int r = 0; r < reps && rc == TC_SUCCESS; r++) {
+        cudaEventRecord(e0, (cudaStream_t)stream);
+        rc = tc_execute(cp, A, B, C, 1.0, 0.0, stream);
+        cudaEventRecord(e1, (cudaStream_t)stream);
+        if (cudaEventSynchronize(e1) != cudaSuccess) { rc = fail(ST_CUDA, "tuning launch failed"); break; }
+        float t = 0;
+        cudaEventElapsedTime(&t, e0, e1);
+        ms = std::min(ms, t);
+      }
+      if (rc != TC_SUCCESS) { tc_plan_destroy(cp); break; }
+      log.push_back({v, ms});
+      if (!best || ms < best_ms) {
+        tc_plan_destroy(best);
+        best = cp;
+        best_ms = ms;
+      } else {
+        tc_plan_destroy(cp);
+      }
+    }
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    if (rc != TC_SUCCESS) { tc_plan_destroy(best); return rc; }
+    best->tuned = log;
+    *tuned = best;
+    return TC_SUCCESS;
+  } catch (...) {
+    return fail(ST_ALLOC, "exception in tc_plan_tuned");
+  }
+}
+
 tc_status_t tc_plan_restrict(tc_plan_t *sub, const tc_plan_t parent, const char *index,
                              int64_t begin, int64_t len, unsigned flags) {
   if (!sub || !parent || !index) return fail(ST_INVALID_ARG, "NULL argument");
@@ -426,6 +487,7 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
   kp.beta = beta;
   // TMA epilogue when the C view is a legal tensor map and C is only written
   kp.use_tma = plan->tt.tma_ok && plan->opts.tma_epilogue && cfg.kind == KIND_F64_DMMA && beta == 0.0 &&
+               !variants()[cfg.variant].stg &&
                encode_c_map(plan, C, kp.cmap);
   // vector slots need operands aligned to the vector; otherwise the scalar slot tables run
   const bool vx = cfg.vecX > 1 && ((uintptr_t)kp.X % (es * cfg.vecX)) == 0;
@@ -439,7 +501,8 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
   kp.nslotY = (int)(vy ? plan->slotY2.pack.size() : plan->slotY1.pack.size());
   kp.vecY = vy ? cfg.vecY : 1;
   kp.dbg = plan->opts.reserved[0];
-  kp.vecC = plan->cvec == 8 && ((uintptr_t)C % 16) == 0 ? 8 : 1;
+  // C stores in 16-B vectors: 8 BF16 (staged BF16 epilogue) / 2 FP64 (STG drain)
+  kp.vecC = plan->cvec > 1 && ((uintptr_t)C % 16) == 0 ? plan->cvec : 1;
   const KernelEntry ke = kernel_for(cfg);
   const int grid = (int)std::min<int64_t>(cfg.nctas, plan->sms);
   void *args[] = {&kp};
@@ -510,6 +573,7 @@ tc_status_t tc_plan_info(const tc_plan_t plan, char *json, size_t cap, size_t *n
     o << "},\"m\":" << names(g.mdig) << ",\"n\":" << names(g.ndig) << ",\"k\":" << names(g.kdig);
     o << ",\"morder\":" << g.morder << ",\"korder\":" << g.korder;
     o << ",\"variant\":" << g.variant << ",\"BM\":" << v.BM << ",\"BN\":" << v.BN << ",\"BK\":" << v.BK
+      << ",\"WM\":" << v.WM << ",\"WN\":" << v.WN << ",\"stg\":" << v.stg
       << ",\"threads\":" << v.threads() << ",\"stages\":" << v.stages << ",\"occ\":" << v.occ;
     o << ",\"Mt\":" << g.Mt << ",\"Nt\":" << g.Nt << ",\"Kt\":" << g.Kt << ",\"nctas\":" << g.nctas
       << ",\"mtiles\":" << g.mtiles << ",\"ntiles\":" << g.ntiles << ",\"nsteps\":" << g.nsteps
@@ -526,7 +590,14 @@ tc_status_t tc_plan_info(const tc_plan_t plan, char *json, size_t cap, size_t *n
     o << ",\"paper_mapping\":\"" << g.paper_mapping << "\"";
     o << ",\"stats\":{\"cost_mode\":\"" << (plan->stats.cost_mode ? "paper" : "b200")
       << "\",\"raw\":" << plan->stats.raw << ",\"pruned\":" << plan->stats.pruned
-      << ",\"ranked\":" << plan->stats.ranked << ",\"plan_ms\":" << plan->stats.plan_ms << "}";
+      << ",\"ranked\":" << plan->stats.ranked << ",\"plan_ms\":" << plan->stats.plan_ms
+      << ",\"per_variant\":[";
+    for (size_t q = 0; q < plan->stats.per_variant.size(); q++)
+      o << (q ? "," : "") << "[" << plan->stats.per_variant[q].first << "," << plan->stats.per_variant[q].second * 1e3 << "]";
+    o << "],\"tuned\":[";
+    for (size_t q = 0; q < plan->tuned.size(); q++)
+      o << (q ? "," : "") << "[" << plan->tuned[q].first << "," << plan->tuned[q].second << "]";
+    o << "]}";
     o << ",\"host_only\":" << (plan->host_only ? "true" : "false") << "}";
     std::string s = o.str();
     if (needed) *needed = s.size() + 1;

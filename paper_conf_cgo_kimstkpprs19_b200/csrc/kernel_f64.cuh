@@ -17,6 +17,14 @@
 //       (WM/8) x (WN/8) DMMA tiles per k4.
 //   (4) REG -> GMEM: C = alpha * acc + beta * C through separable row / column offsets,
 //       predicated by the tile's row / column bitmasks (correct for any size).
+//       Direct variants store from the fragments.  DEFERRED variants (STG) park the raw
+//       accumulators in a per-warp smem staging tile and go straight on with the next tile;
+//       the same warp drains the parked tile a few columns per k4 step of the next tile's
+//       mainloop (lane = tile row: coalesced along C's FVI, 16 B pairs when C allows), so
+//       the C write of tile i is issued in the shadow of tile i+1's DMMAs and no register of
+//       an in-flight store is overwritten by the next tile's accumulators (the near-ridge
+//       K = 24 CCSD(T) and the memory-bound ML contractions, where the C write is most of the
+//       traffic).  No barrier is involved: each warp owns its staging region.
 // CTAs are persistent (grid = 148 x CTAs/SM, tiles round-robin): the producers run up to
 // STAGES k-steps ahead ACROSS tile boundaries, so tile i's epilogue stores overlap tile
 // i+1's loads — the overlap the K = 24 CCSD(T) contractions need (SURVEY 7.2 part 1).
@@ -119,7 +127,7 @@ struct SmemLayout {
   static constexpr int YS = ((BN * PK > BK * PN) ? BN * PK : BK * PN) + 2;
 };
 
-template <int BM, int BN, int BK, int WM, int WN, int STAGES, int PW>
+template <int BM, int BN, int BK, int WM, int WN, int STAGES, int PW, bool STG = false>
 struct F64Kernel {
   static constexpr int WARPS_M = BM / WM, WARPS_N = BN / WN;
   static constexpr int CWARPS = WARPS_M * WARPS_N;            // consumer warps
@@ -128,20 +136,26 @@ struct F64Kernel {
   static constexpr int EX = (BM * BK + PW * 32 - 1) / (PW * 32);  // X slots per producer thread
   static constexpr int EY = (BN * BK + PW * 32 - 1) / (PW * 32);
   using L = SmemLayout<BM, BN, BK>;
-  // ring + barriers + tables; the optional TMA staging box starts at the next 1 KB boundary
-  static constexpr size_t base_bytes() {
+  // deferred epilogue: per consumer warp a [WN][SP] staging tile (lane = row, SP = 36
+  // doubles: the fragment writes take the 2-wavefront minimum, the row reads are contiguous)
+  static constexpr int SP = 36;
+  static constexpr size_t ring_bytes() {
     return sizeof(double) * (size_t)STAGES * (L::XS + L::YS) + 16 * (size_t)STAGES + 12 * (size_t)(BM + BN);
   }
-  static constexpr size_t kStagingOffset =      // in doubles
-      ((sizeof(double) * (size_t)STAGES * (L::XS + L::YS) + 16 * (size_t)STAGES + 12 * (size_t)(BM + BN) +
-        1023) / 1024) * 1024 / 8;
+  static constexpr size_t kStageOffset = (ring_bytes() + 127) / 128 * 128;   // bytes
+  static constexpr size_t stg_bytes() { return STG ? 8 * (size_t)CWARPS * WN * SP : 0; }
+  static constexpr size_t base_bytes() { return kStageOffset + stg_bytes(); }
+  // ring + barriers + tables; the optional TMA staging box starts at the next 1 KB boundary
+  static constexpr size_t kStagingOffset = (base_bytes() + 1023) / 1024 * 1024 / 8;   // in doubles
   static constexpr size_t smem_bytes(bool tma) {
     return tma ? kStagingOffset * 8 + 8 * (size_t)BM * BN : base_bytes();
   }
   static_assert(BK % 4 == 0 && BK <= 64, "BK");
   static_assert(WM % 8 == 0 && WN % 8 == 0, "warp tile");
+  static_assert(BM % WM == 0 && BN % WN == 0, "warp grid");
   static_assert(BM <= 64 * kMaskWords && BN <= 64 * kMaskWords, "tile masks");
   static_assert(L::XS < 8192 && L::YS < 8192, "13-bit smem offsets");
+  static_assert(!STG || WM == 32, "deferred epilogue: one lane per warp-tile row");
 };
 
 // (mt, nt) of tile t with grouped rasterisation (group_m m-tiles share a band of n-tiles).
@@ -281,10 +295,52 @@ __device__ __forceinline__ void load_slots(int32_t (&rel)[E], uint32_t (&pack)[E
   }
 }
 
-template <int BM, int BN, int BK, int WM, int WN, int STAGES, int PW, int MINB, bool XK, bool YK>
-__global__ void __launch_bounds__(F64Kernel<BM, BN, BK, WM, WN, STAGES, PW>::THREADS, MINB)
+// Deferred epilogue (STG variants): drain columns [c0, c0 + NC) of the warp's parked tile.
+// Lane l owns tile row wm * 32 + l (its C offset Cr, validity rok); column c of the warp
+// tile is tile column n0 + c (C offset relCn, validity bit of cmask).  VC: 16-B pairs (lane
+// pairs share a column: lanes 0-15 take rows 2l, 2l + 1 of column c, lanes 16-31 of c + 1).
+template <int WN, int SP, int NC, bool VC>
+__device__ __forceinline__ void drain_cols(const double *__restrict__ st, int c0, int lane, double *Cr, bool rok,
+                                           const int64_t *relCn, int n0, const uint64_t (&cmask)[kMaskWords],
+                                           double alpha, double beta, bool plain) {
+  if (VC) {
+#pragma unroll
+    for (int d = 0; d < NC; d += 2) {
+      const int c = c0 + d + (lane >> 4);
+      if (c < WN && rok && bit_of(cmask, n0 + c)) {
+        double2 v = *reinterpret_cast<const double2 *>(st + c * SP + 2 * (lane & 15));
+        double2 *dst = reinterpret_cast<double2 *>(Cr + relCn[n0 + c]);
+        if (!plain) {
+          if (beta != 0.0) {
+            const double2 o = *dst;
+            v.x = fma(beta, o.x, alpha * v.x);
+            v.y = fma(beta, o.y, alpha * v.y);
+          } else {
+            v.x *= alpha;
+            v.y *= alpha;
+          }
+        }
+        *dst = v;
+      }
+    }
+  } else {
+#pragma unroll
+    for (int d = 0; d < NC; d++) {
+      const int c = c0 + d;
+      if (c < WN && rok && bit_of(cmask, n0 + c)) {
+        double v = st[c * SP + lane];
+        double *dst = Cr + relCn[n0 + c];
+        if (!plain) v = beta != 0.0 ? fma(beta, *dst, alpha * v) : alpha * v;
+        *dst = v;
+      }
+    }
+  }
+}
+
+template <int BM, int BN, int BK, int WM, int WN, int STAGES, int PW, int MINB, bool XK, bool YK, bool STG>
+__global__ void __launch_bounds__(F64Kernel<BM, BN, BK, WM, WN, STAGES, PW, STG>::THREADS, MINB)
 tc_f64_dmma_kernel(const __grid_constant__ KParams p) {
-  using K = F64Kernel<BM, BN, BK, WM, WN, STAGES, PW>;
+  using K = F64Kernel<BM, BN, BK, WM, WN, STAGES, PW, STG>;
   using L = typename K::L;
   constexpr int MI = K::MI, NJ = K::NJ, CW = K::CWARPS;
   extern __shared__ __align__(1024) double smem[];
@@ -297,6 +353,8 @@ tc_f64_dmma_kernel(const __grid_constant__ KParams p) {
   int32_t *boxN = boxM + BM;
   // [BM * BN] C staging box of the TMA epilogue: present only when launched with it
   double *sC = smem + K::kStagingOffset;
+  // [STG] this consumer warp's deferred-epilogue staging tile
+  double *stg_base = reinterpret_cast<double *>(reinterpret_cast<char *>(smem) + K::kStageOffset);
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int ntl = (p.ntotal - (int)blockIdx.x + (int)gridDim.x - 1) / (int)gridDim.x;
@@ -315,6 +373,7 @@ tc_f64_dmma_kernel(const __grid_constant__ KParams p) {
       mbar_init(bar0 + 8 * s, PW * 32);               // full: every producer thread
       mbar_init(bar0 + 8 * (STAGES + s), CW);         // empty: one arrive per consumer warp
     }
+
     asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
   }
   __syncthreads();
@@ -384,6 +443,24 @@ tc_f64_dmma_kernel(const __grid_constant__ KParams p) {
   int64_t roff[MI];
 #pragma unroll
   for (int i = 0; i < MI; i++) roff[i] = relCm[wm * WM + i * 8 + g];
+  // [STG] deferred epilogue state: the parked tile's C row pointer (this lane's row),
+  // row validity, column mask and the next column to drain
+  double *const stg = stg_base + warp * WN * K::SP;
+  const bool plain = alpha == 1.0 && beta == 0.0;
+  const bool vc = STG && p.vecC == 2;
+  const int drow = wm * WM + (vc ? 2 * (lane & 15) : lane);   // tile row this lane drains
+  const int64_t droff = STG ? relCm[drow] : 0;
+  double *dCr = C;
+  bool drok = false, pend = false;
+  uint64_t dmn[kMaskWords] = {0, 0};
+  int dcol = 0;
+  // columns per k4 step so that a parked tile is drained within one k-step of the next tile
+  constexpr int KQ = BK / 4;
+  constexpr int DQ = ((WN + KQ - 1) / KQ + 1) / 2 * 2;
+  auto drain = [&](int c0) {
+    if (vc) drain_cols<WN, K::SP, DQ, true>(stg, c0, lane, dCr, drok, relCn, wn * WN, dmn, alpha, beta, plain);
+    else drain_cols<WN, K::SP, DQ, false>(stg, c0, lane, dCr, drok, relCn, wn * WN, dmn, alpha, beta, plain);
+  };
   // TMA epilogue: box offsets of tile-local rows / columns come from smem tables
   const bool use_tma = p.use_tma && beta == 0.0;
   const uint32_t sCaddr = (uint32_t)__cvta_generic_to_shared(sC);
@@ -421,6 +498,11 @@ tc_f64_dmma_kernel(const __grid_constant__ KParams p) {
       for (int i = 0; i < MI; i++)
 #pragma unroll
         for (int jj = 0; jj < NJ; jj++) dmma884(acc[i][jj][0], acc[i][jj][1], a[i], b[jj]);
+      // [STG] a few columns of the parked tile per k4 step, in the shadow of the DMMAs
+      if (STG && pend && dcol < WN) {
+        drain(dcol);
+        dcol += DQ;
+      }
     }
     __syncwarp();
     if (lane == 0) mbar_arrive(bar0 + 8 * (STAGES + s));
@@ -430,7 +512,29 @@ tc_f64_dmma_kernel(const __grid_constant__ KParams p) {
 #pragma unroll
       for (int i = 0; i < MI; i++) rbits |= (uint32_t)bit_of(mm, wm * WM + i * 8 + g) << i;
       double *Ct = C + (cm + cn);
-      if (use_tma) {
+      if (STG) {
+        // finish the previous parked tile, then park this one (raw accumulators; the drain
+        // applies alpha / beta) and record where it goes
+        if (pend) {
+          for (; dcol < WN; dcol += DQ) drain(dcol);
+        }
+        __syncwarp();
+#pragma unroll
+        for (int jj = 0; jj < NJ; jj++)
+#pragma unroll
+          for (int h = 0; h < 2; h++) {
+            double *col = stg + (jj * 8 + 2 * t + h) * K::SP + g;
+#pragma unroll
+            for (int i = 0; i < MI; i++) col[i * 8] = acc[i][jj][h];
+          }
+        __syncwarp();
+        dCr = Ct + droff;
+        drok = bit_of(mm, drow);
+        dmn[0] = mn[0];
+        dmn[1] = mn[1];
+        pend = true;
+        dcol = 0;
+        (void)rbits;      } else if (use_tma) {
         // stage alpha * acc as the tile's box in smem, one elected thread TMA-stores it;
         // the hardware clips the box at the tensor bounds
         if (threadIdx.x == 0) tma_wait_read();     // previous tile's store has read sC
@@ -454,7 +558,15 @@ tc_f64_dmma_kernel(const __grid_constant__ KParams p) {
         if (threadIdx.x == 0) tma_store(&p.cmap, p.c_rank, crd, sCaddr);
       } else if (beta == 0.0) {
         // predicated stores (no branches); alpha == 1 skips the FP64-pipe multiply
-        const bool a1 = alpha == 1.0;
+        if (alpha != 1.0) {
+#pragma unroll
+          for (int i = 0; i < MI; i++)
+#pragma unroll
+            for (int jj = 0; jj < NJ; jj++) {
+              acc[i][jj][0] *= alpha;
+              acc[i][jj][1] *= alpha;
+            }
+        }
 #pragma unroll
         for (int jj = 0; jj < NJ; jj++)
 #pragma unroll
@@ -463,8 +575,7 @@ tc_f64_dmma_kernel(const __grid_constant__ KParams p) {
             const uint32_t ok = bit_of(mn, cidx) ? rbits : 0u;
             double *col = Ct + relCn[cidx];
 #pragma unroll
-            for (int i = 0; i < MI; i++)
-              st_pred(col + roff[i], a1 ? acc[i][jj][h] : alpha * acc[i][jj][h], (ok >> i) & 1);
+            for (int i = 0; i < MI; i++) st_pred(col + roff[i], acc[i][jj][h], (ok >> i) & 1);
           }
       } else {
 #pragma unroll
@@ -486,6 +597,9 @@ tc_f64_dmma_kernel(const __grid_constant__ KParams p) {
       step = 0;
       ++lt;
     }
+  }
+  if (STG && pend) {
+    for (; dcol < WN; dcol += DQ) drain(dcol);
   }
   if (use_tma && threadIdx.x == 0) tma_wait_all();   // the last box must be read out
 }

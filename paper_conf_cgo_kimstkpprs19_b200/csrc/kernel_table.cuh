@@ -1,40 +1,45 @@
-// kernel_table.cuh — the compiled FP64 kernel instances, one row per tiles.cpp variant.
+// kernel_table.cuh — the compiled FP64 kernel instances, one row of variants.def each.
 // Each kernels_<XK><YK>.cu instantiates the table for one pair of smem layouts, so the
 // 4 x |variants| instances compile in parallel translation units.
-// Consumer warps own 32 x 32 warp tiles (64 accumulator registers); a 4-warp producer
-// group keeps its load slots in registers.  Warps per SM stay <= 16 so that no instance
-// has fewer than 128 registers per thread (the register file is 16 K per sub-partition).
-// Shared memory = BM x BN C staging box (TMA epilogue) + STAGES ring stages; the stage
-// counts keep MINB CTAs resident within 227 KB.
+// Consumer warps own WM x WN warp tiles (at most 64 accumulator registers); a 4-warp producer
+// group keeps its load slots in registers.  Warps per SM stay <= 16 so that no instance has
+// fewer than 128 registers per thread (the register file is 16 K per sub-partition).
+// Shared memory = STAGES ring stages (+ the staged-epilogue tile for STG variants, + the
+// BM x BN TMA box when the optional TMA epilogue is on); the stage counts keep OCC CTAs
+// resident within 227 KB.
 #pragma once
 #include "kernel_f64.cuh"
 
 namespace tc {
 
+struct F64Instance {
+  const void *fn;
+  int threads;
+  size_t smem;       // without the TMA staging box
+  size_t smem_tma;   // with it
+};
+
 template <bool XK, bool YK>
-const void *kernel_ptr(int v) {
+F64Instance f64_instance(int v) {
   switch (v) {
-    //                                           BM   BN  BK  WM  WN  ST PW MINB
-    case 0: return (const void *)&tc_f64_dmma_kernel<128, 64, 16, 32, 32, 3, 4, 1, XK, YK>;
-    case 1: return (const void *)&tc_f64_dmma_kernel<64, 128, 16, 32, 32, 3, 4, 1, XK, YK>;
-    case 2: return (const void *)&tc_f64_dmma_kernel<64, 64, 16, 32, 32, 4, 4, 2, XK, YK>;
-    case 3: return (const void *)&tc_f64_dmma_kernel<64, 64, 24, 32, 32, 3, 4, 2, XK, YK>;
-    case 4: return (const void *)&tc_f64_dmma_kernel<128, 64, 24, 32, 32, 3, 4, 1, XK, YK>;
-    case 5: return (const void *)&tc_f64_dmma_kernel<64, 128, 24, 32, 32, 3, 4, 1, XK, YK>;
-    case 6: return (const void *)&tc_f64_dmma_kernel<128, 32, 16, 32, 32, 4, 4, 2, XK, YK>;
-    case 7: return (const void *)&tc_f64_dmma_kernel<32, 128, 16, 32, 32, 4, 4, 2, XK, YK>;
-    case 8: return (const void *)&tc_f64_dmma_kernel<128, 32, 24, 32, 32, 3, 4, 1, XK, YK>;
-    case 9: return (const void *)&tc_f64_dmma_kernel<32, 128, 24, 32, 32, 3, 4, 1, XK, YK>;
-    case 10: return (const void *)&tc_f64_dmma_kernel<64, 64, 8, 32, 32, 4, 4, 2, XK, YK>;
+#define TC_F64_VARIANT(id, BM, BN, BK, WM, WN, ST, PW, OCC, STG)                                   \
+  case id: {                                                                                       \
+    using K = F64Kernel<BM, BN, BK, WM, WN, ST, PW, STG>;                                         \
+    static_assert(K::smem_bytes(false) <= 227 * 1024, "variant exceeds shared memory");           \
+    return {(const void *)&tc_f64_dmma_kernel<BM, BN, BK, WM, WN, ST, PW, OCC, XK, YK, STG>,      \
+            K::THREADS, K::smem_bytes(false), K::smem_bytes(true)};                               \
   }
-  return nullptr;
+#include "variants.def"
+#undef TC_F64_VARIANT
+  }
+  return {nullptr, 0, 0, 0};
 }
 
 // defined in kernels_00.cu / _01 / _10 / _11
-const void *kernel_ptr_00(int v);
-const void *kernel_ptr_01(int v);
-const void *kernel_ptr_10(int v);
-const void *kernel_ptr_11(int v);
+F64Instance f64_instance_00(int v);
+F64Instance f64_instance_01(int v);
+F64Instance f64_instance_10(int v);
+F64Instance f64_instance_11(int v);
 // defined in kernels_bf16.cu (BF16 tcgen05 variants; smem bytes and block size out)
 const void *kernel_ptr_bf16(int v, bool xk, bool yk, size_t *smem, int *threads);
 

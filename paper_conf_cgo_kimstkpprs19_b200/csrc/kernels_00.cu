@@ -2,5 +2,5 @@
 #include "kernel_table.cuh"
 
 namespace tc {
-const void *kernel_ptr_00(int v) { return kernel_ptr<false, false>(v); }
+F64Instance f64_instance_00(int v) { return f64_instance<false, false>(v); }
 }  // namespace tc

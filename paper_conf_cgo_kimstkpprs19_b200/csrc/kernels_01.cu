@@ -2,5 +2,5 @@
 #include "kernel_table.cuh"
 
 namespace tc {
-const void *kernel_ptr_01(int v) { return kernel_ptr<false, true>(v); }
+F64Instance f64_instance_01(int v) { return f64_instance<false, true>(v); }
 }  // namespace tc

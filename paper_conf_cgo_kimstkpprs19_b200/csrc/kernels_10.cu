@@ -2,5 +2,5 @@
 #include "kernel_table.cuh"
 
 namespace tc {
-const void *kernel_ptr_10(int v) { return kernel_ptr<true, false>(v); }
+F64Instance f64_instance_10(int v) { return f64_instance<true, false>(v); }
 }  // namespace tc

@@ -2,5 +2,5 @@
 #include "kernel_table.cuh"
 
 namespace tc {
-const void *kernel_ptr_11(int v) { return kernel_ptr<true, true>(v); }
+F64Instance f64_instance_11(int v) { return f64_instance<true, true>(v); }
 }  // namespace tc

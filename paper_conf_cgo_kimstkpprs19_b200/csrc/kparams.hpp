@@ -78,8 +78,8 @@ struct KParams {
   int nslotX, nslotY;
   int vecX, vecY;           // elements per slot (16-B cp.async at 2 FP64 / 8 BF16)
   int dbg;                  // TEMPORARY experiment knob
-  int vecC;                 // BF16: 8 => tile rows come in aligned C-contiguous runs of 8
-                            // (staged epilogue with 16-B stores); 1 => per-element stores
+  int vecC;                 // C vector (elements): BF16 8 / FP64 STG 2 => tile rows come in aligned
+                            // C-contiguous runs of vecC (16-B stores); 1 => per-element stores
 };
 
 }  // namespace tc

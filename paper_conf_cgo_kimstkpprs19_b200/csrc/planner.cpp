@@ -104,6 +104,13 @@ double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *
   double t_tile;
   if (umma) {
     t_tile = std::max({t_main, epi_umma, c_tile});
+  } else if (v.stg) {
+    // staged epilogue: the consumers only write the raw tile to smem (2 wavefronts per
+    // fragment store); the producers drain it between their cp.async issues, so the C write
+    // overlaps the next tile's mainloop; the producers' LSU issue carries loads + drain
+    const double sts = (double)warps * MI * NJ * 2 * 2;
+    const double drain = (double)v.BM * v.BN * es / 128.0 + std::ceil((double)cfg.Mt * cfg.Nt / 32.0) * 4.0;
+    t_tile = std::max({t_main + sts, c_tile, steps * ldgsts + drain});
   } else {
     const double t_epi = std::max(epi, c_tile);
     t_tile = std::max(t_main, t_epi) + std::min(t_main, t_epi) / v.occ;
@@ -343,6 +350,8 @@ static Status choose_b200(const Contraction &c, int kind, int forced_variant, Co
     if (forced_variant >= 0 && vi != forced_variant) continue;
     if (variants()[vi].kind != kind) continue;
     const auto &v = variants()[vi];
+    bool vfound = false;
+    Config vbest;
     auto ms = enum_side(c, mx, c0, v.BM);
     auto ns = enum_side(c, ny, -1, v.BN);
     auto ks = enum_side(c, kx, kfirst, v.BK);
@@ -389,17 +398,22 @@ static Status choose_b200(const Contraction &c, int kind, int forced_variant, Co
             if (!fits(cfg, v)) { st.pruned++; continue; }
             cfg.variant = vi;
             // bound: the FP64-pipe time of the padded work alone (no smem / memory terms)
-            if (found) {
+            if (vfound) {
               const double tiles = std::ceil((double)cfg.nctas / (kSMs * v.occ));
               const double lb = tiles * v.occ * (double)cfg.nsteps * v.BM * v.BN * v.BK /
                                 fma_per_clk(v.kind) / kClk + kLaunch;
-              if (lb > best.t_pred) { st.pruned++; continue; }
+              if (lb > vbest.t_pred) { st.pruned++; continue; }
             }
             model_time(c, cfg, v, &cache);
             st.ranked++;
-            if (!found || better(cfg, best)) { best = cfg; found = true; }
+            if (!vfound || better(cfg, vbest)) { vbest = cfg; vfound = true; }
           }
+    if (!vfound) continue;
+    st.per_variant.push_back({vi, vbest.t_pred});
+    if (!found || better(vbest, best)) { best = vbest; found = true; }
   }
+  std::stable_sort(st.per_variant.begin(), st.per_variant.end(),
+                   [](const auto &a, const auto &b) { return a.second < b.second; });
   return found ? ST_OK : ST_NO_CONFIG;
 }
 

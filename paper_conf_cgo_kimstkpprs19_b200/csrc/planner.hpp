@@ -25,6 +25,10 @@ struct PlanStats {
   int64_t ranked = 0;    // cost-model evaluations
   double plan_ms = 0;
   int cost_mode = 0;
+  // best predicted time per kernel variant (variant id, seconds), ascending: the candidate
+  // set of measured tuning (tc_plan_tuned; the paper's "auto-tuned across a selected set",
+  // P:L346-348)
+  std::vector<std::pair<int, double>> per_variant;
 };
 
 struct ForcedTiles {

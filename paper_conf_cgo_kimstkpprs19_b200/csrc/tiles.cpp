@@ -7,24 +7,18 @@
 namespace tc {
 
 const std::vector<Variant> &variants() {
-  // BM, BN, BK, WM, WN, stages, producer warps, CTAs/SM (= __launch_bounds__ min blocks;
-  // smem and registers checked with ptxas -v).  Must match kernels_*.cu.
-  static const std::vector<Variant> v = {
-      {128, 64, 16, 32, 32, 3, 4, 1},   // 0
-      {64, 128, 16, 32, 32, 3, 4, 1},   // 1
-      {64, 64, 16, 32, 32, 4, 4, 2},    // 2
-      {64, 64, 24, 32, 32, 3, 4, 2},    // 3
-      {128, 64, 24, 32, 32, 3, 4, 1},   // 4
-      {64, 128, 24, 32, 32, 3, 4, 1},   // 5
-      {128, 32, 16, 32, 32, 4, 4, 2},   // 6
-      {32, 128, 16, 32, 32, 4, 4, 2},   // 7
-      {128, 32, 24, 32, 32, 3, 4, 1},   // 8
-      {32, 128, 24, 32, 32, 3, 4, 1},   // 9
-      {64, 64, 8, 32, 32, 4, 4, 2},     // 10
-      // BF16 x BF16 -> FP32 on tcgen05 (kernel_bf16.cuh): BM = 128 (UMMA M), BK = 64
-      {128, 64, 64, 32, 32, 6, 4, 1, KIND_BF16_UMMA},    // 11
-      {128, 128, 64, 32, 32, 5, 4, 1, KIND_BF16_UMMA},   // 12
-  };
+  // FP64 shapes from variants.def (must match the kernel instances of kernel_table.cuh);
+  // BF16 x BF16 -> FP32 on tcgen05 (kernel_bf16.cuh): BM = 128 (UMMA M), BK = 64.
+  static const std::vector<Variant> v = [] {
+    std::vector<Variant> t(kNumVariants);
+#define TC_F64_VARIANT(id, BM, BN, BK, WM, WN, ST, PW, OCC, STG) \
+  t[id] = Variant{BM, BN, BK, WM, WN, ST, PW, OCC, KIND_F64_DMMA, STG};
+#include "variants.def"
+#undef TC_F64_VARIANT
+    t[11] = Variant{128, 64, 64, 32, 32, 6, 4, 1, KIND_BF16_UMMA};
+    t[12] = Variant{128, 128, 64, 32, 32, 5, 4, 1, KIND_BF16_UMMA};
+    return t;
+  }();
   return v;
 }
 

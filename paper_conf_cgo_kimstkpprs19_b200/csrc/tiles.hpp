@@ -13,9 +13,12 @@ namespace tc {
 // Compiled kernel shapes (kernel_f64.cuh template instances, api.cu kernel table).
 enum Kind { KIND_F64_DMMA = 0, KIND_BF16_UMMA = 1 };
 
+constexpr int kNumVariants = 21;             // ids 0..20 (variants.def + the BF16 ids 11, 12)
+
 struct Variant {
-  int BM, BN, BK, WM, WN, stages, pw, occ;   // pw = producer warps
+  int BM = 0, BN = 0, BK = 0, WM = 0, WN = 0, stages = 0, pw = 0, occ = 0;   // pw = producer warps
   int kind = KIND_F64_DMMA;
+  int stg = 0;                                // 1: staged epilogue drained by the producers
   int threads() const { return kind == KIND_BF16_UMMA ? 13 * 32 : ((BM / WM) * (BN / WN) + pw) * 32; }
   int cwarps() const { return kind == KIND_BF16_UMMA ? 8 : (BM / WM) * (BN / WN); }
   int esize() const { return kind == KIND_BF16_UMMA ? 2 : 8; }

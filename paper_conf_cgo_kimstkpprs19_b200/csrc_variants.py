@@ -1,3 +1,16 @@
-"""Compiled kernel variants (tiles.cpp variants(), kernel_table.cuh, kernels_bf16.cu)."""
-NUM_VARIANTS = 11                 # FP64 DMMA variants: ids 0 .. NUM_VARIANTS-1
+"""Compiled kernel variants, read from csrc/variants.def (the list tiles.cpp and
+kernel_table.cuh are generated from) so the tests cannot drift from the library."""
+import os
+import re
+
+_DEF = os.path.join(os.path.dirname(os.path.abspath(__file__)), "csrc", "variants.def")
+_ROW = re.compile(r"^TC_F64_VARIANT\(\s*(\d+)((?:\s*,\s*\d+){9})\s*\)", re.M)
+
+F64_SHAPES = {}
+for _m in _ROW.finditer(open(_DEF).read()):
+    _v = [int(x) for x in _m.group(2).split(",")[1:]]
+    F64_SHAPES[int(_m.group(1))] = dict(zip(("BM", "BN", "BK", "WM", "WN", "stages", "pw", "occ", "stg"), _v))
+
+F64_VARIANTS = tuple(sorted(F64_SHAPES))            # FP64 DMMA variants (direct + staged)
+STG_VARIANTS = tuple(v for v in F64_VARIANTS if F64_SHAPES[v]["stg"])
 BF16_VARIANTS = (11, 12)          # BF16 tcgen05 variants (BM = 128, BK = 64; BN = 64 / 128)

@@ -10,7 +10,7 @@ import oracle
 import tcinputs
 from paper_conf_cgo_kimstkpprs19_b200 import binding as tc
 from paper_conf_cgo_kimstkpprs19_b200 import build
-from paper_conf_cgo_kimstkpprs19_b200.csrc_variants import NUM_VARIANTS
+from paper_conf_cgo_kimstkpprs19_b200.csrc_variants import F64_VARIANTS, STG_VARIANTS
 from tests.layouts import PRIME_EXT, layouts_one_contraction, layouts_two_contractions
 
 pytestmark = pytest.mark.gpu
@@ -95,13 +95,25 @@ def test_alpha_beta_and_nan_c():
 
 
 @pytest.mark.parametrize("tma", [True, False])
-@pytest.mark.parametrize("variant", range(NUM_VARIANTS))
+@pytest.mark.parametrize("variant", F64_VARIANTS)
 def test_every_kernel_variant(variant, tma):
     # both epilogues: TMA box store (cp.async.bulk.tensor) and predicated direct stores
     check_case("abcdef-gdab-efgc", "a:10;b:6;c:7;d:10;e:5;f:6;g:11", seed=variant, integer=True,
                variant=variant, tma=tma)
     check_case("abcd-aebf-dfce", "a:18;b:9;c:13;d:20;e:19;f:3", seed=variant, variant=variant, tma=tma)
     check_case("abcd-aebf-fdec", "a:16;b:24;c:8;d:40;e:24;f:9", seed=variant, variant=variant, tma=tma)
+
+
+@pytest.mark.parametrize("variant", STG_VARIANTS)
+def test_staged_epilogue_alpha_beta(variant):
+    # the producers' drain applies alpha / beta: 16-B pairs (C's FVI tile and extent even)
+    # and the scalar path (odd FVI extent), partial tiles on every side, several tiles per CTA
+    check_case("abcd-aebf-dfce", "a:36;b:7;c:9;d:30;e:6;f:5", seed=variant, alpha=0.5, beta=-1.25,
+               variant=variant)
+    check_case("abcd-aebf-dfce", "a:35;b:7;c:9;d:30;e:6;f:5", seed=variant, integer=True, alpha=2.0,
+               beta=1.0, variant=variant)
+    check_case("abcdef-gdab-efgc", "a:24;b:6;c:7;d:10;e:5;f:6;g:24", seed=variant, integer=True,
+               variant=variant)
 
 
 def test_paper_cost_mode_runs():
@@ -186,3 +198,25 @@ def test_execute_host_end_to_end():
     p.execute_host(A, B, C, ws)
     want, S = oracle.contract(expr, ext, A.numpy(), B.numpy(), with_scale=True)
     assert np.all(np.abs(C.numpy() - want) <= TAU64 * S)
+
+
+def test_measured_tuning_returns_a_correct_plan():
+    # tc_plan_tuned: times the top-k variants' best configs on the
+    # caller's tensors and returns the fastest as a new plan; the result must stay exact
+    expr, ext = "abcdef-gdab-efgc", "a:24;b:16;c:16;d:24;e:16;f:16;g:24"
+    p = tc.plan(expr, ext)
+    A = tcinputs.integers_np(p.numel("A"), 11)
+    B = tcinputs.integers_np(p.numel("B"), 12)
+    dA = torch.as_tensor(A, device="cuda")
+    dB = torch.as_tensor(B, device="cuda")
+    dC = torch.empty(p.numel("C"), dtype=torch.float64, device="cuda")
+    t = p.tuned(dA, dB, dC, topk=3, reps=2)
+    info = t.info()
+    assert len(info["stats"]["tuned"]) == 3
+    assert info["variant"] in [v for v, _ in info["stats"]["tuned"]]
+    dC.fill_(float("nan"))
+    t.execute(dA, dB, dC)
+    torch.cuda.synchronize()
+    assert np.array_equal(dC.cpu().numpy(), oracle.contract(expr, ext, A, B))
+    with pytest.raises(tc.TcError):
+        p.tuned(dA, dB, dC, topk=0)

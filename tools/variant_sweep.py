@@ -10,7 +10,7 @@ import torch  # noqa: E402
 
 import tcinputs  # noqa: E402
 from paper_conf_cgo_kimstkpprs19_b200 import binding as tc  # noqa: E402
-from paper_conf_cgo_kimstkpprs19_b200.csrc_variants import NUM_VARIANTS  # noqa: E402
+from paper_conf_cgo_kimstkpprs19_b200.csrc_variants import F64_VARIANTS  # noqa: E402
 
 
 def time_plan(p, A, B, C, flush, reps=5):
@@ -41,15 +41,17 @@ def main():
         B = tcinputs.uniform(p0.numel("B"), 2000 + case.id, device="cuda")
         C = torch.empty(p0.numel("C"), dtype=torch.float64, device="cuda")
         best = p0.info()["variant"]
-        for v in range(NUM_VARIANTS):
+        vs = [int(x) for x in os.environ["TC_VARIANTS"].split(",")] if os.environ.get("TC_VARIANTS") else F64_VARIANTS
+        tmas = (False, True) if os.environ.get("TC_SWEEP_TMA") else (False,)
+        for v, tma in [(v, t) for v in vs for t in tmas]:
             try:
-                p = tc.plan(case.expr, case.extents, variant=v)
+                p = tc.plan(case.expr, case.extents, variant=v, tma=tma)
             except tc.TcError as e:
                 print(json.dumps({"id": case.id, "variant": v, "error": str(e)}))
                 continue
             i = p.info()
             ms = time_plan(p, A, B, C, flush)
-            print(json.dumps({"id": case.id, "variant": v, "chosen": v == best, "ms": round(ms, 4),
+            print(json.dumps({"id": case.id, "variant": v, "tma": tma, "chosen": v == best, "ms": round(ms, 4),
                               "pred_ms": round(i["t_pred_ms"], 4), "comp": round(i["t_comp_ms"], 4),
                               "mem": round(i["t_mem_ms"], 4), "l2": round(i["t_l2_ms"], 4),
                               "gflops": round(p.flops / ms / 1e6, 1), "Mt": i["Mt"], "Nt": i["Nt"],
