@@ -50,6 +50,13 @@ def parse_args():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of oracle work")
+    ap.add_argument("--suites", default="ccsdt,membound",
+                    help="extra workloads reported inside the same JSON line (BASELINE configs 3/4): "
+                         "ccsdt = CCSD(T) 6D sweep N=24..48 FP64, membound = memory-bound TCCG cases in "
+                         "FP32 (split TF32) / TF32 / BF16 vs the HBM roofline; '' = none")
+    ap.add_argument("--profile", action="store_true",
+                    help="after the timed region, launch every case once inside cudaProfilerStart/Stop "
+                         "(for `ncu --profile-from-start off`); writes gpurun_out/profile_cases.json")
     return ap.parse_args()
 
 
@@ -196,6 +203,81 @@ class Clocks:
 
 
 # ---------------------------------------------------------------- GPU run
+# ---------------------------------------------------------------- extra suites (configs 3, 4)
+_TDT = {"f64": "float64", "f32": "float32", "tf32": "float32", "bf16": "bfloat16"}
+_ES = {"f64": 8, "f32": 4, "tf32": 4, "bf16": 2}
+
+
+def time_one(p, A, B, C, steps, warmup, flush, stream):
+    """Median device time (ms) of one tc_execute over `steps` launches, CUDA events on the
+    launch stream, L2 flushed (outside the events) before every launch."""
+    import torch
+    ts = []
+    for i in range(warmup + steps):
+        flush.zero_()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        p.execute(A, B, C)
+        e1.record(stream)
+        e1.synchronize()
+        if i >= warmup:
+            ts.append(e0.elapsed_time(e1))
+    ts.sort()
+    return ts[len(ts) // 2]
+
+
+def run_suite(name, args, flush, stream, dev, hbm):
+    """One extra workload: per case plan (+ measured top-k tuning like the main suite), time,
+    roofline fraction against min(pipe peak, I * HBM) — pipe = FP64 DMMA for f64; the
+    memory-bound cases are reported against HBM bandwidth (algorithmic bytes / time)."""
+    import torch
+    from paper_conf_cgo_kimstkpprs19_b200 import binding as tc
+    rows = []
+    if name == "ccsdt":
+        # BASELINE config 3: sd_t_d1 / sd_t_d2 6D contractions at uniform extents 24..48, FP64
+        todo = [(tcinputs.ccsdt(n, e, 100 + n), "f64") for e in ("abcdef-gdab-efgc", "abcdef-dega-gfbc")
+                for n in (24, 32, 40, 48)]
+    else:
+        # BASELINE config 4: the memory-bound TCCG cases (#1-8 ML tensor x matrix, #18 ab-ac-cb)
+        mb = [c for c in tcinputs.tccg48() if c.id <= 8 or c.id == 18]
+        todo = [(c, dt) for dt in ("f32", "tf32", "bf16") for c in mb]
+    for c, dt in todo:
+        tdt = getattr(torch, _TDT[dt])
+        p = tc.plan(c.expr, c.extents, dtype=dt, cost=args.cost)
+        A = tcinputs.uniform(p.numel("A"), 1000 + c.id, device=dev).to(tdt)
+        B = tcinputs.uniform(p.numel("B"), 2000 + c.id, device=dev).to(tdt)
+        C = torch.empty(p.numel("C"), dtype=tdt, device=dev)
+        if args.tune > 0:
+            p = p.tuned(A, B, C, topk=args.tune, reps=2)
+        ms = time_one(p, A, B, C, max(3, min(args.steps, 5)), 2, flush, stream)
+        byts = _ES[dt] * (p.numel("A") + p.numel("B") + p.numel("C"))
+        gbs = byts / (ms * 1e-3) / 1e9
+        r = {"expr": c.expr, "extents": c.extents, "dtype": dt, "ms": round(ms, 5),
+             "gflops": round(p.flops / ms / 1e6, 2), "gbs": round(gbs, 1),
+             "variant": p.info()["variant"]}
+        if dt == "f64":
+            attain = min(FP64_PEAK_TFLOPS * 1e12, p.flops / byts * hbm)
+            r["roofline_frac"] = round(p.flops / (ms * 1e-3) / attain, 4)
+        else:
+            r["hbm_frac"] = round(gbs * 1e9 / hbm, 4)
+        rows.append(r)
+        del A, B, C, p
+        torch.cuda.empty_cache()
+    out = {"cases": rows}
+    if name == "ccsdt":
+        out["workload"] = "CCSD(T) sd_t_d2 abcdef-gdab-efgc and sd_t_d1 abcdef-dega-gfbc, all extents N, FP64"
+        out["geomean_gflops"] = round(geomean([r["gflops"] for r in rows]), 2)
+        out["geomean_roofline_frac"] = round(geomean([r["roofline_frac"] for r in rows]), 4)
+    else:
+        out["workload"] = "memory-bound TCCG #1-8, #18 in FP32 (split TF32), TF32, BF16; HBM roofline"
+        for dt in ("f32", "tf32", "bf16"):
+            sel = [r for r in rows if r["dtype"] == dt]
+            out[f"geomean_hbm_frac_{dt}"] = round(geomean([r["hbm_frac"] for r in sel]), 4)
+            out[f"geomean_gflops_{dt}"] = round(geomean([r["gflops"] for r in sel]), 2)
+    return out
+
+
 def run_libtc(args):
     import torch
     import torch.distributed as dist
@@ -212,6 +294,12 @@ def run_libtc(args):
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     cases = select_cases(args.cases)
     dev = torch.device("cuda", local)
+
+    def kname(p):
+        i = p.info()
+        return (f"tc_f64_dmma_kernel<{i['BM']},{i['BN']},{i['BK']},{i['WM']},{i['WN']},{i['stages']},4,"
+                f"{i['occ']},{i['xKmajor']},{i['yKmajor']},{i['stg']}>")
+
     stream = torch.cuda.current_stream()
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
 
@@ -283,6 +371,22 @@ def run_libtc(args):
         torch.cuda.synchronize()
         t_wall = time.perf_counter() - t_wall
         clocks.mark_end()
+    if args.profile and rank == 0:
+        # one launch per case inside a profiler range (ncu --profile-from-start off); the
+        # order of the captured launches is the order of profile_cases.json
+        rows = []
+        for (c, p, A, B, C, sh) in work:
+            flush.zero_()
+            torch.cuda.synchronize()
+            torch.cuda.cudart().cudaProfilerStart()
+            (sh.plan if sh is not None else p).execute(A, B, C)
+            torch.cuda.synchronize()
+            torch.cuda.cudart().cudaProfilerStop()
+            rows.append({"case": c.id, "kernel": kname((sh.plan if sh is not None else p)),
+                         "flops": p.flops,
+                         "alg_bytes": 8 * (p.numel("A") + p.numel("B") + p.numel("C"))})
+        with open(os.path.join(ROOT, "gpurun_out", "profile_cases.json"), "w") as f:
+            json.dump(rows, f)
     med = []
     for ts in times:
         s = sorted(ts)
@@ -303,10 +407,6 @@ def run_libtc(args):
     ms_step = sum(med)
 
     # dominant kernel (largest share of the step) -> roofline
-    def kname(p):
-        i = p.info()
-        return (f"tc_f64_dmma_kernel<{i['BM']},{i['BN']},{i['BK']},{i['WM']},{i['WN']},{i['stages']},4,"
-                f"{i['occ']},{i['xKmajor']},{i['yKmajor']},{i['stg']}>")
 
     share = {}
     for w, ms in zip(work, med):
@@ -318,13 +418,18 @@ def run_libtc(args):
     dflops, dms = share[dom]
     achieved = dflops / (dms * 1e-3) / 1e12
     dom_cases = [w[0].id for w in work if kname(run_plan(w)) == dom]
-    traffic = None
+    # DRAM bytes per launch of the dominant kernel from the committed `ncu --set full` capture
+    # (tools/ncu_traffic.py -> profiles/ncu_traffic.json): mean over the dominant cases whose
+    # captured kernel is the one that ran here (tuning can pick another variant on another box)
+    traffic, traffic_alg = None, None
     prof = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(prof):
         try:
-            t = json.load(open(prof))
-            if t.get("kernel") == dom and t.get("case") in dom_cases:
-                traffic = t.get("dram_bytes_per_launch")
+            t = {r["case"]: r for r in json.load(open(prof))["launches"]}
+            hit = [t[i] for i in dom_cases if i in t and t[i]["kernel"] == dom]
+            if hit:
+                traffic = round(sum(r["dram_bytes"] for r in hit) / len(hit))
+                traffic_alg = round(sum(r["alg_bytes"] for r in hit) / len(hit))
         except Exception:
             traffic = None
     roof = {"bound": "tensor", "achieved": round(achieved, 3), "peak": FP64_PEAK_TFLOPS,
@@ -332,6 +437,9 @@ def run_libtc(args):
             "kernel": dom, "cases": dom_cases,
             "peak_source": "measured FP64 DMMA peak (tools/peaks.cu, profiles/r01_peaks.json); "
                            f"derived 148x64x2x1.965GHz = {FP64_PEAK_DERIVED:.2f}",
+            "traffic_cases": "mean dram__bytes_read+write per launch over the dominant cases "
+                             "captured in profiles/ncu_traffic.json",
+            "alg_bytes_per_launch": traffic_alg,
             "launches_per_step": len(dom_cases),
             "share_of_step": round(dms / ms_step, 4)}
 
@@ -377,6 +485,11 @@ def run_libtc(args):
                "how": "tc_execute_host per case: pinned host A,B -> device, kernel, C -> host, "
                       "stream sync; wall clock, best of 2"}
 
+    suites = {}
+    if world == 1 and args.suites:
+        for name in args.suites.split(","):
+            suites[name] = run_suite(name, args, flush, stream, dev, hbm)
+
     cpu = None
     if not args.no_cpu and rank == 0 and world == 1:
         import oracle
@@ -410,6 +523,7 @@ def run_libtc(args):
                                 "launched 1+3 times on the case's own tensors, fastest kept "
                                 "(outside the timed region; P:L346-348)"},
                 "wall_s_timed": round(t_wall, 3),
+                "suites": suites,
                 "per_case": per_case}
         print(json.dumps(line), flush=True)
     if world > 1:

@@ -20,6 +20,16 @@ _SO = os.path.join(_HERE, "libtc.so")
 STATUS = ["TC_SUCCESS", "TC_ERR_INVALID_ARG", "TC_ERR_PARSE", "TC_ERR_INDEX", "TC_ERR_EXTENT",
           "TC_ERR_UNSUPPORTED", "TC_ERR_NO_CONFIG", "TC_ERR_CUDA", "TC_ERR_ALLOC"]
 DTYPES = {"f64": 0, "f32": 1, "tf32": 2, "bf16": 3}
+# torch storage dtype per plan dtype (tf32 and f32 both store FP32)
+def _tdt(name):
+    def get():
+        import torch
+        return getattr(torch, name)
+    return get
+
+
+_TORCH_DTYPE = {"f64": _tdt("float64"), "f32": _tdt("float32"), "tf32": _tdt("float32"),
+                "bf16": _tdt("bfloat16")}
 COST = {"b200": 0, "paper": 1}
 SLAB_A, SLAB_B, SLAB_C = 1, 2, 4
 
@@ -166,9 +176,12 @@ class Plan:
 
     def execute(self, A, B, C, alpha=1.0, beta=0.0, stream=None):
         """C = alpha * sum A*B + beta * C on torch CUDA tensors (current stream)."""
+        want = _TORCH_DTYPE[self.dtype]()
         for name, t, w in (("A", A, "A"), ("B", B, "B"), ("C", C, "C")):
             if not t.is_cuda or not t.is_contiguous():
                 raise TcError(1, f"{name} must be a contiguous CUDA tensor")
+            if t.dtype != want:
+                raise TcError(1, f"{name} is {t.dtype}, the plan's dtype {self.dtype!r} needs {want}")
         self.execute_ptr(A.data_ptr(), B.data_ptr(), C.data_ptr(), alpha, beta, stream)
         return C
 

@@ -8,9 +8,9 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 SO = os.path.join(HERE, "libtc.so")
 SOURCES = ["api.cu", "contraction.cpp", "planner.cpp", "tiles.cpp", "kernels_00.cu", "kernels_01.cu",
-           "kernels_10.cu", "kernels_11.cu", "kernels_bf16.cu"]
+           "kernels_10.cu", "kernels_11.cu", "kernels_umma.cu"]
 HEADERS = ["contraction.hpp", "planner.hpp", "kparams.hpp", "kernel_f64.cuh", "tiles.hpp", "variants.def",
-           "kernel_table.cuh", "kernel_bf16.cuh"]
+           "kernel_table.cuh", "kernel_umma.cuh"]
 NVCC_FLAGS = ["-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo",
               "-Xcompiler", "-fPIC", "-shared"]
 

@@ -38,13 +38,19 @@ struct KernelEntry {
   size_t smem_tma;   // with it
 };
 
+// Kernel family of a dtype: FP64 -> DMMA; BF16 / TF32 / FP32 (split TF32) -> tcgen05.
+int kind_of(int dtype) {
+  return dtype == TC_BF16 ? KIND_BF16_UMMA : dtype == TC_TF32 ? KIND_TF32_UMMA
+       : dtype == TC_F32 ? KIND_F32X3_UMMA : KIND_F64_DMMA;
+}
+
 // The instance for the plan's variant and smem layouts (kernel_table.cuh).
 KernelEntry kernel_for(const Config &cfg) {
   const Variant &v = variants()[cfg.variant];
-  if (v.kind == KIND_BF16_UMMA) {
+  if (is_umma(v.kind)) {
     size_t smem = 0;
     int threads = 0;
-    const void *fn = kernel_ptr_bf16(cfg.variant, cfg.xKmajor, cfg.yKmajor, &smem, &threads);
+    const void *fn = kernel_ptr_umma(cfg.variant, cfg.xKmajor, cfg.yKmajor, &smem, &threads);
     return {fn, threads, smem, smem};
   }
   const F64Instance k = cfg.xKmajor ? (cfg.yKmajor ? f64_instance_11(cfg.variant) : f64_instance_10(cfg.variant))
@@ -96,7 +102,7 @@ void build_host_tables(tc_plan_s *P) {
   P->slotY1 = build_slots(c, cfg, cfg.Y, 1, cfg.yKmajor, v.BN, v.BK);
   if (cfg.vecX > 1) P->slotX2 = build_slots(c, cfg, cfg.X, cfg.vecX, cfg.xKmajor, v.BM, v.BK);
   if (cfg.vecY > 1) P->slotY2 = build_slots(c, cfg, cfg.Y, cfg.vecY, cfg.yKmajor, v.BN, v.BK);
-  P->cvec = cfg.kind == KIND_BF16_UMMA ? c_vec_width(c, cfg, 8) : (v.stg ? c_vec_width(c, cfg, 2) : 1);
+  P->cvec = is_umma(cfg.kind) ? c_vec_width(c, cfg, 8) : (v.stg ? c_vec_width(c, cfg, 2) : 1);
   KParams &kp = P->kp;
   std::memset(&kp, 0, sizeof(kp));
   kp.mtiles = (int)cfg.mtiles;
@@ -220,7 +226,7 @@ tc_status_t finish_plan(tc_plan_s *P, tc_plan_t *out) {
   normalize(P->c, !P->opts.no_fusion && !ft.on);
   const int fv = P->opts.variant > 0 ? P->opts.variant - 1 : -1;
   if (fv >= (int)variants().size()) { delete P; return fail(ST_INVALID_ARG, "variant out of range"); }
-  const int kind = P->dtype == TC_BF16 ? KIND_BF16_UMMA : KIND_F64_DMMA;
+  const int kind = kind_of(P->dtype);
   if (fv >= 0 && variants()[fv].kind != kind) { delete P; return fail(ST_INVALID_ARG, "variant is not built for this dtype"); }
   Status s = choose(P->c, kind, P->opts.cost_mode, fv, ft, P->cfg, P->stats, err);
   if (s != ST_OK) { delete P; return fail(s, err); }
@@ -238,7 +244,7 @@ tc_status_t finish_plan(tc_plan_s *P, tc_plan_t *out) {
   return TC_SUCCESS;
 }
 
-size_t elem_bytes(const tc_plan_s *P) { return P->dtype == TC_BF16 ? 2 : 8; }
+size_t elem_bytes(const tc_plan_s *P) { return (size_t)kind_esize(kind_of(P->dtype)); }
 
 bool overlaps(const void *a, size_t na, const void *b, size_t nb) {
   const char *x = (const char *)a, *y = (const char *)b;
@@ -290,7 +296,7 @@ bool encode_c_map(const tc_plan_s *P, void *C, TmaDesc &out) {
 
 extern "C" {
 
-const char *tc_version(void) { return "libtc 0.3 (sm_100a, FP64 DMMA + BF16 tcgen05, persistent)"; }
+const char *tc_version(void) { return "libtc 0.4 (sm_100a, FP64 DMMA + BF16/TF32/FP32-split tcgen05, persistent)"; }
 
 const char *tc_status_string(tc_status_t s) {
   switch (s) {
@@ -336,8 +342,8 @@ tc_status_t tc_plan_ex(tc_plan_t *plan, const char *expr, const char *extents, t
     std::string err;
     Status s = parse(expr, extents, P->parsed, err);
     if (s != ST_OK) { delete P; return fail(s, err); }
-    if (dtype != TC_F64 && dtype != TC_BF16)
-      { delete P; return fail(ST_UNSUPPORTED, "only TC_F64 and TC_BF16 are built in this version"); }
+    if (dtype != TC_F64 && dtype != TC_BF16 && dtype != TC_TF32 && dtype != TC_F32)
+      { delete P; return fail(ST_UNSUPPORTED, "dtype must be TC_F64, TC_F32, TC_TF32 or TC_BF16"); }
     if (opts && (opts->cost_mode < 0 || opts->cost_mode > 1)) { delete P; return fail(ST_INVALID_ARG, "cost_mode"); }
     P->dtype = dtype;
     return finish_plan(P, plan);
@@ -501,7 +507,8 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
   kp.nslotY = (int)(vy ? plan->slotY2.pack.size() : plan->slotY1.pack.size());
   kp.vecY = vy ? cfg.vecY : 1;
   kp.dbg = plan->opts.reserved[0];
-  // C stores in 16-B vectors: 8 BF16 (staged BF16 epilogue) / 2 FP64 (STG drain)
+  // C stores in 16-B vectors: 8 elements (staged UMMA epilogue: one 16-B BF16 or two 16-B FP32
+  // stores) / 2 FP64 (STG drain)
   kp.vecC = plan->cvec > 1 && ((uintptr_t)C % 16) == 0 ? plan->cvec : 1;
   const KernelEntry ke = kernel_for(cfg);
   const int grid = (int)std::min<int64_t>(cfg.nctas, plan->sms);
@@ -556,7 +563,8 @@ tc_status_t tc_plan_info(const tc_plan_t plan, char *json, size_t cap, size_t *n
       for (size_t i = 0; i < l.size(); i++) s += (i ? ",\"" : "\"") + c.ix[l[i]].name + "\"";
       return s + "]";
     };
-    o << "{\"dtype\":\"" << (g.kind == KIND_BF16_UMMA ? "bf16" : "f64") << "\",\"X\":\"" << (g.X == 1 ? "A" : "B") << "\"";
+    static const char *dn[4] = {"f64", "bf16", "tf32", "f32"};
+    o << "{\"dtype\":\"" << dn[g.kind] << "\",\"X\":\"" << (g.X == 1 ? "A" : "B") << "\"";
     o << ",\"indices\":[";
     for (size_t i = 0; i < c.ix.size(); i++) {
       const char *cls = c.ix[i].cls == EXT_A ? "extA" : c.ix[i].cls == EXT_B ? "extB" : "int";

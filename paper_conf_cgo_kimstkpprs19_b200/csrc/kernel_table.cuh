@@ -40,7 +40,7 @@ F64Instance f64_instance_00(int v);
 F64Instance f64_instance_01(int v);
 F64Instance f64_instance_10(int v);
 F64Instance f64_instance_11(int v);
-// defined in kernels_bf16.cu (BF16 tcgen05 variants; smem bytes and block size out)
-const void *kernel_ptr_bf16(int v, bool xk, bool yk, size_t *smem, int *threads);
+// defined in kernels_umma.cu (BF16 / TF32 / F32X3 tcgen05 variants; smem bytes and block size out)
+const void *kernel_ptr_umma(int v, bool xk, bool yk, size_t *smem, int *threads);
 
 }  // namespace tc

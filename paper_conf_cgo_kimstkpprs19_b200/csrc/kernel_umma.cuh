@@ -18,6 +18,7 @@
 #pragma once
 #include <cuda_bf16.h>
 #include <cstdint>
+#include <type_traits>
 
 #include "kernel_f64.cuh"   // cp.async / mbarrier helpers, tile_coords, bit_of
 #include "kparams.hpp"
@@ -39,12 +40,19 @@ __device__ __forceinline__ void tc05_commit(uint32_t bar) {
   asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n" ::"r"(bar)
                : "memory");
 }
-__device__ __forceinline__ void tc05_mma_bf16(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
-                                              uint32_t accumulate) {
-  asm volatile(
-      "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
-      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(d_tmem),
-      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate) : "memory");
+template <bool TF32>
+__device__ __forceinline__ void tc05_mma(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
+                                         uint32_t accumulate) {
+  if constexpr (TF32)
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(d_tmem),
+        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate) : "memory");
+  else
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(d_tmem),
+        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate) : "memory");
 }
 __device__ __forceinline__ void tc05_ld16(uint32_t taddr, uint32_t (&v)[16]) {
   asm volatile(
@@ -66,26 +74,26 @@ __device__ __forceinline__ void cp_async8v_full(uint32_t dst, const void *src) {
 // Register-cached slots (4- or 8-element vectors): this thread's slots first + i * 128 of
 // one operand; `cnt` of the E entries are real.  Interior tile and full k-step: no bounds
 // work; otherwise each slot tests its k bit and its row bit and zero-fills.
-template <int E>
-__device__ __forceinline__ void bf16_load_slots(int32_t (&rel)[E], uint32_t (&soff)[E], const int32_t *__restrict__ r,
+template <int E, int ES>
+__device__ __forceinline__ void umma_load_slots(int32_t (&rel)[E], uint32_t (&soff)[E], const int32_t *__restrict__ r,
                                                 const uint32_t *__restrict__ pk, int n, int first, int stride) {
 #pragma unroll
   for (int i = 0; i < E; i++) {
     const int q = first + i * stride;
     rel[i] = q < n ? __ldg(r + q) : 0;
-    soff[i] = q < n ? 2u * (__ldg(pk + q) & 0x3FFF) : 0u;   // smem byte offset in the stage
+    soff[i] = q < n ? (uint32_t)ES * (__ldg(pk + q) & 0x3FFF) : 0u;   // smem byte offset in the stage
   }
 }
 
 // One operand, one (tile, step): this thread's `cnt` cached 16-B slots.  Interior tile and
 // full k-step (fast): straight copies.  Otherwise each slot re-reads its packed (k, row) from
 // the slot table, tests the step's k mask and the tile's row mask and zero-fills.
-template <int E>
-__device__ __forceinline__ void bf16_issue(const __nv_bfloat16 *__restrict__ src, uint32_t sdst,
+template <int E, typename T>
+__device__ __forceinline__ void umma_issue(const T *__restrict__ src, uint32_t sdst,
                                            const int32_t (&rel)[E], const uint32_t (&soff)[E], int cnt,
                                            int64_t base, bool fast, uint64_t kmask, const uint64_t (&rmask)[kMaskWords],
                                            const uint32_t *__restrict__ pack, int first, int stride) {
-  const __nv_bfloat16 *b = src + base;
+  const T *b = src + base;
   if (fast) {
 #pragma unroll
     for (int i = 0; i < E; i++)
@@ -105,14 +113,14 @@ __device__ __forceinline__ void bf16_issue(const __nv_bfloat16 *__restrict__ src
 
 // Generic producer path (any vector width, slot tables read from global memory): every slot
 // tests its k bit and its row bit and zero-fills when out of range.
-template <int PW>
-__device__ __forceinline__ void bf16_issue_generic_t(const KParams &p, const __nv_bfloat16 *__restrict__ X,
-                                                     const __nv_bfloat16 *__restrict__ Y, int pt, uint32_t dx,
+template <int PW, typename T>
+__device__ __forceinline__ void umma_issue_generic_t(const KParams &p, const T *__restrict__ X,
+                                                     const T *__restrict__ Y, int pt, uint32_t dx,
                                                      uint32_t dy, int64_t bx, int64_t by, uint64_t km,
                                                      const uint64_t (&mm)[kMaskWords],
                                                      const uint64_t (&mn)[kMaskWords]) {
   for (int side = 0; side < 2; side++) {
-    const __nv_bfloat16 *src = side ? Y : X;
+    const T *src = side ? Y : X;
     const int32_t *rel = side ? p.relY : p.relX;
     const uint32_t *pack = side ? p.packY : p.packX;
     const int n = side ? p.nslotY : p.nslotX, vec = side ? p.vecY : p.vecX;
@@ -123,11 +131,12 @@ __device__ __forceinline__ void bf16_issue_generic_t(const KParams &p, const __n
       const uint32_t pk = __ldg(pack + q);
       const int k = (pk >> 14) & 63, m = pk >> 20;
       const bool ok = ((km >> k) & 1) && ((((m < 64) ? rm[0] : rm[1]) >> (m & 63)) & 1);
-      const __nv_bfloat16 *g = ok ? src + (base + __ldg(rel + q)) : src;
-      const uint32_t d = dst0 + 2u * (pk & 0x3FFF);
-      if (vec == 8) cp_async16v(d, g, ok ? 16 : 0);
-      else if (vec == 4) cp_async8v(d, g, ok ? 8 : 0);
-      else if (vec == 2) cp_async4(d, g, ok ? 4 : 0);
+      const T *g = ok ? src + (base + __ldg(rel + q)) : src;
+      const uint32_t d = dst0 + (uint32_t)sizeof(T) * (pk & 0x3FFF);
+      const int bytes = vec * (int)sizeof(T);
+      if (bytes == 16) cp_async16v(d, g, ok ? 16 : 0);
+      else if (bytes == 8) cp_async8v(d, g, ok ? 8 : 0);
+      else if (bytes == 4) cp_async4(d, g, ok ? 4 : 0);
       else {   // single elements: plain load / store (cp.async has no 2-byte form)
         const unsigned short v = ok ? *reinterpret_cast<const unsigned short *>(g) : (unsigned short)0;
         asm volatile("st.shared.u16 [%0], %1;\n" ::"r"(d), "h"(v) : "memory");
@@ -164,43 +173,63 @@ __device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint
          ((uint64_t)((sbo >> 4) & 0x3FFF) << 32) | (1ull << 46) | (2ull << 61);
 }
 
-template <int BN, int STAGES>
-struct Bf16Kernel {
-  static constexpr int BM = 128, BK = 64;            // one UMMA M = 128, four K = 16 per stage
+// KIND (tiles.hpp): 1 = BF16 (kind::f16), 2 = TF32 on FP32 storage (kind::tf32),
+// 3 = FP32 as split TF32: SW split warps rewrite each landed stage as hi = tf32 truncation
+// (in place) and lo = x - hi (a second plane), and the MMA warp issues hi*hi + hi*lo + lo*hi.
+template <int KIND, int BN, int STAGES>
+struct UmmaKernel {
+  using T = typename std::conditional<KIND == 1, __nv_bfloat16, float>::type;
+  static constexpr int ES = KIND == 1 ? 2 : 4;       // element bytes
+  static constexpr bool SPLIT = KIND == 3;
+  static constexpr int BM = 128, BK = 128 / ES;      // one UMMA M = 128; 128-B k rows
+  static constexpr int KI = 32 / ES;                 // K per MMA instruction (f16: 16, tf32: 8)
   static constexpr int EW = 8, PW = 4;               // epilogue warps, producer warps
-  static constexpr int THREADS = (EW + PW + 1) * 32; // + one MMA warp
-  static constexpr int XS = BM * BK, YS = BN * BK;   // elements per stage (1 KB multiples)
+  static constexpr int SW = SPLIT ? 4 : 0;           // split warps
+  static constexpr int THREADS = (EW + PW + 1 + SW) * 32; // + one MMA warp
+  static constexpr int XS = BM * BK, YS = BN * BK;   // elements per stage plane (1 KB multiples)
+  static constexpr int PLANES = SPLIT ? 2 : 1;       // hi (in place) + lo
   static constexpr int NBUF = 512 / BN;              // FP32 accumulators in flight (all of TMEM)
   static constexpr int TMEM_COLS = NBUF * BN;
   static constexpr size_t smem_bytes() {
-    return 1024 + 2 * (size_t)STAGES * (XS + YS) + 8 * (2 * STAGES + 2 * NBUF) + 16 + 8 * (size_t)(BM + BN) +
-           4 * (size_t)EW * 32 * 32;   // + per-epilogue-warp FP32 staging (32 x 32)
+    return 1024 + (size_t)ES * PLANES * STAGES * (XS + YS) + 8 * (3 * STAGES + 2 * NBUF) + 16 +
+           8 * (size_t)(BM + BN) + 4 * (size_t)EW * 32 * 32;   // + per-epilogue-warp FP32 staging (32 x 32)
   }
   // register-cached slots per producer thread (16-B vectors)
-  static constexpr int EX = BM * BK / 8 / (PW * 32), EY = BN * BK / 8 / (PW * 32);
-  static_assert(BN % 16 == 0 && BN <= 128, "BN");
+  static constexpr int EX = BM * BK * ES / 16 / (PW * 32), EY = BN * BK * ES / 16 / (PW * 32);
+  static_assert(BN % 32 == 0 && BN <= 128, "BN");
   static_assert(TMEM_COLS >= 32 && (TMEM_COLS & (TMEM_COLS - 1)) == 0, "TMEM allocation");
+  static_assert(smem_bytes() <= 232448, "smem");
 };
 
-// UMMA instruction descriptor: BF16 x BF16 -> F32, M = 128, N = BN, majors per operand.
-__host__ __device__ constexpr uint32_t umma_idesc_bf16(int n, bool a_mn, bool b_mn) {
-  return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)a_mn << 15) | ((uint32_t)b_mn << 16) |
-         ((uint32_t)(n >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
+// UMMA instruction descriptor: BF16 x BF16 or TF32 x TF32 -> F32 (c_format 1 at [4,6),
+// a/b_format at [7,10) / [10,13): BF16 = 1, TF32 = 2), M = 128, N = BN, majors per operand.
+__host__ __device__ constexpr uint32_t umma_idesc(int fmt, int n, bool a_mn, bool b_mn) {
+  return (1u << 4) | ((uint32_t)fmt << 7) | ((uint32_t)fmt << 10) | ((uint32_t)a_mn << 15) |
+         ((uint32_t)b_mn << 16) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
 }
 
-template <int BN, int STAGES, bool XK, bool YK>
-__global__ void __launch_bounds__(Bf16Kernel<BN, STAGES>::THREADS, 1)
-tc_bf16_umma_kernel(const __grid_constant__ KParams p) {
-  using K = Bf16Kernel<BN, STAGES>;
-  constexpr int BM = K::BM, BK = K::BK;
+__device__ __forceinline__ void st_out(__nv_bfloat16 *d, float v) { *d = __float2bfloat16_rn(v); }
+__device__ __forceinline__ void st_out(float *d, float v) { *d = v; }
+__device__ __forceinline__ float ld_out(const __nv_bfloat16 *d) { return __bfloat162float(*d); }
+__device__ __forceinline__ float ld_out(const float *d) { return *d; }
+
+template <int KIND, int BN, int STAGES, bool XK, bool YK>
+__global__ void __launch_bounds__(UmmaKernel<KIND, BN, STAGES>::THREADS, 1)
+tc_umma_kernel(const __grid_constant__ KParams p) {
+  using K = UmmaKernel<KIND, BN, STAGES>;
+  using T = typename K::T;
+  constexpr int BM = K::BM, BK = K::BK, ES = K::ES;
   extern __shared__ __align__(1024) unsigned char smem_dyn[];
   // the 128-B swizzle atoms (8 rows x 128 B) must sit on 1 KB boundaries
   unsigned char *smem_raw =
       smem_dyn + ((1024u - ((uint32_t)__cvta_generic_to_shared(smem_dyn) & 1023u)) & 1023u);
-  __nv_bfloat16 *sX = reinterpret_cast<__nv_bfloat16 *>(smem_raw);
-  __nv_bfloat16 *sY = sX + STAGES * K::XS;
-  uint64_t *bars = reinterpret_cast<uint64_t *>(sY + STAGES * K::YS);  // full, empty, tfull[2], tempty[2]
-  uint32_t *tmem_holder = reinterpret_cast<uint32_t *>(bars + 2 * STAGES + 2 * K::NBUF);
+  // stage planes: [X hi | Y hi] x STAGES, then (SPLIT) the lo planes at + LO bytes
+  T *sX = reinterpret_cast<T *>(smem_raw);
+  T *sY = sX + STAGES * K::XS;
+  constexpr uint32_t LO = (uint32_t)ES * STAGES * (K::XS + K::YS);
+  // full, empty, tfull[NBUF], tempty[NBUF], split[STAGES]
+  uint64_t *bars = reinterpret_cast<uint64_t *>(smem_raw + (size_t)LO * K::PLANES);
+  uint32_t *tmem_holder = reinterpret_cast<uint32_t *>(bars + 3 * STAGES + 2 * K::NBUF);
   int64_t *relCm = reinterpret_cast<int64_t *>(tmem_holder + 4);
   int64_t *relCn = relCm + BM;
   float *stage = reinterpret_cast<float *>(relCn + BN);   // [EW][32 columns][32 rows]
@@ -211,10 +240,10 @@ tc_bf16_umma_kernel(const __grid_constant__ KParams p) {
   const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(smem_raw);
   const uint32_t bar0 = (uint32_t)__cvta_generic_to_shared(bars);
   const uint32_t FULL = bar0, EMPTY = bar0 + 8 * STAGES, TFULL = bar0 + 16 * STAGES,
-                 TEMPTY = TFULL + 8 * K::NBUF;
+                 TEMPTY = TFULL + 8 * K::NBUF, SPLITB = TEMPTY + 8 * K::NBUF;
 
   // ---- once per CTA ------------------------------------------------------------------------
-  for (int i = tid; i < STAGES * (K::XS + K::YS) / 8; i += K::THREADS)
+  for (int i = tid; i < (int)(LO * K::PLANES / 16); i += K::THREADS)
     reinterpret_cast<uint4 *>(smem_raw)[i] = make_uint4(0, 0, 0, 0);
   for (int r = tid; r < BM; r += K::THREADS) relCm[r] = p.relCm[r];
   for (int r = tid; r < BN; r += K::THREADS) relCn[r] = p.relCn[r];
@@ -227,6 +256,7 @@ tc_bf16_umma_kernel(const __grid_constant__ KParams p) {
       mbar_init(TFULL + 8 * b, 1);           // tcgen05.commit after a tile's last MMA
       mbar_init(TEMPTY + 8 * b, K::EW);      // one arrive per epilogue warp
     }
+    for (int s = 0; s < STAGES; s++) mbar_init(SPLITB + 8 * s, K::SW > 0 ? K::SW : 1);   // split warps
     asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
   }
   if (warp == K::EW + K::PW) {               // the MMA warp owns the TMEM allocation
@@ -243,17 +273,17 @@ tc_bf16_umma_kernel(const __grid_constant__ KParams p) {
   if (warp >= K::EW && warp < K::EW + K::PW) {
     // ======================= producers ===================================================
     const int pt = tid - K::EW * 32;
-    const __nv_bfloat16 *__restrict__ X = static_cast<const __nv_bfloat16 *>(p.X);
-    const __nv_bfloat16 *__restrict__ Y = static_cast<const __nv_bfloat16 *>(p.Y);
+    const T *__restrict__ X = static_cast<const T *>(p.X);
+    const T *__restrict__ Y = static_cast<const T *>(p.Y);
     // fast path: both operands in 16-B vectors, slots cached in registers
-    const bool cached = p.vecX == 8 && p.vecY == 8 && p.nslotX <= K::EX * K::PW * 32 &&
+    const bool cached = p.vecX == 16 / ES && p.vecY == 16 / ES && p.nslotX <= K::EX * K::PW * 32 &&
                         p.nslotY <= K::EY * K::PW * 32;
     int32_t rx[K::EX], ry[K::EY];
     uint32_t px[K::EX], py[K::EY];
     int cx = 0, cy = 0;
     if (cached) {
-      bf16_load_slots(rx, px, p.relX, p.packX, p.nslotX, pt, K::PW * 32);
-      bf16_load_slots(ry, py, p.relY, p.packY, p.nslotY, pt, K::PW * 32);
+      umma_load_slots<K::EX, ES>(rx, px, p.relX, p.packX, p.nslotX, pt, K::PW * 32);
+      umma_load_slots<K::EY, ES>(ry, py, p.relY, p.packY, p.nslotY, pt, K::PW * 32);
       cx = (p.nslotX - pt + K::PW * 32 - 1) / (K::PW * 32);
       cy = (p.nslotY - pt + K::PW * 32 - 1) / (K::PW * 32);
     }
@@ -274,17 +304,17 @@ tc_bf16_umma_kernel(const __grid_constant__ KParams p) {
       const uint64_t(&mm)[kMaskWords] = cur.mm;
       const uint64_t(&mn)[kMaskWords] = cur.mn;
       const int64_t bx = cur.ox + ks.sx(), by = cur.oy + ks.sy();
-      const uint32_t dx = sbase + 2u * (uint32_t)(s * K::XS);
-      const uint32_t dy = sbase + 2u * (uint32_t)(STAGES * K::XS + s * K::YS);
+      const uint32_t dx = sbase + (uint32_t)ES * (uint32_t)(s * K::XS);
+      const uint32_t dy = sbase + (uint32_t)ES * (uint32_t)(STAGES * K::XS + s * K::YS);
       if (p.dbg & 8) {
         mbar_arrive(FULL + 8 * s);
       } else if (cached) {
-        bf16_issue<K::EX>(X, dx, rx, px, cx, bx, fm && fk, km, mm, p.packX, pt, K::PW * 32);
-        bf16_issue<K::EY>(Y, dy, ry, py, cy, by, fn && fk, km, mn, p.packY, pt, K::PW * 32);
+        umma_issue<K::EX>(X, dx, rx, px, cx, bx, fm && fk, km, mm, p.packX, pt, K::PW * 32);
+        umma_issue<K::EY>(Y, dy, ry, py, cy, by, fn && fk, km, mn, p.packY, pt, K::PW * 32);
         mbar_arrive_cp_async(FULL + 8 * s);
       } else {
-        bf16_issue_generic_t<K::PW>(p, X, Y, pt, dx, dy, bx, by, km, mm, mn);
-        if (p.vecX == 1 || p.vecY == 1) {
+        umma_issue_generic_t<K::PW>(p, X, Y, pt, dx, dy, bx, by, km, mm, mn);
+        if (ES == 2 && (p.vecX == 1 || p.vecY == 1)) {
           // plain stores are published by a release arrive once this thread's copies landed
           asm volatile("cp.async.wait_all;\n" ::: "memory");
           mbar_arrive(FULL + 8 * s);
@@ -300,32 +330,45 @@ tc_bf16_umma_kernel(const __grid_constant__ KParams p) {
     }
   } else if (warp == K::EW + K::PW) {
     // ======================= MMA issuer ===================================================
-    constexpr uint32_t IDESC = umma_idesc_bf16(BN, !XK, !YK);
+    constexpr uint32_t IDESC = umma_idesc(ES == 2 ? 1 : 2, BN, !XK, !YK);
     // canonical no-swizzle layouts (bytes): K-major LBO = 128 (k groups), SBO = 1024 (8-row
     // groups); MN-major SBO = 128 (8-row groups), LBO = rows/8 * 128 (k groups)
     // 128-B swizzled layouts (tiles.hpp smem_off): K-major = 8-row x 128-B atoms stacked
     // along M/N (SBO = 1 KB; K = 16 advances the start by 32 B inside the atom); MN-major =
     // 64-element x 8-k atoms, MN atoms at LBO = 1 KB, 8-k groups at SBO = BMN/64 KB
-    constexpr uint32_t A_LBO = XK ? 16 : 1024, A_SBO = XK ? 1024 : (BM / 64) * 1024;
-    constexpr uint32_t B_LBO = YK ? 16 : 1024, B_SBO = YK ? 1024 : (BN / 64) * 1024;
-    constexpr uint32_t A_KSTEP = XK ? 32 : 2 * A_SBO, B_KSTEP = YK ? 32 : 2 * B_SBO;  // per K = 16
+    // (E = 128 / ES elements per 128-B row; one MMA consumes K = KI = 32 B of k: 16 BF16 =
+    // two 8-k atom groups, 8 TF32 = one)
+    constexpr int E = 128 / ES;
+    constexpr uint32_t A_LBO = XK ? 16 : 1024, A_SBO = XK ? 1024 : (BM / E) * 1024;
+    constexpr uint32_t B_LBO = YK ? 16 : 1024, B_SBO = YK ? 1024 : (BN / E) * 1024;
+    constexpr uint32_t A_KSTEP = XK ? 32 : (K::KI / 8) * A_SBO, B_KSTEP = YK ? 32 : (K::KI / 8) * B_SBO;
     int step = 0, lt = 0;
     for (int j = 0; j < total; j++) {
       const int s = j % STAGES;
       const int buf = lt % K::NBUF;
       if (step == 0 && lt >= K::NBUF) mbar_wait(TEMPTY + 8 * buf, ((lt / K::NBUF) & 1) ^ 1);
-      mbar_wait(FULL + 8 * s, (j / STAGES) & 1);
+      if (K::SPLIT) mbar_wait(SPLITB + 8 * s, (j / STAGES) & 1);
+      else mbar_wait(FULL + 8 * s, (j / STAGES) & 1);
       // the stage was written through the generic proxy (cp.async / st.shared); the MMA
       // reads it through the async proxy
       if (!(p.dbg & 16)) asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
       tc05_fence_after();
       if (lane == 0) {
-        const uint32_t ax = sbase + 2u * (uint32_t)(s * K::XS);
-        const uint32_t by = sbase + 2u * (uint32_t)(STAGES * K::XS + s * K::YS);
+        const uint32_t ax = sbase + (uint32_t)ES * (uint32_t)(s * K::XS);
+        const uint32_t by = sbase + (uint32_t)ES * (uint32_t)(STAGES * K::XS + s * K::YS);
+        const uint32_t d = tmem + (uint32_t)(buf * BN);
 #pragma unroll
-        for (int kk = 0; kk < BK / 16; kk++)
-          if (!(p.dbg & 2)) tc05_mma_bf16(tmem + (uint32_t)(buf * BN), umma_desc(ax + kk * A_KSTEP, A_LBO, A_SBO),
-                        umma_desc(by + kk * B_KSTEP, B_LBO, B_SBO), IDESC, (step > 0 || kk > 0) ? 1u : 0u);
+        for (int kk = 0; kk < BK / K::KI; kk++) {
+          const uint64_t ah = umma_desc(ax + kk * A_KSTEP, A_LBO, A_SBO);
+          const uint64_t bh = umma_desc(by + kk * B_KSTEP, B_LBO, B_SBO);
+          if (K::SPLIT) {   // small terms first: lo*hi, hi*lo, then hi*hi
+            tc05_mma<true>(d, umma_desc(ax + LO + kk * A_KSTEP, A_LBO, A_SBO), bh, IDESC, (step > 0 || kk > 0) ? 1u : 0u);
+            tc05_mma<true>(d, ah, umma_desc(by + LO + kk * B_KSTEP, B_LBO, B_SBO), IDESC, 1u);
+            tc05_mma<true>(d, ah, bh, IDESC, 1u);
+          } else if (!(p.dbg & 2)) {
+            tc05_mma<ES == 4>(d, ah, bh, IDESC, (step > 0 || kk > 0) ? 1u : 0u);
+          }
+        }
         if (p.dbg & 64) mbar_arrive(EMPTY + 8 * s);
         else tc05_commit(EMPTY + 8 * s);                      // smem stage free once MMAs read it
         if (step + 1 == p.nsteps) tc05_commit(TFULL + 8 * buf);   // accumulator ready
@@ -333,11 +376,40 @@ tc_bf16_umma_kernel(const __grid_constant__ KParams p) {
       __syncwarp();
       if (++step == p.nsteps) { step = 0; ++lt; }
     }
+  } else if (K::SPLIT && warp > K::EW + K::PW) {
+    // ======================= split warps (F32X3) ==========================================
+    // once a stage has landed: x -> hi = x with the low 13 mantissa bits cleared (exactly the
+    // TF32 value the MMA reads) in place, lo = x - hi (exact in FP32) into the lo plane
+    const int st = tid - (K::EW + K::PW + 1) * 32;
+    constexpr int N4 = (K::XS + K::YS) / 4;          // float4 per stage plane
+    for (int j = 0; j < total; j++) {
+      const int s = j % STAGES;
+      mbar_wait(FULL + 8 * s, (j / STAGES) & 1);
+      float4 *hx = reinterpret_cast<float4 *>(smem_raw) + (size_t)s * (K::XS / 4);
+      float4 *hy = reinterpret_cast<float4 *>(smem_raw) + (size_t)STAGES * (K::XS / 4) + (size_t)s * (K::YS / 4);
+#pragma unroll 4
+      for (int i = st; i < N4; i += K::SW * 32) {
+        float4 *h = i < K::XS / 4 ? hx + i : hy + (i - K::XS / 4);
+        float4 *l = reinterpret_cast<float4 *>(reinterpret_cast<unsigned char *>(h) + LO);
+        const float4 x = *h;
+        float4 hi, lo;
+        hi.x = __uint_as_float(__float_as_uint(x.x) & 0xFFFFE000u); lo.x = x.x - hi.x;
+        hi.y = __uint_as_float(__float_as_uint(x.y) & 0xFFFFE000u); lo.y = x.y - hi.y;
+        hi.z = __uint_as_float(__float_as_uint(x.z) & 0xFFFFE000u); lo.z = x.z - hi.z;
+        hi.w = __uint_as_float(__float_as_uint(x.w) & 0xFFFFE000u); lo.w = x.w - hi.w;
+        *h = hi;
+        *l = lo;
+      }
+      // generic-proxy writes -> visible to the MMA's async-proxy reads
+      asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
+      __syncwarp();
+      if (lane == 0) mbar_arrive(SPLITB + 8 * s);
+    }
   } else if (warp < K::EW) {
     // ======================= epilogue =====================================================
     // warp w drains TMEM lane quarter w % 4 (tile rows 32(w%4) .. +31; one row per thread)
-    // and column half w / 4; FP32 arithmetic on the FP32 accumulator, RNE to BF16
-    __nv_bfloat16 *__restrict__ C = static_cast<__nv_bfloat16 *>(p.C);
+    // and column half w / 4; FP32 arithmetic on the FP32 accumulator, stored as T (BF16: RNE)
+    T *__restrict__ C = static_cast<T *>(p.C);
     const float alpha = (float)p.alpha, beta = (float)p.beta;
     const int quarter = warp & 3, half = warp >> 2;
     const int row = quarter * 32 + lane;               // TMEM lane = tile row m
@@ -367,10 +439,10 @@ tc_bf16_umma_kernel(const __grid_constant__ KParams p) {
       const uint64_t rm0 = nrm0, rm1 = nrm1, cm0 = ncm0, cm1 = ncm1;
       if (lt + 1 < ntl) fetch(lt + 1);
       const bool rok = ((row < 64 ? rm0 : rm1) >> (row & 63)) & 1;
-      __nv_bfloat16 *Crow = C + (coff + roff);
+      T *Crow = C + (coff + roff);
       const bool cfull = cm0 == p.fullN[0] && cm1 == p.fullN[1];
       const bool gok = ((grow < 64 ? rm0 : rm1) >> (grow & 63)) & 1;
-      __nv_bfloat16 *Cg = C + (coff + goff);
+      T *Cg = C + (coff + goff);
       if (p.dbg & 256) mbar_wait(TFULL + 8 * buf, (lt / K::NBUF) & 1);
       else mbar_wait_sleep(TFULL + 8 * buf, (lt / K::NBUF) & 1);
       tc05_fence_after();
@@ -405,6 +477,19 @@ tc_bf16_umma_kernel(const __grid_constant__ KParams p) {
             if (ok[i]) {
               float r[8] = {alpha * d[i][0].x, alpha * d[i][0].y, alpha * d[i][0].z, alpha * d[i][0].w,
                             alpha * d[i][1].x, alpha * d[i][1].y, alpha * d[i][1].z, alpha * d[i][1].w};
+              if constexpr (ES == 4) {
+                float4 *dst = reinterpret_cast<float4 *>(Cg + rc[i]);
+                if (beta != 0.0f) {
+                  const float4 o0 = dst[0], o1 = dst[1];
+                  r[0] = fmaf(beta, o0.x, r[0]); r[1] = fmaf(beta, o0.y, r[1]);
+                  r[2] = fmaf(beta, o0.z, r[2]); r[3] = fmaf(beta, o0.w, r[3]);
+                  r[4] = fmaf(beta, o1.x, r[4]); r[5] = fmaf(beta, o1.y, r[5]);
+                  r[6] = fmaf(beta, o1.z, r[6]); r[7] = fmaf(beta, o1.w, r[7]);
+                }
+                dst[0] = make_float4(r[0], r[1], r[2], r[3]);
+                dst[1] = make_float4(r[4], r[5], r[6], r[7]);
+                continue;
+              }
               uint4 *dst = reinterpret_cast<uint4 *>(Cg + rc[i]);
               if (beta != 0.0f) {
                 const uint4 o = *dst;
@@ -431,16 +516,16 @@ tc_bf16_umma_kernel(const __grid_constant__ KParams p) {
 #pragma unroll
             for (int q = 0; q < W; q++)
               if (half * HC + c0 + q < p.Nt)               // (the full mask covers Nt columns)
-                Crow[relCn[half * HC + c0 + q]] = __float2bfloat16_rn(alpha * __uint_as_float(v[q]));
+                st_out(Crow + relCn[half * HC + c0 + q], alpha * __uint_as_float(v[q]));
           } else {
 #pragma unroll
             for (int q = 0; q < W; q++) {
               const int c = half * HC + c0 + q;
               if (((c < 64 ? cm0 : cm1) >> (c & 63)) & 1) {
-                __nv_bfloat16 *dst = Crow + relCn[c];
+                T *dst = Crow + relCn[c];
                 float r = alpha * __uint_as_float(v[q]);
-                if (beta != 0.0f) r = fmaf(beta, __bfloat162float(*dst), r);
-                *dst = __float2bfloat16_rn(r);
+                if (beta != 0.0f) r = fmaf(beta, ld_out(dst), r);
+                st_out(dst, r);
               }
             }
           }

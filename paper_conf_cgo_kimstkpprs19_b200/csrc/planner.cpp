@@ -24,7 +24,10 @@ static int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 // multiply-adds per clock per SM of the kernel family's MMA pipe: DMMA 64 (measured), BF16
 // tcgen05 4096 (2.25 PFLOP/s dense nominal at 1.86 GHz; MEASURED_PEAKS.json has cuBLAS's
 // sustained figure)
-static double fma_per_clk(int kind) { return kind == KIND_BF16_UMMA ? 4096.0 : kFmaPerClk; }
+// TF32 half the BF16 rate; F32X3 issues three TF32 MMAs per k-step
+static double fma_per_clk(int kind) {
+  return kind == KIND_BF16_UMMA ? 4096.0 : kind == KIND_TF32_UMMA ? 2048.0 : kind == KIND_F32X3_UMMA ? 2048.0 / 3 : kFmaPerClk;
+}
 
 int64_t contiguous_run(const Contraction &c, int t, const std::vector<int> &T) {
   // cal_Cont: elements contiguous in memory within the tile hyper-rectangle
@@ -58,7 +61,7 @@ static std::pair<double, double> operand_sim(const Contraction &c, const Config 
     if (it != cache->end()) return it->second;
   }
   const SlotTable st = build_slots(c, cfg, t, vec, kmaj, BMN, BK);
-  const int es = cfg.kind == KIND_BF16_UMMA ? 2 : 8;
+  const int es = kind_esize(cfg.kind);
   const std::pair<double, double> r{slot_wavefronts(st, vec, es, cfg.kind), slot_sectors(st, vec, es)};
   if (cache) (*cache)[key] = r;
   return r;
@@ -70,8 +73,8 @@ double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *
   const double nctas = (double)cfg.nctas, steps = (double)cfg.nsteps;
   // per CTA-step pipe cycles on one SM: FP64 (DMMA) and shared memory
   const double dmma = (double)v.BM * v.BN * v.BK / fma_per_clk(v.kind);
-  const bool umma = v.kind == KIND_BF16_UMMA;
-  const int maxv = cfg.kind == KIND_BF16_UMMA ? 8 : 2;   // 16 B per cp.async
+  const bool umma = is_umma(v.kind);
+  const int maxv = 16 / kind_esize(cfg.kind);   // 16 B per cp.async
   cfg.vecX = vec_width(c, cfg, cfg.X, maxv);
   cfg.vecY = vec_width(c, cfg, cfg.Y, maxv);
   const auto sx = operand_sim(c, cfg, cfg.X, cfg.vecX, cfg.xKmajor, v.BM, v.BK, cache);
@@ -517,7 +520,7 @@ static Status choose_paper(const Contraction &c, int kind, int forced_variant, C
         const double TBy = (double)tprod(y.tb), REGy = (double)tprod(y.reg);
         const double TBk = (double)tprod(k);
         // P:L172 hardware constraints (V100: 48 KB smem per block, 255 registers/thread)
-        const double smem = (kind == KIND_BF16_UMMA ? 2.0 : 8.0) * (TBx * TBk * REGx + TBy * TBk * REGy);
+        const double smem = (double)kind_esize(kind) * (TBx * TBk * REGx + TBy * TBk * REGy);
         bool ok = smem <= 48 * 1024 && REGx * REGy <= 64 && TBx * TBy <= 1024;
         // enough thread blocks (R16: at least one wave of the running GPU)
         ok &= (double)cfg.nctas >= kSMs;

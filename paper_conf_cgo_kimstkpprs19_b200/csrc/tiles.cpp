@@ -17,6 +17,12 @@ const std::vector<Variant> &variants() {
 #undef TC_F64_VARIANT
     t[11] = Variant{128, 64, 64, 32, 32, 6, 4, 1, KIND_BF16_UMMA};
     t[12] = Variant{128, 128, 64, 32, 32, 5, 4, 1, KIND_BF16_UMMA};
+    // TF32 (FP32 storage): same 128-B rows, BK = 32 elements
+    t[21] = Variant{128, 64, 32, 32, 32, 6, 4, 1, KIND_TF32_UMMA};
+    t[22] = Variant{128, 128, 32, 32, 32, 5, 4, 1, KIND_TF32_UMMA};
+    // FP32 as split TF32 (hi + lo planes per stage: twice the smem per stage)
+    t[23] = Variant{128, 64, 32, 32, 32, 3, 4, 1, KIND_F32X3_UMMA};
+    t[24] = Variant{128, 128, 32, 32, 32, 2, 4, 1, KIND_F32X3_UMMA};
     return t;
   }();
   return v;
@@ -110,8 +116,8 @@ SlotTable build_slots(const Contraction &c, const Config &cfg, int t, int vec, b
     }
     mul[p] = m;
   }
-  // packed slot: smem offset (elements) | k | row; FP64: 13 | 6 | 13 bits, BF16: 14 | 6 | 12
-  const int kshift = cfg.kind == KIND_BF16_UMMA ? 14 : 13, mshift = cfg.kind == KIND_BF16_UMMA ? 20 : 19;
+  // packed slot: smem offset (elements) | k | row; FP64: 13 | 6 | 13 bits, UMMA: 14 | 6 | 12
+  const int kshift = is_umma(cfg.kind) ? 14 : 13, mshift = is_umma(cfg.kind) ? 20 : 19;
   std::vector<int> d(r, 0);
   for (;;) {
     int mn = 0, k = 0;

@@ -11,38 +11,47 @@
 namespace tc {
 
 // Compiled kernel shapes (kernel_f64.cuh template instances, api.cu kernel table).
-enum Kind { KIND_F64_DMMA = 0, KIND_BF16_UMMA = 1 };
+// F64: DMMA register tiles (kernel_f64.cuh).  The others share the tcgen05 kernel
+// (kernel_umma.cuh): BF16 = kind::f16, TF32 = kind::tf32 on FP32 storage, F32X3 = FP32 data
+// as a 3-pass split TF32 product (hi*hi + hi*lo + lo*hi, near-FP32 accuracy).
+enum Kind { KIND_F64_DMMA = 0, KIND_BF16_UMMA = 1, KIND_TF32_UMMA = 2, KIND_F32X3_UMMA = 3 };
+inline bool is_umma(int kind) { return kind != KIND_F64_DMMA; }
+inline int kind_esize(int kind) { return kind == KIND_F64_DMMA ? 8 : kind == KIND_BF16_UMMA ? 2 : 4; }
 
-constexpr int kNumVariants = 21;             // ids 0..20 (variants.def + the BF16 ids 11, 12)
+constexpr int kNumVariants = 25;   // ids 0..20 (variants.def + BF16 11, 12) + TF32 21, 22 + F32X3 23, 24
 
 struct Variant {
   int BM = 0, BN = 0, BK = 0, WM = 0, WN = 0, stages = 0, pw = 0, occ = 0;   // pw = producer warps
   int kind = KIND_F64_DMMA;
   int stg = 0;                                // 1: staged epilogue drained by the producers
-  int threads() const { return kind == KIND_BF16_UMMA ? 13 * 32 : ((BM / WM) * (BN / WN) + pw) * 32; }
-  int cwarps() const { return kind == KIND_BF16_UMMA ? 8 : (BM / WM) * (BN / WN); }
-  int esize() const { return kind == KIND_BF16_UMMA ? 2 : 8; }
+  int threads() const {
+    return kind == KIND_F32X3_UMMA ? 17 * 32 : is_umma(kind) ? 13 * 32 : ((BM / WM) * (BN / WN) + pw) * 32;
+  }
+  int cwarps() const { return is_umma(kind) ? 8 : (BM / WM) * (BN / WN); }
+  int esize() const { return kind_esize(kind); }
 };
 const std::vector<Variant> &variants();
 
 // Smem offset (in elements) of element (row mn, k) of one operand stage.
 //  FP64 (kernel_f64.cuh SmemLayout): pitch 4 (mod 16) doubles, k- or mn-contiguous.
-//  BF16 (kernel_bf16.cuh): UMMA 128-B swizzled layouts (stage base 1 KB aligned); the 16-B
-//  chunk index inside a 128-B row is XORed with the row's index inside its 8-row atom.
-//  K-major (BK = 64 = one 128-B row): row mn at (mn/8) KB + (mn%8) 128 B, k along the row.
-//  MN-major: atom (mn/64, k/8) at ((k/8) (BMN/64) + mn/64) KB, row k%8, mn%64 along the row.
+//  UMMA kinds (kernel_umma.cuh): 128-B swizzled layouts (stage base 1 KB aligned); the 16-B
+//  chunk index inside a 128-B row is XORed with the row's index inside its 8-row atom.  With
+//  E = 128 / esize elements per 128-B row (BF16 64, TF32 32):
+//  K-major (BK = E = one 128-B row): row mn at (mn/8) KB + (mn%8) 128 B, k along the row.
+//  MN-major: atom (mn/E, k/8) at ((k/8) (BMN/E) + mn/E) KB, row k%8, mn%E along the row.
 inline int smem_off(int kind, bool kmajor, int mn, int k, int BMN, int BK) {
-  if (kind == KIND_BF16_UMMA) {
+  if (is_umma(kind)) {
+    const int es = kind_esize(kind), E = 128 / es;
     int byte;
     if (kmajor) {
-      const int r = mn % 8;
-      byte = (mn / 8) * 1024 + r * 128 + ((((k * 2) >> 4) ^ r) << 4) + (k * 2 & 15);
+      const int r = mn % 8, kb = k * es;
+      byte = (mn / 8) * 1024 + r * 128 + (((kb >> 4) ^ r) << 4) + (kb & 15);
     } else {
-      const int r = k % 8, e = mn % 64;
-      byte = ((k / 8) * (BMN / 64) + mn / 64) * 1024 + r * 128 + ((((e * 2) >> 4) ^ r) << 4) + (e * 2 & 15);
+      const int r = k % 8, eb = (mn % E) * es;
+      byte = ((k / 8) * (BMN / E) + mn / E) * 1024 + r * 128 + (((eb >> 4) ^ r) << 4) + (eb & 15);
     }
     (void)BK;
-    return byte / 2;
+    return byte / es;
   }
   return kmajor ? mn * (BK + 4) + k : k * (BMN + 4) + mn;
 }
@@ -92,8 +101,8 @@ double slot_wavefronts(const SlotTable &s, int vec, int esize = 8, int kind = KI
 // Global-memory 32-B sectors one stage of loads touches (sum over warp instructions of the
 // distinct sectors of 32 consecutive slots; the tile origin is taken as sector-aligned).
 double slot_sectors(const SlotTable &s, int vec, int esize = 8);
-// Smem offset field of a packed slot (13 bits for FP64, 14 bits for BF16).
-inline uint32_t slot_off(uint32_t pack, int kind) { return kind == KIND_BF16_UMMA ? (pack & 0x3FFF) : (pack & 8191); }
+// Smem offset field of a packed slot (13 bits for FP64, 14 bits for the UMMA kinds).
+inline uint32_t slot_off(uint32_t pack, int kind) { return is_umma(kind) ? (pack & 0x3FFF) : (pack & 8191); }
 
 // Device-side tables for one configuration.
 struct TileTables {

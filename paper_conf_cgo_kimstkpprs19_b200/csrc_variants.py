@@ -14,3 +14,5 @@ for _m in _ROW.finditer(open(_DEF).read()):
 F64_VARIANTS = tuple(sorted(F64_SHAPES))            # FP64 DMMA variants (direct + staged)
 STG_VARIANTS = tuple(v for v in F64_VARIANTS if F64_SHAPES[v]["stg"])
 BF16_VARIANTS = (11, 12)          # BF16 tcgen05 variants (BM = 128, BK = 64; BN = 64 / 128)
+TF32_VARIANTS = (21, 22)          # TF32 tcgen05 (FP32 storage; BK = 32; BN = 64 / 128)
+F32_VARIANTS = (23, 24)           # FP32 as split TF32 (hi*hi + hi*lo + lo*hi; BN = 64 / 128)

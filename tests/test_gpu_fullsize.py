@@ -68,3 +68,28 @@ def test_tccg_full_size_rank1_every_element(cid):
     # S[x] = sum |A B| = want (all factors positive); tau * S plus the closed form's own
     # rounding (a product of <= 8 factors: 8 ulp)
     assert np.all(np.abs(got - want) <= (TAU64 + 16 * 2.2e-16) * np.abs(want))
+
+
+@pytest.mark.parametrize("n,expr", [(48, "abcdef-gdab-efgc"), (40, "abcdef-dega-gfbc")])
+def test_ccsdt_max_size_sampled(n, expr):
+    # BASELINE config 3 at its largest extent: |C| = 48^6 = 1.2e10 FP64 elements (97.8 GB) —
+    # past 2^31 elements, so every 64-bit offset path of the tables and the epilogue runs
+    case = tcinputs.ccsdt(n, expr, 100 + n)
+    p = tc.plan(case.expr, case.extents)
+    A = tcinputs.uniform(p.numel("A"), 1000 + case.id, device="cuda")
+    B = tcinputs.uniform(p.numel("B"), 2000 + case.id, device="cuda")
+    C = torch.full((p.numel("C"),), float("nan"), dtype=torch.float64, device="cuda")
+    p.execute(A, B, C)
+    torch.cuda.synchronize()
+    nC = C.numel()
+    rng = np.random.default_rng(n)
+    idx = np.unique(np.concatenate([rng.integers(0, nC, 2000), np.arange(128), np.arange(nC - 128, nC),
+                                    (np.int64(1) << 31) + np.arange(-64, 64)]))
+    got = C[torch.as_tensor(idx, device="cuda")].cpu().numpy()
+    want, S = oracle.sample(case.expr, case.extents, A.cpu().numpy(), B.cpu().numpy(), idx,
+                            with_scale=True)
+    bad = np.flatnonzero(~(np.abs(got - want) <= TAU64 * S))
+    assert bad.size == 0, (n, idx[bad[:5]], got[bad[:5]], want[bad[:5]])
+    assert not bool(torch.isnan(C).any())   # every element was written
+    del C
+    torch.cuda.empty_cache()

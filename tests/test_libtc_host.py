@@ -132,9 +132,15 @@ def test_errors_are_status_codes():
     with pytest.raises(tc.TcError) as e:
         tc.plan("abcd-aebf-dfc", "a:2;b:2;c:2;d:2;e:2;f:2", host_only=True)
     assert e.value.status == "TC_ERR_INDEX" and "exactly two" in e.value.detail
-    with pytest.raises(tc.TcError) as e:
-        tc.plan("ab-ac-cb", "a:2;b:2;c:2", dtype="f32", host_only=True)
-    assert e.value.status == "TC_ERR_UNSUPPORTED"
+    import ctypes
+    h = ctypes.c_void_p()
+    st = tc.lib().tc_plan(ctypes.byref(h), b"ab-ac-cb", b"a:2;b:2;c:2", 7)   # no such dtype
+    assert tc.lib().tc_status_string(st).decode() == "TC_ERR_UNSUPPORTED" and not h.value
+    for dt in ("f32", "tf32", "bf16"):                 # every dtype of the header is built
+        assert tc.plan("ab-ac-cb", "a:2;b:2;c:2", dtype=dt, host_only=True).info()["dtype"] == dt
+    with pytest.raises(tc.TcError) as e:              # a BF16 variant for a TF32 plan
+        tc.plan("ab-ac-cb", "a:2;b:2;c:2", dtype="tf32", host_only=True, variant=11)
+    assert e.value.status == "TC_ERR_INVALID_ARG"
     with pytest.raises(tc.TcError) as e:              # an FP64 variant for a BF16 plan
         tc.plan("ab-ac-cb", "a:2;b:2;c:2", dtype="bf16", host_only=True, variant=0)
     assert e.value.status == "TC_ERR_INVALID_ARG"
