@@ -62,7 +62,9 @@ typedef struct tc_plan_opts {
   int no_fusion;     /* 1: do not merge adjacent indices (row a2)                            */
   int tma_epilogue;  /* 1: stage C tiles in smem and store them with TMA (cp.async.bulk.tensor)
                         when C is a legal tensor map and beta == 0; 0 (default): direct stores */
-  int reserved[7];
+  int morder;        /* 0: planner's choice; 1: m digits in C order (C's FVI first); 2: in the X
+                        operand's memory order (its FVI first) — tests of both epilogues   */
+  int reserved[6];
 } tc_plan_opts;
 
 /*

@@ -44,7 +44,7 @@ class TcError(RuntimeError):
 class _Opts(ctypes.Structure):
     _fields_ = [("cost_mode", ctypes.c_int), ("host_only", ctypes.c_int), ("variant", ctypes.c_int),
                 ("force_tiles", ctypes.c_char_p), ("no_fusion", ctypes.c_int), ("tma_epilogue", ctypes.c_int),
-                ("reserved", ctypes.c_int * 7)]
+                ("morder", ctypes.c_int), ("reserved", ctypes.c_int * 6)]
 
 
 _lib = None
@@ -197,8 +197,10 @@ class Plan:
 
 def plan(expr: str, extents: str, dtype: str = "f64", cost: str = "b200", host_only: bool = False,
          variant: int | None = None, force_tiles: str | None = None, fusion: bool = True,
-         tma: bool = False, dbg: int = 0) -> Plan:
+         tma: bool = False, dbg: int = 0, morder: str | None = None) -> Plan:
+    """morder: None = planner's choice, "C" = m digits in C order, "X" = in the X operand's order."""
     o = _Opts()
+    o.morder = {None: 0, "C": 1, "X": 2}[morder]
     o.reserved[0] = int(dbg)
     o.tma_epilogue = int(tma)
     o.cost_mode = COST[cost]

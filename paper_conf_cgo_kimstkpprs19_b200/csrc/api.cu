@@ -102,7 +102,8 @@ void build_host_tables(tc_plan_s *P) {
   P->slotY1 = build_slots(c, cfg, cfg.Y, 1, cfg.yKmajor, v.BN, v.BK);
   if (cfg.vecX > 1) P->slotX2 = build_slots(c, cfg, cfg.X, cfg.vecX, cfg.xKmajor, v.BM, v.BK);
   if (cfg.vecY > 1) P->slotY2 = build_slots(c, cfg, cfg.Y, cfg.vecY, cfg.yKmajor, v.BN, v.BK);
-  P->cvec = is_umma(cfg.kind) ? c_vec_width(c, cfg, 8) : (v.stg ? c_vec_width(c, cfg, 2) : 1);
+  int cs0 = 1, ct0 = 1;
+  P->cvec = is_umma(cfg.kind) ? c_run_rows(c, cfg, 8, &cs0, &ct0) : (v.stg ? c_vec_width(c, cfg, 2) : 1);
   KParams &kp = P->kp;
   std::memset(&kp, 0, sizeof(kp));
   kp.mtiles = (int)cfg.mtiles;
@@ -122,6 +123,11 @@ void build_host_tables(tc_plan_s *P) {
   kp.kbase = P->tt.kbase;
   kp.nouter = (int)P->tt.kouter.size();
   kp.Mt = (int)cfg.Mt;
+  kp.cs0 = cs0;
+  kp.nmma = v.BN;
+  kp.kmma = v.BK;
+  if (is_umma(cfg.kind)) umma_trim(cfg, v, &kp.nmma, &kp.kmma);
+  kp.ct0 = ct0;
   kp.Nt = (int)cfg.Nt;
   kp.c_rank = (int)c.t[0].idx.size();
 }
@@ -221,6 +227,8 @@ tc_status_t finish_plan(tc_plan_s *P, tc_plan_t *out) {
   std::string err;
   ForcedTiles ft;
   if (!parse_force(P->opts.force_tiles, ft)) { delete P; return fail(ST_INVALID_ARG, "malformed force_tiles"); }
+  if (P->opts.morder < 0 || P->opts.morder > 2) { delete P; return fail(ST_INVALID_ARG, "morder must be 0, 1 or 2"); }
+  ft.morder = P->opts.morder - 1;
   // forced tiles name the original indices: plan without fusion so the names survive
   P->c = P->parsed;
   normalize(P->c, !P->opts.no_fusion && !ft.on);
@@ -586,7 +594,7 @@ tc_status_t tc_plan_info(const tc_plan_t plan, char *json, size_t cap, size_t *n
     o << ",\"Mt\":" << g.Mt << ",\"Nt\":" << g.Nt << ",\"Kt\":" << g.Kt << ",\"nctas\":" << g.nctas
       << ",\"mtiles\":" << g.mtiles << ",\"ntiles\":" << g.ntiles << ",\"nsteps\":" << g.nsteps
       << ",\"grid\":" << std::min<int64_t>(g.nctas, plan->sms);
-    o << ",\"vecX\":" << g.vecX << ",\"vecY\":" << g.vecY << ",\"vecC\":" << plan->cvec << ",\"xKmajor\":" << g.xKmajor
+    o << ",\"vecX\":" << g.vecX << ",\"vecY\":" << g.vecY << ",\"vecC\":" << plan->cvec << ",\"cs0\":" << plan->kp.cs0 << ",\"xKmajor\":" << g.xKmajor
       << ",\"yKmajor\":" << g.yKmajor << ",\"wfX\":" << g.wfX << ",\"wfY\":" << g.wfY;
     char buf[512];
     std::snprintf(buf, sizeof buf,

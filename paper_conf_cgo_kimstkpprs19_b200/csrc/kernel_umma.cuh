@@ -168,9 +168,12 @@ __device__ __forceinline__ void tc05_ld(uint32_t taddr, uint32_t (&v)[W]) {
 // UMMA shared-memory descriptor, 128-B swizzle (SM100 layout: start>>4 [0,14), LBO>>4
 // [16,30), SBO>>4 [32,46), version 1 [46,48), base offset 0 [49,52), layout type
 // SWIZZLE_128B = 2 [61,64)).
+// MN-major FP32 (TF32) operands use SWIZZLE_128B_BASE32B = 1 instead: 4-row x 128-B atoms
+// whose 32-B granules are XORed with the row (CUTLASS Layout_MN_SW128_32B_Atom).
+template <int LAYOUT = 2>
 __device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
   return (uint64_t)((saddr >> 4) & 0x3FFF) | ((uint64_t)((lbo >> 4) & 0x3FFF) << 16) |
-         ((uint64_t)((sbo >> 4) & 0x3FFF) << 32) | (1ull << 46) | (2ull << 61);
+         ((uint64_t)((sbo >> 4) & 0x3FFF) << 32) | (1ull << 46) | ((uint64_t)LAYOUT << 61);
 }
 
 // KIND (tiles.hpp): 1 = BF16 (kind::f16), 2 = TF32 on FP32 storage (kind::tf32),
@@ -192,7 +195,7 @@ struct UmmaKernel {
   static constexpr int TMEM_COLS = NBUF * BN;
   static constexpr size_t smem_bytes() {
     return 1024 + (size_t)ES * PLANES * STAGES * (XS + YS) + 8 * (3 * STAGES + 2 * NBUF) + 16 +
-           8 * (size_t)(BM + BN) + 4 * (size_t)EW * 32 * 32;   // + per-epilogue-warp FP32 staging (32 x 32)
+           8 * (size_t)(BM + BN) + 16 + 4 * (size_t)EW * 32 * 32;   // + per-epilogue-warp FP32 staging (32 x 32)
   }
   // register-cached slots per producer thread (16-B vectors)
   static constexpr int EX = BM * BK * ES / 16 / (PW * 32), EY = BN * BK * ES / 16 / (PW * 32);
@@ -213,6 +216,38 @@ __device__ __forceinline__ void st_out(float *d, float v) { *d = v; }
 __device__ __forceinline__ float ld_out(const __nv_bfloat16 *d) { return __bfloat162float(*d); }
 __device__ __forceinline__ float ld_out(const float *d) { return *d; }
 
+// 8 consecutive C elements (16-B aligned): C = x + beta * C (x already scaled by alpha)
+__device__ __forceinline__ void store_run8(float *dst, float (&x)[8], float beta) {
+  float4 *d = reinterpret_cast<float4 *>(dst);
+  if (beta != 0.0f) {
+    const float4 o0 = d[0], o1 = d[1];
+    x[0] = fmaf(beta, o0.x, x[0]); x[1] = fmaf(beta, o0.y, x[1]); x[2] = fmaf(beta, o0.z, x[2]);
+    x[3] = fmaf(beta, o0.w, x[3]); x[4] = fmaf(beta, o1.x, x[4]); x[5] = fmaf(beta, o1.y, x[5]);
+    x[6] = fmaf(beta, o1.z, x[6]); x[7] = fmaf(beta, o1.w, x[7]);
+  }
+  d[0] = make_float4(x[0], x[1], x[2], x[3]);
+  d[1] = make_float4(x[4], x[5], x[6], x[7]);
+}
+__device__ __forceinline__ void store_run8(__nv_bfloat16 *dst, float (&x)[8], float beta) {
+  uint4 *d = reinterpret_cast<uint4 *>(dst);
+  if (beta != 0.0f) {
+    const uint4 o = *d;
+    const uint32_t ow[4] = {o.x, o.y, o.z, o.w};
+#pragma unroll
+    for (int j = 0; j < 4; j++) {
+      x[2 * j] = fmaf(beta, __uint_as_float(ow[j] << 16), x[2 * j]);
+      x[2 * j + 1] = fmaf(beta, __uint_as_float(ow[j] & 0xFFFF0000u), x[2 * j + 1]);
+    }
+  }
+  uint32_t w[4];
+#pragma unroll
+  for (int j = 0; j < 4; j++) {
+    const __nv_bfloat162 b2 = __floats2bfloat162_rn(x[2 * j], x[2 * j + 1]);
+    w[j] = *reinterpret_cast<const uint32_t *>(&b2);
+  }
+  *d = make_uint4(w[0], w[1], w[2], w[3]);
+}
+
 template <int KIND, int BN, int STAGES, bool XK, bool YK>
 __global__ void __launch_bounds__(UmmaKernel<KIND, BN, STAGES>::THREADS, 1)
 tc_umma_kernel(const __grid_constant__ KParams p) {
@@ -228,11 +263,14 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
   T *sY = sX + STAGES * K::XS;
   constexpr uint32_t LO = (uint32_t)ES * STAGES * (K::XS + K::YS);
   // full, empty, tfull[NBUF], tempty[NBUF], split[STAGES]
-  uint64_t *bars = reinterpret_cast<uint64_t *>(smem_raw + (size_t)LO * K::PLANES);
+  // [EW][32 columns][32 rows] FP32 epilogue staging right after the planes (1 KB aligned),
+  // then the barriers and tables
+  float *stage = reinterpret_cast<float *>(smem_raw + (size_t)LO * K::PLANES);
+  uint64_t *bars = reinterpret_cast<uint64_t *>(stage + K::EW * 32 * 32);
   uint32_t *tmem_holder = reinterpret_cast<uint32_t *>(bars + 3 * STAGES + 2 * K::NBUF);
   int64_t *relCm = reinterpret_cast<int64_t *>(tmem_holder + 4);
   int64_t *relCn = relCm + BM;
-  float *stage = reinterpret_cast<float *>(relCn + BN);   // [EW][32 columns][32 rows]
+
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int ntl = (p.ntotal - (int)blockIdx.x + (int)gridDim.x - 1) / (int)gridDim.x;
@@ -330,18 +368,24 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
     }
   } else if (warp == K::EW + K::PW) {
     // ======================= MMA issuer ===================================================
-    constexpr uint32_t IDESC = umma_idesc(ES == 2 ? 1 : 2, BN, !XK, !YK);
+    // N and the number of K-instructions trimmed to the plan's tile (host: umma_trim): a
+    // 24-column tile issues N = 32 (K-major Y) instead of BN, a 36-deep k step 3 of 4
+    const uint32_t IDESC = umma_idesc(ES == 2 ? 1 : 2, p.nmma, !XK, !YK);
+    const int kmma = p.kmma;
     // canonical no-swizzle layouts (bytes): K-major LBO = 128 (k groups), SBO = 1024 (8-row
     // groups); MN-major SBO = 128 (8-row groups), LBO = rows/8 * 128 (k groups)
     // 128-B swizzled layouts (tiles.hpp smem_off): K-major = 8-row x 128-B atoms stacked
     // along M/N (SBO = 1 KB; K = 16 advances the start by 32 B inside the atom); MN-major =
     // 64-element x 8-k atoms, MN atoms at LBO = 1 KB, 8-k groups at SBO = BMN/64 KB
-    // (E = 128 / ES elements per 128-B row; one MMA consumes K = KI = 32 B of k: 16 BF16 =
-    // two 8-k atom groups, 8 TF32 = one)
+    // (E = 128 / ES elements per 128-B row; one MMA consumes K = KI = 32 B of k.  BF16
+    // MN-major: 8-k x 128-B atoms (1 KB), K = 16 = two k groups.  TF32 MN-major
+    // (SWIZZLE_128B_BASE32B): 4-k x 128-B atoms (512 B), K = 8 = two k groups.)
     constexpr int E = 128 / ES;
-    constexpr uint32_t A_LBO = XK ? 16 : 1024, A_SBO = XK ? 1024 : (BM / E) * 1024;
-    constexpr uint32_t B_LBO = YK ? 16 : 1024, B_SBO = YK ? 1024 : (BN / E) * 1024;
-    constexpr uint32_t A_KSTEP = XK ? 32 : (K::KI / 8) * A_SBO, B_KSTEP = YK ? 32 : (K::KI / 8) * B_SBO;
+    constexpr uint32_t ATOM = ES == 4 ? 512 : 1024, KG = ES == 4 ? 4 : 8;   // MN-major atom bytes, k rows
+    constexpr int XL = XK || ES == 2 ? 2 : 1, YL = YK || ES == 2 ? 2 : 1;   // descriptor layout types
+    constexpr uint32_t A_LBO = XK ? 16 : ATOM, A_SBO = XK ? 1024 : (BM / E) * ATOM;
+    constexpr uint32_t B_LBO = YK ? 16 : ATOM, B_SBO = YK ? 1024 : (BN / E) * ATOM;
+    constexpr uint32_t A_KSTEP = XK ? 32 : (K::KI / KG) * A_SBO, B_KSTEP = YK ? 32 : (K::KI / KG) * B_SBO;
     int step = 0, lt = 0;
     for (int j = 0; j < total; j++) {
       const int s = j % STAGES;
@@ -359,11 +403,12 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
         const uint32_t d = tmem + (uint32_t)(buf * BN);
 #pragma unroll
         for (int kk = 0; kk < BK / K::KI; kk++) {
-          const uint64_t ah = umma_desc(ax + kk * A_KSTEP, A_LBO, A_SBO);
-          const uint64_t bh = umma_desc(by + kk * B_KSTEP, B_LBO, B_SBO);
+          if (kk >= kmma) break;
+          const uint64_t ah = umma_desc<XL>(ax + kk * A_KSTEP, A_LBO, A_SBO);
+          const uint64_t bh = umma_desc<YL>(by + kk * B_KSTEP, B_LBO, B_SBO);
           if (K::SPLIT) {   // small terms first: lo*hi, hi*lo, then hi*hi
-            tc05_mma<true>(d, umma_desc(ax + LO + kk * A_KSTEP, A_LBO, A_SBO), bh, IDESC, (step > 0 || kk > 0) ? 1u : 0u);
-            tc05_mma<true>(d, ah, umma_desc(by + LO + kk * B_KSTEP, B_LBO, B_SBO), IDESC, 1u);
+            tc05_mma<true>(d, umma_desc<XL>(ax + LO + kk * A_KSTEP, A_LBO, A_SBO), bh, IDESC, (step > 0 || kk > 0) ? 1u : 0u);
+            tc05_mma<true>(d, ah, umma_desc<YL>(by + LO + kk * B_KSTEP, B_LBO, B_SBO), IDESC, 1u);
             tc05_mma<true>(d, ah, bh, IDESC, 1u);
           } else if (!(p.dbg & 2)) {
             tc05_mma<ES == 4>(d, ah, bh, IDESC, (step > 0 || kk > 0) ? 1u : 0u);
@@ -433,6 +478,22 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
       ncm1 = p.tileN[nt].mask[1];
     };
     if (ntl > 0) fetch(0);
+    // CTA-wide staged path (cs0 > 1): thread -> (run, first column, column step).  With
+    // nruns | 256 (the host guarantees it for this path) every thread keeps one run: rows
+    // rr + cs0 * i, i < 8, of columns rcol0, rcol0 + rcstep, ...
+    int rr = 0, rcol0 = 0, rcstep = 1;
+    int64_t rroff = 0;
+    const int rs0 = p.cs0;
+    if (p.vecC == 8 && p.cs0 > 1) {
+      const int nruns = p.Mt >> 3, t8 = p.ct0 >> 3;
+      const int etid = warp * 32 + lane;
+      const int run = etid % nruns;
+      const int lo = run % rs0, tq = run / rs0;
+      rr = lo + rs0 * (8 * (tq % t8) + p.ct0 * (tq / t8));
+      rcol0 = etid / nruns;
+      rcstep = K::EW * 32 / nruns;
+      rroff = relCm[rr];
+    }
     for (int lt = 0; lt < ntl; lt++) {
       const int buf = lt % K::NBUF;
       const int64_t coff = ncoff;
@@ -446,6 +507,35 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
       if (p.dbg & 256) mbar_wait(TFULL + 8 * buf, (lt / K::NBUF) & 1);
       else mbar_wait_sleep(TFULL + 8 * buf, (lt / K::NBUF) & 1);
       tc05_fence_after();
+      if (p.vecC == 8 && p.cs0 > 1) {
+        // CTA-wide staged epilogue: C's FVI is an inner m digit (tile-row stride cs0), so the
+        // 8 C-contiguous elements of a run live in rows r, r + cs0, ..., r + 7 cs0 of
+        // different warps.  Per 64-column pass all eight warps park their TMEM rows in smem
+        // ([column][row] FP32), then each thread stores whole runs: 16-B (BF16) / 2 x 16-B
+        // (FP32) stores along C's FVI, whatever the m digit order (the X loads keep theirs).
+        const bool rrok = ((rr < 64 ? rm0 : rm1) >> (rr & 63)) & 1;
+        T *Cr = C + (coff + rroff);
+        for (int pc = 0; pc < BN && pc < p.Nt; pc += 64) {
+          uint32_t v[32];
+          tc05_ld<32>(tmem + ((uint32_t)(quarter * 32) << 16) + (uint32_t)(buf * BN + pc + half * 32), v);
+#pragma unroll
+          for (int q = 0; q < 32; q++) stage[(half * 32 + q) * 128 + row] = __uint_as_float(v[q]);
+          asm volatile("bar.sync 1, %0;\n" ::"r"(K::EW * 32) : "memory");
+          // this thread's run (fixed for the kernel when nruns divides the 256 threads)
+          const int ncols = min(64, p.Nt - pc);
+          if (rrok) {
+            for (int col = rcol0; col < ncols; col += rcstep) {
+              const int c = pc + col;
+              if (!(((c < 64 ? cm0 : cm1) >> (c & 63)) & 1)) continue;
+              float x[8];
+#pragma unroll
+              for (int i = 0; i < 8; i++) x[i] = alpha * stage[col * 128 + rr + rs0 * i];
+              store_run8(Cr + relCn[c], x, beta);
+            }
+          }
+          asm volatile("bar.sync 1, %0;\n" ::"r"(K::EW * 32) : "memory");
+        }
+      } else
 #pragma unroll
       for (int c0 = 0; c0 < HC; c0 += 32 > HC ? HC : 32) {
         constexpr int W = 32 > HC ? HC : 32;

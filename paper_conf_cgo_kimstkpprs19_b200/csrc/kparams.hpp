@@ -80,6 +80,9 @@ struct KParams {
   int dbg;                  // TEMPORARY experiment knob
   int vecC;                 // C vector (elements): BF16 8 / FP64 STG 2 => tile rows come in aligned
                             // C-contiguous runs of vecC (16-B stores); 1 => per-element stores
+  int nmma, kmma;           // UMMA: instruction N (<= BN) and K-instructions per stage (<= BK / KI)
+  int cs0, ct0;             // UMMA: tile-row stride and tile of C's FVI among the m digits
+                            // (cs0 == 1: C's FVI leads m; the runs are consecutive rows)
 };
 
 }  // namespace tc

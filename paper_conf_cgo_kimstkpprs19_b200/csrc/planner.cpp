@@ -72,7 +72,12 @@ double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *
   finish_counts(c, cfg);
   const double nctas = (double)cfg.nctas, steps = (double)cfg.nsteps;
   // per CTA-step pipe cycles on one SM: FP64 (DMMA) and shared memory
-  const double dmma = (double)v.BM * v.BN * v.BK / fma_per_clk(v.kind);
+  double dmma = (double)v.BM * v.BN * v.BK / fma_per_clk(v.kind);
+  if (is_umma(v.kind)) {   // the kernel trims N and the K instructions to the tile
+    int nm, km;
+    umma_trim(cfg, v, &nm, &km);
+    dmma = (double)v.BM * nm * km * (32 / v.esize()) / fma_per_clk(v.kind);
+  }
   const bool umma = is_umma(v.kind);
   const int maxv = 16 / kind_esize(cfg.kind);   // 16 B per cp.async
   cfg.vecX = vec_width(c, cfg, cfg.X, maxv);
@@ -131,6 +136,11 @@ double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *
   if (c.t[0].idx.empty()) eS = 1;
   else if (!cfg.mdig.empty() && cfg.mdig[0] == c.t[0].idx[0])
     eS = sector_eff(std::min<int64_t>(srun, cfg.T[cfg.mdig[0]]), es);
+  else if (umma) {
+    // staged epilogue: C's FVI anywhere in m, runs of 8 C-contiguous elements per store
+    int s0, t0;
+    if (c_run_rows(c, cfg, 8, &s0, &t0) == 8) eS = sector_eff(std::min<int64_t>(32, t0), es);
+  }
   const double bx = es * c.numel(cfg.X), by = es * c.numel(cfg.Y), bc = es * c.numel(0);
   double rx = 1, ry = 1;
   if (bx + by > 0.5 * kL2Bytes) {
@@ -300,6 +310,10 @@ std::string tiling_str(const Contraction &c, const Tiling &t) {
 bool better(const Config &a, const Config &b) {
   // deterministic: cost, then more CTAs, then larger tile, then variant / order ids
   if (a.t_pred != b.t_pred) return a.t_pred < b.t_pred;
+  // the same bounding term: the one with less pressure on the others (e.g. an L2-bound tie
+  // between a scalar and a vectorised load order goes to the vectorised one)
+  const double sa = a.t_comp + a.t_mem + a.t_l2, sb = b.t_comp + b.t_mem + b.t_l2;
+  if (sa != sb) return sa < sb;
   if (a.nctas != b.nctas) return a.nctas > b.nctas;
   if (a.Mt * a.Nt != b.Mt * b.Nt) return a.Mt * a.Nt > b.Mt * b.Nt;
   if (a.variant != b.variant) return a.variant < b.variant;
@@ -313,9 +327,10 @@ bool fits(const Config &cfg, const Variant &v) {
 }
 
 // The distinct (morder, korder) digit-order options of a contraction.
-std::vector<Config> order_options(const Contraction &c, int kind) {
+std::vector<Config> order_options(const Contraction &c, int kind, int only_morder = -1) {
   std::vector<Config> out;
   for (int mo = 0; mo < 2; mo++)
+    if (only_morder < 0 || mo == only_morder)
     for (int ko = 0; ko < 2; ko++) {
       Config cfg;
       cfg.morder = mo;
@@ -332,7 +347,8 @@ std::vector<Config> order_options(const Contraction &c, int kind) {
 }  // namespace
 
 // ---------------------------------------------------------------- B200 mode
-static Status choose_b200(const Contraction &c, int kind, int forced_variant, Config &best, PlanStats &st) {
+static Status choose_b200(const Contraction &c, int kind, int forced_variant, int only_morder, Config &best,
+                          PlanStats &st) {
   WfCache cache;
   Config base;
   base.kind = kind;
@@ -347,7 +363,7 @@ static Status choose_b200(const Contraction &c, int kind, int forced_variant, Co
   int kfirst = -1;
   if (!c.t[base.X].idx.empty() && c.ix[c.t[base.X].idx[0]].cls == INTL) kfirst = c.t[base.X].idx[0];
   else if (!c.t[base.Y].idx.empty() && c.ix[c.t[base.Y].idx[0]].cls == INTL) kfirst = c.t[base.Y].idx[0];
-  const auto orders = order_options(c, kind);
+  const auto orders = order_options(c, kind, only_morder);
   bool found = false;
   for (int vi = 0; vi < (int)variants().size(); vi++) {
     if (forced_variant >= 0 && vi != forced_variant) continue;
@@ -557,7 +573,7 @@ static Status choose_forced(const Contraction &c, int kind, const ForcedTiles &f
                             Config &best, std::string &err) {
   WfCache cache;
   bool found = false;
-  for (const auto &o : order_options(c, kind)) {
+  for (const auto &o : order_options(c, kind, ft.morder)) {
     Config cfg = o;
     cfg.T.assign(c.ix.size(), 1);
     for (size_t id = 0; id < c.ix.size(); id++) {
@@ -588,12 +604,12 @@ Status choose(const Contraction &c, int kind, int cost_mode, int forced_variant,
   Status s;
   if (ft.on) s = choose_forced(c, kind, ft, forced_variant, out, err);
   else if (cost_mode == 1) s = choose_paper(c, kind, forced_variant, out, stats);
-  else s = choose_b200(c, kind, forced_variant, out, stats);
+  else s = choose_b200(c, kind, forced_variant, ft.morder, out, stats);
   if (s == ST_NO_CONFIG && !ft.on && cost_mode == 1) {
     // the paper's value sets can leave nothing after pruning (tiny problems): fall back to
     // the B200 enumeration so that every legal contraction gets a plan (R13)
     PlanStats st2;
-    s = choose_b200(c, kind, forced_variant, out, st2);
+    s = choose_b200(c, kind, forced_variant, ft.morder, out, st2);
     stats.ranked += st2.ranked;
   }
   if (s != ST_OK && err.empty()) err = "no legal configuration";

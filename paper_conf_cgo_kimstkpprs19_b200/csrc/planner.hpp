@@ -34,6 +34,7 @@ struct PlanStats {
 struct ForcedTiles {
   bool on = false;
   std::map<std::string, int> tile;  // by index name
+  int morder = -1;                  // >= 0: only this m digit order (tests of both epilogues)
 };
 
 // Choose a configuration.  forced_variant < 0: planner's choice.

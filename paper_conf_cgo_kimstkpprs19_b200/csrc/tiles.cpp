@@ -93,6 +93,33 @@ int c_vec_width(const Contraction &c, const Config &cfg, int maxv) {
   return 1;
 }
 
+int c_run_rows(const Contraction &c, const Config &cfg, int w, int *s0, int *t0) {
+  const auto &v = c.t[0];
+  *s0 = 1;
+  *t0 = 1;
+  if (v.idx.empty() || v.stride[0] != 1) return 1;
+  const int f = v.idx[0];
+  int stride = 1;
+  bool found = false;
+  for (int id : cfg.mdig) {
+    if (id == f) { found = true; break; }
+    stride *= cfg.T[id];
+  }
+  if (!found) return 1;
+  bool ok = cfg.T[f] % w == 0 && c.ix[f].n % w == 0 && v.base % w == 0;
+  for (size_t p = 1; p < v.stride.size(); p++) ok &= v.stride[p] % w == 0;
+  // the CTA-wide staged path gives every one of its 256 threads one run: Mt / w runs must
+  // divide 256
+  if (stride > 1) {
+    const int64_t nr = cfg.Mt / w;
+    ok &= cfg.Mt % w == 0 && nr > 0 && nr <= 256 && (nr & (nr - 1)) == 0;
+  }
+  if (!ok) return 1;
+  *s0 = stride;
+  *t0 = cfg.T[f];
+  return w;
+}
+
 bool vec_possible(const Contraction &c, const Config &cfg, int t) { return vec_width(c, cfg, t, 2) == 2; }
 
 SlotTable build_slots(const Contraction &c, const Config &cfg, int t, int vec, bool kmajor,

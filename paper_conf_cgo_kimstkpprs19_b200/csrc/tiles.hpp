@@ -38,7 +38,8 @@ const std::vector<Variant> &variants();
 //  chunk index inside a 128-B row is XORed with the row's index inside its 8-row atom.  With
 //  E = 128 / esize elements per 128-B row (BF16 64, TF32 32):
 //  K-major (BK = E = one 128-B row): row mn at (mn/8) KB + (mn%8) 128 B, k along the row.
-//  MN-major: atom (mn/E, k/8) at ((k/8) (BMN/E) + mn/E) KB, row k%8, mn%E along the row.
+//  MN-major: atom (mn/E, k/8) at ((k/8) (BMN/E) + mn/E) KB, row k%8, mn%E along the row;
+//  4-byte elements use 4-row atoms with 32-B granules instead (see below).
 inline int smem_off(int kind, bool kmajor, int mn, int k, int BMN, int BK) {
   if (is_umma(kind)) {
     const int es = kind_esize(kind), E = 128 / es;
@@ -46,6 +47,11 @@ inline int smem_off(int kind, bool kmajor, int mn, int k, int BMN, int BK) {
     if (kmajor) {
       const int r = mn % 8, kb = k * es;
       byte = (mn / 8) * 1024 + r * 128 + (((kb >> 4) ^ r) << 4) + (kb & 15);
+    } else if (es == 4) {
+      // FP32 / TF32 MN-major (SWIZZLE_128B_BASE32B): 4-k x 128-B atoms of 512 B, atom
+      // (mn/32, k/4) at ((k/4) (BMN/32) + mn/32) 512 B, row k%4, the 32-B granule XORed with it
+      const int r = k % 4, eb = (mn % E) * es;
+      byte = ((k / 4) * (BMN / E) + mn / E) * 512 + r * 128 + (((eb >> 5) ^ r) << 5) + (eb & 31);
     } else {
       const int r = k % 8, eb = (mn % E) * es;
       byte = ((k / 8) * (BMN / E) + mn / E) * 1024 + r * 128 + (((eb >> 4) ^ r) << 4) + (eb & 15);
@@ -87,6 +93,22 @@ int vec_width(const Contraction &c, const Config &cfg, int t, int maxv);
 // w-aligned C elements: C's FVI is the first m digit, its tile, its extent, C's base and
 // every other C stride are multiples of w.
 int c_vec_width(const Contraction &c, const Config &cfg, int maxv);
+// UMMA instruction trimming for a plan: N = Nt rounded up to 16 (K-major Y) or to a whole
+// 128-B swizzle atom (MN-major Y: 64 BF16 / 32 FP32 columns), capped at BN; K instructions
+// per stage = ceil(Kt / KI), KI = 32 B of k (16 BF16 / 8 TF32).
+inline void umma_trim(const Config &cfg, const Variant &v, int *nmma, int *kmma) {
+  const int es = kind_esize(v.kind), ki = 32 / es, nq = cfg.yKmajor ? 16 : 128 / es;
+  const int n = (int)((cfg.Nt + nq - 1) / nq * nq);
+  *nmma = n < v.BN ? n : v.BN;
+  const int k = (int)((cfg.Kt + ki - 1) / ki);
+  *kmma = k < v.BK / ki ? k : v.BK / ki;
+}
+
+// UMMA staged epilogue (kernel_umma.cuh): C's FVI f may sit anywhere among the m digits.
+// Returns w (or 1) such that every w consecutive values of f's tile digit (w-aligned) are w
+// consecutive, w-aligned C elements; *s0 = tile-row stride of f (product of the tiles of
+// the m digits before it), *t0 = f's tile.  Rows r = lo + s0 (w j + t0 hi) start the runs.
+int c_run_rows(const Contraction &c, const Config &cfg, int w, int *s0, int *t0);
 
 struct SlotTable {
   std::vector<int64_t> rel;    // element offset inside (tile, step)

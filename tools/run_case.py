@@ -15,7 +15,7 @@ cost = sys.argv[3] if len(sys.argv) > 3 else "b200"
 variant = int(sys.argv[4]) if len(sys.argv) > 4 else None
 case = [c for c in tcinputs.tccg48() if c.id == cid][0] if cid > 0 else tcinputs.eq1()
 dtype = os.environ.get("TC_DTYPE", "f64")
-tdt = torch.bfloat16 if dtype == "bf16" else torch.float64
+tdt = {"bf16": torch.bfloat16, "f32": torch.float32, "tf32": torch.float32}.get(dtype, torch.float64)
 p = tc.plan(case.expr, case.extents, cost=cost, variant=variant, dtype=dtype)
 A = tcinputs.uniform(p.numel("A"), 1000 + cid, device="cuda").to(tdt)
 B = tcinputs.uniform(p.numel("B"), 2000 + cid, device="cuda").to(tdt)
