@@ -15,7 +15,7 @@ import json
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-_SO = os.path.join(_HERE, "libtc.so")
+_SO = os.environ.get("LIBTC_SO") or os.path.join(_HERE, "libtc.so")   # (A/B builds)
 
 STATUS = ["TC_SUCCESS", "TC_ERR_INVALID_ARG", "TC_ERR_PARSE", "TC_ERR_INDEX", "TC_ERR_EXTENT",
           "TC_ERR_UNSUPPORTED", "TC_ERR_NO_CONFIG", "TC_ERR_CUDA", "TC_ERR_ALLOC"]

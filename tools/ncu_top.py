@@ -30,10 +30,18 @@ src = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-so
                      capture_output=True, text=True).stdout
 r = list(csv.reader(io.StringIO(src)))
 h = r[1]
-rows = r[2:]
+rows = [x for x in r[2:] if len(x) == len(h) and x[0] != h[0]]
 ia, isrc = h.index("Address"), h.index("Source")
 iss, iex = h.index("Warp Stall Sampling (All Samples)"), h.index("Instructions Executed")
-tot = sum(float(x[iss] or 0) for x in rows)
+def num(v):
+    try:
+        return float(v or 0)
+    except ValueError:
+        return 0.0
+
+
+rows = [x for x in rows if num(x[iss]) or num(x[iex])]
+tot = sum(num(x[iss]) for x in rows)
 print("stall samples", tot)
-for x in sorted(rows, key=lambda x: -float(x[iss] or 0))[:ntop]:
+for x in sorted(rows, key=lambda x: -num(x[iss]))[:ntop]:
     print(f"  {int(x[ia], 16) & 0xffff:#06x} {x[isrc][:70]:70s} {x[iss]:>7s} {x[iex]}")
