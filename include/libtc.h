@@ -117,6 +117,19 @@ tc_status_t tc_execute_host(const tc_plan_t plan, const void *A_host, const void
 tc_status_t tc_plan_tuned(tc_plan_t *tuned, const tc_plan_t plan, const void *A, const void *B,
                           void *C, int topk, int reps, tc_stream_t stream);
 
+/*
+ * Plan cache (the paper's deployment model is "plan once, run many",
+ * P:L77, L300): returns the cached plan of (expr, extents, dtype, opts, current device) —
+ * the strings as given, byte for byte — or plans it with tc_plan_ex and caches it.  The
+ * returned handle is a new reference: release it with tc_plan_destroy (plans are reference
+ * counted; the cache holds one reference until tc_plan_cache_clear).  Thread-safe.  Errors:
+ * as tc_plan_ex (nothing is cached on failure).
+ */
+tc_status_t tc_plan_cached(tc_plan_t *plan, const char *expr, const char *extents, tc_dtype_t dtype,
+                           const tc_plan_opts *opts /* nullable */);
+size_t tc_plan_cache_size(void);   /* plans currently cached                                   */
+void tc_plan_cache_clear(void);    /* drop the cache's references (live handles stay valid)    */
+
 /* Flags of tc_plan_restrict: the operand passed to tc_execute is the compact slab itself. */
 #define TC_SLAB_A 1u
 #define TC_SLAB_B 2u
@@ -138,7 +151,7 @@ tc_status_t tc_plan_info(const tc_plan_t plan, char *json, size_t cap, size_t *n
 
 double tc_plan_flops(const tc_plan_t plan);          /* 2 * prod(all extents) (R5)       */
 int64_t tc_plan_numel(const tc_plan_t plan, int t);  /* elements of 0=C, 1=A, 2=B        */
-void tc_plan_destroy(tc_plan_t plan);                /* NULL-safe                        */
+void tc_plan_destroy(tc_plan_t plan);                /* NULL-safe; releases one reference */
 const char *tc_status_string(tc_status_t status);
 const char *tc_last_error(void);                     /* thread-local detail string       */
 const char *tc_version(void);

@@ -84,6 +84,10 @@ def lib():
         L.tc_status_string.restype = cp
         L.tc_last_error.restype = cp
         L.tc_version.restype = cp
+        L.tc_plan_cached.argtypes = [ctypes.POINTER(vp), cp, cp, ctypes.c_int, ctypes.POINTER(_Opts)]
+        L.tc_plan_cached.restype = ctypes.c_int
+        L.tc_plan_cache_size.restype = ctypes.c_size_t
+        L.tc_plan_cache_clear.restype = None
         L.tc_check.argtypes = [cp, cp]
         L.tc_check.restype = ctypes.c_int
         _lib = L
@@ -193,6 +197,39 @@ class Plan:
                                      ctypes.c_size_t(workspace.numel() * workspace.element_size()),
                                      _stream_ptr(stream)))
         return C
+
+
+def _opts(cost, host_only, variant, force_tiles, fusion, tma, dbg, morder) -> _Opts:
+    o = _Opts()
+    o.morder = {None: 0, "C": 1, "X": 2}[morder]
+    o.reserved[0] = int(dbg)
+    o.tma_epilogue = int(tma)
+    o.cost_mode = COST[cost]
+    o.host_only = int(host_only)
+    o.variant = 0 if variant is None else int(variant) + 1
+    o.force_tiles = force_tiles.encode() if force_tiles else None
+    o.no_fusion = int(not fusion)
+    return o
+
+
+def plan_cached(expr: str, extents: str, dtype: str = "f64", cost: str = "b200", host_only: bool = False,
+                variant: int | None = None, force_tiles: str | None = None, fusion: bool = True,
+                tma: bool = False, dbg: int = 0, morder: str | None = None) -> Plan:
+    """tc_plan_cached: the process-wide cached plan of these arguments (planned on first use)."""
+    o = _opts(cost, host_only, variant, force_tiles, fusion, tma, dbg, morder)
+    h = ctypes.c_void_p()
+    _raise(lib().tc_plan_cached(ctypes.byref(h), expr.encode(), extents.encode(), DTYPES[dtype], ctypes.byref(o)))
+    p = Plan(h, expr, extents, dtype)
+    p._opts = o
+    return p
+
+
+def plan_cache_size() -> int:
+    return int(lib().tc_plan_cache_size())
+
+
+def plan_cache_clear() -> None:
+    lib().tc_plan_cache_clear()
 
 
 def plan(expr: str, extents: str, dtype: str = "f64", cost: str = "b200", host_only: bool = False,

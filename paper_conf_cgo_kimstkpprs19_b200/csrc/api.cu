@@ -5,7 +5,10 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <atomic>
 #include <cmath>
+#include <map>
+#include <mutex>
 #include <cstdio>
 #include <cstring>
 #include <new>
@@ -61,6 +64,7 @@ KernelEntry kernel_for(const Config &cfg) {
 }  // namespace
 
 struct tc_plan_s {
+  std::atomic<int> refs{1};   // tc_plan_destroy releases one; the plan cache holds one
   Contraction parsed;      // as parsed (before normalisation) — restriction starts here
   Contraction c;           // normalised (dropped extent-1 indices, fused runs)
   int dtype = 0;
@@ -366,7 +370,70 @@ tc_status_t tc_plan(tc_plan_t *plan, const char *expr, const char *extents, tc_d
   return tc_plan_ex(plan, expr, extents, dtype, nullptr);
 }
 
-void tc_plan_destroy(tc_plan_t plan) { delete plan; }
+void tc_plan_destroy(tc_plan_t plan) {
+  if (plan && plan->refs.fetch_sub(1) == 1) delete plan;
+}
+
+// ---------------------------------------------------------------- plan cache (NEXT-1)
+namespace {
+std::mutex g_cache_mu;
+std::map<std::string, tc_plan_t> &plan_cache() {
+  static std::map<std::string, tc_plan_t> m;
+  return m;
+}
+std::string cache_key(const char *expr, const char *extents, tc_dtype_t dtype, const tc_plan_opts *o,
+                      int dev) {
+  std::ostringstream k;
+  k << expr << '\x1f' << extents << '\x1f' << (int)dtype << '\x1f' << dev;
+  if (o)
+    k << '\x1f' << o->cost_mode << ',' << o->host_only << ',' << o->variant << ',' << o->no_fusion << ','
+      << o->tma_epilogue << ',' << o->morder << ',' << o->reserved[0] << ','
+      << (o->force_tiles ? o->force_tiles : "");
+  return k.str();
+}
+}  // namespace
+
+tc_status_t tc_plan_cached(tc_plan_t *plan, const char *expr, const char *extents, tc_dtype_t dtype,
+                           const tc_plan_opts *opts) {
+  if (!plan || !expr || !extents) return fail(ST_INVALID_ARG, "NULL argument");
+  *plan = nullptr;
+  try {
+    int dev = -1;
+    if (!(opts && opts->host_only) && cudaGetDevice(&dev) != cudaSuccess) {
+      cudaGetLastError();
+      dev = -1;
+    }
+    const std::string key = cache_key(expr, extents, dtype, opts, dev);
+    std::lock_guard<std::mutex> lock(g_cache_mu);
+    auto &m = plan_cache();
+    auto it = m.find(key);
+    if (it != m.end()) {
+      it->second->refs.fetch_add(1);
+      *plan = it->second;
+      return TC_SUCCESS;
+    }
+    tc_plan_t p = nullptr;
+    tc_status_t st = tc_plan_ex(&p, expr, extents, dtype, opts);
+    if (st != TC_SUCCESS) return st;
+    p->refs.fetch_add(1);   // the cache's reference
+    m[key] = p;
+    *plan = p;
+    return TC_SUCCESS;
+  } catch (...) {
+    return fail(ST_ALLOC, "exception in tc_plan_cached");
+  }
+}
+
+size_t tc_plan_cache_size(void) {
+  std::lock_guard<std::mutex> lock(g_cache_mu);
+  return plan_cache().size();
+}
+
+void tc_plan_cache_clear(void) {
+  std::lock_guard<std::mutex> lock(g_cache_mu);
+  for (auto &kv : plan_cache()) tc_plan_destroy(kv.second);
+  plan_cache().clear();
+}
 
 double tc_plan_flops(const tc_plan_t plan) { return plan ? plan->parsed.flops() : 0.0; }
 

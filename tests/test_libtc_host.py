@@ -148,3 +148,24 @@ def test_errors_are_status_codes():
     with pytest.raises(tc.TcError) as e:
         p.execute_ptr(16, 32, 64)
     assert e.value.status == "TC_ERR_CUDA"          # host_only plans cannot execute
+
+
+def test_plan_cache_reuse_and_refcounts():
+    # NEXT-1: plan once, run many — same arguments => the same plan object
+    tc.plan_cache_clear()
+    e, x = "abcd-aebf-dfce", "a:24;b:16;c:24;d:16;e:16;f:24"
+    p1 = tc.plan_cached(e, x, host_only=True)
+    p2 = tc.plan_cached(e, x, host_only=True)
+    assert p1.handle.value == p2.handle.value and tc.plan_cache_size() == 1
+    p3 = tc.plan_cached(e, x, dtype="bf16", host_only=True)        # another key
+    p4 = tc.plan_cached(e, x, host_only=True, variant=3)
+    assert len({p1.handle.value, p3.handle.value, p4.handle.value}) == 3 and tc.plan_cache_size() == 3
+    assert p1.info() == tc.plan(e, x, host_only=True).info() | {"stats": p1.info()["stats"]}
+    # dropping every Python handle and the cache frees nothing twice; live handles stay valid
+    del p2
+    tc.plan_cache_clear()
+    assert tc.plan_cache_size() == 0 and p1.info()["dtype"] == "f64" and p3.info()["dtype"] == "bf16"
+    # failures are not cached
+    with pytest.raises(tc.TcError):
+        tc.plan_cached("ab-ac-cd", "a:2;b:2;c:2;d:2", host_only=True)
+    assert tc.plan_cache_size() == 0
