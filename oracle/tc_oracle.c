@@ -122,10 +122,12 @@ static int parse_all(Spec *s, const char *expr, const char *extents) {
         if (occurs(s, t, id) > 1) return E_INDEX;
   /* 3. limits: rank <= 8 per tensor, <= 16 distinct indices */
   if (too_many) return E_UNSUP;
-  /* 4. each index in exactly two of the three tensors */
+  /* 4. each index in exactly two of the three tensors, or in all three: a batch
+        (Hadamard) index, SURVEY 8(f) NEXT-3 — C[..h..] = sum A[..h..] B[..h..] for every h,
+        which the loop below already computes (h is decoded from C and read in A and B) */
   for (int id = 0; id < s->nidx; id++) {
     int c = occurs(s, 0, id) + occurs(s, 1, id) + occurs(s, 2, id);
-    if (c != 2) return E_INDEX;
+    if (c != 2 && c != 3) return E_INDEX;
   }
   /* 5. extents syntax: "name:int;name:int" */
   char names[64][MAX_NAME]; long long vals[64]; int nent = 0;

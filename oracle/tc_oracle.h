@@ -9,8 +9,9 @@
  * Definition (Section II, eq. (1) and the sum below it):
  *     C[a,b,c,d] = sum_{e,f} A[a,e,b,f] * B[d,f,c,e]
  * generalised by the Einstein convention: every index that does not appear in
- * C is summed.  Every index appears in exactly two of the three tensors.  The
- * update reading is C = alpha * sum + beta * C (reading R3; beta == 0 => the
+ * C is summed.  Every index appears in exactly two of the three tensors, or in
+ * all three: a batch (Hadamard) index (reading R31), which is
+ * not summed — C[..h..] = sum A[..h..] * B[..h..] for each h.  The update reading is C = alpha * sum + beta * C (reading R3; beta == 0 => the
  * old C is never read).
  * Storage: the FIRST listed index of each tensor is the fastest
  * varying index (stride 1); offset = sum_k i_k * prod_{j<k} N_j.

@@ -127,6 +127,15 @@ void build_host_tables(tc_plan_s *P) {
   kp.kbase = P->tt.kbase;
   kp.nouter = (int)P->tt.kouter.size();
   kp.Mt = (int)cfg.Mt;
+  kp.nbdim = 0;
+  for (size_t id = 0; id < c.ix.size(); id++) {
+    if (c.ix[id].cls != BATCH) continue;
+    const int i = kp.nbdim++;
+    kp.bext[i] = (int)c.ix[id].n;
+    kp.bsX[i] = c.stride_of(cfg.X, (int)id);
+    kp.bsY[i] = c.stride_of(cfg.Y, (int)id);
+    kp.bsC[i] = c.stride_of(0, (int)id);
+  }
   kp.cs0 = cs0;
   kp.nmma = v.BN;
   kp.kmma = v.BK;
@@ -240,6 +249,14 @@ tc_status_t finish_plan(tc_plan_s *P, tc_plan_t *out) {
   if (fv >= (int)variants().size()) { delete P; return fail(ST_INVALID_ARG, "variant out of range"); }
   const int kind = kind_of(P->dtype);
   if (fv >= 0 && variants()[fv].kind != kind) { delete P; return fail(ST_INVALID_ARG, "variant is not built for this dtype"); }
+  {
+    int nb = 0;
+    for (auto &ix : P->c.ix) nb += ix.cls == BATCH;
+    if (nb > kMaxBatch || P->c.nbatch() > 65535) {
+      delete P;
+      return fail(ST_UNSUPPORTED, "more than 4 batch indices or more than 65535 batch values");
+    }
+  }
   Status s = choose(P->c, kind, P->opts.cost_mode, fv, ft, P->cfg, P->stats, err);
   if (s != ST_OK) { delete P; return fail(s, err); }
   build_host_tables(P);
@@ -568,6 +585,7 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
   kp.beta = beta;
   // TMA epilogue when the C view is a legal tensor map and C is only written
   kp.use_tma = plan->tt.tma_ok && plan->opts.tma_epilogue && cfg.kind == KIND_F64_DMMA && beta == 0.0 &&
+               kp.nbdim == 0 &&
                !variants()[cfg.variant].stg &&
                encode_c_map(plan, C, kp.cmap);
   // vector slots need operands aligned to the vector; otherwise the scalar slot tables run
@@ -586,9 +604,11 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
   // stores) / 2 FP64 (STG drain)
   kp.vecC = plan->cvec > 1 && ((uintptr_t)C % 16) == 0 ? plan->cvec : 1;
   const KernelEntry ke = kernel_for(cfg);
-  const int grid = (int)std::min<int64_t>(cfg.nctas, plan->sms);
+  // persistent CTAs: one wave over all batch slabs (grid y = batch values, R31)
+  const int64_t nb = plan->c.nbatch();
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(cfg.nctas, (plan->sms + nb - 1) / nb));
   void *args[] = {&kp};
-  cudaError_t e = cudaLaunchKernel(ke.fn, dim3(grid), dim3(ke.threads), args,
+  cudaError_t e = cudaLaunchKernel(ke.fn, dim3(grid, (unsigned)nb), dim3(ke.threads), args,
                                    kp.use_tma ? ke.smem_tma : ke.smem, (cudaStream_t)stream);
   if (e != cudaSuccess) return fail(ST_CUDA, std::string("launch: ") + cudaGetErrorString(e));
   return TC_SUCCESS;
@@ -642,7 +662,8 @@ tc_status_t tc_plan_info(const tc_plan_t plan, char *json, size_t cap, size_t *n
     o << "{\"dtype\":\"" << dn[g.kind] << "\",\"X\":\"" << (g.X == 1 ? "A" : "B") << "\"";
     o << ",\"indices\":[";
     for (size_t i = 0; i < c.ix.size(); i++) {
-      const char *cls = c.ix[i].cls == EXT_A ? "extA" : c.ix[i].cls == EXT_B ? "extB" : "int";
+      const char *cls = c.ix[i].cls == EXT_A ? "extA" : c.ix[i].cls == EXT_B ? "extB"
+                      : c.ix[i].cls == BATCH ? "batch" : "int";
       o << (i ? "," : "") << "{\"name\":\"" << c.ix[i].name << "\",\"n\":" << c.ix[i].n
         << ",\"cls\":\"" << cls << "\",\"tile\":" << g.T[i] << "}";
     }
@@ -660,7 +681,8 @@ tc_status_t tc_plan_info(const tc_plan_t plan, char *json, size_t cap, size_t *n
       << ",\"threads\":" << v.threads() << ",\"stages\":" << v.stages << ",\"occ\":" << v.occ;
     o << ",\"Mt\":" << g.Mt << ",\"Nt\":" << g.Nt << ",\"Kt\":" << g.Kt << ",\"nctas\":" << g.nctas
       << ",\"mtiles\":" << g.mtiles << ",\"ntiles\":" << g.ntiles << ",\"nsteps\":" << g.nsteps
-      << ",\"grid\":" << std::min<int64_t>(g.nctas, plan->sms);
+      << ",\"grid\":" << std::max<int64_t>(1, std::min<int64_t>(g.nctas, (plan->sms + c.nbatch() - 1) / c.nbatch()))
+      << ",\"nbatch\":" << c.nbatch();
     o << ",\"vecX\":" << g.vecX << ",\"vecY\":" << g.vecY << ",\"vecC\":" << plan->cvec << ",\"cs0\":" << plan->kp.cs0 << ",\"xKmajor\":" << g.xKmajor
       << ",\"yKmajor\":" << g.yKmajor << ",\"wfX\":" << g.wfX << ",\"wfY\":" << g.wfY;
     char buf[512];

@@ -103,10 +103,10 @@ Status parse(const char *expr, const char *extents, Contraction &out, std::strin
     for (size_t i = 0; i < L[t].size(); i++)
       for (size_t j = i + 1; j < L[t].size(); j++)
         if (L[t][i] == L[t][j]) { err = "index '" + L[t][i] + "' repeated in one tensor"; return ST_INDEX; }
-  // each index in exactly two tensors
+  // each index in exactly two tensors, or in all three (a batch index, R31)
   for (auto &nm : order)
-    if (count[nm] != 2) {
-      err = "index '" + nm + "' must occur in exactly two tensors (found " +
+    if (count[nm] != 2 && count[nm] != 3) {
+      err = "index '" + nm + "' must occur in exactly two tensors, or in all three (found " +
             std::to_string(count[nm]) + ")";
       return ST_INDEX;
     }
@@ -179,7 +179,8 @@ Status parse(const char *expr, const char *extents, Contraction &out, std::strin
   }
   for (size_t id = 0; id < out.ix.size(); id++) {
     bool inC = out.pos_in(0, (int)id) >= 0, inA = out.pos_in(1, (int)id) >= 0;
-    out.ix[id].cls = !inC ? INTL : (inA ? EXT_A : EXT_B);
+    const bool inB = out.pos_in(2, (int)id) >= 0;
+    out.ix[id].cls = !inC ? INTL : (inA && inB ? BATCH : inA ? EXT_A : EXT_B);
   }
   return ST_OK;
 }

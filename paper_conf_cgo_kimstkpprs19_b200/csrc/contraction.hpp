@@ -14,7 +14,10 @@ enum Status {
 
 // Reuse class of an index: each index is a reuse direction of the one tensor that
 // does not contain it.
-enum Cls { EXT_A = 0, EXT_B = 1, INTL = 2 };
+// BATCH (R31): an index of C, A and B — a Hadamard index, not
+// summed; the kernels run one slab of C per batch value (grid y).
+enum Cls { EXT_A = 0, EXT_B = 1, INTL = 2, BATCH = 3 };
+inline bool is_ext(int cls) { return cls == EXT_A || cls == EXT_B; }
 
 constexpr int kMaxRank = 8;
 constexpr int kMaxIdx = 16;
@@ -49,6 +52,18 @@ struct Contraction {
   int64_t numel(int t) const {
     int64_t n = 1;
     for (int id : this->t[t].idx) n *= ix[id].n;
+    return n;
+  }
+  // C's first non-batch index (the "C FVI" the tiling maps first), or -1
+  int c_fvi() const {
+    for (int id : this->t[0].idx)
+      if (ix[id].cls != BATCH) return id;
+    return -1;
+  }
+  // product of the batch extents (1 without batch indices)
+  int64_t nbatch() const {
+    int64_t n = 1;
+    for (auto &i : ix) if (i.cls == BATCH) n *= i.n;
     return n;
   }
   double flops() const {

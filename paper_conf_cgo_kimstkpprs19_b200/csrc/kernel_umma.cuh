@@ -311,8 +311,10 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
   if (warp >= K::EW && warp < K::EW + K::PW) {
     // ======================= producers ===================================================
     const int pt = tid - K::EW * 32;
-    const T *__restrict__ X = static_cast<const T *>(p.X);
-    const T *__restrict__ Y = static_cast<const T *>(p.Y);
+    int64_t box_, boy_, boc_;
+    batch_offsets(p, box_, boy_, boc_);
+    const T *__restrict__ X = static_cast<const T *>(p.X) + box_;
+    const T *__restrict__ Y = static_cast<const T *>(p.Y) + boy_;
     // fast path: both operands in 16-B vectors, slots cached in registers
     const bool cached = p.vecX == 16 / ES && p.vecY == 16 / ES && p.nslotX <= K::EX * K::PW * 32 &&
                         p.nslotY <= K::EY * K::PW * 32;
@@ -454,7 +456,9 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
     // ======================= epilogue =====================================================
     // warp w drains TMEM lane quarter w % 4 (tile rows 32(w%4) .. +31; one row per thread)
     // and column half w / 4; FP32 arithmetic on the FP32 accumulator, stored as T (BF16: RNE)
-    T *__restrict__ C = static_cast<T *>(p.C);
+    int64_t box_, boy_, boc_;
+    batch_offsets(p, box_, boy_, boc_);
+    T *__restrict__ C = static_cast<T *>(p.C) + boc_;
     const float alpha = (float)p.alpha, beta = (float)p.beta;
     const int quarter = warp & 3, half = warp >> 2;
     const int row = quarter * 32 + lane;               // TMEM lane = tile row m

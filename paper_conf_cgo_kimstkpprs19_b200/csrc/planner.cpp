@@ -70,7 +70,7 @@ static std::pair<double, double> operand_sim(const Contraction &c, const Config 
 // ---------------------------------------------------------------- B200 cost model
 double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *cache) {
   finish_counts(c, cfg);
-  const double nctas = (double)cfg.nctas, steps = (double)cfg.nsteps;
+  const double nctas = (double)cfg.nctas * (double)c.nbatch(), steps = (double)cfg.nsteps;
   // per CTA-step pipe cycles on one SM: FP64 (DMMA) and shared memory
   double dmma = (double)v.BM * v.BN * v.BK / fma_per_clk(v.kind);
   if (is_umma(v.kind)) {   // the kernel trims N and the K instructions to the tile
@@ -356,10 +356,10 @@ static Status choose_b200(const Contraction &c, int kind, int forced_variant, in
   base.T.assign(c.ix.size(), 1);
   // Alg. 2 walks each input's index list; C's FVI is mapped first on the X side
   std::vector<int> mx, ny, kx;
-  for (int id : c.t[base.X].idx) if (c.ix[id].cls != INTL) mx.push_back(id);
-  for (int id : c.t[base.Y].idx) if (c.ix[id].cls != INTL) ny.push_back(id);
+  for (int id : c.t[base.X].idx) if (is_ext(c.ix[id].cls)) mx.push_back(id);
+  for (int id : c.t[base.Y].idx) if (is_ext(c.ix[id].cls)) ny.push_back(id);
   for (int id : c.t[base.X].idx) if (c.ix[id].cls == INTL) kx.push_back(id);
-  const int c0 = c.t[0].idx.empty() ? -1 : c.t[0].idx[0];
+  const int c0 = c.c_fvi();
   int kfirst = -1;
   if (!c.t[base.X].idx.empty() && c.ix[c.t[base.X].idx[0]].cls == INTL) kfirst = c.t[base.X].idx[0];
   else if (!c.t[base.Y].idx.empty() && c.ix[c.t[base.Y].idx[0]].cls == INTL) kfirst = c.t[base.Y].idx[0];
@@ -418,7 +418,7 @@ static Status choose_b200(const Contraction &c, int kind, int forced_variant, in
             cfg.variant = vi;
             // bound: the FP64-pipe time of the padded work alone (no smem / memory terms)
             if (vfound) {
-              const double tiles = std::ceil((double)cfg.nctas / (kSMs * v.occ));
+              const double tiles = std::ceil((double)cfg.nctas * (double)c.nbatch() / (kSMs * v.occ));
               const double lb = tiles * v.occ * (double)cfg.nsteps * v.BM * v.BN * v.BK /
                                 fma_per_clk(v.kind) / kClk + kLaunch;
               if (lb > vbest.t_pred) { st.pruned++; continue; }
@@ -447,10 +447,10 @@ static Status choose_paper(const Contraction &c, int kind, int forced_variant, C
   digit_orders(c, base);
   base.T.assign(c.ix.size(), 1);
   const int X = base.X, Y = base.Y;
-  const int c0 = c.t[0].idx.empty() ? -1 : c.t[0].idx[0];
+  const int c0 = c.c_fvi();
   std::vector<int> xe, ye, ki;
-  for (int id : c.t[X].idx) if (c.ix[id].cls != INTL) xe.push_back(id);
-  for (int id : c.t[Y].idx) if (c.ix[id].cls != INTL) ye.push_back(id);
+  for (int id : c.t[X].idx) if (is_ext(c.ix[id].cls)) xe.push_back(id);
+  for (int id : c.t[Y].idx) if (is_ext(c.ix[id].cls)) ye.push_back(id);
   for (int id : c.t[X].idx) if (c.ix[id].cls == INTL) ki.push_back(id);
   const int64_t TBS[3] = {4, 8, 16}, REGS[4] = {2, 4, 6, 8};
 
@@ -500,7 +500,7 @@ static Status choose_paper(const Contraction &c, int kind, int forced_variant, C
     for (auto &u : uniq) out.push_back({u.first, u.second});
     return out;
   };
-  const int yfvi = (!c.t[Y].idx.empty() && c.ix[c.t[Y].idx[0]].cls != INTL) ? c.t[Y].idx[0] : -1;
+  const int yfvi = (!c.t[Y].idx.empty() && is_ext(c.ix[c.t[Y].idx[0]].cls)) ? c.t[Y].idx[0] : -1;
   auto px = enum_tb_reg(xe, c0, -1);
   auto py = enum_tb_reg(ye, -1, yfvi);
   std::set<Tiling> kset;

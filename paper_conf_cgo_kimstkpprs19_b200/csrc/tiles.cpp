@@ -31,7 +31,11 @@ const std::vector<Variant> &variants() {
 static int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
 void digit_orders(const Contraction &c, Config &cfg) {
-  cfg.X = c.t[0].idx.empty() ? 1 : (c.pos_in(1, c.t[0].idx[0]) >= 0 ? 1 : 2);
+  // X = the input holding C's FVI — the first non-batch index of C
+  int cf = -1;
+  for (int id : c.t[0].idx)
+    if (c.ix[id].cls != BATCH) { cf = id; break; }
+  cfg.X = cf < 0 ? 1 : (c.pos_in(1, cf) >= 0 ? 1 : 2);
   cfg.Y = 3 - cfg.X;
   cfg.mdig.clear();
   cfg.ndig.clear();
@@ -40,12 +44,12 @@ void digit_orders(const Contraction &c, Config &cfg) {
   // m: C order puts C's FVI first (coalesced C rows); X order follows X's memory
   // (coalesced, vectorisable X loads)
   if (cfg.morder == 0) {
-    for (int id : c.t[0].idx) if (c.pos_in(cfg.X, id) >= 0) cfg.mdig.push_back(id);
+    for (int id : c.t[0].idx) if (c.pos_in(cfg.X, id) >= 0 && is_ext(c.ix[id].cls)) cfg.mdig.push_back(id);
   } else {
-    for (int id : xv) if (c.ix[id].cls != INTL) cfg.mdig.push_back(id);
+    for (int id : xv) if (is_ext(c.ix[id].cls)) cfg.mdig.push_back(id);
   }
   // n: Y's memory order (C's FVI is never on the n side)
-  for (int id : yv) if (c.ix[id].cls != INTL) cfg.ndig.push_back(id);
+  for (int id : yv) if (is_ext(c.ix[id].cls)) cfg.ndig.push_back(id);
   // k: X's or Y's order of the internal indices
   for (int id : (cfg.korder == 0 ? xv : yv)) if (c.ix[id].cls == INTL) cfg.kdig.push_back(id);
   // smem layout: k-contiguous iff the operand's FVI is internal

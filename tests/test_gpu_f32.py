@@ -176,3 +176,19 @@ def test_umma_inner_fvi_epilogue(dtype, layout):
         check_f32(expr, ext, dtype, seed=layout, integer=True, morder="X")
         check_f32(expr, ext, dtype, seed=layout, integer=True, alpha=2.0, beta=1.0, morder="X")
         check_f32(expr, ext, dtype, seed=layout, alpha=0.5, beta=-1.25, morder="X")
+
+
+@pytest.mark.parametrize("dtype", ["f32", "tf32", "bf16"])
+@pytest.mark.parametrize("expr,ext", [("hij-hik-hkj", "h:3;i:130;j:64;k:70"),
+                                      ("abcd-aebd-ecd", "a:24;b:6;c:40;d:3;e:50"),
+                                      ("abc-ab-cb", "a:30;b:4;c:50"), ("ab-ab-ab", "a:5;b:7")])
+def test_umma_batch_indices(dtype, expr, ext):
+    if dtype == "bf16":
+        from tests.test_gpu_bf16 import check_bf16
+        check_bf16(expr, ext, seed=1, integer=True)
+        check_bf16(expr, ext, seed=2, integer=True, alpha=2.0, beta=1.0)
+        check_bf16(expr, ext, seed=3)
+    else:
+        check_f32(expr, ext, dtype, seed=1, integer=True)
+        check_f32(expr, ext, dtype, seed=2, integer=True, alpha=2.0, beta=1.0)
+        check_f32(expr, ext, dtype, seed=3)

@@ -220,3 +220,24 @@ def test_measured_tuning_returns_a_correct_plan():
     assert np.array_equal(dC.cpu().numpy(), oracle.contract(expr, ext, A, B))
     with pytest.raises(tc.TcError):
         p.tuned(dA, dB, dC, topk=0)
+
+
+# Batch (Hadamard) indices (R31): grid y walks the batch slabs
+BATCH = [
+    ("hij-hik-hkj", "h:3;i:40;j:50;k:60"),          # batched GEMM, batch index fastest
+    ("ijh-ikh-kjh", "h:7;i:64;j:72;k:32"),          # batch index slowest
+    ("abcd-aebd-ecd", "a:24;b:6;c:40;d:3;e:50"),
+    ("abcd-dbea-ecb", "a:16;b:3;c:24;d:9;e:20"),    # batch in the middle of every tensor
+    ("ab-ab-ab", "a:5;b:7"),                        # pure Hadamard product
+    ("abc-ab-cb", "a:30;b:4;c:50"),                 # batched outer product
+    ("C[h,g,i] = A[g,k,h] * B[k,i,g,h]", "h:2;g:3;i:40;k:50"),
+]
+
+
+@pytest.mark.parametrize("expr,ext", BATCH)
+def test_batch_indices(expr, ext):
+    check_case(expr, ext, seed=7, integer=True)
+    check_case(expr, ext, seed=8)
+    check_case(expr, ext, seed=9, alpha=0.5, beta=-1.5)
+    for v in (2, 13, 19):                           # direct, staged and wide warp tiles
+        check_case(expr, ext, seed=10, integer=True, variant=v)

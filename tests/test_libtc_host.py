@@ -169,3 +169,18 @@ def test_plan_cache_reuse_and_refcounts():
     with pytest.raises(tc.TcError):
         tc.plan_cached("ab-ac-cd", "a:2;b:2;c:2;d:2", host_only=True)
     assert tc.plan_cache_size() == 0
+
+
+def test_batch_index_classification_and_limits():
+    # an index of C, A and B is a batch (Hadamard) index: neither m, n nor k (R31)
+    i = tc.plan("abcd-aebd-ecd", "a:24;b:6;c:40;d:3;e:50", host_only=True).info()
+    cls = {d["name"]: d["cls"] for d in i["indices"]}
+    assert cls == {"a": "extA", "b": "extA", "c": "extB", "d": "batch", "e": "int"}
+    assert "d" not in i["m"] + i["n"] + i["k"] and i["nbatch"] == 3
+    assert tc.plan("ab-ab-ab", "a:5;b:7", host_only=True).info()["nbatch"] == 35
+    with pytest.raises(tc.TcError) as e:                       # > 65535 batch slabs
+        tc.plan("abc-abc-abc", "a:100;b:100;c:10", host_only=True)
+    assert e.value.status == "TC_ERR_UNSUPPORTED"
+    with pytest.raises(tc.TcError) as e:                       # > 4 batch indices
+        tc.plan("abcde-abcde-abcde", "a:2;b:2;c:2;d:2;e:2", host_only=True)
+    assert e.value.status == "TC_ERR_UNSUPPORTED"

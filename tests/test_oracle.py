@@ -282,3 +282,33 @@ def test_f32_path_rounds_once():
     B = np.array([1.0, 1.0], dtype=np.float32)
     r = oracle.contract("a-ac-c", "a:1;c:2", A, B, dtype="f32")
     assert r[0] == np.float32(1.0 + 2 ** -30)
+
+
+# Batch (Hadamard) indices (R31): an index in C, A and B is
+# not summed.  Pinned against torch.einsum and against per-slice TTGT (explicit slicing).
+BATCH_CASES = [
+    ("hij-hik-hkj", {"h": 3, "i": 4, "j": 5, "k": 6}),        # batched GEMM, batch fastest
+    ("ijh-ikh-kjh", {"h": 3, "i": 4, "j": 5, "k": 2}),        # batch slowest
+    ("abcd-aebd-ecd", {"a": 2, "b": 3, "c": 4, "d": 3, "e": 5}),
+    ("ab-ab-ab", {"a": 5, "b": 7}),                            # pure Hadamard product
+    ("abc-ab-cb", {"a": 3, "b": 4, "c": 5}),                   # batched outer product
+    ("C[h,g,i] = A[g,k,h] * B[k,i,g,h]", {"h": 2, "g": 3, "i": 4, "k": 5}),
+]
+
+
+@pytest.mark.parametrize("expr,ext", BATCH_CASES)
+def test_batch_indices_vs_einsum_and_sliced_ttgt(expr, ext):
+    import re
+    if "[" in expr:
+        c, a, b = ("".join(re.findall(r"[a-z]", t)) for t in
+                   re.match(r"C\[(.*)\] = A\[(.*)\] \* B\[(.*)\]", expr).groups())
+    else:
+        c, a, b = tcinputs.split_expr(expr)
+    es = _ext_str(ext, a + b)
+    A = tcinputs.uniform_np(tcinputs.numel(a, ext), 31)
+    B = tcinputs.uniform_np(tcinputs.numel(b, ext), 32)
+    got, S = oracle.contract(expr, es, A, B, with_scale=True)
+    assert np.all(np.abs(got - einsum_ref(c, a, b, ext, A, B)) <= TAU64 * S)
+    Ai, Bi = tcinputs.integers_np(A.size, 33), tcinputs.integers_np(B.size, 34)
+    from tests.ttgt import batched_ttgt
+    assert np.array_equal(oracle.contract(expr, es, Ai, Bi), batched_ttgt(c, a, b, ext, Ai, Bi))

@@ -48,3 +48,24 @@ def einsum_ref(c_idx: str, a_idx: str, b_idx: str, ext: dict, A, B) -> np.ndarra
     bn = torch.as_tensor(_nd(B, b_idx, ext), dtype=torch.float64)
     eq = f"{a_idx[::-1]},{b_idx[::-1]}->{c_idx[::-1]}"
     return torch.einsum(eq, an, bn).reshape(-1).numpy()
+
+
+def batched_ttgt(c_idx: str, a_idx: str, b_idx: str, ext: dict, A, B) -> np.ndarray:
+    """Batch (Hadamard) indices — in C, A and B — by explicit slicing: for every combination
+    of the batch indices, take the A, B slices, contract them with ``ttgt`` and write the C
+    slice (R31: C[..h..] = sum A[..h..] B[..h..] for each h)."""
+    import itertools
+    bat = [x for x in c_idx if x in a_idx and x in b_idx]
+    if not bat:
+        return ttgt(c_idx, a_idx, b_idx, ext, A, B)
+    an, bn = _nd(A, a_idx, ext), _nd(B, b_idx, ext)
+    cn = np.zeros([ext[x] for x in reversed(c_idx)])
+    ra, rb, rc = list(reversed(a_idx)), list(reversed(b_idx)), list(reversed(c_idx))
+    for combo in itertools.product(*[range(ext[x]) for x in bat]):
+        sel = dict(zip(bat, combo))
+        sa = an[tuple(sel.get(x, slice(None)) for x in ra)]
+        sb = bn[tuple(sel.get(x, slice(None)) for x in rb)]
+        c2, a2, b2 = ("".join(x for x in s if x not in bat) for s in (c_idx, a_idx, b_idx))
+        flat = ttgt(c2, a2, b2, ext, np.ascontiguousarray(sa).reshape(-1), np.ascontiguousarray(sb).reshape(-1))
+        cn[tuple(sel.get(x, slice(None)) for x in rc)] = _nd(flat, c2, ext)
+    return cn.reshape(-1)
