@@ -78,6 +78,11 @@ struct tc_plan_s {
   TileTables tt;
   SlotTable slotX1, slotY1, slotX2, slotY2;   // scalar and cfg.vecX / cfg.vecY wide slots
   int cvec = 1;            // c_vec_width of the plan (16-B C stores when > 1)
+  // batch (Hadamard) indices (R31): extent and element strides in X, Y, C.  tc_execute
+  // launches the kernel once per batch slab with the operands offset to it — the kernels
+  // carry no batch code (the FP64 variants run at their 128-register cap).
+  struct BatchDim { int64_t n, sX, sY, sC; };
+  std::vector<BatchDim> batch;
   std::vector<std::pair<int, double>> tuned;   // tc_plan_tuned: (variant, measured ms) per candidate
   KParams kp{};            // device pointers filled in; X/Y/C/alpha/beta/slots set per call
   void *dev = nullptr;     // one device buffer with every table
@@ -127,15 +132,11 @@ void build_host_tables(tc_plan_s *P) {
   kp.kbase = P->tt.kbase;
   kp.nouter = (int)P->tt.kouter.size();
   kp.Mt = (int)cfg.Mt;
-  kp.nbdim = 0;
-  for (size_t id = 0; id < c.ix.size(); id++) {
-    if (c.ix[id].cls != BATCH) continue;
-    const int i = kp.nbdim++;
-    kp.bext[i] = (int)c.ix[id].n;
-    kp.bsX[i] = c.stride_of(cfg.X, (int)id);
-    kp.bsY[i] = c.stride_of(cfg.Y, (int)id);
-    kp.bsC[i] = c.stride_of(0, (int)id);
-  }
+  P->batch.clear();
+  for (size_t id = 0; id < c.ix.size(); id++)
+    if (c.ix[id].cls == BATCH)
+      P->batch.push_back({c.ix[id].n, c.stride_of(cfg.X, (int)id), c.stride_of(cfg.Y, (int)id),
+                          c.stride_of(0, (int)id)});
   kp.cs0 = cs0;
   kp.nmma = v.BN;
   kp.kmma = v.BK;
@@ -252,7 +253,7 @@ tc_status_t finish_plan(tc_plan_s *P, tc_plan_t *out) {
   {
     int nb = 0;
     for (auto &ix : P->c.ix) nb += ix.cls == BATCH;
-    if (nb > kMaxBatch || P->c.nbatch() > 65535) {
+    if (nb > 4 || P->c.nbatch() > 65535) {
       delete P;
       return fail(ST_UNSUPPORTED, "more than 4 batch indices or more than 65535 batch values");
     }
@@ -585,7 +586,7 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
   kp.beta = beta;
   // TMA epilogue when the C view is a legal tensor map and C is only written
   kp.use_tma = plan->tt.tma_ok && plan->opts.tma_epilogue && cfg.kind == KIND_F64_DMMA && beta == 0.0 &&
-               kp.nbdim == 0 &&
+               plan->batch.empty() &&
                !variants()[cfg.variant].stg &&
                encode_c_map(plan, C, kp.cmap);
   // vector slots need operands aligned to the vector; otherwise the scalar slot tables run
@@ -604,13 +605,29 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
   // stores) / 2 FP64 (STG drain)
   kp.vecC = plan->cvec > 1 && ((uintptr_t)C % 16) == 0 ? plan->cvec : 1;
   const KernelEntry ke = kernel_for(cfg);
-  // persistent CTAs: one wave over all batch slabs (grid y = batch values, R31)
-  const int64_t nb = plan->c.nbatch();
-  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(cfg.nctas, (plan->sms + nb - 1) / nb));
+  const int grid = (int)std::min<int64_t>(cfg.nctas, plan->sms);
   void *args[] = {&kp};
-  cudaError_t e = cudaLaunchKernel(ke.fn, dim3(grid, (unsigned)nb), dim3(ke.threads), args,
-                                   kp.use_tma ? ke.smem_tma : ke.smem, (cudaStream_t)stream);
-  if (e != cudaSuccess) return fail(ST_CUDA, std::string("launch: ") + cudaGetErrorString(e));
+  const int64_t nb = plan->c.nbatch();
+  const char *X0 = static_cast<const char *>(kp.X), *Y0 = static_cast<const char *>(kp.Y);
+  char *C0 = static_cast<char *>(kp.C);
+  for (int64_t b = 0; b < nb; b++) {
+    if (!plan->batch.empty()) {   // batch slab b (mixed radix, first batch index fastest)
+      int64_t r = b, ox = 0, oy = 0, oc = 0;
+      for (const auto &d : plan->batch) {
+        const int64_t i = r % d.n;
+        r /= d.n;
+        ox += i * d.sX;
+        oy += i * d.sY;
+        oc += i * d.sC;
+      }
+      kp.X = X0 + es * ox;
+      kp.Y = Y0 + es * oy;
+      kp.C = C0 + es * oc;
+    }
+    cudaError_t e = cudaLaunchKernel(ke.fn, dim3(grid), dim3(ke.threads), args,
+                                     kp.use_tma ? ke.smem_tma : ke.smem, (cudaStream_t)stream);
+    if (e != cudaSuccess) return fail(ST_CUDA, std::string("launch: ") + cudaGetErrorString(e));
+  }
   return TC_SUCCESS;
 }
 
@@ -681,7 +698,7 @@ tc_status_t tc_plan_info(const tc_plan_t plan, char *json, size_t cap, size_t *n
       << ",\"threads\":" << v.threads() << ",\"stages\":" << v.stages << ",\"occ\":" << v.occ;
     o << ",\"Mt\":" << g.Mt << ",\"Nt\":" << g.Nt << ",\"Kt\":" << g.Kt << ",\"nctas\":" << g.nctas
       << ",\"mtiles\":" << g.mtiles << ",\"ntiles\":" << g.ntiles << ",\"nsteps\":" << g.nsteps
-      << ",\"grid\":" << std::max<int64_t>(1, std::min<int64_t>(g.nctas, (plan->sms + c.nbatch() - 1) / c.nbatch()))
+      << ",\"grid\":" << std::min<int64_t>(g.nctas, plan->sms)
       << ",\"nbatch\":" << c.nbatch();
     o << ",\"vecX\":" << g.vecX << ",\"vecY\":" << g.vecY << ",\"vecC\":" << plan->cvec << ",\"cs0\":" << plan->kp.cs0 << ",\"xKmajor\":" << g.xKmajor
       << ",\"yKmajor\":" << g.yKmajor << ",\"wfX\":" << g.wfX << ",\"wfY\":" << g.wfY;

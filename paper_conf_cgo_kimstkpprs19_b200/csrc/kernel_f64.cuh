@@ -158,19 +158,6 @@ struct F64Kernel {
   static_assert(!STG || WM == 32, "deferred epilogue: one lane per warp-tile row");
 };
 
-// Element offsets of this CTA's batch slab (blockIdx.y) in X, Y and C.
-__device__ __forceinline__ void batch_offsets(const KParams &p, int64_t &ox, int64_t &oy, int64_t &oc) {
-  ox = oy = oc = 0;
-  int r = (int)blockIdx.y;
-  for (int i = 0; i < p.nbdim; i++) {
-    const int d = r % p.bext[i];
-    r /= p.bext[i];
-    ox += d * p.bsX[i];
-    oy += d * p.bsY[i];
-    oc += d * p.bsC[i];
-  }
-}
-
 // (mt, nt) of tile t with grouped rasterisation (group_m m-tiles share a band of n-tiles).
 __device__ __forceinline__ void tile_coords(const KParams &p, int t, int &mt, int &nt) {
   const int per_group = p.group_m * p.ntiles;
@@ -394,10 +381,8 @@ tc_f64_dmma_kernel(const __grid_constant__ KParams p) {
   if (warp >= CW) {
     // ======================= producer warps ===============================================
     const int ptid = tid - CW * 32;
-    int64_t box_, boy_, boc_;
-    batch_offsets(p, box_, boy_, boc_);
-    const double *__restrict__ X = static_cast<const double *>(p.X) + box_;
-    const double *__restrict__ Y = static_cast<const double *>(p.Y) + boy_;
+    const double *__restrict__ X = static_cast<const double *>(p.X);
+    const double *__restrict__ Y = static_cast<const double *>(p.Y);
     int32_t rx[K::EX], ry[K::EY];
     uint32_t px[K::EX], py[K::EY];
     load_slots(rx, px, p.relX, p.packX, p.nslotX, ptid, PW * 32, L::XS - 2);
@@ -438,9 +423,7 @@ tc_f64_dmma_kernel(const __grid_constant__ KParams p) {
   }
 
   // ======================= consumer warps =================================================
-  int64_t box_, boy_, boc_;
-  batch_offsets(p, box_, boy_, boc_);
-  double *__restrict__ C = static_cast<double *>(p.C) + boc_;
+  double *__restrict__ C = static_cast<double *>(p.C);
   const int wm = warp % K::WARPS_M, wn = warp / K::WARPS_M;
   const int g = lane >> 2, t = lane & 3;
   // fragment offsets (compile-time layouts): A(m, k) and B(k, n)

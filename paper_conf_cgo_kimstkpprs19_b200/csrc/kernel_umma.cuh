@@ -311,10 +311,8 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
   if (warp >= K::EW && warp < K::EW + K::PW) {
     // ======================= producers ===================================================
     const int pt = tid - K::EW * 32;
-    int64_t box_, boy_, boc_;
-    batch_offsets(p, box_, boy_, boc_);
-    const T *__restrict__ X = static_cast<const T *>(p.X) + box_;
-    const T *__restrict__ Y = static_cast<const T *>(p.Y) + boy_;
+    const T *__restrict__ X = static_cast<const T *>(p.X);
+    const T *__restrict__ Y = static_cast<const T *>(p.Y);
     // fast path: both operands in 16-B vectors, slots cached in registers
     const bool cached = p.vecX == 16 / ES && p.vecY == 16 / ES && p.nslotX <= K::EX * K::PW * 32 &&
                         p.nslotY <= K::EY * K::PW * 32;
@@ -336,7 +334,7 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
     int step = 0, lt = 0;
     for (int j = 0; j < total; j++) {
       const int s = j % STAGES;
-      if (j >= STAGES) mbar_wait(EMPTY + 8 * s, ((j / STAGES) & 1) ^ 1);
+      if (j >= STAGES && !(p.dbg & 16384)) mbar_wait(EMPTY + 8 * s, ((j / STAGES) & 1) ^ 1);
       if (step + 1 == p.nsteps && lt + 1 < ntl) ProdTile::prefetch(p, (int)blockIdx.x + (lt + 1) * (int)gridDim.x);
       const uint64_t km = ks.mask(p);
       const bool fk = km == p.fullK;
@@ -392,9 +390,9 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
     for (int j = 0; j < total; j++) {
       const int s = j % STAGES;
       const int buf = lt % K::NBUF;
-      if (step == 0 && lt >= K::NBUF) mbar_wait(TEMPTY + 8 * buf, ((lt / K::NBUF) & 1) ^ 1);
+      if (step == 0 && lt >= K::NBUF && !(p.dbg & 32768)) mbar_wait(TEMPTY + 8 * buf, ((lt / K::NBUF) & 1) ^ 1);
       if (K::SPLIT) mbar_wait(SPLITB + 8 * s, (j / STAGES) & 1);
-      else mbar_wait(FULL + 8 * s, (j / STAGES) & 1);
+      else if (!(p.dbg & 32768)) mbar_wait(FULL + 8 * s, (j / STAGES) & 1);
       // the stage was written through the generic proxy (cp.async / st.shared); the MMA
       // reads it through the async proxy
       if (!(p.dbg & 16)) asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
@@ -456,9 +454,7 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
     // ======================= epilogue =====================================================
     // warp w drains TMEM lane quarter w % 4 (tile rows 32(w%4) .. +31; one row per thread)
     // and column half w / 4; FP32 arithmetic on the FP32 accumulator, stored as T (BF16: RNE)
-    int64_t box_, boy_, boc_;
-    batch_offsets(p, box_, boy_, boc_);
-    T *__restrict__ C = static_cast<T *>(p.C) + boc_;
+    T *__restrict__ C = static_cast<T *>(p.C);
     const float alpha = (float)p.alpha, beta = (float)p.beta;
     const int quarter = warp & 3, half = warp >> 2;
     const int row = quarter * 32 + lane;               // TMEM lane = tile row m

@@ -39,8 +39,6 @@ struct alignas(64) TmaDesc {
   unsigned char bytes[128];
 };
 
-constexpr int kMaxBatch = 4;   // batch (Hadamard) indices per contraction (grid y)
-
 struct KParams {
   TmaDesc cmap;             // TMA descriptor of C (tile box = the C tile), if use_tma
   int use_tma;              // 1: epilogue stages the C tile in smem and TMA-stores it
@@ -82,11 +80,6 @@ struct KParams {
   int dbg;                  // TEMPORARY experiment knob
   int vecC;                 // C vector (elements): BF16 8 / FP64 STG 2 => tile rows come in aligned
                             // C-contiguous runs of vecC (16-B stores); 1 => per-element stores
-  // batch indices: blockIdx.y in mixed radix over bext (first
-  // fastest) selects one C slab; X, Y and C move by the batch strides
-  int nbdim;
-  int bext[kMaxBatch];
-  int64_t bsX[kMaxBatch], bsY[kMaxBatch], bsC[kMaxBatch];
   int nmma, kmma;           // UMMA: instruction N (<= BN) and K-instructions per stage (<= BK / KI)
   int cs0, ct0;             // UMMA: tile-row stride and tile of C's FVI among the m digits
                             // (cs0 == 1: C's FVI leads m; the runs are consecutive rows)
