@@ -334,7 +334,7 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
     int step = 0, lt = 0;
     for (int j = 0; j < total; j++) {
       const int s = j % STAGES;
-      if (j >= STAGES && !(p.dbg & 16384)) mbar_wait(EMPTY + 8 * s, ((j / STAGES) & 1) ^ 1);
+      if (j >= STAGES) mbar_wait(EMPTY + 8 * s, ((j / STAGES) & 1) ^ 1);
       if (step + 1 == p.nsteps && lt + 1 < ntl) ProdTile::prefetch(p, (int)blockIdx.x + (lt + 1) * (int)gridDim.x);
       const uint64_t km = ks.mask(p);
       const bool fk = km == p.fullK;
@@ -390,9 +390,9 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
     for (int j = 0; j < total; j++) {
       const int s = j % STAGES;
       const int buf = lt % K::NBUF;
-      if (step == 0 && lt >= K::NBUF && !(p.dbg & 32768)) mbar_wait(TEMPTY + 8 * buf, ((lt / K::NBUF) & 1) ^ 1);
+      if (step == 0 && lt >= K::NBUF) mbar_wait(TEMPTY + 8 * buf, ((lt / K::NBUF) & 1) ^ 1);
       if (K::SPLIT) mbar_wait(SPLITB + 8 * s, (j / STAGES) & 1);
-      else if (!(p.dbg & 32768)) mbar_wait(FULL + 8 * s, (j / STAGES) & 1);
+      else mbar_wait(FULL + 8 * s, (j / STAGES) & 1);
       // the stage was written through the generic proxy (cp.async / st.shared); the MMA
       // reads it through the async proxy
       if (!(p.dbg & 16)) asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
