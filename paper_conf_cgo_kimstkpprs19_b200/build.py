@@ -30,7 +30,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if force or _stale():
         from concurrent.futures import ThreadPoolExecutor
         nvcc = os.path.join(os.environ.get("CUDA_HOME", "/usr/local/cuda"), "bin", "nvcc")
-        objdir = os.path.join(HERE, "build")
+        # (a side build, e.g. tools/trace_umma.py's -DTC_TRACE library, keeps its own objects)
+        objdir = os.path.join(HERE, "build") if SO == os.path.join(HERE, "libtc.so") else os.path.dirname(SO)
         os.makedirs(objdir, exist_ok=True)
         cflags = [f for f in NVCC_FLAGS if f != "-shared"]
 

@@ -248,6 +248,22 @@ __device__ __forceinline__ void store_run8(__nv_bfloat16 *dst, float (&x)[8], fl
   *d = make_uint4(w[0], w[1], w[2], w[3]);
 }
 
+// Development trace (dbg & 4096): CTA 0 records clock64() at the hand-off points of the first
+// 1024 stages / tiles into the C buffer (which then holds no result): [0..) producer warp 0
+// after its EMPTY wait, [1024..) after its FULL arrive, [2048..) MMA after its FULL wait,
+// [3072..) MMA after its commits, [4096..) epilogue warp 0 after TFULL, [5120..) after TEMPTY,
+// [6144..) producer warp 0 at the loop top, [7168..) after its tile switch.
+// Compiled in only with -DTC_TRACE (tools/trace_umma.py builds such a libtc on the side).
+#ifdef TC_TRACE
+constexpr bool kTrace = true;
+#else
+constexpr bool kTrace = false;
+#endif
+__device__ __forceinline__ void trace_at(const KParams &p, int slot, int j) {
+  if (kTrace && (p.dbg & 4096) && blockIdx.x == 0 && j < 1024)
+    static_cast<unsigned long long *>(p.C)[slot * 1024 + j] = clock64();
+}
+
 template <int KIND, int BN, int STAGES, bool XK, bool YK>
 __global__ void __launch_bounds__(UmmaKernel<KIND, BN, STAGES>::THREADS, 1)
 tc_umma_kernel(const __grid_constant__ KParams p) {
@@ -334,7 +350,9 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
     int step = 0, lt = 0;
     for (int j = 0; j < total; j++) {
       const int s = j % STAGES;
+      if (pt == 0) trace_at(p, 6, j);
       if (j >= STAGES) mbar_wait(EMPTY + 8 * s, ((j / STAGES) & 1) ^ 1);
+      if (pt == 0) trace_at(p, 0, j);
       if (step + 1 == p.nsteps && lt + 1 < ntl) ProdTile::prefetch(p, (int)blockIdx.x + (lt + 1) * (int)gridDim.x);
       const uint64_t km = ks.mask(p);
       const bool fk = km == p.fullK;
@@ -360,10 +378,12 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
           mbar_arrive_cp_async(FULL + 8 * s);
         }
       }
+      if (pt == 0) trace_at(p, 1, j);
       ks.advance(p);
       if (++step == p.nsteps) {
         step = 0;
         if (++lt < ntl) cur.fetch(p, (int)blockIdx.x + lt * (int)gridDim.x);
+        if (pt == 0) trace_at(p, 7, j);
       }
     }
   } else if (warp == K::EW + K::PW) {
@@ -393,6 +413,7 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
       if (step == 0 && lt >= K::NBUF) mbar_wait(TEMPTY + 8 * buf, ((lt / K::NBUF) & 1) ^ 1);
       if (K::SPLIT) mbar_wait(SPLITB + 8 * s, (j / STAGES) & 1);
       else mbar_wait(FULL + 8 * s, (j / STAGES) & 1);
+      if (lane == 0) trace_at(p, 2, j);
       // the stage was written through the generic proxy (cp.async / st.shared); the MMA
       // reads it through the async proxy
       if (!(p.dbg & 16)) asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
@@ -417,6 +438,7 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
         if (p.dbg & 64) mbar_arrive(EMPTY + 8 * s);
         else tc05_commit(EMPTY + 8 * s);                      // smem stage free once MMAs read it
         if (step + 1 == p.nsteps) tc05_commit(TFULL + 8 * buf);   // accumulator ready
+        trace_at(p, 3, j);
       }
       __syncwarp();
       if (++step == p.nsteps) { step = 0; ++lt; }
@@ -507,7 +529,9 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
       if (p.dbg & 256) mbar_wait(TFULL + 8 * buf, (lt / K::NBUF) & 1);
       else mbar_wait_sleep(TFULL + 8 * buf, (lt / K::NBUF) & 1);
       tc05_fence_after();
-      if (p.vecC == 8 && p.cs0 > 1) {
+      if (kTrace && (p.dbg & 4096)) {
+        if (warp == 0 && lane == 0) trace_at(p, 4, lt);
+      } else if (p.vecC == 8 && p.cs0 > 1) {
         // CTA-wide staged epilogue: C's FVI is an inner m digit (tile-row stride cs0), so the
         // 8 C-contiguous elements of a run live in rows r, r + cs0, ..., r + 7 cs0 of
         // different warps.  Per 64-column pass all eight warps park their TMEM rows in smem
@@ -624,6 +648,7 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
       tc05_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(TEMPTY + 8 * buf);
+      if (warp == 0 && lane == 0) trace_at(p, 5, lt);
     }
   }
   __syncthreads();
