@@ -45,7 +45,7 @@ def parse_args():
     ap.add_argument("--impl", default="libtc", choices=["libtc", "reference"])
     ap.add_argument("--cases", default="")
     ap.add_argument("--cost", default="b200", choices=["b200", "paper"])
-    ap.add_argument("--tune", type=int, default=4,
+    ap.add_argument("--tune", type=int, default=8,
                     help="measured tuning (tc_plan_tuned) over the model's top-k variants; 0 = model only")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")

@@ -93,3 +93,55 @@ def test_ccsdt_max_size_sampled(n, expr):
     assert not bool(torch.isnan(C).any())   # every element was written
     del C
     torch.cuda.empty_cache()
+
+
+@pytest.mark.parametrize("cid", [1, 8, 12, 18, 30, 33, 40])
+def test_tuned_plans_as_bench_times_them(cid):
+    # bench.py times tc_plan_tuned plans (top-8 variants measured); check those, sampled
+    case = [c for c in tcinputs.tccg48() if c.id == cid][0]
+    p = tc.plan(case.expr, case.extents)
+    A = tcinputs.uniform(p.numel("A"), 1000 + case.id, device="cuda")
+    B = tcinputs.uniform(p.numel("B"), 2000 + case.id, device="cuda")
+    C = torch.empty(p.numel("C"), dtype=torch.float64, device="cuda")
+    p = p.tuned(A, B, C, topk=8, reps=1)
+    C.fill_(float("nan"))
+    p.execute(A, B, C)
+    torch.cuda.synchronize()
+    n = C.numel()
+    idx = np.unique(np.concatenate([np.random.default_rng(cid).integers(0, n, 1500), np.arange(64),
+                                    np.arange(n - 64, n)]))
+    got = C[torch.as_tensor(idx, device="cuda")].cpu().numpy()
+    want, S = oracle.sample(case.expr, case.extents, A.cpu().numpy(), B.cpu().numpy(), idx, with_scale=True)
+    assert np.all(np.abs(got - want) <= TAU64 * S), (cid, p.info()["variant"])
+    assert torch.isfinite(C).all()
+
+
+@pytest.mark.parametrize("dtype", ["bf16", "tf32", "f32"])
+@pytest.mark.parametrize("cid", [1, 4, 6, 7])
+def test_membound_suite_full_size_sampled(dtype, cid):
+    # BASELINE config 4 at full size in the bench's launch configuration (tuned plan)
+    case = [c for c in tcinputs.tccg48() if c.id == cid][0]
+    tdt = torch.bfloat16 if dtype == "bf16" else torch.float32
+    p = tc.plan(case.expr, case.extents, dtype=dtype)
+    A = tcinputs.uniform(p.numel("A"), 1000 + cid, device="cuda").to(tdt)
+    B = tcinputs.uniform(p.numel("B"), 2000 + cid, device="cuda").to(tdt)
+    C = torch.empty(p.numel("C"), dtype=tdt, device="cuda")
+    p = p.tuned(A, B, C, topk=8, reps=1)
+    C.fill_(float("nan"))
+    p.execute(A, B, C)
+    torch.cuda.synchronize()
+    n = C.numel()
+    idx = np.unique(np.concatenate([np.random.default_rng(cid).integers(0, n, 2000), np.arange(64),
+                                    np.arange(n - 64, n)]))
+    got = C[torch.as_tensor(idx, device="cuda")].float().cpu().numpy().astype(np.float64)
+    exact, S = oracle.sample(case.expr, case.extents, A.double().cpu().numpy(), B.double().cpu().numpy(),
+                             idx, with_scale=True)
+    K = p.flops / 2 / n
+    if dtype == "f32":
+        tol = 1e-5 * S
+    elif dtype == "tf32":
+        tol = 2.0 ** -9 * S + 2.0 ** -23 * np.abs(exact)
+    else:   # DESIGN R21 / test_gpu_bf16: one BF16 ulp of the result + FP32 accumulation
+        tol = 2.0 ** -8 * np.abs(exact) + K * 2.0 ** -23 * S
+    bad = np.flatnonzero(~(np.abs(got - exact) <= tol))
+    assert bad.size == 0, (cid, dtype, idx[bad[:5]], got[bad[:5]], exact[bad[:5]])
