@@ -289,8 +289,11 @@ def run_libtc(args):
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if world != args.gpus:
         raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    # the sharded path (C slabs + NCCL input broadcast); TC_BENCH_FORCE_DIST=1 takes it at
+    # world size 1 too (a one-GPU check of the multi-GPU code path under torchrun)
+    sharded = world > 1 or os.environ.get("TC_BENCH_FORCE_DIST") == "1"
     torch.cuda.set_device(local)
-    if world > 1:
+    if sharded:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     cases = select_cases(args.cases)
     dev = torch.device("cuda", local)
@@ -309,12 +312,12 @@ def run_libtc(args):
     for c in cases:
         t0 = time.perf_counter()
         p = tc.plan(c.expr, c.extents, cost=args.cost)
-        if world > 1:
+        if sharded:
             sh = tcdist.shard_plan(p, c.expr, c.extents, world, rank)
         t_plan += time.perf_counter() - t0
         A = tcinputs.uniform(p.numel("A"), 1000 + c.id, device=dev)
         B = tcinputs.uniform(p.numel("B"), 2000 + c.id, device=dev)
-        if world == 1:
+        if not sharded:
             C = torch.empty(p.numel("C"), dtype=torch.float64, device=dev)
             if args.tune > 0:
                 t0 = time.perf_counter()
@@ -332,7 +335,7 @@ def run_libtc(args):
     def one(i, record):
         c, p, A, B, C, sh = work[i]
         flush.zero_()
-        if world > 1:
+        if sharded:
             dist.barrier()
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
@@ -354,7 +357,7 @@ def run_libtc(args):
             for i in range(len(work)):
                 one(i, rec)
         torch.cuda.synchronize()
-        if world > 1:
+        if sharded:
             dist.barrier()
         torch.cuda.synchronize()
         clocks.mark_start()
@@ -366,7 +369,7 @@ def run_libtc(args):
             torch.cuda.synchronize()
             for i, (e0, e1) in enumerate(rec):
                 times[i].append(e0.elapsed_time(e1))
-        if world > 1:
+        if sharded:
             dist.barrier()
         torch.cuda.synchronize()
         t_wall = time.perf_counter() - t_wall
@@ -391,7 +394,7 @@ def run_libtc(args):
     for ts in times:
         s = sorted(ts)
         med.append(s[len(s) // 2])
-    if world > 1:
+    if sharded:
         t = torch.tensor(med, dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         med = t.tolist()
@@ -505,13 +508,13 @@ def run_libtc(args):
     if rank == 0:
         line = {"metric": METRIC, "value": round(value, 2), "unit": UNIT, "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_step, 4),
-                "higher_is_better": True, "scaling": "strong" if world > 1 else "weak",
+                "higher_is_better": True, "scaling": "strong" if sharded else "weak",
                 "vs_baseline": None, "dtype": "f64", "data": "synthetic",
                 "config": {"workload": "TCCG-48 suite (SURVEY App. A extents), FP64, alpha=1, beta=0",
                            "cases": len(cases), "cost_model": args.cost,
                            "l2": "flushed before every launch (256 MiB memset, outside events)",
                            "timing": "CUDA events per launch on the launch stream; median of steps",
-                           "parallelism": f"C-slab shard x{world}" if world > 1 else "single GPU"},
+                           "parallelism": f"C-slab shard x{world}" if sharded else "single GPU"},
                 "roofline": roof,
                 "roofline_geomean_frac": round(geomean(fr), 4),
                 "cpu_baseline": cpu, "e2e": e2e,
@@ -526,7 +529,7 @@ def run_libtc(args):
                 "suites": suites,
                 "per_case": per_case}
         print(json.dumps(line), flush=True)
-    if world > 1:
+    if sharded:
         dist.destroy_process_group()
 
 
