@@ -241,3 +241,19 @@ def test_batch_indices(expr, ext):
     check_case(expr, ext, seed=9, alpha=0.5, beta=-1.5)
     for v in (2, 13, 19):                           # direct, staged and wide warp tiles
         check_case(expr, ext, seed=10, integer=True, variant=v)
+
+
+def test_cached_plan_executes_and_is_shared():
+    # NEXT-1: tc_plan_cached returns the same plan for the same arguments; it runs like any plan
+    tc.plan_cache_clear()
+    e, x = "abcd-aebf-dfce", "a:24;b:16;c:24;d:16;e:16;f:24"
+    p1 = tc.plan_cached(e, x)
+    p2 = tc.plan_cached(e, x)
+    assert p1.handle.value == p2.handle.value and tc.plan_cache_size() == 1
+    A = tcinputs.integers_np(p1.numel("A"), 5)
+    B = tcinputs.integers_np(p1.numel("B"), 6)
+    got = run_gpu(p2, A, B)
+    assert np.array_equal(got, oracle.contract(e, x, A, B))
+    del p1
+    tc.plan_cache_clear()
+    assert np.array_equal(run_gpu(p2, A, B), got)   # the caller's reference outlives the cache
