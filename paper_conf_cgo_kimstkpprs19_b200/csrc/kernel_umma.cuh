@@ -189,7 +189,9 @@ struct UmmaKernel {
   static constexpr int EW = 8;                       // epilogue warps
   // producer warps: their cp.async issue is the stage's critical path (tools/trace_umma.py);
   // 8 instead of 4 measured +43 % on BF16 ab-ac-cb and +15 % on the memory-bound BF16 suite
-  // (12 spill in the epilogue); the split kind keeps 4 (its split warps take the registers)
+  // (12 spill in the epilogue)
+  // (17 warps: 5 on one SM sub-partition cap the registers at 96; 16-warp splits with 7 or 3
+  // producers measured worse for FP32)
   static constexpr int PW = SPLIT ? 4 : 8;
   static constexpr int SW = SPLIT ? 4 : 0;           // split warps
   static constexpr int THREADS = (EW + PW + 1 + SW) * 32; // + one MMA warp
@@ -202,7 +204,8 @@ struct UmmaKernel {
            8 * (size_t)(BM + BN) + 16 + 4 * (size_t)EW * 32 * 32;   // + per-epilogue-warp FP32 staging (32 x 32)
   }
   // register-cached slots per producer thread (16-B vectors)
-  static constexpr int EX = BM * BK * ES / 16 / (PW * 32), EY = BN * BK * ES / 16 / (PW * 32);
+  static constexpr int EX = (BM * BK * ES / 16 + PW * 32 - 1) / (PW * 32);
+  static constexpr int EY = (BN * BK * ES / 16 + PW * 32 - 1) / (PW * 32);
   static_assert(BN % 32 == 0 && BN <= 128, "BN");
   static_assert(TMEM_COLS >= 32 && (TMEM_COLS & (TMEM_COLS - 1)) == 0, "TMEM allocation");
   static_assert(smem_bytes() <= 232448, "smem");
@@ -357,7 +360,7 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
       if (pt == 0) trace_at(p, 6, j);
       if (j >= STAGES) mbar_wait(EMPTY + 8 * s, ((j / STAGES) & 1) ^ 1);
       if (pt == 0) trace_at(p, 0, j);
-      if (step + 1 == p.nsteps && lt + 1 < ntl) ProdTile::prefetch(p, (int)blockIdx.x + (lt + 1) * (int)gridDim.x);
+      // (no prefetch.global.L1 of the next tile's records here: measured slower)
       const uint64_t km = ks.mask(p);
       const bool fk = km == p.fullK;
       const bool fm = cur.fm, fn = cur.fn;

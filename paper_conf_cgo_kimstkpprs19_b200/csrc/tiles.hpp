@@ -25,7 +25,7 @@ struct Variant {
   int kind = KIND_F64_DMMA;
   int stg = 0;                                // 1: staged epilogue drained by the producers
   int threads() const {
-    return is_umma(kind) ? 17 * 32 : ((BM / WM) * (BN / WN) + pw) * 32;   // UMMA: 8 + 8 + 1 (+4 split - 4 producers)
+    return is_umma(kind) ? 17 * 32 : ((BM / WM) * (BN / WN) + pw) * 32;   // UMMA: 8 + 8 + 1 (split: 8 + 4 + 1 + 4)
   }
   int cwarps() const { return is_umma(kind) ? 8 : (BM / WM) * (BN / WN); }
   int esize() const { return kind_esize(kind); }
