@@ -54,6 +54,8 @@ def parse_args():
                     help="extra workloads reported inside the same JSON line (BASELINE configs 3/4): "
                          "ccsdt = CCSD(T) 6D sweep N=24..48 FP64, membound = memory-bound TCCG cases in "
                          "FP32 (split TF32) / TF32 / BF16 vs the HBM roofline; '' = none")
+    ap.add_argument("--no-scale6d", action="store_true",
+                    help="skip the config-5 6D contraction (sd_t_d2, N = 40) timed at every world size")
     ap.add_argument("--profile", action="store_true",
                     help="after the timed region, launch every case once inside cudaProfilerStart/Stop "
                          "(for `ncu --profile-from-start off`); writes gpurun_out/profile_cases.json")
@@ -488,6 +490,47 @@ def run_libtc(args):
                "how": "tc_execute_host per case: pinned host A,B -> device, kernel, C -> host, "
                       "stream sync; wall clock, best of 2"}
 
+    # BASELINE config 5 / SURVEY 8(e): the large 6D contraction (sd_t_d2, all extents 40) sharded
+    # on its largest external index — the case the >= 85 % scaling target is stated for.
+    # Reported at every N (max over ranks) with and without the input broadcast.
+    scale6d = None
+    if not args.no_scale6d:
+        c6 = tcinputs.ccsdt(40, "abcdef-gdab-efgc", 140)
+        p6 = tc.plan(c6.expr, c6.extents, cost=args.cost)
+        A6 = tcinputs.uniform(p6.numel("A"), 1140, device=dev)
+        B6 = tcinputs.uniform(p6.numel("B"), 2140, device=dev)
+        sh6 = tcdist.shard_plan(p6, c6.expr, c6.extents, world, rank) if sharded else None
+        run6 = sh6.plan if sh6 is not None else p6
+        C6 = torch.empty(sh6.c_numel if sh6 is not None else p6.numel("C"), dtype=torch.float64, device=dev)
+        tot, comp = [], []
+        for it in range(args.warmup + max(3, min(args.steps, 5))):
+            flush.zero_()
+            if sharded:
+                dist.barrier()
+            ev = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
+            ev[0].record(stream)
+            if sharded:
+                tcdist.broadcast_inputs(A6, B6, src=0)
+            ev[1].record(stream)
+            if run6 is not None:
+                run6.execute(A6, B6, C6)
+            ev[2].record(stream)
+            torch.cuda.synchronize()
+            if it >= args.warmup:
+                tot.append(ev[0].elapsed_time(ev[2]))
+                comp.append(ev[1].elapsed_time(ev[2]))
+        t6 = torch.tensor([sorted(tot)[len(tot) // 2], sorted(comp)[len(comp) // 2]], dtype=torch.float64, device=dev)
+        if sharded:
+            dist.all_reduce(t6, op=dist.ReduceOp.MAX)
+        scale6d = {"expr": c6.expr, "extents": c6.extents, "n_gpus": world,
+                   "ms": round(t6[0].item(), 4), "gflops": round(p6.flops / t6[0].item() / 1e6, 2),
+                   "ms_compute_only": round(t6[1].item(), 4),
+                   "gflops_compute_only": round(p6.flops / t6[1].item() / 1e6, 2),
+                   "how": "C slab on the largest external index per rank, NCCL broadcast of A and B "
+                          "inside the first interval; time = max over ranks (SURVEY 8(e))"}
+        del A6, B6, C6
+        torch.cuda.empty_cache()
+
     suites = {}
     if world == 1 and args.suites:
         for name in args.suites.split(","):
@@ -527,6 +570,7 @@ def run_libtc(args):
                                 "(outside the timed region; P:L346-348)"},
                 "wall_s_timed": round(t_wall, 3),
                 "suites": suites,
+                "scale6d": scale6d,
                 "per_case": per_case}
         print(json.dumps(line), flush=True)
     if sharded:
