@@ -502,6 +502,8 @@ def run_libtc(args):
         sh6 = tcdist.shard_plan(p6, c6.expr, c6.extents, world, rank) if sharded else None
         run6 = sh6.plan if sh6 is not None else p6
         C6 = torch.empty(sh6.c_numel if sh6 is not None else p6.numel("C"), dtype=torch.float64, device=dev)
+        if args.tune > 0 and run6 is not None:   # the same measured top-k as every other case
+            run6 = run6.tuned(A6, B6, C6, topk=args.tune, reps=2)
         tot, comp = [], []
         for it in range(args.warmup + max(3, min(args.steps, 5))):
             flush.zero_()
