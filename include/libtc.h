@@ -93,6 +93,20 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
                        double beta, tc_stream_t stream);
 
 /*
+ * Grouped contractions into one output (first step; the CCSD(T) triples
+ * of P:L27, L330 accumulate the 9 sd_t_d1 and 9 sd_t_d2 contractions into one t3):
+ *   C = alpha * sum_{i<n} (sum_int A_i*B_i under plans[i]) + beta * C
+ * plans[i] may contract differently shaped A_i, B_i, but every plan must give C the same
+ * layout (extents and element strides per position, origin, dtype, device): otherwise
+ * TC_ERR_INVALID_ARG before anything is launched.  A[i], B[i] are DEVICE pointers as for
+ * tc_execute; C is written by plans[0] with beta and accumulated (beta = 1) by the rest, all
+ * on `stream` in order (capturable into a CUDA graph).  Errors: TC_ERR_INVALID_ARG (n < 1,
+ * NULL arrays or entries, layout mismatch), then as tc_execute for each entry.
+ */
+tc_status_t tc_execute_group(const tc_plan_t *plans, const void *const *A, const void *const *B,
+                             int n, void *C, double alpha, double beta, tc_stream_t stream);
+
+/*
  * End-to-end call with HOST buffers (used for bench.py's "e2e" figure): copies A, B (and C
  * when beta != 0) from host memory into the caller-provided device workspace, runs
  * tc_execute, copies C back, and synchronises `stream`.  workspace must hold

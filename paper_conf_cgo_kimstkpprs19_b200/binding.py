@@ -64,6 +64,9 @@ def lib():
         L.tc_plan.restype = ctypes.c_int
         L.tc_execute.argtypes = [vp, vp, vp, vp, dbl, dbl, vp]
         L.tc_execute.restype = ctypes.c_int
+        L.tc_execute_group.argtypes = [ctypes.POINTER(vp), ctypes.POINTER(vp), ctypes.POINTER(vp),
+                                       ctypes.c_int, vp, dbl, dbl, vp]
+        L.tc_execute_group.restype = ctypes.c_int
         L.tc_execute_host.argtypes = [vp, vp, vp, vp, dbl, dbl, vp, ctypes.c_size_t, vp]
         L.tc_execute_host.restype = ctypes.c_int
         L.tc_plan_workspace_bytes.argtypes = [vp]
@@ -222,6 +225,28 @@ def plan_cached(expr: str, extents: str, dtype: str = "f64", cost: str = "b200",
     p = Plan(h, expr, extents, dtype)
     p._opts = o
     return p
+
+
+def execute_group_ptr(plans, A, B, C: int, alpha=1.0, beta=0.0, stream=None):
+    """tc_execute_group on raw device pointers: C = alpha * sum_i plans[i](A[i], B[i]) + beta * C."""
+    n = len(plans)
+    if len(A) != n or len(B) != n:
+        raise TcError(1, "plans, A and B must have the same length")
+    arr = ctypes.c_void_p * max(n, 1)
+    _raise(lib().tc_execute_group(arr(*[p._h for p in plans]), arr(*[ctypes.c_void_p(a) for a in A]),
+                                  arr(*[ctypes.c_void_p(b) for b in B]), int(n), ctypes.c_void_p(C),
+                                  float(alpha), float(beta), _stream_ptr(stream)))
+
+
+def execute_group(plans, A, B, C, alpha=1.0, beta=0.0, stream=None):
+    """Grouped contractions into one C (CCSD(T) triples pattern) on torch
+    CUDA tensors: C = alpha * sum_i plans[i](A[i], B[i]) + beta * C."""
+    for name, t in [("C", C)] + [(f"A[{i}]", a) for i, a in enumerate(A)] + [(f"B[{i}]", b) for i, b in enumerate(B)]:
+        if not t.is_cuda or not t.is_contiguous():
+            raise TcError(1, f"{name} must be a contiguous CUDA tensor")
+    execute_group_ptr(plans, [a.data_ptr() for a in A], [b.data_ptr() for b in B], C.data_ptr(),
+                      alpha, beta, stream)
+    return C
 
 
 def plan_cache_size() -> int:

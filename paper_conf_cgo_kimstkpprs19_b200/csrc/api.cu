@@ -631,6 +631,29 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
   return TC_SUCCESS;
 }
 
+tc_status_t tc_execute_group(const tc_plan_t *plans, const void *const *A, const void *const *B,
+                             int n, void *C, double alpha, double beta, tc_stream_t stream) {
+  if (!plans || !A || !B || !C || n < 1) return fail(ST_INVALID_ARG, "NULL array or n < 1");
+  for (int i = 0; i < n; i++)
+    if (!plans[i] || !A[i] || !B[i]) return fail(ST_INVALID_ARG, "NULL plan or tensor pointer in group");
+  // every member must see the same C: extents and strides per position, origin, dtype, device
+  const Contraction &c0 = plans[0]->parsed;
+  for (int i = 1; i < n; i++) {
+    const Contraction &ci = plans[i]->parsed;
+    bool same = plans[i]->dtype == plans[0]->dtype && plans[i]->device == plans[0]->device &&
+                ci.t[0].idx.size() == c0.t[0].idx.size() && ci.t[0].base == c0.t[0].base &&
+                ci.parent_numel[0] == c0.parent_numel[0];
+    for (size_t k = 0; same && k < c0.t[0].idx.size(); k++)
+      same = ci.ix[ci.t[0].idx[k]].n == c0.ix[c0.t[0].idx[k]].n && ci.t[0].stride[k] == c0.t[0].stride[k];
+    if (!same) return fail(ST_INVALID_ARG, "group member " + std::to_string(i) + " gives C another layout");
+  }
+  for (int i = 0; i < n; i++) {
+    tc_status_t st = tc_execute(plans[i], A[i], B[i], C, alpha, i == 0 ? beta : 1.0, stream);
+    if (st != TC_SUCCESS) return st;
+  }
+  return TC_SUCCESS;
+}
+
 size_t tc_plan_workspace_bytes(const tc_plan_t plan) {
   if (!plan) return 0;
   auto al = [](size_t x) { return (x + 255) & ~(size_t)255; };

@@ -184,3 +184,37 @@ def test_batch_index_classification_and_limits():
     with pytest.raises(tc.TcError) as e:                       # > 4 batch indices
         tc.plan("abcde-abcde-abcde", "a:2;b:2;c:2;d:2;e:2", host_only=True)
     assert e.value.status == "TC_ERR_UNSUPPORTED"
+
+
+def test_execute_group_validation_host():
+    """tc_execute_group checks, before any launch, that every member gives C the same layout
+    (SURVEY 8(f) NEXT-4): the 18 CCSD(T) triples pass validation and reach tc_execute (which
+    refuses host_only plans with TC_ERR_CUDA); a member with another C layout is refused with
+    TC_ERR_INVALID_ARG; so are n < 1 and a dtype mismatch."""
+    ext = "a:6;b:5;c:7;d:6;e:5;f:7;g:9"
+    exprs = [c.expr for c in tcinputs.tccg48() if c.group.startswith("CCSDT")]
+    plans = [tc.plan(e, ext, host_only=True) for e in exprs]
+    big = 1 << 40
+    A = [big + i * (1 << 30) for i in range(len(plans))]
+    B = [2 * big + i * (1 << 30) for i in range(len(plans))]
+    C = 3 * big
+    with pytest.raises(tc.TcError) as e:
+        tc.execute_group_ptr(plans, A, B, C)
+    assert e.value.status == "TC_ERR_CUDA"                                  # reached tc_execute
+    other = tc.plan("abcdef-gdab-efgc", "a:6;b:5;c:7;d:6;e:5;f:8;g:9", host_only=True)
+    for bad in (plans + [other], [other] + plans[:2]):
+        with pytest.raises(tc.TcError) as e:
+            tc.execute_group_ptr(bad, A[:len(bad)] + [big] * (len(bad) - len(A)),
+                                 B[:len(bad)] + [big] * (len(bad) - len(B)), C)
+        assert e.value.status == "TC_ERR_INVALID_ARG"
+    perm = tc.plan("bacdef-gdab-efgc", ext, host_only=True)
+    with pytest.raises(tc.TcError) as e:                           # C positions permuted
+        tc.execute_group_ptr([plans[0], perm], A[:2], B[:2], C)    
+    assert e.value.status == "TC_ERR_INVALID_ARG"
+    f32 = tc.plan(exprs[0], ext, dtype="f32", host_only=True)
+    with pytest.raises(tc.TcError) as e:
+        tc.execute_group_ptr([plans[0], f32], A[:2], B[:2], C)
+    assert e.value.status == "TC_ERR_INVALID_ARG"
+    with pytest.raises(tc.TcError) as e:
+        tc.execute_group_ptr([], [], [], C)
+    assert e.value.status == "TC_ERR_INVALID_ARG"
