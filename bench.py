@@ -50,10 +50,11 @@ def parse_args():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of oracle work")
-    ap.add_argument("--suites", default="ccsdt,membound",
+    ap.add_argument("--suites", default="ccsdt,membound,triples",
                     help="extra workloads reported inside the same JSON line (BASELINE configs 3/4): "
                          "ccsdt = CCSD(T) 6D sweep N=24..48 FP64, membound = memory-bound TCCG cases in "
-                         "FP32 (split TF32) / TF32 / BF16 vs the HBM roofline; '' = none")
+                         "FP32 (split TF32) / TF32 / BF16 vs the HBM roofline, triples = the 18 CCSD(T) "
+                         "contractions into one t3 (tc_execute_group); '' = none")
     ap.add_argument("--no-scale6d", action="store_true",
                     help="skip the config-5 6D contraction (sd_t_d2, N = 40) timed at every world size")
     ap.add_argument("--profile", action="store_true",
@@ -229,6 +230,47 @@ def time_one(p, A, B, C, steps, warmup, flush, stream):
     return ts[len(ts) // 2]
 
 
+def run_triples(args, flush, stream, dev, hbm):
+    """CCSD(T) triples: the 18 sd_t_d1 / sd_t_d2 contractions of TCCG-48
+    (#31-48) accumulated into one t3 by tc_execute_group, FP64, uniform extents N.  The
+    roofline is that of the fused ideal (inputs read once, t3 written once): min(FP64 peak,
+    I * HBM) — the headroom the on-chip fusion (t3 written once, not 18 times) would take."""
+    import torch
+    from paper_conf_cgo_kimstkpprs19_b200 import binding as tc
+    exprs = [c.expr for c in tcinputs.tccg48() if c.group.startswith("CCSDT")]
+    rows = []
+    for n in (16, 24):
+        ext = ";".join(f"{x}:{n}" for x in "abcdefg")
+        plans = [tc.plan(e, ext, cost=args.cost) for e in exprs]
+        A = [tcinputs.uniform(p.numel("A"), 1000 + i, device=dev) for i, p in enumerate(plans)]
+        B = [tcinputs.uniform(p.numel("B"), 2000 + i, device=dev) for i, p in enumerate(plans)]
+        C = torch.empty(plans[0].numel("C"), dtype=torch.float64, device=dev)
+        ts = []
+        for it in range(2 + max(3, min(args.steps, 5))):
+            flush.zero_()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            tc.execute_group(plans, A, B, C)
+            e1.record(stream)
+            e1.synchronize()
+            if it >= 2:
+                ts.append(e0.elapsed_time(e1))
+        ms = sorted(ts)[len(ts) // 2]
+        flops = sum(p.flops for p in plans)
+        byts_fused = 8 * (sum(p.numel("A") + p.numel("B") for p in plans) + C.numel())
+        byts_group = 8 * (sum(p.numel("A") + p.numel("B") for p in plans) + (2 * len(plans) - 1) * C.numel())
+        attain = min(FP64_PEAK_TFLOPS * 1e12, flops / byts_fused * hbm)
+        rows.append({"extents": ext, "contractions": len(plans), "ms": round(ms, 4),
+                     "gflops": round(flops / ms / 1e6, 2),
+                     "roofline_frac_vs_fused": round(flops / (ms * 1e-3) / attain, 4),
+                     "hbm_frac_of_group_bytes": round(byts_group / (ms * 1e-3) / hbm, 4)})
+        del A, B, C, plans
+        torch.cuda.empty_cache()
+    return {"workload": "CCSD(T) triples: TCCG-48 #31-48 into one t3 (tc_execute_group, beta=1 "
+                        "after the first), FP64, all extents N; L2 flushed before each group",
+            "cases": rows}
+
+
 def run_suite(name, args, flush, stream, dev, hbm):
     """One extra workload: per case plan (+ measured top-k tuning like the main suite), time,
     roofline fraction against min(pipe peak, I * HBM) — pipe = FP64 DMMA for f64; the
@@ -236,6 +278,8 @@ def run_suite(name, args, flush, stream, dev, hbm):
     import torch
     from paper_conf_cgo_kimstkpprs19_b200 import binding as tc
     rows = []
+    if name == "triples":
+        return run_triples(args, flush, stream, dev, hbm)
     if name == "ccsdt":
         # BASELINE config 3: sd_t_d1 / sd_t_d2 6D contractions at uniform extents 24..48, FP64
         todo = [(tcinputs.ccsdt(n, e, 100 + n), "f64") for e in ("abcdef-gdab-efgc", "abcdef-dega-gfbc")
