@@ -245,6 +245,10 @@ def run_triples(args, flush, stream, dev, hbm):
         A = [tcinputs.uniform(p.numel("A"), 1000 + i, device=dev) for i, p in enumerate(plans)]
         B = [tcinputs.uniform(p.numel("B"), 2000 + i, device=dev) for i, p in enumerate(plans)]
         C = torch.empty(plans[0].numel("C"), dtype=torch.float64, device=dev)
+        if args.tune > 0:   # member 0 writes t3 (beta = 0); the rest accumulate: tuned at beta = 1
+            C.zero_()
+            plans = [p.tuned(A[i], B[i], C, topk=args.tune, reps=2, beta=0.0 if i == 0 else 1.0)
+                     for i, p in enumerate(plans)]
         ts = []
         for it in range(2 + max(3, min(args.steps, 5))):
             flush.zero_()
@@ -267,7 +271,8 @@ def run_triples(args, flush, stream, dev, hbm):
         del A, B, C, plans
         torch.cuda.empty_cache()
     return {"workload": "CCSD(T) triples: TCCG-48 #31-48 into one t3 (tc_execute_group, beta=1 "
-                        "after the first), FP64, all extents N; L2 flushed before each group",
+                        "after the first), FP64, all extents N; L2 flushed before each group; "
+                        "members tuned top-k at their own beta (tc_plan_tuned_beta)",
             "cases": rows}
 
 

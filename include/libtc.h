@@ -130,6 +130,12 @@ tc_status_t tc_execute_host(const tc_plan_t plan, const void *A_host, const void
  */
 tc_status_t tc_plan_tuned(tc_plan_t *tuned, const tc_plan_t plan, const void *A, const void *B,
                           void *C, int topk, int reps, tc_stream_t stream);
+/* As tc_plan_tuned, but the candidates are timed as C = A*B + beta*C (C's contents change:
+   it is read and accumulated into).  For plans that will run with beta != 0 — the
+   accumulating members of tc_execute_group — whose best variant differs from beta = 0's
+   (reading C at the tile end costs 3-8x, unevenly across variants; R33). */
+tc_status_t tc_plan_tuned_beta(tc_plan_t *tuned, const tc_plan_t plan, const void *A, const void *B,
+                               void *C, int topk, int reps, double beta, tc_stream_t stream);
 
 /*
  * Plan cache (the paper's deployment model is "plan once, run many",

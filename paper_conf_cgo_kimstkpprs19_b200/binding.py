@@ -75,6 +75,8 @@ def lib():
         L.tc_plan_restrict.restype = ctypes.c_int
         L.tc_plan_tuned.argtypes = [ctypes.POINTER(vp), vp, vp, vp, vp, ctypes.c_int, ctypes.c_int, vp]
         L.tc_plan_tuned.restype = ctypes.c_int
+        L.tc_plan_tuned_beta.argtypes = [ctypes.POINTER(vp), vp, vp, vp, vp, ctypes.c_int, ctypes.c_int, dbl, vp]
+        L.tc_plan_tuned_beta.restype = ctypes.c_int
         L.tc_plan_info.argtypes = [vp, ctypes.c_char_p, ctypes.c_size_t, ctypes.POINTER(ctypes.c_size_t)]
         L.tc_plan_info.restype = ctypes.c_int
         L.tc_plan_flops.argtypes = [vp]
@@ -165,16 +167,17 @@ class Plan:
                                       int(length), int(flags)))
         return Plan(h, self.expr, f"{self.extents}|{index}[{begin}:{begin + length}]", self.dtype)
 
-    def tuned(self, A, B, C, topk: int = 4, reps: int = 3, stream=None) -> "Plan":
+    def tuned(self, A, B, C, topk: int = 4, reps: int = 3, stream=None, beta: float = 0.0) -> "Plan":
         """tc_plan_tuned: time the best configs of the top-k variants on these tensors (C is
-        overwritten) and return the fastest as a new plan."""
+        overwritten; with beta != 0, tc_plan_tuned_beta: C is accumulated into) and return
+        the fastest as a new plan."""
         for name, t in (("A", A), ("B", B), ("C", C)):
             if not t.is_cuda or not t.is_contiguous():
                 raise TcError(1, f"{name} must be a contiguous CUDA tensor")
         h = ctypes.c_void_p()
-        _raise(lib().tc_plan_tuned(ctypes.byref(h), self._h, ctypes.c_void_p(A.data_ptr()),
-                                   ctypes.c_void_p(B.data_ptr()), ctypes.c_void_p(C.data_ptr()),
-                                   int(topk), int(reps), _stream_ptr(stream)))
+        _raise(lib().tc_plan_tuned_beta(ctypes.byref(h), self._h, ctypes.c_void_p(A.data_ptr()),
+                                        ctypes.c_void_p(B.data_ptr()), ctypes.c_void_p(C.data_ptr()),
+                                        int(topk), int(reps), float(beta), _stream_ptr(stream)))
         return Plan(h, self.expr, self.extents, self.dtype)
 
     def execute_ptr(self, A: int, B: int, C: int, alpha=1.0, beta=0.0, stream=None):

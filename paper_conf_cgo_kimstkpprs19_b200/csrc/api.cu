@@ -462,6 +462,11 @@ int64_t tc_plan_numel(const tc_plan_t plan, int t) {
 
 tc_status_t tc_plan_tuned(tc_plan_t *tuned, const tc_plan_t plan, const void *A, const void *B, void *C,
                           int topk, int reps, tc_stream_t stream) {
+  return tc_plan_tuned_beta(tuned, plan, A, B, C, topk, reps, 0.0, stream);
+}
+
+tc_status_t tc_plan_tuned_beta(tc_plan_t *tuned, const tc_plan_t plan, const void *A, const void *B, void *C,
+                               int topk, int reps, double beta, tc_stream_t stream) {
   if (!tuned || !plan || !A || !B || !C) return fail(ST_INVALID_ARG, "NULL argument");
   *tuned = nullptr;
   if (plan->host_only || !plan->dev) return fail(ST_CUDA, "plan was made host_only");
@@ -492,11 +497,11 @@ tc_status_t tc_plan_tuned(tc_plan_t *tuned, const tc_plan_t plan, const void *A,
       if (rc != TC_SUCCESS) break;
       cp->stats.per_variant = plan->stats.per_variant;
       // one warm-up, then the minimum over reps single launches (C is overwritten)
-      rc = tc_execute(cp, A, B, C, 1.0, 0.0, stream);
+      rc = tc_execute(cp, A, B, C, 1.0, beta, stream);
       float ms = 1e30f;
       for (int r = 0; r < reps && rc == TC_SUCCESS; r++) {
         cudaEventRecord(e0, (cudaStream_t)stream);
-        rc = tc_execute(cp, A, B, C, 1.0, 0.0, stream);
+        rc = tc_execute(cp, A, B, C, 1.0, beta, stream);
         cudaEventRecord(e1, (cudaStream_t)stream);
         if (cudaEventSynchronize(e1) != cudaSuccess) { rc = fail(ST_CUDA, "tuning launch failed"); break; }
         float t = 0;
@@ -520,7 +525,7 @@ tc_status_t tc_plan_tuned(tc_plan_t *tuned, const tc_plan_t plan, const void *A,
     *tuned = best;
     return TC_SUCCESS;
   } catch (...) {
-    return fail(ST_ALLOC, "exception in tc_plan_tuned");
+    return fail(ST_ALLOC, "exception in tc_plan_tuned_beta");
   }
 }
 

@@ -90,3 +90,22 @@ def test_group_in_cuda_graph():
     torch.cuda.synchronize()
     want, _ = _oracle_sum(exprs, A, B, None, 1.0, 0.0)
     assert np.array_equal(dC.cpu().numpy(), want)
+
+
+def test_group_with_members_tuned_at_beta1():
+    """tc_plan_tuned_beta: accumulating members tuned at beta = 1 still compute the group."""
+    exprs = _triples()
+    plans = [tc.plan(e, EXT) for e in exprs]
+    A, B = _inputs(exprs, tcinputs.integers_np, plans)
+    dA = [torch.as_tensor(np.ascontiguousarray(a), device="cuda") for a in A]
+    dB = [torch.as_tensor(np.ascontiguousarray(b), device="cuda") for b in B]
+    n = plans[0].numel("C")
+    dC = torch.zeros(n, dtype=torch.float64, device="cuda")
+    plans = [p.tuned(dA[i], dB[i], dC, topk=3, reps=1, beta=0.0 if i == 0 else 1.0)
+             for i, p in enumerate(plans)]
+    assert all(len(p.info()["stats"]["tuned"]) >= 1 for p in plans)
+    dC.fill_(float("nan"))
+    tc.execute_group(plans, dA, dB, dC)
+    torch.cuda.synchronize()
+    want, _ = _oracle_sum(exprs, A, B, None, 1.0, 0.0)
+    assert np.array_equal(dC.cpu().numpy(), want)
