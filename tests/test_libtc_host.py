@@ -218,3 +218,15 @@ def test_execute_group_validation_host():
     with pytest.raises(tc.TcError) as e:
         tc.execute_group_ptr([], [], [], C)
     assert e.value.status == "TC_ERR_INVALID_ARG"
+
+
+def test_plan_tuned_beta_errors_host():
+    """tc_plan_tuned_beta validates like tc_plan_tuned: NULL tensors / topk < 1 are
+    TC_ERR_INVALID_ARG, a host_only plan is TC_ERR_CUDA; *tuned stays NULL."""
+    p = tc.plan("abcdef-gdab-efgc", "a:6;b:5;c:7;d:6;e:5;f:7;g:9", host_only=True)
+    L = tc.lib()
+    h = ctypes.c_void_p()
+    x = ctypes.c_void_p(1 << 40)
+    assert L.tc_plan_tuned_beta(ctypes.byref(h), p._h, None, x, x, 2, 1, 1.0, None) == 1
+    assert L.tc_plan_tuned_beta(ctypes.byref(h), p._h, x, x, x, 0, 1, 1.0, None) == 7   # host_only first
+    assert not h.value
