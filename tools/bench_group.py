@@ -18,7 +18,7 @@ def run(ext, reps=20):
     B = [torch.rand(p.numel("B"), dtype=torch.float64, device="cuda") for p in plans]
     C = torch.zeros(plans[0].numel("C"), dtype=torch.float64, device="cuda")
     s = torch.cuda.Stream()
-    flops = sum(tc.lib().tc_plan_flops(p.handle if hasattr(p, "handle") else p._h) for p in plans)
+    flops = sum(p.flops for p in plans)
     out = {"extents": ext, "contractions": len(plans), "gflop": flops / 1e9, "c_bytes": C.numel() * 8}
     with torch.cuda.stream(s):
         for _ in range(3):
