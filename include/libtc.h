@@ -5,7 +5,8 @@
  * The operation (Section II, eq. (1) and the sum below it):
  *     C[a,b,c,d] = sum_{e,f} A[a,e,b,f] * B[d,f,c,e]
  * generalised with the Einstein convention to any expression in which every index
- * occurs in exactly two of the three tensors, and with the update
+ * occurs in exactly two of the three tensors — or in all three: a batch (Hadamard)
+ * index, not summed (reading R31) — and with the update
  *     C = alpha * sum_int A * B + beta * C          (beta == 0: C is never read)
  * (reading R3).  No transposed intermediate is ever created.
  *
@@ -34,8 +35,9 @@ typedef enum {
   TC_SUCCESS = 0,
   TC_ERR_INVALID_ARG = 1, /* NULL pointer/handle, C overlaps A or B, wrong device, bad opts */
   TC_ERR_PARSE = 2,       /* malformed expression or extents string                          */
-  TC_ERR_INDEX = 3,       /* index in one tensor only or in all three, repeated in a tensor,
-                             extent missing / duplicated / naming an unknown index           */
+  TC_ERR_INDEX = 3,       /* index in one tensor only (an index in all three is a legal batch
+                             index, R31), repeated in a tensor, extent missing / duplicated /
+                             naming an unknown index                                         */
   TC_ERR_EXTENT = 4,      /* extent < 1, or an element count overflows int64                 */
   TC_ERR_UNSUPPORTED = 5, /* rank > 8, > 16 distinct indices, extent > 2^31-1, dtype not built */
   TC_ERR_NO_CONFIG = 6,   /* planner found no legal configuration (a bug)                    */
@@ -64,7 +66,7 @@ typedef struct tc_plan_opts {
                         when C is a legal tensor map and beta == 0; 0 (default): direct stores */
   int morder;        /* 0: planner's choice; 1: m digits in C order (C's FVI first); 2: in the X
                         operand's memory order (its FVI first) — tests of both epilogues   */
-  int reserved[6];
+  int reserved[6];   /* must be zero (TC_ERR_INVALID_ARG otherwise)                         */
 } tc_plan_opts;
 
 /*

@@ -23,8 +23,41 @@ import subprocess
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-_SO = os.path.join(_HERE, "libtc_oracle.so")
 _SRC = os.path.join(_HERE, "tc_oracle.c")
+# gcc flags of SURVEY 8(d) / BASELINE.md: the plain loop at -O3 for this host's own ISA;
+# -ffp-contract=off so each term is a plain multiply followed by a plain add
+CFLAGS = ["-O3", "-march=native", "-fopenmp", "-ffp-contract=off", "-fPIC", "-shared"]
+
+
+def cpu_model() -> str:
+    """The host CPU's model name (/proc/cpuinfo), for the bench line."""
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def _host_key() -> str:
+    # -march=native code is only valid on the CPU it was compiled for: one library per host
+    # ISA (the tree travels to the GPU box, where the oracle is rebuilt for that host)
+    import hashlib
+    flags = ""
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("flags"):
+                    flags = line
+                    break
+    except OSError:
+        pass
+    return hashlib.sha1((cpu_model() + flags).encode()).hexdigest()[:12]
+
+
+_SO = os.path.join(_HERE, f"libtc_oracle_{_host_key()}.so")
 
 STATUS = {0: "TC_SUCCESS", 1: "TC_ERR_INVALID_ARG", 2: "TC_ERR_PARSE", 3: "TC_ERR_INDEX",
           4: "TC_ERR_EXTENT", 5: "TC_ERR_UNSUPPORTED"}
@@ -33,10 +66,12 @@ _NP = {"f64": np.float64, "f32": np.float32, "tf32": np.float32, "bf16": np.uint
 
 
 def build(force: bool = False) -> str:
-    """Compile the oracle (plain C, -ffp-contract=off so each term is mul-then-add)."""
+    """Compile the oracle (plain C, -O3 -march=native, -ffp-contract=off so each term is
+    mul-then-add) for this host."""
     if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(_SRC):
-        subprocess.check_call(["gcc", "-O2", "-fopenmp", "-ffp-contract=off", "-fPIC", "-shared",
-                               "-o", _SO, _SRC, "-lm"])
+        tmp = f"{_SO}.{os.getpid()}.tmp"
+        subprocess.check_call(["gcc"] + CFLAGS + ["-o", tmp, _SRC, "-lm"])
+        os.replace(tmp, _SO)
     return _SO
 
 

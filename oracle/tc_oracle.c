@@ -3,7 +3,8 @@
  * See tc_oracle.h for the definition followed (eq. (1),
  * L138/L145/L149) and for who may load this library.  Shares no code with libtc.
  *
- * Build: gcc -O2 -fopenmp -ffp-contract=off -fPIC -shared -o libtc_oracle.so tc_oracle.c -lm
+ * Build: gcc -O3 -march=native -fopenmp -ffp-contract=off -fPIC -shared -o libtc_oracle_<host>.so
+ *        tc_oracle.c -lm   (oracle/__init__.py builds one library per host CPU)
  * (-ffp-contract=off: every term is a plain multiply followed by a plain add.)
  */
 #include "tc_oracle.h"

@@ -205,10 +205,9 @@ class Plan:
         return C
 
 
-def _opts(cost, host_only, variant, force_tiles, fusion, tma, dbg, morder) -> _Opts:
+def _opts(cost, host_only, variant, force_tiles, fusion, tma, morder) -> _Opts:
     o = _Opts()
     o.morder = {None: 0, "C": 1, "X": 2}[morder]
-    o.reserved[0] = int(dbg)
     o.tma_epilogue = int(tma)
     o.cost_mode = COST[cost]
     o.host_only = int(host_only)
@@ -220,9 +219,9 @@ def _opts(cost, host_only, variant, force_tiles, fusion, tma, dbg, morder) -> _O
 
 def plan_cached(expr: str, extents: str, dtype: str = "f64", cost: str = "b200", host_only: bool = False,
                 variant: int | None = None, force_tiles: str | None = None, fusion: bool = True,
-                tma: bool = False, dbg: int = 0, morder: str | None = None) -> Plan:
+                tma: bool = False, morder: str | None = None) -> Plan:
     """tc_plan_cached: the process-wide cached plan of these arguments (planned on first use)."""
-    o = _opts(cost, host_only, variant, force_tiles, fusion, tma, dbg, morder)
+    o = _opts(cost, host_only, variant, force_tiles, fusion, tma, morder)
     h = ctypes.c_void_p()
     _raise(lib().tc_plan_cached(ctypes.byref(h), expr.encode(), extents.encode(), DTYPES[dtype], ctypes.byref(o)))
     p = Plan(h, expr, extents, dtype)
@@ -262,17 +261,9 @@ def plan_cache_clear() -> None:
 
 def plan(expr: str, extents: str, dtype: str = "f64", cost: str = "b200", host_only: bool = False,
          variant: int | None = None, force_tiles: str | None = None, fusion: bool = True,
-         tma: bool = False, dbg: int = 0, morder: str | None = None) -> Plan:
+         tma: bool = False, morder: str | None = None) -> Plan:
     """morder: None = planner's choice, "C" = m digits in C order, "X" = in the X operand's order."""
-    o = _Opts()
-    o.morder = {None: 0, "C": 1, "X": 2}[morder]
-    o.reserved[0] = int(dbg)
-    o.tma_epilogue = int(tma)
-    o.cost_mode = COST[cost]
-    o.host_only = int(host_only)
-    o.variant = 0 if variant is None else int(variant) + 1
-    o.force_tiles = force_tiles.encode() if force_tiles else None
-    o.no_fusion = int(not fusion)
+    o = _opts(cost, host_only, variant, force_tiles, fusion, tma, morder)
     h = ctypes.c_void_p()
     _raise(lib().tc_plan_ex(ctypes.byref(h), expr.encode(), extents.encode(), DTYPES[dtype], ctypes.byref(o)))
     p = Plan(h, expr, extents, dtype)

@@ -206,7 +206,13 @@ Status upload(tc_plan_s *P, std::string &err) {
   const KernelEntry ke = kernel_for(P->cfg);
   const bool tma = P->tt.tma_ok && P->opts.tma_epilogue && P->cfg.kind == KIND_F64_DMMA &&
                    !variants()[P->cfg.variant].stg;
-  e = cudaFuncSetAttribute(ke.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(tma ? ke.smem_tma : ke.smem));
+  // The attribute belongs to the kernel instance, which many plans share: always set the
+  // largest size any plan of the instance may launch with (the TMA staging box when it fits),
+  // so a later plan without the TMA epilogue cannot shrink it under an earlier plan's launch.
+  const size_t kMaxSmem = 227 * 1024;
+  const size_t smem_max = ke.smem_tma <= kMaxSmem ? std::max(ke.smem, ke.smem_tma) : ke.smem;
+  if (tma && ke.smem_tma > smem_max) { err = "TMA epilogue staging exceeds shared memory"; return ST_UNSUPPORTED; }
+  e = cudaFuncSetAttribute(ke.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_max);
   if (e != cudaSuccess) { err = std::string("cudaFuncSetAttribute: ") + cudaGetErrorString(e); return ST_CUDA; }
   int occ = 0;
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ke.fn, ke.threads, tma ? ke.smem_tma : ke.smem);
@@ -242,6 +248,8 @@ tc_status_t finish_plan(tc_plan_s *P, tc_plan_t *out) {
   ForcedTiles ft;
   if (!parse_force(P->opts.force_tiles, ft)) { delete P; return fail(ST_INVALID_ARG, "malformed force_tiles"); }
   if (P->opts.morder < 0 || P->opts.morder > 2) { delete P; return fail(ST_INVALID_ARG, "morder must be 0, 1 or 2"); }
+  for (int r : P->opts.reserved)
+    if (r != 0) { delete P; return fail(ST_INVALID_ARG, "tc_plan_opts.reserved[] must be zero"); }
   ft.morder = P->opts.morder - 1;
   // forced tiles name the original indices: plan without fusion so the names survive
   P->c = P->parsed;
@@ -471,6 +479,11 @@ tc_status_t tc_plan_tuned_beta(tc_plan_t *tuned, const tc_plan_t plan, const voi
   *tuned = nullptr;
   if (plan->host_only || !plan->dev) return fail(ST_CUDA, "plan was made host_only");
   if (topk < 1 || reps < 1) return fail(ST_INVALID_ARG, "topk and reps must be >= 1");
+  {
+    int cur = -1;
+    if (cudaGetDevice(&cur) != cudaSuccess || cur != plan->device)
+      return fail(ST_INVALID_ARG, "current device differs from the plan's device");
+  }
   try {
     // candidates: the best configuration of each of the top-k variants by predicted time
     std::vector<int> cand;
@@ -538,7 +551,8 @@ tc_status_t tc_plan_restrict(tc_plan_t *sub, const tc_plan_t parent, const char 
     int id = -1;
     for (size_t i = 0; i < pc.ix.size(); i++) if (pc.ix[i].name == index) id = (int)i;
     if (id < 0) return fail(ST_INDEX, std::string("unknown index '") + index + "'");
-    if (begin < 0 || len < 1 || begin + len > pc.ix[id].n) return fail(ST_EXTENT, "slab out of range");
+    if (begin < 0 || len < 1 || len > pc.ix[id].n || begin > pc.ix[id].n - len)   // (no int64 overflow)
+      return fail(ST_EXTENT, "slab out of range");
     tc_plan_s *P = new tc_plan_s();
     P->opts = parent->opts;
     P->force_tiles = parent->force_tiles;
@@ -571,8 +585,10 @@ tc_status_t tc_plan_restrict(tc_plan_t *sub, const tc_plan_t parent, const char 
   }
 }
 
-tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void *C, double alpha,
-                       double beta, tc_stream_t stream) {
+namespace {
+// Everything tc_execute checks before it launches (also run for every member of a group
+// before the group's first launch, so a bad member leaves C untouched).
+tc_status_t check_execute(const tc_plan_t plan, const void *A, const void *B, const void *C) {
   if (!plan || !A || !B || !C) return fail(ST_INVALID_ARG, "NULL plan or tensor pointer");
   if (plan->host_only || !plan->dev) return fail(ST_CUDA, "plan was made host_only");
   const size_t es = elem_bytes(plan);
@@ -582,6 +598,15 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
   int cur = -1;
   if (cudaGetDevice(&cur) != cudaSuccess || cur != plan->device)
     return fail(ST_INVALID_ARG, "current device differs from the plan's device");
+  return TC_SUCCESS;
+}
+}  // namespace
+
+tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void *C, double alpha,
+                       double beta, tc_stream_t stream) {
+  const tc_status_t chk = check_execute(plan, A, B, C);
+  if (chk != TC_SUCCESS) return chk;
+  const size_t es = elem_bytes(plan);
   KParams kp = plan->kp;
   const Config &cfg = plan->cfg;
   kp.X = cfg.X == 1 ? A : B;
@@ -605,7 +630,6 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
   kp.packY = vy ? plan->d_packY2 : plan->d_packY1;
   kp.nslotY = (int)(vy ? plan->slotY2.pack.size() : plan->slotY1.pack.size());
   kp.vecY = vy ? cfg.vecY : 1;
-  kp.dbg = plan->opts.reserved[0];
   // C stores in 16-B vectors: 8 elements (staged UMMA epilogue: one 16-B BF16 or two 16-B FP32
   // stores) / 2 FP64 (STG drain)
   kp.vecC = plan->cvec > 1 && ((uintptr_t)C % 16) == 0 ? plan->cvec : 1;
@@ -651,6 +675,13 @@ tc_status_t tc_execute_group(const tc_plan_t *plans, const void *const *A, const
     for (size_t k = 0; same && k < c0.t[0].idx.size(); k++)
       same = ci.ix[ci.t[0].idx[k]].n == c0.ix[c0.t[0].idx[k]].n && ci.t[0].stride[k] == c0.t[0].stride[k];
     if (!same) return fail(ST_INVALID_ARG, "group member " + std::to_string(i) + " gives C another layout");
+  }
+  for (int i = 0; i < n; i++) {
+    const tc_status_t chk = check_execute(plans[i], A[i], B[i], C);
+    if (chk != TC_SUCCESS) {
+      g_err = "group member " + std::to_string(i) + ": " + g_err;
+      return chk;
+    }
   }
   for (int i = 0; i < n; i++) {
     tc_status_t st = tc_execute(plans[i], A[i], B[i], C, alpha, i == 0 ? beta : 1.0, stream);

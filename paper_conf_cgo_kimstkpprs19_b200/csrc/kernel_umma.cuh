@@ -255,19 +255,19 @@ __device__ __forceinline__ void store_run8(__nv_bfloat16 *dst, float (&x)[8], fl
   *d = make_uint4(w[0], w[1], w[2], w[3]);
 }
 
-// Development trace (dbg & 4096): CTA 0 records clock64() at the hand-off points of the first
-// 1024 stages / tiles into the C buffer (which then holds no result): [0..) producer warp 0
-// after its EMPTY wait, [1024..) after its FULL arrive, [2048..) MMA after its FULL wait,
-// [3072..) MMA after its commits, [4096..) epilogue warp 0 after TFULL, [5120..) after TEMPTY,
-// [6144..) producer warp 0 at the loop top, [7168..) after its tile switch.
-// Compiled in only with -DTC_TRACE (tools/trace_umma.py builds such a libtc on the side).
+// Development trace: CTA 0 records clock64() at the hand-off points of the first 1024 stages
+// / tiles into the C buffer (which then holds no result): [0..) producer warp 0 after its
+// EMPTY wait, [1024..) after its FULL arrive, [2048..) MMA after its FULL wait, [3072..) MMA
+// after its commits, [4096..) epilogue warp 0 after TFULL, [5120..) after TEMPTY, [6144..)
+// producer warp 0 at the loop top, [7168..) after its tile switch.  Compiled in only in a
+// -DTC_TRACE side build (tools/trace_umma.py); the shipped library has no trace code.
 #ifdef TC_TRACE
 constexpr bool kTrace = true;
 #else
 constexpr bool kTrace = false;
 #endif
 __device__ __forceinline__ void trace_at(const KParams &p, int slot, int j) {
-  if (kTrace && (p.dbg & 4096) && blockIdx.x == 0 && j < 1024)
+  if (kTrace && blockIdx.x == 0 && j < 1024)
     static_cast<unsigned long long *>(p.C)[slot * 1024 + j] = clock64();
 }
 
@@ -369,9 +369,7 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
       const int64_t bx = cur.ox + ks.sx(), by = cur.oy + ks.sy();
       const uint32_t dx = sbase + (uint32_t)ES * (uint32_t)(s * K::XS);
       const uint32_t dy = sbase + (uint32_t)ES * (uint32_t)(STAGES * K::XS + s * K::YS);
-      if (p.dbg & 8) {
-        mbar_arrive(FULL + 8 * s);
-      } else if (cached) {
+      if (cached) {
         umma_issue<K::EX>(X, dx, rx, px, cx, bx, fm && fk, km, mm, p.packX, pt, K::PW * 32);
         umma_issue<K::EY>(Y, dy, ry, py, cy, by, fn && fk, km, mn, p.packY, pt, K::PW * 32);
         mbar_arrive_cp_async(FULL + 8 * s);
@@ -423,7 +421,7 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
       if (lane == 0) trace_at(p, 2, j);
       // the stage was written through the generic proxy (cp.async / st.shared); the MMA
       // reads it through the async proxy
-      if (!(p.dbg & 16)) asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
+      asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
       tc05_fence_after();
       if (lane == 0) {
         const uint32_t ax = sbase + (uint32_t)ES * (uint32_t)(s * K::XS);
@@ -438,12 +436,11 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
             tc05_mma<true>(d, umma_desc<XL>(ax + LO + kk * A_KSTEP, A_LBO, A_SBO), bh, IDESC, (step > 0 || kk > 0) ? 1u : 0u);
             tc05_mma<true>(d, ah, umma_desc<YL>(by + LO + kk * B_KSTEP, B_LBO, B_SBO), IDESC, 1u);
             tc05_mma<true>(d, ah, bh, IDESC, 1u);
-          } else if (!(p.dbg & 2)) {
+          } else {
             tc05_mma<ES == 4>(d, ah, bh, IDESC, (step > 0 || kk > 0) ? 1u : 0u);
           }
         }
-        if (p.dbg & 64) mbar_arrive(EMPTY + 8 * s);
-        else tc05_commit(EMPTY + 8 * s);                      // smem stage free once MMAs read it
+        tc05_commit(EMPTY + 8 * s);                           // smem stage free once MMAs read it
         if (step + 1 == p.nsteps) tc05_commit(TFULL + 8 * buf);   // accumulator ready
         trace_at(p, 3, j);
       }
@@ -533,10 +530,9 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
       const bool cfull = cm0 == p.fullN[0] && cm1 == p.fullN[1];
       const bool gok = ((grow < 64 ? rm0 : rm1) >> (grow & 63)) & 1;
       T *Cg = C + (coff + goff);
-      if (p.dbg & 256) mbar_wait(TFULL + 8 * buf, (lt / K::NBUF) & 1);
-      else mbar_wait_sleep(TFULL + 8 * buf, (lt / K::NBUF) & 1);
+      mbar_wait_sleep(TFULL + 8 * buf, (lt / K::NBUF) & 1);
       tc05_fence_after();
-      if (kTrace && (p.dbg & 4096)) {
+      if (kTrace) {
         if (warp == 0 && lane == 0) trace_at(p, 4, lt);
       } else if (p.vecC == 8 && p.cs0 > 1) {
         // CTA-wide staged epilogue: C's FVI is an inner m digit (tile-row stride cs0), so the
@@ -571,7 +567,6 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
       for (int c0 = 0; c0 < HC; c0 += 32 > HC ? HC : 32) {
         constexpr int W = 32 > HC ? HC : 32;
         if (half * HC + c0 >= p.Nt) break;             // columns past the tile's Nt: padding
-        if (p.dbg & 4) break;
         uint32_t v[W];
         tc05_ld<W>(tmem + ((uint32_t)(quarter * 32) << 16) + (uint32_t)(buf * BN + half * HC + c0), v);
         if (p.vecC == 8) {
@@ -627,8 +622,7 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
                 const __nv_bfloat162 b2 = __floats2bfloat162_rn(r[2 * j], r[2 * j + 1]);
                 w[j] = *reinterpret_cast<const uint32_t *>(&b2);
               }
-              if (!(p.dbg & 1)) *dst = make_uint4(w[0], w[1], w[2], w[3]);
-              else if (w[0] == 12345u) *dst = make_uint4(w[0], w[1], w[2], w[3]);
+              *dst = make_uint4(w[0], w[1], w[2], w[3]);
             }
           }
           __syncwarp();

@@ -77,7 +77,6 @@ struct KParams {
   const uint32_t *packY;
   int nslotX, nslotY;
   int vecX, vecY;           // elements per slot (16-B cp.async at 2 FP64 / 8 BF16)
-  int dbg;                  // TEMPORARY experiment knob
   int vecC;                 // C vector (elements): BF16 8 / FP64 STG 2 => tile rows come in aligned
                             // C-contiguous runs of vecC (16-B stores); 1 => per-element stores
   int nmma, kmma;           // UMMA: instruction N (<= BN) and K-instructions per stage (<= BK / KI)

@@ -524,6 +524,9 @@ static Status choose_paper(const Contraction &c, int kind, int forced_variant, C
   if (kset.empty()) kset.insert(Tiling());
   st.raw = (int64_t)px.size() * py.size() * kset.size();
   bool found = false;
+  // best B200-model time per variant over the configs the paper's rules keep: the candidate
+  // list of measured tuning (tc_plan_tuned) in paper mode too
+  std::map<int, double> vbest;
   for (auto &x : px)
     for (auto &y : py)
       for (auto &k : kset) {
@@ -551,6 +554,8 @@ static Status choose_paper(const Contraction &c, int kind, int forced_variant, C
             Config t = cfg;
             t.variant = vi;
             model_time(c, t, variants()[vi], &cache);
+            auto vb = vbest.find(vi);
+            if (vb == vbest.end() || t.t_pred < vb->second) vbest[vi] = t.t_pred;
             if (vi_best < 0 || better(t, fit)) { fit = t; vi_best = vi; }
           }
         }
@@ -565,6 +570,9 @@ static Status choose_paper(const Contraction &c, int kind, int forced_variant, C
                          (fit.paper_cost == best.paper_cost && better(fit, best));
         if (win) { best = fit; found = true; }
       }
+  for (auto &kv : vbest) st.per_variant.push_back(kv);
+  std::stable_sort(st.per_variant.begin(), st.per_variant.end(),
+                   [](const auto &a, const auto &b) { return a.second < b.second; });
   return found ? ST_OK : ST_NO_CONFIG;
 }
 
@@ -611,6 +619,7 @@ Status choose(const Contraction &c, int kind, int cost_mode, int forced_variant,
     PlanStats st2;
     s = choose_b200(c, kind, forced_variant, ft.morder, out, st2);
     stats.ranked += st2.ranked;
+    stats.per_variant = st2.per_variant;
   }
   if (s != ST_OK && err.empty()) err = "no legal configuration";
   stats.plan_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();

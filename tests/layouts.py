@@ -28,5 +28,7 @@ def layouts_two_contractions():
     return out
 
 
-# distinct small extents, so a transposed index cannot alias another one
-PRIME_EXT = {"a": 2, "b": 3, "c": 5, "d": 7, "k": 3, "l": 5}
+# pairwise DISTINCT small primes, so a transposed index cannot alias another one (no two
+# indices of any layout share an extent: a swapped pair of indices changes the shape)
+PRIME_EXT = {"a": 2, "b": 3, "c": 5, "d": 7, "k": 11, "l": 13}
+assert len(set(PRIME_EXT.values())) == len(PRIME_EXT)

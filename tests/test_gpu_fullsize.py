@@ -1,7 +1,14 @@
-"""Full-size parity: every TCCG-48 contraction at the benchmark extents,
-in the exact launch configuration bench.py times (same plan, same seeded device inputs),
-checked against the CPU oracle on sampled outputs (random + first + last elements), and
-against the rank-1 closed form on EVERY output element for a subset.  Needs a B200."""
+"""Full-size parity: every workload bench.py times, at its full extents and in the exact
+launch configuration bench.py times it in (same planning, same measured top-k tuning, same
+seeded device inputs, same alpha / beta), checked against the CPU oracle on sampled outputs:
+2^16 random elements plus EVERY element of the first and the last C tile of the plan
+(SURVEY 8(d) "Parity for the large cases"), and against the rank-1 closed form on every
+output element for a subset.  Needs a B200.
+
+Covered: TCCG-48 FP64 (model plan and tuned plan), the CCSD(T) sweep of config 3 at
+N = 24..48 (beta = 0) and TCCG #31-48 at beta = 1 (NWChem-style t3 accumulation),
+the memory-bound suite of config 4 (#1-8, #18 in FP32 / TF32 / BF16) and the FP32 SD2
+family of Figs. 6/7 (sd_t_d2, TCCG #40-48, single precision)."""
 import numpy as np
 import pytest
 import torch
@@ -13,6 +20,9 @@ from paper_conf_cgo_kimstkpprs19_b200 import build
 
 pytestmark = pytest.mark.gpu
 TAU64 = 1e-12
+NSAMPLE = 1 << 16
+TUNE_TOPK = 8          # bench.py --tune default
+_TDT = {"f64": torch.float64, "f32": torch.float32, "tf32": torch.float32, "bf16": torch.bfloat16}
 
 
 @pytest.fixture(scope="module", autouse=True)
@@ -23,24 +33,153 @@ def _dev():
     torch.cuda.set_device(0)
 
 
+def tile_indices(p, last: bool) -> np.ndarray:
+    """C linear indices of every element of the plan's first (origin) or last C tile, from
+    the plan's own (normalised) C view: index extents, tiles and strides (tc_plan_info)."""
+    info = p.info()
+    ix = {d["name"]: d for d in info["indices"]}
+    cv = info["tensors"]["C"]
+    off = np.array([cv["base"]], dtype=np.int64)
+    for name, stride in zip(cv["idx"], cv["stride"]):
+        n, t = ix[name]["n"], max(1, ix[name]["tile"])
+        o = (n - 1) // t * t if last else 0
+        r = np.arange(o, min(o + t, n), dtype=np.int64) * stride
+        off = (off[:, None] + r[None, :]).reshape(-1)
+    return off
+
+
+def sample_indices(p, n: int, seed: int) -> np.ndarray:
+    rng = np.random.default_rng(seed)
+    return np.unique(np.concatenate([rng.integers(0, n, NSAMPLE), tile_indices(p, False),
+                                     tile_indices(p, True), np.array([0, n - 1])]))
+
+
+def check_sampled(p, case, dtype, A, B, C, C0=None, beta=0.0, seed=0):
+    """Sampled parity of C (device) against the oracle on the same inputs (upcast exactly)."""
+    n = C.numel()
+    idx = sample_indices(p, n, seed)
+    got = C[torch.as_tensor(idx, device=C.device)].double().cpu().numpy()
+    c0 = None if C0 is None else C0.double().cpu().numpy()
+    exact, S = oracle.sample(case.expr, case.extents, A.double().cpu().numpy(), B.double().cpu().numpy(),
+                             idx, C=c0, beta=beta, with_scale=True)
+    K = p.flops / 2 / max(1, p.numel("C"))
+    if dtype == "f64":
+        tol = TAU64 * S
+    elif dtype == "f32":
+        tol = 1e-5 * S                                     # north_star FP32
+    elif dtype == "tf32":                                  # DESIGN R30
+        tol = 2.0 ** -9 * S + 2.0 ** -23 * np.abs(exact)
+    else:                                                  # one BF16 ulp + FP32 accumulation
+        tol = 2.0 ** -8 * np.abs(exact) + K * 2.0 ** -23 * S
+    bad = np.flatnonzero(~(np.abs(got - exact) <= tol))
+    assert bad.size == 0, (case.expr, dtype, idx[bad[:5]], got[bad[:5]], exact[bad[:5]], p.info()["variant"])
+    return idx.size
+
+
+def inputs(p, case, dtype, dev="cuda"):
+    tdt = _TDT[dtype]
+    A = tcinputs.uniform(p.numel("A"), 1000 + case.id, device=dev).to(tdt)
+    B = tcinputs.uniform(p.numel("B"), 2000 + case.id, device=dev).to(tdt)
+    return A, B
+
+
+def run_tuned(case, dtype="f64", beta=0.0, tune=True):
+    """Plan + tune exactly as bench.py does, then one execute on NaN-prefilled C (beta = 0) or
+    on the seeded C_in (beta != 0); returns what check_sampled needs."""
+    tdt = _TDT[dtype]
+    p = tc.plan(case.expr, case.extents, dtype=dtype)
+    A, B = inputs(p, case, dtype)
+    C = torch.empty(p.numel("C"), dtype=tdt, device="cuda")
+    C0 = None
+    if beta != 0.0:
+        C0 = tcinputs.uniform(p.numel("C"), 3000 + case.id, device="cuda").to(tdt)
+    if tune:
+        if beta != 0.0:
+            C.copy_(C0)
+        p = p.tuned(A, B, C, topk=TUNE_TOPK, reps=1, beta=beta)
+    if beta != 0.0:
+        C.copy_(C0)
+    else:
+        C.fill_(float("nan"))
+    p.execute(A, B, C, beta=beta)
+    torch.cuda.synchronize()
+    return p, A, B, C, C0
+
+
+@pytest.mark.parametrize("tuned", [False, True], ids=["model", "tuned"])
 @pytest.mark.parametrize("case", tcinputs.tccg48(), ids=lambda c: f"tccg{c.id}")
-def test_tccg_full_size_sampled(case):
+def test_tccg_full_size_sampled(case, tuned):
+    p, A, B, C, _ = run_tuned(case, tune=tuned)
+    check_sampled(p, case, "f64", A, B, C, seed=case.id)
+    assert torch.isfinite(C).all()          # every element was written
+    del A, B, C
+
+
+@pytest.mark.parametrize("case", [c for c in tcinputs.tccg48() if c.id >= 31], ids=lambda c: f"tccg{c.id}")
+def test_ccsdt_tccg_beta1_tuned(case):
+    # CCSD(T) sd_t_d1 / d2 accumulating into t3 (beta = 1, P:L344; SURVEY 8(d) config 3),
+    # planned and tuned at beta = 1 as bench.py's ccsdt suite and the triples group run them
+    p, A, B, C, C0 = run_tuned(case, beta=1.0)
+    check_sampled(p, case, "f64", A, B, C, C0=C0, beta=1.0, seed=case.id)
+
+
+# (beta = 1 rows at N <= 32: the oracle needs the whole C_in on the host, and at N = 48 a
+# second 97.8 GB C_in does not fit the GPU next to C)
+@pytest.mark.parametrize("n,beta", [(24, 0.0), (32, 0.0), (40, 0.0), (48, 0.0), (24, 1.0), (32, 1.0)])
+@pytest.mark.parametrize("expr", ["abcdef-gdab-efgc", "abcdef-dega-gfbc"])
+def test_ccsdt_sweep_tuned(expr, n, beta):
+    # bench.py's ccsdt suite (BASELINE config 3), each row in its own launch configuration
+    case = tcinputs.ccsdt(n, expr, 100 + n)
+    p, A, B, C, C0 = run_tuned(case, beta=beta)
+    check_sampled(p, case, "f64", A, B, C, C0=C0, beta=beta, seed=n)
+    if beta == 0.0:
+        assert not bool(torch.isnan(C).any())
+    del A, B, C, C0
+    torch.cuda.empty_cache()
+
+
+@pytest.mark.parametrize("n,expr", [(48, "abcdef-gdab-efgc"), (40, "abcdef-dega-gfbc")])
+def test_ccsdt_max_size_int64_offsets(n, expr):
+    # |C| = 48^6 = 1.2e10 FP64 elements (97.8 GB), past 2^31: every 64-bit offset path of the
+    # tables and the epilogue runs; elements around 2^31 and 2^32 are sampled explicitly
+    case = tcinputs.ccsdt(n, expr, 100 + n)
     p = tc.plan(case.expr, case.extents)
-    A = tcinputs.uniform(p.numel("A"), 1000 + case.id, device="cuda")
-    B = tcinputs.uniform(p.numel("B"), 2000 + case.id, device="cuda")
+    A, B = inputs(p, case, "f64")
     C = torch.full((p.numel("C"),), float("nan"), dtype=torch.float64, device="cuda")
     p.execute(A, B, C)
     torch.cuda.synchronize()
-    n = C.numel()
-    rng = np.random.default_rng(case.id)
-    idx = np.unique(np.concatenate([rng.integers(0, n, 1500), np.arange(min(n, 256)),
-                                    np.arange(max(0, n - 256), n)]))
+    nC = C.numel()
+    idx = np.unique(np.concatenate([sample_indices(p, nC, n), (np.int64(1) << 31) + np.arange(-64, 64),
+                                    (np.int64(1) << 32) + np.arange(-64, 64)]))
     got = C[torch.as_tensor(idx, device="cuda")].cpu().numpy()
-    want, S = oracle.sample(case.expr, case.extents, A.cpu().numpy(), B.cpu().numpy(), idx,
-                            with_scale=True)
+    want, S = oracle.sample(case.expr, case.extents, A.cpu().numpy(), B.cpu().numpy(), idx, with_scale=True)
     bad = np.flatnonzero(~(np.abs(got - want) <= TAU64 * S))
-    assert bad.size == 0, (case.id, idx[bad[:5]], got[bad[:5]], want[bad[:5]])
-    assert torch.isfinite(C).all()          # every element was written
+    assert bad.size == 0, (n, idx[bad[:5]], got[bad[:5]], want[bad[:5]])
+    assert not bool(torch.isnan(C).any())   # every element was written
+    del C
+    torch.cuda.empty_cache()
+
+
+@pytest.mark.parametrize("dtype", ["bf16", "tf32", "f32"])
+@pytest.mark.parametrize("cid", [1, 2, 3, 4, 5, 6, 7, 8, 18])
+def test_membound_suite_full_size_tuned(dtype, cid):
+    # bench.py's membound suite (BASELINE config 4), every row, tuned as the bench tunes it
+    case = [c for c in tcinputs.tccg48() if c.id == cid][0]
+    p, A, B, C, _ = run_tuned(case, dtype=dtype)
+    check_sampled(p, case, dtype, A, B, C, seed=cid)
+    assert not bool(torch.isnan(C.float()).any())
+
+
+@pytest.mark.parametrize("cid", list(range(40, 49)))
+def test_sd2_f32_family_full_size(cid):
+    # Figs. 6/7 (P:L346-348): the SD2 CCSD(T) subset in single precision — TCCG #40-48
+    # (sd_t_d2, e.g. SD2_1 = abcdef-gdab-efgc, P:L353) at the suite's extents, FP32 through
+    # the split-TF32 tcgen05 path, model plan and tuned plan
+    case = [c for c in tcinputs.tccg48() if c.id == cid][0]
+    for tune in (False, True):
+        p, A, B, C, _ = run_tuned(case, dtype="f32", tune=tune)
+        check_sampled(p, case, "f32", A, B, C, seed=cid)
+        assert not bool(torch.isnan(C).any())
 
 
 @pytest.mark.parametrize("cid", [1, 6, 9, 12, 13, 16, 18, 31, 40, 48])
@@ -68,80 +207,3 @@ def test_tccg_full_size_rank1_every_element(cid):
     # S[x] = sum |A B| = want (all factors positive); tau * S plus the closed form's own
     # rounding (a product of <= 8 factors: 8 ulp)
     assert np.all(np.abs(got - want) <= (TAU64 + 16 * 2.2e-16) * np.abs(want))
-
-
-@pytest.mark.parametrize("n,expr", [(48, "abcdef-gdab-efgc"), (40, "abcdef-dega-gfbc")])
-def test_ccsdt_max_size_sampled(n, expr):
-    # BASELINE config 3 at its largest extent: |C| = 48^6 = 1.2e10 FP64 elements (97.8 GB) —
-    # past 2^31 elements, so every 64-bit offset path of the tables and the epilogue runs
-    case = tcinputs.ccsdt(n, expr, 100 + n)
-    p = tc.plan(case.expr, case.extents)
-    A = tcinputs.uniform(p.numel("A"), 1000 + case.id, device="cuda")
-    B = tcinputs.uniform(p.numel("B"), 2000 + case.id, device="cuda")
-    C = torch.full((p.numel("C"),), float("nan"), dtype=torch.float64, device="cuda")
-    p.execute(A, B, C)
-    torch.cuda.synchronize()
-    nC = C.numel()
-    rng = np.random.default_rng(n)
-    idx = np.unique(np.concatenate([rng.integers(0, nC, 2000), np.arange(128), np.arange(nC - 128, nC),
-                                    (np.int64(1) << 31) + np.arange(-64, 64)]))
-    got = C[torch.as_tensor(idx, device="cuda")].cpu().numpy()
-    want, S = oracle.sample(case.expr, case.extents, A.cpu().numpy(), B.cpu().numpy(), idx,
-                            with_scale=True)
-    bad = np.flatnonzero(~(np.abs(got - want) <= TAU64 * S))
-    assert bad.size == 0, (n, idx[bad[:5]], got[bad[:5]], want[bad[:5]])
-    assert not bool(torch.isnan(C).any())   # every element was written
-    del C
-    torch.cuda.empty_cache()
-
-
-@pytest.mark.parametrize("cid", [1, 8, 12, 18, 30, 33, 40])
-def test_tuned_plans_as_bench_times_them(cid):
-    # bench.py times tc_plan_tuned plans (top-8 variants measured); check those, sampled
-    case = [c for c in tcinputs.tccg48() if c.id == cid][0]
-    p = tc.plan(case.expr, case.extents)
-    A = tcinputs.uniform(p.numel("A"), 1000 + case.id, device="cuda")
-    B = tcinputs.uniform(p.numel("B"), 2000 + case.id, device="cuda")
-    C = torch.empty(p.numel("C"), dtype=torch.float64, device="cuda")
-    p = p.tuned(A, B, C, topk=8, reps=1)
-    C.fill_(float("nan"))
-    p.execute(A, B, C)
-    torch.cuda.synchronize()
-    n = C.numel()
-    idx = np.unique(np.concatenate([np.random.default_rng(cid).integers(0, n, 1500), np.arange(64),
-                                    np.arange(n - 64, n)]))
-    got = C[torch.as_tensor(idx, device="cuda")].cpu().numpy()
-    want, S = oracle.sample(case.expr, case.extents, A.cpu().numpy(), B.cpu().numpy(), idx, with_scale=True)
-    assert np.all(np.abs(got - want) <= TAU64 * S), (cid, p.info()["variant"])
-    assert torch.isfinite(C).all()
-
-
-@pytest.mark.parametrize("dtype", ["bf16", "tf32", "f32"])
-@pytest.mark.parametrize("cid", [1, 4, 6, 7])
-def test_membound_suite_full_size_sampled(dtype, cid):
-    # BASELINE config 4 at full size in the bench's launch configuration (tuned plan)
-    case = [c for c in tcinputs.tccg48() if c.id == cid][0]
-    tdt = torch.bfloat16 if dtype == "bf16" else torch.float32
-    p = tc.plan(case.expr, case.extents, dtype=dtype)
-    A = tcinputs.uniform(p.numel("A"), 1000 + cid, device="cuda").to(tdt)
-    B = tcinputs.uniform(p.numel("B"), 2000 + cid, device="cuda").to(tdt)
-    C = torch.empty(p.numel("C"), dtype=tdt, device="cuda")
-    p = p.tuned(A, B, C, topk=8, reps=1)
-    C.fill_(float("nan"))
-    p.execute(A, B, C)
-    torch.cuda.synchronize()
-    n = C.numel()
-    idx = np.unique(np.concatenate([np.random.default_rng(cid).integers(0, n, 2000), np.arange(64),
-                                    np.arange(n - 64, n)]))
-    got = C[torch.as_tensor(idx, device="cuda")].float().cpu().numpy().astype(np.float64)
-    exact, S = oracle.sample(case.expr, case.extents, A.double().cpu().numpy(), B.double().cpu().numpy(),
-                             idx, with_scale=True)
-    K = p.flops / 2 / n
-    if dtype == "f32":
-        tol = 1e-5 * S
-    elif dtype == "tf32":
-        tol = 2.0 ** -9 * S + 2.0 ** -23 * np.abs(exact)
-    else:   # DESIGN R21 / test_gpu_bf16: one BF16 ulp of the result + FP32 accumulation
-        tol = 2.0 ** -8 * np.abs(exact) + K * 2.0 ** -23 * S
-    bad = np.flatnonzero(~(np.abs(got - exact) <= tol))
-    assert bad.size == 0, (cid, dtype, idx[bad[:5]], got[bad[:5]], exact[bad[:5]])

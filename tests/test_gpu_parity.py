@@ -257,3 +257,18 @@ def test_cached_plan_executes_and_is_shared():
     del p1
     tc.plan_cache_clear()
     assert np.array_equal(run_gpu(p2, A, B), got)   # the caller's reference outlives the cache
+
+
+def test_tma_plan_survives_a_later_plain_plan_on_the_same_kernel():
+    """The dynamic-smem attribute belongs to the kernel instance that many plans share: a TMA
+    epilogue plan, then a plan WITHOUT it on the same variant and layouts, then the TMA plan
+    again must still launch and be right (the later plan used to shrink the limit)."""
+    expr, ext = "abcd-aebf-dfce", "a:16;b:16;c:16;d:16;e:16;f:16"
+    A, B = tcinputs.uniform_np(16 ** 4, 11), tcinputs.uniform_np(16 ** 4, 12)
+    want, S = oracle.contract(expr, ext, A, B, with_scale=True)
+    for v in (3, 0):
+        p_tma = tc.plan(expr, ext, variant=v, tma=True)
+        p_plain = tc.plan(expr, ext, variant=v, tma=False)
+        for p in (p_tma, p_plain, p_tma):
+            got = run_gpu(p, A, B)
+            assert np.all(np.abs(got - want) <= TAU64 * S), (v, p is p_tma)

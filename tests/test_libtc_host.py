@@ -230,3 +230,27 @@ def test_plan_tuned_beta_errors_host():
     assert L.tc_plan_tuned_beta(ctypes.byref(h), p._h, None, x, x, 2, 1, 1.0, None) == 1
     assert L.tc_plan_tuned_beta(ctypes.byref(h), p._h, x, x, x, 0, 1, 1.0, None) == 7   # host_only first
     assert not h.value
+
+
+def test_reserved_opts_rejected_and_restrict_overflow():
+    """tc_plan_opts.reserved[] must be zero (no hidden switches reach the kernels); a slab
+    whose begin + len would overflow int64 is TC_ERR_EXTENT, not an out-of-bounds plan."""
+    o = tc._opts("b200", True, None, None, True, False, None)
+    o.reserved[0] = 64
+    h = ctypes.c_void_p()
+    st = tc.lib().tc_plan_ex(ctypes.byref(h), b"ab-ac-cb", b"a:8;b:8;c:8", 0, ctypes.byref(o))
+    assert tc.STATUS[st] == "TC_ERR_INVALID_ARG" and not h.value
+    p = tc.plan("ab-ac-cb", "a:8;b:8;c:8", host_only=True)
+    for begin, length in (((1 << 63) - 2, 4), (7, 2), (-1, 1), (0, 0)):
+        with pytest.raises(tc.TcError) as e:
+            p.restrict("a", begin, length)
+        assert e.value.status == "TC_ERR_EXTENT"
+
+
+def test_paper_mode_lists_tuning_candidates():
+    """Paper-mode plans carry the B200-ranked per-variant candidates too, so measured tuning
+    (tc_plan_tuned) has more than the planned variant to time in either cost mode."""
+    for ext in ("a:16;b:16;c:16;d:16;e:16;f:16", "a:2;b:2;c:2;d:2;e:2;f:2"):   # (2: paper sets prune all)
+        i = tc.plan("abcd-aebf-dfce", ext, cost="paper", host_only=True).info()
+        pv = i["stats"]["per_variant"]
+        assert len(pv) >= 2 and [t for _, t in pv] == sorted(t for _, t in pv)

@@ -21,7 +21,7 @@ def main():
     for case in tcinputs.tccg48():
         if ids and case.id not in ids:
             continue
-        p = tc.plan(case.expr, case.extents, cost=cost, dtype=dtype, dbg=int(os.environ.get("TC_DBG", "0")))
+        p = tc.plan(case.expr, case.extents, cost=cost, dtype=dtype)
         info = p.info()
         A = tcinputs.uniform(p.numel("A"), 1000 + case.id, device="cuda").to(tdt)
         B = tcinputs.uniform(p.numel("B"), 2000 + case.id, device="cuda").to(tdt)

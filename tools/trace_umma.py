@@ -1,6 +1,6 @@
-"""Per-stage hand-off timeline of the tcgen05 kernel (dbg & 4096 trace, CTA 0, clock64).
+"""Per-stage hand-off timeline of the tcgen05 kernel (-DTC_TRACE side build, CTA 0, clock64).
 Builds a -DTC_TRACE libtc on the side (build/trace/libtc.so) and loads it instead.
-usage: python tools/trace_umma.py <case> <dtype> [extra dbg]"""
+usage: python tools/trace_umma.py <case> <dtype>"""
 import os
 import sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
@@ -18,10 +18,9 @@ import tcinputs  # noqa: E402
 from paper_conf_cgo_kimstkpprs19_b200 import binding as tc  # noqa: E402
 
 cid, dt = int(sys.argv[1]), sys.argv[2]
-extra = int(sys.argv[3]) if len(sys.argv) > 3 else 0
 case = [c for c in tcinputs.tccg48() if c.id == cid][0]
 tdt = {"bf16": torch.bfloat16, "f32": torch.float32, "tf32": torch.float32}[dt]
-p = tc.plan(case.expr, case.extents, dtype=dt, dbg=4096 | extra)
+p = tc.plan(case.expr, case.extents, dtype=dt)
 A = tcinputs.uniform(p.numel("A"), 1, device="cuda").to(tdt)
 B = tcinputs.uniform(p.numel("B"), 2, device="cuda").to(tdt)
 C = torch.zeros(max(p.numel("C"), 8 * 1024 * 8 // tdt.itemsize + 64), dtype=tdt, device="cuda")
