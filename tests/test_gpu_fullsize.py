@@ -149,8 +149,8 @@ def test_ccsdt_max_size_int64_offsets(n, expr):
     p.execute(A, B, C)
     torch.cuda.synchronize()
     nC = C.numel()
-    idx = np.unique(np.concatenate([sample_indices(p, nC, n), (np.int64(1) << 31) + np.arange(-64, 64),
-                                    (np.int64(1) << 32) + np.arange(-64, 64)]))
+    extra = [(np.int64(1) << s) + np.arange(-64, 64) for s in (31, 32) if (1 << s) + 64 <= nC]
+    idx = np.unique(np.concatenate([sample_indices(p, nC, n)] + extra))
     got = C[torch.as_tensor(idx, device="cuda")].cpu().numpy()
     want, S = oracle.sample(case.expr, case.extents, A.cpu().numpy(), B.cpu().numpy(), idx, with_scale=True)
     bad = np.flatnonzero(~(np.abs(got - want) <= TAU64 * S))
