@@ -109,6 +109,31 @@ tc_status_t tc_execute_group(const tc_plan_t *plans, const void *const *A, const
                              int n, void *C, double alpha, double beta, tc_stream_t stream);
 
 /*
+ * FUSED grouped contraction (R34): the same sum as
+ * tc_execute_group,
+ *   C = alpha * sum_{i<n} (sum_int A_i*B_i under plans[i]) + beta * C,
+ * run as ONE persistent FP64 kernel that keeps each C tile on chip across all n members and
+ * stores it once (the CCSD(T) triples of P:L27, L330, L344: 18 contractions into t3, which
+ * the paper and tc_execute_group run as 18 kernels each reading and writing t3).
+ * tc_group_plan: plans[i] (FP64, all giving C the same layout as in tc_execute_group, no
+ * batch index, n <= 32) are read, not kept; the group owns its own tables (device memory on
+ * the current device, or none when the plans are host_only — then tc_group_execute fails).
+ * The common C tile is chosen so that every member's tile is at most 64 x 64 (rows = the C
+ * indices of the operand holding C's FVI); TC_ERR_UNSUPPORTED when no such tile exists.
+ * tc_group_execute: A[i], B[i] device pointers as for tc_execute on plans[i]; asynchronous on
+ * `stream`, no allocation; beta == 0 => C is only written.  Errors: TC_ERR_INVALID_ARG (NULL,
+ * C overlapping any A_i / B_i, wrong device), TC_ERR_CUDA (launch, host_only group).
+ */
+typedef struct tc_group_s *tc_group_t;
+tc_status_t tc_group_plan(tc_group_t *group, const tc_plan_t *plans, int n);
+tc_status_t tc_group_execute(const tc_group_t group, const void *const *A, const void *const *B, void *C,
+                             double alpha, double beta, tc_stream_t stream);
+/* JSON: the C tile (T per C position), tiles, BK, per-member Mt / Nt / Kt / k-steps and the
+   simulated shared-memory wavefronts of its stage loads and box flush. */
+tc_status_t tc_group_info(const tc_group_t group, char *json, size_t cap, size_t *needed);
+void tc_group_destroy(tc_group_t group);                /* NULL-safe                       */
+
+/*
  * End-to-end call with HOST buffers (used for bench.py's "e2e" figure): copies A, B (and C
  * when beta != 0) from host memory into the caller-provided device workspace, runs
  * tc_execute, copies C back, and synchronises `stream`.  workspace must hold

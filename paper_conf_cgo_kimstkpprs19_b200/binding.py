@@ -93,6 +93,14 @@ def lib():
         L.tc_plan_cached.restype = ctypes.c_int
         L.tc_plan_cache_size.restype = ctypes.c_size_t
         L.tc_plan_cache_clear.restype = None
+        L.tc_group_plan.argtypes = [ctypes.POINTER(vp), ctypes.POINTER(vp), ctypes.c_int]
+        L.tc_group_plan.restype = ctypes.c_int
+        L.tc_group_execute.argtypes = [vp, ctypes.POINTER(vp), ctypes.POINTER(vp), vp, dbl, dbl, vp]
+        L.tc_group_execute.restype = ctypes.c_int
+        L.tc_group_info.argtypes = [vp, ctypes.c_char_p, ctypes.c_size_t, ctypes.POINTER(ctypes.c_size_t)]
+        L.tc_group_info.restype = ctypes.c_int
+        L.tc_group_destroy.argtypes = [vp]
+        L.tc_group_destroy.restype = None
         L.tc_check.argtypes = [cp, cp]
         L.tc_check.restype = ctypes.c_int
         _lib = L
@@ -249,6 +257,59 @@ def execute_group(plans, A, B, C, alpha=1.0, beta=0.0, stream=None):
     execute_group_ptr(plans, [a.data_ptr() for a in A], [b.data_ptr() for b in B], C.data_ptr(),
                       alpha, beta, stream)
     return C
+
+
+class GroupPlan:
+    """A fused grouped contraction (tc_group_t): one kernel computes
+    C = alpha * sum_i plans[i](A[i], B[i]) + beta * C with every C tile kept on chip across the
+    members and stored once."""
+
+    def __init__(self, handle: ctypes.c_void_p, n: int):
+        self._h = handle
+        self.n = n
+        self._info = None
+
+    def __del__(self):
+        h = getattr(self, "_h", None)
+        if h and _lib is not None:
+            _lib.tc_group_destroy(h)
+            self._h = None
+
+    def info(self) -> dict:
+        if self._info is None:
+            need = ctypes.c_size_t(0)
+            _raise(lib().tc_group_info(self._h, None, 0, ctypes.byref(need)))
+            buf = ctypes.create_string_buffer(need.value)
+            _raise(lib().tc_group_info(self._h, buf, need.value, ctypes.byref(need)))
+            self._info = json.loads(buf.value.decode())
+        return self._info
+
+    def execute_ptr(self, A, B, C: int, alpha=1.0, beta=0.0, stream=None):
+        if len(A) != self.n or len(B) != self.n:
+            raise TcError(1, f"the group has {self.n} members")
+        arr = ctypes.c_void_p * self.n
+        _raise(lib().tc_group_execute(self._h, arr(*[ctypes.c_void_p(a) for a in A]),
+                                      arr(*[ctypes.c_void_p(b) for b in B]), ctypes.c_void_p(C),
+                                      float(alpha), float(beta), _stream_ptr(stream)))
+
+    def execute(self, A, B, C, alpha=1.0, beta=0.0, stream=None):
+        import torch
+        for name, t in [("C", C)] + [(f"A[{i}]", a) for i, a in enumerate(A)] + [(f"B[{i}]", b) for i, b in enumerate(B)]:
+            if not t.is_cuda or not t.is_contiguous():
+                raise TcError(1, f"{name} must be a contiguous CUDA tensor")
+            if t.dtype != torch.float64:
+                raise TcError(1, f"{name} is {t.dtype}; fused groups are FP64")
+        self.execute_ptr([a.data_ptr() for a in A], [b.data_ptr() for b in B], C.data_ptr(), alpha, beta, stream)
+        return C
+
+
+def plan_group(plans) -> GroupPlan:
+    """tc_group_plan: fuse the member plans (all giving C one layout) into one kernel."""
+    n = len(plans)
+    arr = ctypes.c_void_p * max(n, 1)
+    h = ctypes.c_void_p()
+    _raise(lib().tc_group_plan(ctypes.byref(h), arr(*[p._h for p in plans]), int(n)))
+    return GroupPlan(h, n)
 
 
 def plan_cache_size() -> int:

@@ -22,6 +22,7 @@
 #include "kparams.hpp"
 #include "planner.hpp"
 #include "tiles.hpp"
+#include "plan_internal.hpp"
 
 using namespace tc;
 
@@ -32,6 +33,14 @@ tc_status_t fail(Status s, const std::string &msg) {
   g_err = msg;
   return (tc_status_t)s;
 }
+}  // namespace
+
+namespace tc {
+tc_status_t set_error(Status s, const std::string &msg) { return fail(s, msg); }
+std::string &last_error_string() { return g_err; }
+}  // namespace tc
+
+namespace {
 
 // ---------------------------------------------------------------- kernel table
 struct KernelEntry {
@@ -63,42 +72,6 @@ KernelEntry kernel_for(const Config &cfg) {
 
 }  // namespace
 
-struct tc_plan_s {
-  std::atomic<int> refs{1};   // tc_plan_destroy releases one; the plan cache holds one
-  Contraction parsed;      // as parsed (before normalisation) — restriction starts here
-  Contraction c;           // normalised (dropped extent-1 indices, fused runs)
-  int dtype = 0;
-  int device = -1;
-  int sms = 148;
-  bool host_only = false;
-  Config cfg;
-  PlanStats stats;
-  tc_plan_opts opts{};
-  std::string force_tiles;
-  TileTables tt;
-  SlotTable slotX1, slotY1, slotX2, slotY2;   // scalar and cfg.vecX / cfg.vecY wide slots
-  int cvec = 1;            // c_vec_width of the plan (16-B C stores when > 1)
-  // batch (Hadamard) indices (R31): extent and element strides in X, Y, C.  tc_execute
-  // launches the kernel once per batch slab with the operands offset to it — the kernels
-  // carry no batch code (the FP64 variants run at their 128-register cap).
-  struct BatchDim { int64_t n, sX, sY, sC; };
-  std::vector<BatchDim> batch;
-  std::vector<std::pair<int, double>> tuned;   // tc_plan_tuned: (variant, measured ms) per candidate
-  KParams kp{};            // device pointers filled in; X/Y/C/alpha/beta/slots set per call
-  void *dev = nullptr;     // one device buffer with every table
-  size_t dev_bytes = 0;
-  const int32_t *d_relX1 = nullptr, *d_relY1 = nullptr, *d_relX2 = nullptr, *d_relY2 = nullptr;
-  const uint32_t *d_packX1 = nullptr, *d_packY1 = nullptr, *d_packX2 = nullptr, *d_packY2 = nullptr;
-  ~tc_plan_s() {
-    if (dev) {
-      int cur = -1;
-      cudaGetDevice(&cur);
-      if (cur != device) cudaSetDevice(device);
-      cudaFree(dev);
-      if (cur != device && cur >= 0) cudaSetDevice(cur);
-    }
-  }
-};
 
 namespace {
 

@@ -1,0 +1,483 @@
+// group.cpp — planner of the fused grouped contraction (see group.hpp).
+//
+// Enumerate -> prune -> cost, as for one contraction, but over the tile of the
+// SHARED output: one tile T_p per C position, such that every member's Mt_i (product over
+// the C positions of its operand X_i) and Nt_i fit the 64 x 64 DMMA register tiles; ranked
+// by the number of C tiles (each tile costs every member's k-steps once) and padding.  Per
+// member, the digit orders of rows and columns are chosen by simulating the shared-memory
+// wavefronts of the member's cp.async stage writes and of its flush into the swizzled box.
+#include "group.hpp"
+
+#include <algorithm>
+#include <chrono>
+#include <cmath>
+#include <functional>
+#include <map>
+#include <set>
+
+namespace tc {
+
+namespace {
+
+int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+// Shared-memory wavefronts of a sequence of warp instructions: entries (byte offset, bytes)
+// in lane order, 32 per instruction; a bank (4-byte words, 32 banks) serves one word per
+// wavefront.
+double smem_wavefronts(const std::vector<std::pair<int64_t, int>> &acc) {
+  double total = 0;
+  for (size_t b = 0; b < acc.size(); b += 32) {
+    const size_t e = std::min(acc.size(), b + 32);
+    std::set<int64_t> words[32];
+    int64_t bytes = 0;
+    for (size_t i = b; i < e; i++) {
+      for (int64_t w = acc[i].first / 4; w < (acc[i].first + acc[i].second + 3) / 4; w++) words[w & 31].insert(w);
+      bytes += acc[i].second;
+    }
+    size_t wf = 0;
+    for (auto &s : words) wf = std::max(wf, s.size());
+    total += (double)std::max<int64_t>((int64_t)wf, (bytes + 127) / 128);
+  }
+  return total;
+}
+
+struct Member {
+  const Contraction *c = nullptr;
+  int X = 1, Y = 2;               // tensor ids (1 = A, 2 = B)
+  std::vector<int> mpos, npos;    // C positions held by X / Y
+  std::vector<int> kid;           // internal index ids, in k-digit order
+  std::vector<int> Tk;            // k tile per kid
+  int64_t nsteps = 1;
+};
+
+// Operand description for run building: dims in the operand's memory order.
+struct OpDim {
+  int id;          // member-local index id
+  int cpos;        // C position, or -1 (internal)
+  int64_t tile, n, gstride, sstride;
+};
+
+// smem element offset of (row, k) in a plane: k-major rows of pitch BK + 4, or mn-major k
+// rows of pitch BMN + 4 (4 mod 16 doubles: conflict-free DMMA fragment loads, as in the
+// single-contraction kernel).
+int64_t plane_off(bool kmajor, int64_t row, int64_t k, int BMN, int BK) {
+  return kmajor ? row * (BK + 4) + k : k * (BMN + 4) + row;
+}
+
+// The dims of operand t of member M with the given row-digit order (C positions) and tiles.
+std::vector<OpDim> op_dims(const Member &M, int t, const std::vector<int> &roword, const int32_t *T,
+                           bool kmajor, int BMN, int BK) {
+  const Contraction &c = *M.c;
+  std::vector<OpDim> d;
+  for (size_t j = 0; j < c.t[t].idx.size(); j++) {
+    const int id = c.t[t].idx[j];
+    OpDim o{id, c.pos_in(0, id), 1, c.ix[id].n, c.t[t].stride[j], 0};
+    int64_t mul = 1;
+    if (o.cpos >= 0) {
+      o.tile = T[o.cpos];
+      for (int p : roword) {
+        if (p == o.cpos) break;
+        mul *= T[p];
+      }
+      o.sstride = plane_off(kmajor, mul, 0, BMN, BK);
+    } else {
+      for (size_t q = 0; q < M.kid.size(); q++) {
+        if (M.kid[q] == id) { o.tile = M.Tk[q]; break; }
+        mul *= M.Tk[q];
+      }
+      o.sstride = plane_off(kmajor, 0, mul, BMN, BK);
+    }
+    d.push_back(o);
+  }
+  return d;
+}
+
+struct Runs {
+  std::vector<int32_t> rel;
+  std::vector<uint32_t> soff;
+  std::vector<uint64_t> dig;
+  int runlen = 1, vec = 1;
+};
+
+// Runs along dim 0 (when it is smem-contiguous), enumerated over dims 1.. (first fastest).
+Runs build_runs(const std::vector<OpDim> &d, int64_t base, bool vec_ok, std::string &err, bool &ok) {
+  Runs r;
+  ok = true;
+  if (d.empty()) {
+    r.rel.push_back(0);
+    r.soff.push_back(0);
+    r.dig.push_back(0);
+    return r;
+  }
+  const bool contiguous = d[0].sstride == 1;
+  r.runlen = contiguous ? (int)d[0].tile : 1;
+  const size_t first = contiguous ? 1 : 0;
+  bool ev = vec_ok && contiguous && d[0].tile % 2 == 0 && d[0].n % 2 == 0 && base % 2 == 0;
+  for (size_t j = 1; j < d.size(); j++) ev &= d[j].gstride % 2 == 0;
+  r.vec = ev ? 2 : 1;
+  std::vector<int64_t> dg(d.size(), 0);
+  for (;;) {
+    int64_t rel = 0, so = 0;
+    uint64_t pk = 0;
+    for (size_t j = first; j < d.size(); j++) {
+      rel += dg[j] * d[j].gstride;
+      so += dg[j] * d[j].sstride;
+      pk |= (uint64_t)dg[j] << (8 * j);
+    }
+    if (rel > INT32_MAX || rel < INT32_MIN) { err = "operand tile spans more than 2^31 elements"; ok = false; return r; }
+    r.rel.push_back((int32_t)rel);
+    r.soff.push_back((uint32_t)so);
+    r.dig.push_back(pk);
+    size_t j = first;
+    for (; j < d.size(); j++) {
+      if (++dg[j] < d[j].tile) break;
+      dg[j] = 0;
+    }
+    if (j == d.size()) break;
+  }
+  return r;
+}
+
+// cp.async stage-write wavefronts of one operand: vectors w in order, warp = 32 consecutive w.
+double runs_wavefronts(const Runs &r, int64_t plane_byte0) {
+  std::vector<std::pair<int64_t, int>> acc;
+  const int vpr = r.runlen / r.vec;
+  for (size_t q = 0; q < r.rel.size(); q++)
+    for (int v = 0; v < vpr; v++) acc.push_back({plane_byte0 + 8 * ((int64_t)r.soff[q] + v * r.vec), 8 * r.vec});
+  return smem_wavefronts(acc);
+}
+
+// box offset of every row (column) of a member tile, from the digit order and the tiles
+std::vector<int32_t> row_box(const std::vector<int> &order, const int32_t *T, const int64_t *bst, int BMN) {
+  std::vector<int32_t> out(BMN, -1);
+  int64_t tot = 1;
+  for (int p : order) tot *= T[p];
+  for (int64_t r = 0; r < tot && r < BMN; r++) {
+    int64_t q = r, o = 0;
+    for (int p : order) {
+      o += (q % T[p]) * bst[p];
+      q /= T[p];
+    }
+    out[r] = (int32_t)o;
+  }
+  return out;
+}
+
+// flush wavefronts of one member tile: 4 consumer warps (2 x 2 of 32 x 32), each the DMMA
+// m8n8k4 accumulator layout (lane g = row i*8 + g, t = column pair 2t + h); load + store
+double flush_wavefronts(const std::vector<int32_t> &R, const std::vector<int32_t> &Q) {
+  double total = 0;
+  for (int wm = 0; wm < 2; wm++)
+    for (int wn = 0; wn < 2; wn++)
+      for (int i = 0; i < 4; i++)
+        for (int jj = 0; jj < 4; jj++)
+          for (int h = 0; h < 2; h++) {
+            std::vector<std::pair<int64_t, int>> acc;
+            for (int lane = 0; lane < 32; lane++) {
+              const int g = lane >> 2, t = lane & 3;
+              const int r = R[wm * 32 + i * 8 + g], c = Q[wn * 32 + jj * 8 + 2 * t + h];
+              if (r >= 0 && c >= 0) acc.push_back({8 * (int64_t)gbox_sw(r + c), 8});
+            }
+            if (!acc.empty()) total += 2 * smem_wavefronts(acc);
+          }
+  return total;
+}
+
+std::vector<std::vector<int>> orders_with_first(const std::vector<int> &pos, int first, size_t cap) {
+  std::vector<int> rest;
+  for (int p : pos) if (p != first) rest.push_back(p);
+  std::sort(rest.begin(), rest.end());
+  std::vector<std::vector<int>> out;
+  do {
+    std::vector<int> o;
+    if (first >= 0) o.push_back(first);
+    o.insert(o.end(), rest.begin(), rest.end());
+    out.push_back(o);
+    if (out.size() >= cap) break;
+  } while (std::next_permutation(rest.begin(), rest.end()));
+  return out;
+}
+
+}  // namespace
+
+Status plan_group(const std::vector<const Contraction *> &members, GroupTables &g, std::string &err) {
+  const auto t0 = std::chrono::steady_clock::now();
+  g = GroupTables();
+  const int n = (int)members.size();
+  if (n < 1 || n > kGMaxMembers) { err = "fused group: 1 to 32 members"; return ST_UNSUPPORTED; }
+  const Contraction &c0 = *members[0];
+  const int rank = (int)c0.t[0].idx.size();
+  if (rank < 1 || rank > kGMaxCdims) { err = "fused group: C rank must be 1..8"; return ST_UNSUPPORTED; }
+  g.rank = rank;
+  for (int p = 0; p < rank; p++) {
+    g.N[p] = c0.ix[c0.t[0].idx[p]].n;
+    g.cstride[p] = c0.t[0].stride[p];
+  }
+  g.cbase = c0.t[0].base;
+
+  // ---- members: X = the operand holding C position 0, rows / columns = the C
+  //      positions of X / Y
+  std::vector<Member> M(n);
+  for (int i = 0; i < n; i++) {
+    const Contraction &c = *members[i];
+    M[i].c = &c;
+    for (auto &ix : c.ix)
+      if (ix.cls == BATCH) { err = "fused group: batch indices are not supported"; return ST_UNSUPPORTED; }
+    if ((int)c.t[0].idx.size() != rank) { err = "fused group: C rank differs"; return ST_UNSUPPORTED; }
+    if ((int)c.t[1].idx.size() > kGMaxOpDims || (int)c.t[2].idx.size() > kGMaxOpDims) {
+      err = "fused group: operand rank > 8"; return ST_UNSUPPORTED;
+    }
+    const int id0 = c.t[0].idx[0];
+    M[i].X = c.pos_in(1, id0) >= 0 ? 1 : 2;
+    M[i].Y = 3 - M[i].X;
+    for (int p = 0; p < rank; p++) {
+      const int id = c.t[0].idx[p];
+      (c.pos_in(M[i].X, id) >= 0 ? M[i].mpos : M[i].npos).push_back(p);
+    }
+    // k digits: the operand whose FVI is internal leads (its loads run along k)
+    const auto &xv = c.t[M[i].X].idx, &yv = c.t[M[i].Y].idx;
+    const bool xk = !xv.empty() && c.ix[xv[0]].cls == INTL, yk = !yv.empty() && c.ix[yv[0]].cls == INTL;
+    const auto &ko = (!xk && yk) ? yv : xv;
+    for (int id : ko) if (c.ix[id].cls == INTL) M[i].kid.push_back(id);
+    g.flops += c.flops();
+  }
+
+  // ---- enumerate the C tile: T_p in {powers of two <= 64} u {N_p if <= 64}; prune by the
+  //      member bounds Mt_i, Nt_i <= 64; rank by tiles, then padding, then a longer C run
+  std::vector<std::vector<int32_t>> cand(rank);
+  for (int p = 0; p < rank; p++) {
+    std::set<int32_t> s;
+    for (int t = 1; t <= 64 && t <= g.N[p]; t *= 2) s.insert(t);
+    if (g.N[p] <= 64) s.insert((int32_t)g.N[p]);
+    cand[p].assign(s.begin(), s.end());
+  }
+  int32_t best[kGMaxCdims] = {}, cur[kGMaxCdims] = {};
+  double bestTiles = 0, bestPad = 0;
+  int64_t bestRun = 0;
+  bool found = false;
+  std::vector<int64_t> mprod(n, 1), nprod(n, 1);
+  std::function<void(int)> dfs = [&](int p) {
+    if (p == rank) {
+      double tiles = 1, pad = 0;
+      for (int q = 0; q < rank; q++) {
+        tiles *= (double)cdiv(g.N[q], cur[q]);
+        pad += (double)(cdiv(g.N[q], cur[q]) * cur[q] - g.N[q]) / (double)g.N[q];
+      }
+      const bool win = !found || tiles < bestTiles || (tiles == bestTiles && pad < bestPad) ||
+                       (tiles == bestTiles && pad == bestPad && cur[0] > bestRun);
+      if (win) {
+        std::copy(cur, cur + rank, best);
+        bestTiles = tiles;
+        bestPad = pad;
+        bestRun = cur[0];
+        found = true;
+      }
+      return;
+    }
+    for (int32_t t : cand[p]) {
+      bool ok = true;
+      for (int i = 0; i < n && ok; i++) {
+        const bool inX = std::find(M[i].mpos.begin(), M[i].mpos.end(), p) != M[i].mpos.end();
+        ok = (inX ? mprod[i] : nprod[i]) * t <= (inX ? kGBM : kGBN);
+      }
+      if (!ok) continue;
+      for (int i = 0; i < n; i++) {
+        const bool inX = std::find(M[i].mpos.begin(), M[i].mpos.end(), p) != M[i].mpos.end();
+        (inX ? mprod[i] : nprod[i]) *= t;
+      }
+      cur[p] = t;
+      dfs(p + 1);
+      for (int i = 0; i < n; i++) {
+        const bool inX = std::find(M[i].mpos.begin(), M[i].mpos.end(), p) != M[i].mpos.end();
+        (inX ? mprod[i] : nprod[i]) /= t;
+      }
+    }
+  };
+  dfs(0);
+  if (!found) { err = "fused group: no common C tile fits"; return ST_UNSUPPORTED; }
+  int64_t bst[kGMaxCdims];
+  g.ntiles = 1;
+  g.box = 1;
+  for (int p = 0; p < rank; p++) {
+    g.T[p] = best[p];
+    g.ntl[p] = (int32_t)cdiv(g.N[p], best[p]);
+    g.ntiles *= g.ntl[p];
+    bst[p] = g.box;
+    g.box *= best[p];
+  }
+  if (g.ntiles >= (1ll << 31)) { err = "fused group: more than 2^31 C tiles"; return ST_UNSUPPORTED; }
+
+  // ---- BK (compiled: 16 with 3 stages, 24 with 2): fewest padded k-steps; per member the
+  //      first k digit takes the tile with the fewest steps (largest such), the others fill
+  //      up to BK
+  double bestK = 0;
+  for (int BK : {24, 16}) {
+    double cost = 0;
+    for (auto &m : M) {
+      int64_t prod = 1, steps = 1;
+      for (size_t q = 0; q < m.kid.size(); q++) {
+        const int64_t nk = m.c->ix[m.kid[q]].n;
+        int64_t t;
+        if (q == 0) {
+          t = std::min<int64_t>(nk, BK);
+          const int64_t s = cdiv(nk, t);
+          t = cdiv(nk, s);                // same steps, smallest tile: the padding goes
+        } else {
+          t = std::min<int64_t>(nk, std::max<int64_t>(1, BK / prod));
+        }
+        prod *= t;
+        steps *= cdiv(nk, t);
+      }
+      cost += (double)steps * BK + 4.0 * steps;   // (+ per-step hand-off)
+    }
+    if (bestK == 0 || cost < bestK) { bestK = cost; g.BK = BK; }
+  }
+  g.stages = g.BK == 16 ? 3 : 2;
+  g.variant = g.BK == 16 ? 0 : 1;
+  const int BK = g.BK;
+  for (auto &m : M) {
+    int64_t prod = 1;
+    m.Tk.clear();
+    m.nsteps = 1;
+    for (size_t q = 0; q < m.kid.size(); q++) {
+      const int64_t nk = m.c->ix[m.kid[q]].n;
+      int64_t t;
+      if (q == 0) {
+        t = std::min<int64_t>(nk, BK);
+        t = cdiv(nk, cdiv(nk, t));
+      } else {
+        t = std::min<int64_t>(nk, std::max<int64_t>(1, BK / prod));
+      }
+      m.Tk.push_back((int)t);
+      prod *= t;
+      m.nsteps *= cdiv(nk, t);
+    }
+  }
+
+  // ---- per member: digit orders (simulated smem wavefronts), runs, steps, boxes
+  const int XS = gplane_doubles(kGBM, BK);
+  for (int i = 0; i < n; i++) {
+    Member &m = M[i];
+    const Contraction &c = *m.c;
+    const auto &xv = c.t[m.X].idx, &yv = c.t[m.Y].idx;
+    const bool xkm = !xv.empty() && c.ix[xv[0]].cls == INTL;
+    const bool ykm = !yv.empty() && c.ix[yv[0]].cls == INTL;
+    const int xf = (!xv.empty() && !xkm) ? c.pos_in(0, xv[0]) : -1;   // X's FVI leads the rows
+    const int yf = (!yv.empty() && !ykm) ? c.pos_in(0, yv[0]) : -1;
+    const auto mo = orders_with_first(m.mpos, xf, 120), no = orders_with_first(m.npos, yf, 120);
+    double bestc = 0, bestFl = 0, bestLd = 0;
+    std::vector<int> bm, bn;
+    for (auto &ro : mo)
+      for (auto &co : no) {
+        const auto R = row_box(ro, g.T, bst, kGBM), Q = row_box(co, g.T, bst, kGBN);
+        const double fl = flush_wavefronts(R, Q);
+        std::string e2;
+        bool ok1 = true, ok2 = true;
+        const Runs rx = build_runs(op_dims(m, m.X, ro, g.T, xkm, kGBM, BK), c.t[m.X].base, true, e2, ok1);
+        const Runs ry = build_runs(op_dims(m, m.Y, co, g.T, ykm, kGBN, BK), c.t[m.Y].base, true, e2, ok2);
+        if (!ok1 || !ok2) { err = e2; return ST_UNSUPPORTED; }
+        const double ld = runs_wavefronts(rx, 0) + runs_wavefronts(ry, 8ll * XS);
+        const double cost = fl + ld * (double)m.nsteps;
+        if (bm.empty() || cost < bestc) { bestc = cost; bm = ro; bn = co; bestFl = fl; bestLd = ld; }
+      }
+    g.flushWf.push_back(bestFl);
+    g.loadWf.push_back(bestLd);
+    // device records
+    GMemberDev D{};
+    D.layout = (xkm ? 1 : 0) | (ykm ? 2 : 0);
+    D.xIsA = m.X == 1;
+    auto fill_op = [&](GOperandDev &o, int t, const std::vector<int> &ord, bool km, int BMN) -> bool {
+      const auto dims = op_dims(m, t, ord, g.T, km, BMN, BK);
+      std::string e2;
+      bool ok = true;
+      Runs r = build_runs(dims, c.t[t].base, true, e2, ok);
+      if (!ok) { err = e2; return false; }
+      for (int p = 0; p < rank; p++) o.tstep[p] = (int64_t)g.T[p] * c.stride_of(t, c.t[0].idx[p]);
+      o.run0 = (int32_t)g.runRel.size();
+      o.nrun = (int32_t)r.rel.size();
+      o.runlen = r.runlen;
+      o.vec = r.vec;
+      o.ndim = (int32_t)dims.size();
+      for (int j = 0; j < kGMaxOpDims; j++) o.cpos[j] = j < (int)dims.size() ? dims[j].cpos : -1;
+      g.runRel.insert(g.runRel.end(), r.rel.begin(), r.rel.end());
+      g.runSoff.insert(g.runSoff.end(), r.soff.begin(), r.soff.end());
+      g.runDig.insert(g.runDig.end(), r.dig.begin(), r.dig.end());
+      return true;
+    };
+    if (!fill_op(D.x, m.X, bm, xkm, kGBM) || !fill_op(D.y, m.Y, bn, ykm, kGBN)) return ST_UNSUPPORTED;
+    // k steps: the k-tile grid, first k digit fastest
+    D.step0 = (int32_t)g.steps.size();
+    D.nsteps = (int32_t)m.nsteps;
+    {
+      const size_t nk = m.kid.size();
+      std::vector<int64_t> od(nk, 0);
+      for (;;) {
+        GStepDev s{};
+        s.full = 1;
+        for (size_t q = 0; q < nk; q++) {
+          const int id = m.kid[q];
+          const int64_t o = od[q] * m.Tk[q], lim = std::min<int64_t>(m.Tk[q], c.ix[id].n - o);
+          s.kx += o * c.stride_of(m.X, id);
+          s.ky += o * c.stride_of(m.Y, id);
+          if (lim != m.Tk[q]) s.full = 0;
+          const int jx = c.pos_in(m.X, id), jy = c.pos_in(m.Y, id);
+          s.klimX |= (uint64_t)lim << (8 * jx);
+          s.klimY |= (uint64_t)lim << (8 * jy);
+        }
+        g.steps.push_back(s);
+        size_t q = 0;
+        for (; q < nk; q++) {
+          if (++od[q] < cdiv(c.ix[m.kid[q]].n, m.Tk[q])) break;
+          od[q] = 0;
+        }
+        if (q == nk) break;
+      }
+    }
+    // k padding (Kt < BK): zero the k rows / columns [Kt, BK) of both planes every step
+    int64_t Kt = 1;
+    for (int t : m.Tk) Kt *= t;
+    D.pad0 = (int32_t)g.pad.size();
+    if (Kt < BK) {
+      for (int plane = 0; plane < 2; plane++) {
+        const bool km = plane == 0 ? xkm : ykm;
+        const int BMN = plane == 0 ? kGBM : kGBN;
+        for (int64_t row = 0; row < BMN; row++)
+          for (int64_t k = Kt; k < BK; k++)
+            g.pad.push_back((uint32_t)(8 * (plane_off(km, row, k, BMN, BK) + (plane ? XS : 0))));
+      }
+    }
+    D.npad = (int32_t)g.pad.size() - D.pad0;
+    const auto R = row_box(bm, g.T, bst, kGBM), Q = row_box(bn, g.T, bst, kGBN);
+    g.boxM.insert(g.boxM.end(), R.begin(), R.end());
+    g.boxN.insert(g.boxN.end(), Q.begin(), Q.end());
+    g.mem.push_back(D);
+    int64_t Mt = 1, Nt = 1;
+    for (int p : m.mpos) Mt *= g.T[p];
+    for (int p : m.npos) Nt *= g.T[p];
+    g.Mt.push_back(Mt);
+    g.Nt.push_back(Nt);
+    g.Kt.push_back(Kt);
+    g.padded_flops += 2.0 * (double)g.ntiles * (double)m.nsteps * kGBM * kGBN * BK;
+  }
+
+  // ---- copy-out units: the box in C order, 2 elements per unit when 16-B stores are legal
+  bool u2 = g.T[0] % 2 == 0 && g.N[0] % 2 == 0 && g.cstride[0] == 1 && g.cbase % 2 == 0;
+  for (int p = 1; p < rank; p++) u2 &= g.cstride[p] % 2 == 0;
+  g.uvec = u2 ? 2 : 1;
+  for (int64_t o = 0; o < g.box; o += g.uvec) {
+    int64_t q = o, rel = 0;
+    uint64_t dg = 0;
+    for (int p = 0; p < rank; p++) {
+      const int64_t d = q % g.T[p];
+      q /= g.T[p];
+      rel += d * g.cstride[p];
+      dg |= (uint64_t)d << (8 * p);
+    }
+    g.unitRel.push_back(rel);
+    g.unitDig.push_back(dg);
+  }
+  g.plan_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  return ST_OK;
+}
+
+}  // namespace tc

@@ -254,3 +254,39 @@ def test_paper_mode_lists_tuning_candidates():
         i = tc.plan("abcd-aebf-dfce", ext, cost="paper", host_only=True).info()
         pv = i["stats"]["per_variant"]
         assert len(pv) >= 2 and [t for _, t in pv] == sorted(t for _, t in pv)
+
+
+def test_group_plan_triples_host():
+    """Fused group planning (NEXT-4) of the 18 CCSD(T) triples without a GPU: one 4^6 C tile
+    makes every member a 64 x 64 DMMA tile (3 C indices per operand), BK follows the internal
+    extent, and the simulated flush of every member into the swizzled box is conflict-free
+    (4 warps x 32 accesses x load+store x 2 wavefronts = 512)."""
+    exprs = [c.expr for c in tcinputs.tccg48() if c.group.startswith("CCSDT")]
+    for ext, bk in (("a:24;b:16;c:16;d:24;e:16;f:16;g:24", 24), (";".join(f"{x}:16" for x in "abcdefg"), 16)):
+        g = tc.plan_group([tc.plan(e, ext, host_only=True) for e in exprs])
+        i = g.info()
+        assert i["T"] == [4] * 6 and i["BK"] == bk and i["box"] == 4096
+        assert all(m["Mt"] == 64 and m["Nt"] == 64 and m["nsteps"] == 1 for m in i["per_member"])
+        assert all(m["flush_wf"] == 512 for m in i["per_member"])
+        # FVI runs: 16-B vectors on both operands of every member (aligned extents)
+        assert all(m["vecX"] == 2 and m["vecY"] == 2 for m in i["per_member"])
+        with pytest.raises(tc.TcError) as e:                     # planned, not executable
+            g.execute_ptr([1 << 40] * 18, [1 << 41] * 18, 1 << 42)
+        assert e.value.status == "TC_ERR_CUDA"
+
+
+def test_group_plan_errors_host():
+    ext = "a:6;b:5;c:7;d:6;e:5;f:7;g:9"
+    p = tc.plan("abcdef-gdab-efgc", ext, host_only=True)
+    with pytest.raises(tc.TcError) as e:
+        tc.plan_group([])
+    assert e.value.status == "TC_ERR_INVALID_ARG"
+    with pytest.raises(tc.TcError) as e:                         # C laid out differently
+        tc.plan_group([p, tc.plan("abcdef-gdab-efgc", "a:6;b:5;c:7;d:6;e:5;f:8;g:9", host_only=True)])
+    assert e.value.status == "TC_ERR_INVALID_ARG"
+    with pytest.raises(tc.TcError) as e:                         # batch index
+        tc.plan_group([tc.plan("abc-abd-cbd", "a:4;b:4;c:4;d:4", host_only=True)])
+    assert e.value.status == "TC_ERR_UNSUPPORTED"
+    with pytest.raises(tc.TcError) as e:                         # an operand of rank 9 (> 8)
+        tc.plan_group([tc.plan("abcdefgh-abcdefghi-i", ";".join(f"{x}:2" for x in "abcdefghi"), host_only=True)])
+    assert e.value.status == "TC_ERR_UNSUPPORTED"
