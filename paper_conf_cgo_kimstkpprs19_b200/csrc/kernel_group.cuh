@@ -206,8 +206,9 @@ tc_f64_group_kernel(const __grid_constant__ GParams p) {
         const double *__restrict__ Yb = p.Y[i] + tile.off(M.y.tstep, p.rank);
         const int vx = ((p.vecmask >> (2 * i)) & 1) ? M.x.vec : 1;
         const int vy = ((p.vecmask >> (2 * i + 1)) & 1) ? M.y.vec : 1;
-        const uint64_t Lx = tile.interior ? 0 : g_op_lims(M.x, tile.Lc);
-        const uint64_t Ly = tile.interior ? 0 : g_op_lims(M.y, tile.Lc);
+        // (needed by partial k-steps of interior tiles too)
+        const uint64_t Lx = g_op_lims(M.x, tile.Lc);
+        const uint64_t Ly = g_op_lims(M.y, tile.Lc);
         for (int s = 0; s < M.nsteps; s++, j++) {
           const int st = j % STAGES;
           if (j >= STAGES) mbar_wait(bar0 + 8 * (STAGES + st), ((j / STAGES) & 1) ^ 1);
