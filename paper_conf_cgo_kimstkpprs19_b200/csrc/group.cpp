@@ -4,8 +4,10 @@
 // SHARED output: one tile T_p per C position, such that every member's Mt_i (product over
 // the C positions of its operand X_i) and Nt_i fit the 64 x 64 DMMA register tiles; ranked
 // by the number of C tiles (each tile costs every member's k-steps once) and padding.  Per
-// member, the digit orders of rows and columns are chosen by simulating the shared-memory
-// wavefronts of the member's cp.async stage writes and of its flush into the swizzled box.
+// member and per load mode (TMA boxes / cp.async gathers), the digit order of rows and
+// columns is chosen by simulating the shared-memory wavefronts of the stage writes (cp.async),
+// of the DMMA fragment loads (TMA: swizzled boxes in the operand's own order) and of the
+// member's read-modify-write of the swizzled C box.
 #include "group.hpp"
 
 #include <algorithm>
@@ -26,16 +28,20 @@ int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 // wavefront.
 double smem_wavefronts(const std::vector<std::pair<int64_t, int>> &acc) {
   double total = 0;
+  std::vector<int64_t> words[32];
   for (size_t b = 0; b < acc.size(); b += 32) {
     const size_t e = std::min(acc.size(), b + 32);
-    std::set<int64_t> words[32];
+    for (auto &w : words) w.clear();
     int64_t bytes = 0;
     for (size_t i = b; i < e; i++) {
-      for (int64_t w = acc[i].first / 4; w < (acc[i].first + acc[i].second + 3) / 4; w++) words[w & 31].insert(w);
+      for (int64_t w = acc[i].first / 4; w < (acc[i].first + acc[i].second + 3) / 4; w++) words[w & 31].push_back(w);
       bytes += acc[i].second;
     }
     size_t wf = 0;
-    for (auto &s : words) wf = std::max(wf, s.size());
+    for (auto &s : words) {
+      std::sort(s.begin(), s.end());
+      wf = std::max(wf, (size_t)(std::unique(s.begin(), s.end()) - s.begin()));
+    }
     total += (double)std::max<int64_t>((int64_t)wf, (bytes + 127) / 128);
   }
   return total;
@@ -50,21 +56,31 @@ struct Member {
   int64_t nsteps = 1;
 };
 
-// Operand description for run building: dims in the operand's memory order.
+// Operand description: dims in the operand's memory order.
 struct OpDim {
   int id;          // member-local index id
   int cpos;        // C position, or -1 (internal)
   int64_t tile, n, gstride, sstride;
 };
 
-// smem element offset of (row, k) in a plane: k-major rows of pitch BK + 4, or mn-major k
-// rows of pitch BMN + 4 (4 mod 16 doubles: conflict-free DMMA fragment loads, as in the
-// single-contraction kernel).
+// cp.async planes: smem element offset of (row, k) — k-major rows of pitch BK + 4, or
+// mn-major k rows of pitch BMN + 4 (4 mod 16 doubles: conflict-free DMMA fragment loads, as
+// in the single-contraction kernel).
 int64_t plane_off(bool kmajor, int64_t row, int64_t k, int BMN, int BK) {
   return kmajor ? row * (BK + 4) + k : k * (BMN + 4) + row;
 }
 
-// The dims of operand t of member M with the given row-digit order (C positions) and tiles.
+// row multiplier of C position p in a digit order (product of the tiles before it)
+int64_t row_mul(const std::vector<int> &ord, const int32_t *T, int p) {
+  int64_t mul = 1;
+  for (int q : ord) {
+    if (q == p) break;
+    mul *= T[q];
+  }
+  return mul;
+}
+
+// The dims of operand t of member M (cp.async planes: sstride = smem element stride).
 std::vector<OpDim> op_dims(const Member &M, int t, const std::vector<int> &roword, const int32_t *T,
                            bool kmajor, int BMN, int BK) {
   const Contraction &c = *M.c;
@@ -72,15 +88,11 @@ std::vector<OpDim> op_dims(const Member &M, int t, const std::vector<int> &rowor
   for (size_t j = 0; j < c.t[t].idx.size(); j++) {
     const int id = c.t[t].idx[j];
     OpDim o{id, c.pos_in(0, id), 1, c.ix[id].n, c.t[t].stride[j], 0};
-    int64_t mul = 1;
     if (o.cpos >= 0) {
       o.tile = T[o.cpos];
-      for (int p : roword) {
-        if (p == o.cpos) break;
-        mul *= T[p];
-      }
-      o.sstride = plane_off(kmajor, mul, 0, BMN, BK);
+      o.sstride = plane_off(kmajor, row_mul(roword, T, o.cpos), 0, BMN, BK);
     } else {
+      int64_t mul = 1;
       for (size_t q = 0; q < M.kid.size(); q++) {
         if (M.kid[q] == id) { o.tile = M.Tk[q]; break; }
         mul *= M.Tk[q];
@@ -99,8 +111,9 @@ struct Runs {
   int runlen = 1, vec = 1;
 };
 
-// Runs along dim 0 (when it is smem-contiguous), enumerated over dims 1.. (first fastest).
-Runs build_runs(const std::vector<OpDim> &d, int64_t base, bool vec_ok, std::string &err, bool &ok) {
+// cp.async runs along dim 0 (when it is smem-contiguous), enumerated over dims 1.. (first
+// fastest).
+Runs build_runs(const std::vector<OpDim> &d, int64_t base, std::string &err, bool &ok) {
   Runs r;
   ok = true;
   if (d.empty()) {
@@ -112,7 +125,7 @@ Runs build_runs(const std::vector<OpDim> &d, int64_t base, bool vec_ok, std::str
   const bool contiguous = d[0].sstride == 1;
   r.runlen = contiguous ? (int)d[0].tile : 1;
   const size_t first = contiguous ? 1 : 0;
-  bool ev = vec_ok && contiguous && d[0].tile % 2 == 0 && d[0].n % 2 == 0 && base % 2 == 0;
+  bool ev = contiguous && d[0].tile % 2 == 0 && d[0].n % 2 == 0 && base % 2 == 0;
   for (size_t j = 1; j < d.size(); j++) ev &= d[j].gstride % 2 == 0;
   r.vec = ev ? 2 : 1;
   std::vector<int64_t> dg(d.size(), 0);
@@ -147,24 +160,32 @@ double runs_wavefronts(const Runs &r, int64_t plane_byte0) {
   return smem_wavefronts(acc);
 }
 
+// digit values of row r in a digit order
+std::vector<int64_t> row_digits(int64_t r, const std::vector<int> &order, const int32_t *T) {
+  std::vector<int64_t> d(kGMaxCdims, 0);
+  for (int p : order) {
+    d[p] = r % T[p];
+    r /= T[p];
+  }
+  return d;
+}
+
 // box offset of every row (column) of a member tile, from the digit order and the tiles
 std::vector<int32_t> row_box(const std::vector<int> &order, const int32_t *T, const int64_t *bst, int BMN) {
   std::vector<int32_t> out(BMN, -1);
   int64_t tot = 1;
   for (int p : order) tot *= T[p];
   for (int64_t r = 0; r < tot && r < BMN; r++) {
-    int64_t q = r, o = 0;
-    for (int p : order) {
-      o += (q % T[p]) * bst[p];
-      q /= T[p];
-    }
+    const auto d = row_digits(r, order, T);
+    int64_t o = 0;
+    for (int p : order) o += d[p] * bst[p];
     out[r] = (int32_t)o;
   }
   return out;
 }
 
-// flush wavefronts of one member tile: 4 consumer warps (2 x 2 of 32 x 32), each the DMMA
-// m8n8k4 accumulator layout (lane g = row i*8 + g, t = column pair 2t + h); load + store
+// member RMW of the box: 4 consumer warps (2 x 2 of 32 x 32), each the DMMA m8n8k4
+// accumulator layout (lane g = row i*8 + g, t = column pair 2t + h); load + store
 double flush_wavefronts(const std::vector<int32_t> &R, const std::vector<int32_t> &Q) {
   double total = 0;
   for (int wm = 0; wm < 2; wm++)
@@ -180,6 +201,82 @@ double flush_wavefronts(const std::vector<int32_t> &R, const std::vector<int32_t
             }
             if (!acc.empty()) total += 2 * smem_wavefronts(acc);
           }
+  return total;
+}
+
+// TMA box layout of one operand: the tensor map lists the operand's dims in the order perm
+// (perm[0] = 0, the FVI; dims 1.. permuted — the map's strides need not grow), the box is the
+// tile (a k-FVI box padded to a pitch of 4 mod 8 doubles), dense in smem in the map's order,
+// no swizzle: the order is chosen so that the DMMA fragment loads are conflict-free.
+struct TmaLayout {
+  bool ok = false;
+  std::vector<int> perm;        // map dim j -> operand dim perm[j]
+  std::vector<int64_t> box;     // box extent per map dim
+  std::vector<int64_t> bs;      // element stride inside the box of each OPERAND dim
+  int64_t bytes = 0;
+  int64_t byte(const std::vector<int64_t> &d) const {
+    int64_t o = 0;
+    for (size_t j = 0; j < d.size(); j++) o += d[j] * bs[j];
+    return 8 * o;
+  }
+};
+
+int64_t kpitch(int64_t t) {   // smallest p >= t with p = 4 (mod 8): conflict-free k-major rows
+  int64_t p = t;
+  while (p % 8 != 4) p++;
+  return p;
+}
+
+bool tma_eligible(const std::vector<OpDim> &d, int64_t base) {
+  if (d.empty() || d.size() > (size_t)kGMaxTmaDims || d[0].gstride != 1 || base % 2 != 0) return false;
+  if (d[0].cpos >= 0 && d[0].tile % 2 != 0) return false;          // box dim 0: 16-B multiple
+  for (size_t j = 1; j < d.size(); j++)
+    if (d[j].gstride % 2 != 0 || d[j].gstride * 8 >= (1ll << 40)) return false;
+  for (auto &x : d)
+    if (x.n >= (1ll << 32) || x.tile > 256 || kpitch(x.tile) > 256) return false;
+  return true;
+}
+
+TmaLayout tma_make(const std::vector<OpDim> &d, const std::vector<int> &perm) {
+  TmaLayout L;
+  L.perm = perm;
+  L.box.assign(d.size(), 1);
+  L.bs.assign(d.size(), 0);
+  int64_t m = 1;
+  for (size_t j = 0; j < perm.size(); j++) {
+    const OpDim &x = d[perm[j]];
+    L.box[j] = (j == 0 && x.cpos < 0) ? kpitch(x.tile) : x.tile;
+    L.bs[perm[j]] = m;
+    m *= L.box[j];
+  }
+  L.bytes = 8 * m;
+  L.ok = true;
+  return L;
+}
+
+// DMMA fragment-load wavefronts of one operand tile in smem: per row group i (8 rows) and k4
+// step, thread (g, t) loads element (row 8i + g, k 4kk + t); rowe / ke are element offsets;
+// 32 doubles need >= 2 wavefronts, and each bank pair serves one distinct double per wavefront
+double frag_wavefronts(const std::vector<int64_t> &rowe, const std::vector<int64_t> &ke, int kq) {
+  double total = 0;
+  for (int i = 0; i < 8; i++)
+    for (int kk = 0; kk < kq; kk++) {
+      int64_t seen[16][32];
+      int cnt[16] = {0};
+      int wf = 2;
+      for (int lane = 0; lane < 32; lane++) {
+        const int g = lane >> 2, t = lane & 3;
+        const int64_t a = rowe[i * 8 + g] + ke[kk * 4 + t];
+        const int b = (int)(a & 15);
+        bool dup = false;
+        for (int q = 0; q < cnt[b]; q++) dup |= seen[b][q] == a;
+        if (!dup) {
+          seen[b][cnt[b]++] = a;
+          wf = std::max(wf, cnt[b]);
+        }
+      }
+      total += wf;
+    }
   return total;
 }
 
@@ -251,6 +348,9 @@ Status plan_group(const std::vector<const Contraction *> &members, GroupTables &
     if (g.N[p] <= 64) s.insert((int32_t)g.N[p]);
     cand[p].assign(s.begin(), s.end());
   }
+  std::vector<std::vector<char>> inX(n, std::vector<char>(rank, 0));
+  for (int i = 0; i < n; i++)
+    for (int p : M[i].mpos) inX[i][p] = 1;
   int32_t best[kGMaxCdims] = {}, cur[kGMaxCdims] = {};
   double bestTiles = 0, bestPad = 0;
   int64_t bestRun = 0;
@@ -276,21 +376,12 @@ Status plan_group(const std::vector<const Contraction *> &members, GroupTables &
     }
     for (int32_t t : cand[p]) {
       bool ok = true;
-      for (int i = 0; i < n && ok; i++) {
-        const bool inX = std::find(M[i].mpos.begin(), M[i].mpos.end(), p) != M[i].mpos.end();
-        ok = (inX ? mprod[i] : nprod[i]) * t <= (inX ? kGBM : kGBN);
-      }
+      for (int i = 0; i < n && ok; i++) ok = (inX[i][p] ? mprod[i] : nprod[i]) * t <= (inX[i][p] ? kGBM : kGBN);
       if (!ok) continue;
-      for (int i = 0; i < n; i++) {
-        const bool inX = std::find(M[i].mpos.begin(), M[i].mpos.end(), p) != M[i].mpos.end();
-        (inX ? mprod[i] : nprod[i]) *= t;
-      }
+      for (int i = 0; i < n; i++) (inX[i][p] ? mprod[i] : nprod[i]) *= t;
       cur[p] = t;
       dfs(p + 1);
-      for (int i = 0; i < n; i++) {
-        const bool inX = std::find(M[i].mpos.begin(), M[i].mpos.end(), p) != M[i].mpos.end();
-        (inX ? mprod[i] : nprod[i]) /= t;
-      }
+      for (int i = 0; i < n; i++) (inX[i][p] ? mprod[i] : nprod[i]) /= t;
     }
   };
   dfs(0);
@@ -307,91 +398,146 @@ Status plan_group(const std::vector<const Contraction *> &members, GroupTables &
   }
   if (g.ntiles >= (1ll << 31)) { err = "fused group: more than 2^31 C tiles"; return ST_UNSUPPORTED; }
 
-  // ---- BK (compiled: 16 with 3 stages, 24 with 2): fewest padded k-steps; per member the
-  //      first k digit takes the tile with the fewest steps (largest such), the others fill
-  //      up to BK
-  double bestK = 0;
-  for (int BK : {24, 16}) {
-    double cost = 0;
-    for (auto &m : M) {
-      int64_t prod = 1, steps = 1;
-      for (size_t q = 0; q < m.kid.size(); q++) {
-        const int64_t nk = m.c->ix[m.kid[q]].n;
-        int64_t t;
-        if (q == 0) {
-          t = std::min<int64_t>(nk, BK);
-          const int64_t s = cdiv(nk, t);
-          t = cdiv(nk, s);                // same steps, smallest tile: the padding goes
-        } else {
-          t = std::min<int64_t>(nk, std::max<int64_t>(1, BK / prod));
-        }
-        prod *= t;
-        steps *= cdiv(nk, t);
-      }
-      cost += (double)steps * BK + 4.0 * steps;   // (+ per-step hand-off)
-    }
-    if (bestK == 0 || cost < bestK) { bestK = cost; g.BK = BK; }
-  }
-  g.stages = g.BK == 16 ? 3 : 2;
-  g.variant = g.BK == 16 ? 0 : 1;
-  const int BK = g.BK;
-  for (auto &m : M) {
-    int64_t prod = 1;
-    m.Tk.clear();
-    m.nsteps = 1;
+  // ---- BK (compiled: 16 and 24): fewest padded k-steps; per member the first k digit takes
+  //      the tile with the fewest steps (the smallest such), the others fill up to BK
+  auto ktiles = [&](const Member &m, int BK, std::vector<int> &Tk) {
+    int64_t prod = 1, steps = 1;
+    Tk.clear();
     for (size_t q = 0; q < m.kid.size(); q++) {
       const int64_t nk = m.c->ix[m.kid[q]].n;
       int64_t t;
       if (q == 0) {
         t = std::min<int64_t>(nk, BK);
-        t = cdiv(nk, cdiv(nk, t));
+        t = cdiv(nk, cdiv(nk, t));      // same steps, smallest tile: the padding goes
       } else {
         t = std::min<int64_t>(nk, std::max<int64_t>(1, BK / prod));
       }
-      m.Tk.push_back((int)t);
+      Tk.push_back((int)t);
       prod *= t;
-      m.nsteps *= cdiv(nk, t);
+      steps *= cdiv(nk, t);
     }
+    return steps;
+  };
+  double bestK = 0;
+  for (int BK : {24, 16}) {
+    double cost = 0;
+    std::vector<int> Tk;
+    for (auto &m : M) {
+      const int64_t steps = ktiles(m, BK, Tk);
+      cost += (double)steps * BK + 4.0 * steps;   // (+ per-step hand-off)
+    }
+    if (bestK == 0 || cost < bestK) { bestK = cost; g.BK = BK; }
   }
+  g.variant = g.BK == 16 ? 0 : 1;
+  const int BK = g.BK;
+  for (auto &m : M) m.nsteps = ktiles(m, BK, m.Tk);
 
-  // ---- per member: digit orders (simulated smem wavefronts), runs, steps, boxes
+  // ---- per member: digit orders (simulated smem wavefronts), runs, TMA boxes, steps, tables
   const int XS = gplane_doubles(kGBM, BK);
+  g.tma = true;
+  std::vector<TmaLayout> tlx(n), tly(n);
+  std::vector<std::vector<int>> tord_m(n), tord_n(n), cord_m(n), cord_n(n);
   for (int i = 0; i < n; i++) {
     Member &m = M[i];
     const Contraction &c = *m.c;
     const auto &xv = c.t[m.X].idx, &yv = c.t[m.Y].idx;
     const bool xkm = !xv.empty() && c.ix[xv[0]].cls == INTL;
     const bool ykm = !yv.empty() && c.ix[yv[0]].cls == INTL;
-    const int xf = (!xv.empty() && !xkm) ? c.pos_in(0, xv[0]) : -1;   // X's FVI leads the rows
+    int64_t Kt = 1;
+    for (int t : m.Tk) Kt *= t;
+    const int kq = (int)cdiv(Kt, 4);
+    // (a) cp.async planes: rows led by the operand's FVI (runs are smem-contiguous)
+    const int xf = (!xv.empty() && !xkm) ? c.pos_in(0, xv[0]) : -1;
     const int yf = (!yv.empty() && !ykm) ? c.pos_in(0, yv[0]) : -1;
-    const auto mo = orders_with_first(m.mpos, xf, 120), no = orders_with_first(m.npos, yf, 120);
     double bestc = 0, bestFl = 0, bestLd = 0;
-    std::vector<int> bm, bn;
-    for (auto &ro : mo)
-      for (auto &co : no) {
+    for (auto &ro : orders_with_first(m.mpos, xf, 120))
+      for (auto &co : orders_with_first(m.npos, yf, 120)) {
         const auto R = row_box(ro, g.T, bst, kGBM), Q = row_box(co, g.T, bst, kGBN);
         const double fl = flush_wavefronts(R, Q);
-        std::string e2;
         bool ok1 = true, ok2 = true;
-        const Runs rx = build_runs(op_dims(m, m.X, ro, g.T, xkm, kGBM, BK), c.t[m.X].base, true, e2, ok1);
-        const Runs ry = build_runs(op_dims(m, m.Y, co, g.T, ykm, kGBN, BK), c.t[m.Y].base, true, e2, ok2);
-        if (!ok1 || !ok2) { err = e2; return ST_UNSUPPORTED; }
+        const Runs rx = build_runs(op_dims(m, m.X, ro, g.T, xkm, kGBM, BK), c.t[m.X].base, err, ok1);
+        const Runs ry = build_runs(op_dims(m, m.Y, co, g.T, ykm, kGBN, BK), c.t[m.Y].base, err, ok2);
+        if (!ok1 || !ok2) return ST_UNSUPPORTED;
         const double ld = runs_wavefronts(rx, 0) + runs_wavefronts(ry, 8ll * XS);
         const double cost = fl + ld * (double)m.nsteps;
-        if (bm.empty() || cost < bestc) { bestc = cost; bm = ro; bn = co; bestFl = fl; bestLd = ld; }
+        if (cord_m[i].empty() || cost < bestc) { bestc = cost; cord_m[i] = ro; cord_n[i] = co; bestFl = fl; bestLd = ld; }
       }
     g.flushWf.push_back(bestFl);
     g.loadWf.push_back(bestLd);
-    // device records
+    // (b) TMA boxes (one internal index, Kt a multiple of 4): per operand the map's dim order
+    //     and the row order with the fewest fragment-load wavefronts, then among those the
+    //     pair with the cheapest box read-modify-write
+    const auto dx = op_dims(m, m.X, m.mpos, g.T, false, kGBM, BK), dy = op_dims(m, m.Y, m.npos, g.T, false, kGBN, BK);
+    const bool tok = m.kid.size() <= 1 && Kt % 4 == 0 && tma_eligible(dx, c.t[m.X].base) &&
+                     tma_eligible(dy, c.t[m.Y].base);
+    g.tma = g.tma && tok;
+    double bestT = -1;
+    if (tok) {
+      const int kidx = m.kid.empty() ? -1 : m.kid[0];
+      struct Cand { TmaLayout L; std::vector<int> ord; double wf; };
+      auto search = [&](int t, const std::vector<OpDim> &d, const std::vector<int> &pos, int BMN) {
+        std::vector<int> rest;
+        for (size_t q = 1; q < d.size(); q++) rest.push_back((int)q);
+        std::vector<Cand> all;
+        double bestwf = -1;
+        do {
+          std::vector<int> perm{0};
+          perm.insert(perm.end(), rest.begin(), rest.end());
+          const TmaLayout L = tma_make(d, perm);
+          const int jk = kidx >= 0 ? c.pos_in(t, kidx) : -1;
+          std::vector<int64_t> ke(32, 0);
+          for (int k = 0; k < 32; k++) ke[k] = jk >= 0 ? (k < Kt ? k : 0) * L.bs[jk] : 0;
+          for (auto &ord : orders_with_first(pos, -1, 120)) {
+            std::vector<int64_t> rowe(BMN, 0);
+            int64_t tot = 1;
+            for (int p : ord) tot *= g.T[p];
+            for (int64_t r = 0; r < tot && r < BMN; r++) {
+              const auto dg = row_digits(r, ord, g.T);
+              for (size_t q = 0; q < d.size(); q++)
+                if (d[q].cpos >= 0) rowe[r] += dg[d[q].cpos] * L.bs[q];
+            }
+            const double wf = frag_wavefronts(rowe, ke, (int)cdiv(Kt, 4));
+            if (bestwf < 0 || wf < bestwf) { bestwf = wf; all.clear(); }
+            if (wf == bestwf && all.size() < 16) all.push_back({L, ord, wf});
+          }
+        } while (std::next_permutation(rest.begin(), rest.end()));
+        return all;
+      };
+      const auto cx = search(m.X, dx, m.mpos, kGBM), cy = search(m.Y, dy, m.npos, kGBN);
+      for (auto &a : cx)
+        for (auto &b : cy) {
+          const double cost = flush_wavefronts(row_box(a.ord, g.T, bst, kGBM), row_box(b.ord, g.T, bst, kGBN)) +
+                              (double)m.nsteps * (a.wf + b.wf) * 4;
+          if (bestT < 0 || cost < bestT) {
+            bestT = cost;
+            tlx[i] = a.L;
+            tly[i] = b.L;
+            tord_m[i] = a.ord;
+            tord_n[i] = b.ord;
+          }
+        }
+      g.tma_stage_bytes = (int)std::max<int64_t>(g.tma_stage_bytes, (tlx[i].bytes + 127) / 128 * 128 + tly[i].bytes);
+    }
+    g.fragWf.push_back(bestT);
+  }
+
+  for (int i = 0; i < n; i++) {
+    Member &m = M[i];
+    const Contraction &c = *m.c;
+    const auto &xv = c.t[m.X].idx, &yv = c.t[m.Y].idx;
+    const bool xkm = !xv.empty() && c.ix[xv[0]].cls == INTL;
+    const bool ykm = !yv.empty() && c.ix[yv[0]].cls == INTL;
+    int64_t Kt = 1;
+    for (int t : m.Tk) Kt *= t;
     GMemberDev D{};
-    D.layout = (xkm ? 1 : 0) | (ykm ? 2 : 0);
     D.xIsA = m.X == 1;
+    D.kq = (int32_t)cdiv(Kt, 4);
+    // cp.async side: runs in the cp.async digit order
     auto fill_op = [&](GOperandDev &o, int t, const std::vector<int> &ord, bool km, int BMN) -> bool {
       const auto dims = op_dims(m, t, ord, g.T, km, BMN, BK);
-      std::string e2;
       bool ok = true;
-      Runs r = build_runs(dims, c.t[t].base, true, e2, ok);
-      if (!ok) { err = e2; return false; }
+      Runs r = build_runs(dims, c.t[t].base, err, ok);
+      if (!ok) return false;
       for (int p = 0; p < rank; p++) o.tstep[p] = (int64_t)g.T[p] * c.stride_of(t, c.t[0].idx[p]);
       o.run0 = (int32_t)g.runRel.size();
       o.nrun = (int32_t)r.rel.size();
@@ -402,9 +548,45 @@ Status plan_group(const std::vector<const Contraction *> &members, GroupTables &
       g.runRel.insert(g.runRel.end(), r.rel.begin(), r.rel.end());
       g.runSoff.insert(g.runSoff.end(), r.soff.begin(), r.soff.end());
       g.runDig.insert(g.runDig.end(), r.dig.begin(), r.dig.end());
+      // consumer k addressing, cp.async planes: k is linear in the plane (k-major: 1 element
+      // per k, mn-major: a pitch per k); no chunks, no swizzle
+      o.kch_log2[0] = 30;
+      o.kchunk[0] = 0;
+      o.kmul[0] = 8 * (km ? 1 : BMN + 4);
+      o.swz[0] = 0;
       return true;
     };
-    if (!fill_op(D.x, m.X, bm, xkm, kGBM) || !fill_op(D.y, m.Y, bn, ykm, kGBN)) return ST_UNSUPPORTED;
+    if (!fill_op(D.x, m.X, cord_m[i], xkm, kGBM) || !fill_op(D.y, m.Y, cord_n[i], ykm, kGBN)) return ST_UNSUPPORTED;
+    // TMA side
+    auto fill_tma = [&](GOperandDev &o, int t, const TmaLayout &L, std::vector<GroupTables::TmaSpec> &spec) {
+      GroupTables::TmaSpec s;
+      for (int j = 0; j < kGMaxTmaDims; j++) o.tma_cpos[j] = -1;
+      o.tma_kdim = -1;
+      if (g.tma) {
+        const auto dims = op_dims(m, t, m.X == t ? tord_m[i] : tord_n[i], g.T, false, kGBM, BK);
+        s.rank = (int)dims.size();
+        for (int j = 0; j < s.rank; j++) {   // map dim j = operand dim perm[j]
+          const OpDim &x = dims[L.perm[j]];
+          s.dims[j] = (uint64_t)x.n;
+          if (j > 0) s.strides[j - 1] = (uint64_t)(8 * x.gstride);
+          s.box[j] = (uint32_t)L.box[j];
+          o.tma_cpos[j] = x.cpos;
+          if (x.cpos < 0) o.tma_kdim = j;
+        }
+        s.base = c.t[t].base;
+        o.tma_tx = (int32_t)L.bytes;
+        const int kidx = m.kid.empty() ? -1 : m.kid[0];
+        const int jk = kidx >= 0 ? c.pos_in(t, kidx) : -1;
+        o.kch_log2[1] = 30;                 // one box: k is linear in it
+        o.kchunk[1] = 0;
+        o.kmul[1] = jk >= 0 ? (int32_t)(8 * L.bs[jk]) : 0;
+        o.swz[1] = 0;
+      }
+      spec.push_back(s);
+    };
+    fill_tma(D.x, m.X, tlx[i], g.tmaX);
+    fill_tma(D.y, m.Y, tly[i], g.tmaY);
+    D.tma_yoff = g.tma ? (int32_t)((tlx[i].bytes + 127) / 128 * 128) : 0;
     // k steps: the k-tile grid, first k digit fastest
     D.step0 = (int32_t)g.steps.size();
     D.nsteps = (int32_t)m.nsteps;
@@ -423,6 +605,7 @@ Status plan_group(const std::vector<const Contraction *> &members, GroupTables &
           const int jx = c.pos_in(m.X, id), jy = c.pos_in(m.Y, id);
           s.klimX |= (uint64_t)lim << (8 * jx);
           s.klimY |= (uint64_t)lim << (8 * jy);
+          if (q == 0) s.kc = (int32_t)o;   // (TMA groups have one internal index)
         }
         g.steps.push_back(s);
         size_t q = 0;
@@ -433,9 +616,7 @@ Status plan_group(const std::vector<const Contraction *> &members, GroupTables &
         if (q == nk) break;
       }
     }
-    // k padding (Kt < BK): zero the k rows / columns [Kt, BK) of both planes every step
-    int64_t Kt = 1;
-    for (int t : m.Tk) Kt *= t;
+    // cp.async k padding (Kt < BK): zero the k rows / columns [Kt, BK) of both planes
     D.pad0 = (int32_t)g.pad.size();
     if (Kt < BK) {
       for (int plane = 0; plane < 2; plane++) {
@@ -447,9 +628,49 @@ Status plan_group(const std::vector<const Contraction *> &members, GroupTables &
       }
     }
     D.npad = (int32_t)g.pad.size() - D.pad0;
-    const auto R = row_box(bm, g.T, bst, kGBM), Q = row_box(bn, g.T, bst, kGBN);
-    g.boxM.insert(g.boxM.end(), R.begin(), R.end());
-    g.boxN.insert(g.boxN.end(), Q.begin(), Q.end());
+    // consumer tables per mode: row bytes of X / Y in the plane, box offsets of rows / columns
+    for (int mode = 0; mode < 2; mode++) {
+      const auto &om = mode ? tord_m[i] : cord_m[i];
+      const auto &on = mode ? tord_n[i] : cord_n[i];
+      // rows outside the member's tile load from a valid plane address (0) and are never
+      // written back (box offset -1)
+      std::vector<int32_t> tab(kGCtab, -1);
+      std::fill(tab.begin(), tab.begin() + 128, 0);
+      if (mode == 0 || g.tma) {
+        const auto R = row_box(om, g.T, bst, kGBM), Q = row_box(on, g.T, bst, kGBN);
+        for (int r = 0; r < 64; r++) {
+          tab[128 + r] = R[r];
+          tab[192 + r] = Q[r];
+        }
+        for (int side = 0; side < 2; side++) {
+          const int t = side ? m.Y : m.X;
+          const auto &ord = side ? on : om;
+          int64_t tot = 1;
+          for (int p : ord) tot *= g.T[p];
+          for (int64_t r = 0; r < tot && r < 64; r++) {
+            int64_t b;
+            if (mode == 0) {
+              const bool km = side ? ykm : xkm;
+              int64_t row = 0;
+              const auto dg = row_digits(r, ord, g.T);
+              for (int p : ord) row += dg[p] * row_mul(ord, g.T, p);
+              b = 8 * plane_off(km, row, 0, side ? kGBN : kGBM, BK);
+            } else {
+              const TmaLayout &L = side ? tly[i] : tlx[i];
+              const auto dg = row_digits(r, ord, g.T);
+              std::vector<int64_t> d(c.t[t].idx.size(), 0);
+              for (size_t j = 0; j < d.size(); j++) {
+                const int cp = c.pos_in(0, c.t[t].idx[j]);
+                if (cp >= 0) d[j] = dg[cp];
+              }
+              b = L.byte(d);
+            }
+            tab[side * 64 + r] = (int32_t)b;
+          }
+        }
+      }
+      g.ctab[mode].insert(g.ctab[mode].end(), tab.begin(), tab.end());
+    }
     g.mem.push_back(D);
     int64_t Mt = 1, Nt = 1;
     for (int p : m.mpos) Mt *= g.T[p];
@@ -457,7 +678,7 @@ Status plan_group(const std::vector<const Contraction *> &members, GroupTables &
     g.Mt.push_back(Mt);
     g.Nt.push_back(Nt);
     g.Kt.push_back(Kt);
-    g.padded_flops += 2.0 * (double)g.ntiles * (double)m.nsteps * kGBM * kGBN * BK;
+    g.padded_flops += 2.0 * (double)g.ntiles * (double)m.nsteps * kGBM * kGBN * 4 * cdiv(Kt, 4);
   }
 
   // ---- copy-out units: the box in C order, 2 elements per unit when 16-B stores are legal

@@ -3,17 +3,19 @@
 // The CCSD(T) triples (9 sd_t_d1 + 9 sd_t_d2 contractions, all adding into
 // one t3) run as one persistent kernel.  Per C tile (a hyper-rectangle prod_p T_p of t3,
 // P:L119), for every member i in turn:
-//   (1) PRODUCER warps gather member i's X_i tile (Mt_i x Kt_i) and Y_i tile (Kt_i x Nt_i)
-//       of each k-step with cp.async into a STAGES-deep ring (the paper's step 1),
-//       walking each operand in its own memory order by runs along its FVI;
-//       zero-fill outside the tensors;
-//   (2)+(3) CONSUMER warps multiply with DMMA m8n8k4 register tiles (steps 2-3)
-//       exactly as the single-contraction kernel (kernel_f64.cuh), the smem layout (k- or
-//       mn-major per operand) chosen per member at run time;
-//   then the member's accumulators are added into the C tile's XOR-swizzled smem box (the
-//   digit orders of the member's rows / columns make this conflict-free, group.cpp).
-// After the last member the box leaves for C once: C = alpha * box + beta * C (step 4,
-// P:L84) — t3 is written once instead of 18 times, and read once when beta != 0.
+//   (1) the member's X_i tile (Mt_i x Kt_i) and Y_i tile (Kt_i x Nt_i) of each k-step reach a
+//       STAGES-deep shared-memory ring (the paper's step 1): by TMA — one elected
+//       thread issues cp.async.bulk.tensor boxes over each operand's own index order
+//       (P:L138-145), SWIZZLE_128B / 64B, out-of-range elements zero-filled by the hardware
+//        — or, when some operand cannot be a TMA box, by producer warps gathering runs
+//       along each operand's FVI with cp.async into padded-pitch planes;
+//   (2)+(3) CONSUMER warps run DMMA m8n8k4 register tiles over the stage (steps 2-3,
+//       P:L82-83); fragment addresses come from per-member row / k tables (swizzled for the
+//       TMA planes), so one code path serves every member's layout;
+//   the member's register tile STARTS from the C tile's current values in an XOR-swizzled smem
+//   box and is written back after its last k-step (the DMMAs do the accumulation: no separate
+//   adds on the FP64 pipe).  After the last member the box leaves for C once:
+//   C = alpha * box + beta * C (step 4) — t3 is written once instead of 18 times.
 #pragma once
 #include <cstdint>
 
@@ -22,15 +24,38 @@
 
 namespace tc {
 
+// Ablation side builds only (tools/group_ablation.py compiles libtc with -DTC_GROUP_ABLATE=k;
+// the shipped library has kGAbl = 0): 1 = producers skip the loads, 2 = consumers skip the
+// DMMAs, 3 = consumers skip the box load / store.
+#ifdef TC_GROUP_ABLATE
+constexpr int kGAbl = TC_GROUP_ABLATE;
+#else
+constexpr int kGAbl = 0;
+#endif
+// Hand-off timeline (-DTC_GROUP_TRACE side builds only, tools/group_trace.py): CTA 0, consumer
+// warp 0 / producer warp 0, lane 0, clock64 at slot * 1024 + step of p.trace.
+#ifdef TC_GROUP_TRACE
+#define GTRACE(slot, step)                                                                   \
+  do {                                                                                       \
+    if (blockIdx.x == 0 && (threadIdx.x & 127) == 0 && (step) >= 0 && (step) < 1024)         \
+      p.trace[(slot) * 1024 + (step)] = clock64();                                           \
+  } while (0)
+#else
+#define GTRACE(slot, step) do { } while (0)
+#endif
+
 struct GParams {
+  TmaDesc xmap[kGMaxMembers];      // TMA mode: per member the tensor maps of X_i and Y_i
+  TmaDesc ymap[kGMaxMembers];
   const double *X[kGMaxMembers];   // per member: its X / Y operand (A or B, group.hpp)
   const double *Y[kGMaxMembers];
-  uint64_t vecmask;                // bit 2i: X_i may use 16-B vectors; bit 2i+1: Y_i
+  uint64_t vecmask;                // cp.async: bit 2i: X_i may use 16-B vectors; bit 2i+1: Y_i
   double *C;
   double alpha, beta;
   int nmem, rank, ntiles, nunits;
   int uvec;                        // C elements per copy-out unit (1 or 2, group.cpp)
   int cvec16;                      // 1: units of 2 are stored as one 16-B vector (C aligned)
+  int stage_bytes;                 // TMA: bytes per ring stage (group.hpp tma_stage_bytes)
   int32_t ntl[kGMaxCdims];
   int64_t cstep[kGMaxCdims];       // T_p * C stride of position p
   int64_t N[kGMaxCdims];
@@ -43,21 +68,29 @@ struct GParams {
   const uint32_t *runSoff;
   const uint64_t *runDig;
   const uint32_t *pad;
-  const int32_t *boxM, *boxN;
+  const int32_t *ctab;             // this launch mode's consumer tables (group.hpp)
   const int64_t *unitRel;
   const uint64_t *unitDig;
+  unsigned long long *trace;       // (-DTC_GROUP_TRACE side builds only)
 };
 
-template <int BK, int STAGES>
+template <int BK, int STAGES, bool TMA>
 struct GroupCfg {
-  static constexpr int BM = kGBM, BN = kGBN, WM = 32, WN = 32;
+  static constexpr int BM = kGBM, BN = kGBN;
   static constexpr int CW = 4, PW = 4;                      // consumer / producer warps
   static constexpr int THREADS = (CW + PW) * 32;
   static constexpr int PM = BM + 4, PN = BN + 4, PK = BK + 4;
   static constexpr int XS = (BM * PK > BK * PM ? BM * PK : BK * PM) + 2;   // = gplane_doubles
-  static constexpr int YS = (BN * PK > BK * PN ? BN * PK : BK * PN) + 2;
+  // plane bytes: TMA boxes (1 KB aligned, group.hpp gtma_plane_bytes) or padded-pitch planes
+  // cp.async: padded-pitch planes; TMA: the stage size comes from the plan (p.stage_bytes:
+  // the largest X box + Y box of a member), the Y box right after the member's X box
+  static constexpr int PLANE = 8 * XS;
+  static constexpr int STAGE = 2 * PLANE;
   static constexpr int BOX = BM * BN;
-  static constexpr size_t smem_bytes() { return 8 * ((size_t)STAGES * (XS + YS) + BOX) + 16 * STAGES; }
+  // + 128 B: the ring is aligned to 128 B inside the dynamic smem (TMA destinations)
+  static constexpr size_t smem_bytes(int tma_stage) {
+    return 128 + (size_t)STAGES * (TMA ? tma_stage : STAGE) + 8 * BOX + 16 * STAGES;
+  }
   static_assert(BK % 4 == 0 && BK <= 32, "BK");
 };
 
@@ -78,34 +111,36 @@ __device__ __forceinline__ uint64_t g_op_lims(const GOperandDev &op, uint64_t Lc
   return L;
 }
 
-// Gather one operand tile (one k-step) into a stage plane: vector w = pt + 128 i is vector v
-// of run q; runs lie along the operand's FVI, consecutive threads take consecutive vectors.
-__device__ __forceinline__ void g_gather(const GParams &p, const double *__restrict__ base, uint32_t sdst,
-                                         const GOperandDev &op, int vec, int pt, bool fast, uint64_t L) {
+// ---------------------------------------------------------------- cp.async producer path
+// Gather of one operand tile (one k-step) into a padded-pitch plane, in two phases so that the
+// run-table latency hides behind the stage wait: vector w = pt + 128 e (e < 8 per chunk) is
+// vector v of run q; runs lie along the operand's FVI, consecutive threads take consecutive
+// vectors.
+struct GFetch {
+  int32_t rel[8];     // element offset of the vector in the operand tile
+  uint32_t so[8];     // smem element offset in the plane
+};
+
+__device__ __forceinline__ void g_qv(int w0, int vpr, int &q, int &v, int &dq, int &dv) {
+  q = w0 / vpr;
+  v = w0 - q * vpr;
+  dq = 128 / vpr;
+  dv = 128 - dq * vpr;
+}
+
+__device__ __forceinline__ void g_fetch(const GParams &p, const GOperandDev &op, int vec, int nvec, int pt,
+                                        int chunk, GFetch &f) {
   const int vpr = op.runlen / vec;
-  const int nvec = op.nrun * vpr;
   const int32_t *__restrict__ rr = p.runRel + op.run0;
   const uint32_t *__restrict__ rs = p.runSoff + op.run0;
-  const uint64_t *__restrict__ rd = p.runDig + op.run0;
-  int q = pt / vpr, v = pt - (pt / vpr) * vpr;
-  const int dq = 128 / vpr, dv = 128 - (128 / vpr) * vpr;
-  // bytes checked by SWAR: dims 1.. when runs cover dim 0, else every dim
-  const int jfirst = op.runlen > 1 ? 1 : 0;
-  uint64_t maskH = 0;
-  for (int j = jfirst; j < op.ndim; j++) maskH |= 0x80ull << (8 * j);
-  const int lim0 = (int)(L & 0xFF);
-  for (int w = pt; w < nvec; w += 128) {
-    const int rel = __ldg(rr + q) + v * vec;
-    const uint32_t dst = sdst + 8u * (__ldg(rs + q) + (uint32_t)(v * vec));
-    const double *src = base + rel;
-    if (fast) {
-      if (vec == 2) cp_async16_full(dst, src);
-      else cp_async8_full(dst, src);
-    } else {
-      int nval = g_all_lt(__ldg(rd + q), L, maskH) ? vec : 0;
-      if (op.runlen > 1) nval = min(nval, max(0, lim0 - v * vec));
-      if (vec == 2) cp_async16(dst, nval ? src : base, 8 * nval);
-      else cp_async8(dst, nval ? src : base, 8 * nval);
+  const int w0 = pt + 1024 * chunk;
+  int q, v, dq, dv;
+  g_qv(w0, vpr, q, v, dq, dv);
+#pragma unroll
+  for (int e = 0; e < 8; e++) {
+    if (w0 + 128 * e < nvec) {
+      f.rel[e] = __ldg(rr + q) + v * vec;
+      f.so[e] = __ldg(rs + q) + (uint32_t)(v * vec);
     }
     q += dq;
     v += dv;
@@ -113,30 +148,128 @@ __device__ __forceinline__ void g_gather(const GParams &p, const double *__restr
   }
 }
 
-// One k-step of one member on the consumer warps: DMMA over the stage (compile-time layouts).
-template <int BK, bool XK, bool YK>
-__device__ __forceinline__ void g_mma_step(double (&acc)[4][4][2], const double *__restrict__ xs,
-                                           const double *__restrict__ ys, int wm, int wn, int g, int t) {
-  constexpr int PK = BK + 4, PM = kGBM + 4, PN = kGBN + 4;
-  const int aoff = XK ? (wm * 32 + g) * PK + t : t * PM + wm * 32 + g;
-  const int boff = YK ? (wn * 32 + g) * PK + t : t * PN + wn * 32 + g;
-  constexpr int AI = XK ? 8 * PK : 8, AK = XK ? 4 : 4 * PM;
-  constexpr int BJ = YK ? 8 * PK : 8, BKs = YK ? 4 : 4 * PN;
+__device__ __forceinline__ void g_issue(const GParams &p, const double *__restrict__ base, uint32_t sdst,
+                                        const GOperandDev &op, int vec, int nvec, int pt, int chunk,
+                                        const GFetch &f, bool fast, uint64_t L) {
+  const int w0 = pt + 1024 * chunk;
+  if (fast) {
 #pragma unroll
-  for (int kk = 0; kk < BK / 4; kk++) {
-    double a[4], b[4];
-#pragma unroll
-    for (int i = 0; i < 4; i++) a[i] = xs[aoff + i * AI + kk * AK];
-#pragma unroll
-    for (int j = 0; j < 4; j++) b[j] = ys[boff + j * BJ + kk * BKs];
-#pragma unroll
-    for (int i = 0; i < 4; i++)
-#pragma unroll
-      for (int j = 0; j < 4; j++) dmma884(acc[i][j][0], acc[i][j][1], a[i], b[j]);
+    for (int e = 0; e < 8; e++) {
+      if (w0 + 128 * e < nvec) {
+        if (vec == 2) cp_async16_full(sdst + 8u * f.so[e], base + f.rel[e]);
+        else cp_async8_full(sdst + 8u * f.so[e], base + f.rel[e]);
+      }
+    }
+    return;
+  }
+  // bytes checked by SWAR: dims 1.. when runs cover dim 0, else every dim
+  const int jfirst = op.runlen > 1 ? 1 : 0;
+  uint64_t maskH = 0;
+  for (int j = jfirst; j < op.ndim; j++) maskH |= 0x80ull << (8 * j);
+  const int lim0 = (int)(L & 0xFF);
+  const uint64_t *__restrict__ rd = p.runDig + op.run0;
+  const int vpr = op.runlen / vec;
+  int q, v, dq, dv;
+  g_qv(w0, vpr, q, v, dq, dv);
+  for (int e = 0; e < 8; e++) {
+    if (w0 + 128 * e < nvec) {
+      int nval = g_all_lt(__ldg(rd + q), L, maskH) ? vec : 0;
+      if (op.runlen > 1) nval = min(nval, max(0, lim0 - v * vec));
+      const uint32_t dst = sdst + 8u * f.so[e];
+      if (vec == 2) cp_async16(dst, nval ? base + f.rel[e] : base, 8 * nval);
+      else cp_async8(dst, nval ? base + f.rel[e] : base, 8 * nval);
+    }
+    q += dq;
+    v += dv;
+    if (v >= vpr) { v -= vpr; q++; }
   }
 }
 
-// tile t -> C coordinates (position 0 fastest), packed limits, interior flag, C origin
+// ---------------------------------------------------------------- TMA producer path
+__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(bar), "r"(bytes) : "memory");
+}
+
+// TMA load of one box at crd into smem dst, completing on mbarrier bar
+__device__ __forceinline__ void tma_load(const TmaDesc *map, int rank, const int32_t *crd, uint32_t dst,
+                                         uint32_t bar) {
+  const uint64_t m = reinterpret_cast<uint64_t>(map);
+  switch (rank) {
+    case 1:
+      asm volatile("cp.async.bulk.tensor.1d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2}], [%3];\n"
+                   ::"r"(dst), "l"(m), "r"(crd[0]), "r"(bar) : "memory");
+      break;
+    case 2:
+      asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];\n"
+                   ::"r"(dst), "l"(m), "r"(crd[0]), "r"(crd[1]), "r"(bar) : "memory");
+      break;
+    case 3:
+      asm volatile("cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];\n"
+                   ::"r"(dst), "l"(m), "r"(crd[0]), "r"(crd[1]), "r"(crd[2]), "r"(bar) : "memory");
+      break;
+    case 4:
+      asm volatile("cp.async.bulk.tensor.4d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, %5}], [%6];\n"
+                   ::"r"(dst), "l"(m), "r"(crd[0]), "r"(crd[1]), "r"(crd[2]), "r"(crd[3]), "r"(bar) : "memory");
+      break;
+    default:
+      asm volatile("cp.async.bulk.tensor.5d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, %5, %6}], [%7];\n"
+                   ::"r"(dst), "l"(m), "r"(crd[0]), "r"(crd[1]), "r"(crd[2]), "r"(crd[3]), "r"(crd[4]), "r"(bar)
+                   : "memory");
+      break;
+  }
+}
+
+// the box of one operand for (tile, k-step): coordinates per map dim = the tile origin (C
+// dims) or the k-tile origin (the internal dim)
+__device__ __forceinline__ void g_tma_operand(const TmaDesc *map, const GOperandDev &op, const int32_t *tc,
+                                              const int32_t (&T)[kGMaxCdims], int32_t kc, uint32_t dst,
+                                              uint32_t bar) {
+  int32_t crd[kGMaxTmaDims];
+#pragma unroll
+  for (int j = 0; j < kGMaxTmaDims; j++) {
+    const int cp = op.tma_cpos[j];
+    crd[j] = j == op.tma_kdim ? kc : (cp >= 0 ? tc[cp] * T[cp] : 0);
+  }
+  tma_load(map, op.ndim, crd, dst, bar);
+}
+
+// ---------------------------------------------------------------- consumers
+// One k-step of one member: DMMA over the stage, fragment addresses from the member's row and
+// k byte offsets (swizzled for TMA planes; swz = 0 for padded-pitch planes).
+template <int BK>
+__device__ __forceinline__ void g_mma_step(double (&acc)[4][4][2], const char *__restrict__ xs,
+                                           const char *__restrict__ ys, const uint32_t (&rx)[4],
+                                           const uint32_t (&ry)[4], const uint32_t (&kx)[BK / 4],
+                                           const uint32_t (&ky)[BK / 4], uint32_t swx, uint32_t swy, int kq) {
+#pragma unroll
+  for (int kk = 0; kk < BK / 4; kk++) {
+    if (kk < kq) {
+      double a[4], b[4];
+#pragma unroll
+      for (int i = 0; i < 4; i++) a[i] = *reinterpret_cast<const double *>(xs + gplane_sw(rx[i] + kx[kk], swx));
+#pragma unroll
+      for (int j = 0; j < 4; j++) b[j] = *reinterpret_cast<const double *>(ys + gplane_sw(ry[j] + ky[kk], swy));
+#pragma unroll
+      for (int i = 0; i < 4; i++)
+#pragma unroll
+        for (int j = 0; j < 4; j++) dmma884(acc[i][j][0], acc[i][j][1], a[i], b[j]);
+    }
+  }
+}
+
+// this thread's k byte offsets of one operand (k = 4 kk + t)
+template <int BK>
+__device__ __forceinline__ void g_kbytes(const GOperandDev &op, int mode, int t, uint32_t (&kb)[BK / 4]) {
+  const int l2 = op.kch_log2[mode];
+  const uint32_t chunk = (uint32_t)op.kchunk[mode], mul = (uint32_t)op.kmul[mode];
+#pragma unroll
+  for (int kk = 0; kk < BK / 4; kk++) {
+    const uint32_t k = (uint32_t)(4 * kk + t);
+    kb[kk] = (k >> l2) * chunk + (k & ((1u << l2) - 1u)) * mul;
+  }
+}
+
+// tile t -> C coordinates (position 0 fastest), packed limits, interior flag
 struct GTile {
   int32_t c[kGMaxCdims];
   uint64_t Lc;
@@ -166,42 +299,100 @@ struct GTile {
   }
 };
 
-template <int BK, int STAGES>
-__global__ void __launch_bounds__(GroupCfg<BK, STAGES>::THREADS, 2)
+// per member, per consumer thread: row byte offsets of its fragments and box offsets of its
+// accumulators (group.hpp consumer table)
+struct GRows {
+  uint32_t rx[4], ry[4];
+  int32_t bm[4], bn[4][2];
+  __device__ __forceinline__ void load(const int32_t *__restrict__ tb, int wm, int wn, int g, int t) {
+#pragma unroll
+    for (int a = 0; a < 4; a++) {
+      rx[a] = (uint32_t)__ldg(tb + wm * 32 + a * 8 + g);
+      ry[a] = (uint32_t)__ldg(tb + 64 + wn * 32 + a * 8 + g);
+      bm[a] = __ldg(tb + 128 + wm * 32 + a * 8 + g);
+      bn[a][0] = __ldg(tb + 192 + wn * 32 + a * 8 + 2 * t);
+      bn[a][1] = __ldg(tb + 192 + wn * 32 + a * 8 + 2 * t + 1);
+    }
+  }
+};
+
+template <int BK, int STAGES, bool TMA>
+__global__ void __launch_bounds__(GroupCfg<BK, STAGES, TMA>::THREADS, 2)
 tc_f64_group_kernel(const __grid_constant__ GParams p) {
-  using K = GroupCfg<BK, STAGES>;
-  extern __shared__ __align__(1024) double smem[];
-  // smem: [STAGES][X plane XS | Y plane YS], then the C box, then the barriers
-  double *box = smem + STAGES * (K::XS + K::YS);
+  using K = GroupCfg<BK, STAGES, TMA>;
+  constexpr int MODE = TMA ? 1 : 0;
+  extern __shared__ __align__(128) unsigned char smem_dyn[];
+  // smem: [STAGES][X | Y] (128-B aligned), the C box, the barriers, then (cp.async) the member
+  // records (group_api.cu sizes it)
+  unsigned char *ring = smem_dyn + ((128u - ((uint32_t)__cvta_generic_to_shared(smem_dyn) & 127u)) & 127u);
+  const int SB = TMA ? p.stage_bytes : K::STAGE;   // bytes per stage
+  double *box = reinterpret_cast<double *>(ring + STAGES * SB);
   uint64_t *bars = reinterpret_cast<uint64_t *>(box + K::BOX);   // full[S], empty[S]
+  GMemberDev *smem_mem = reinterpret_cast<GMemberDev *>(bars + 2 * STAGES);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int ntl = (p.ntiles - (int)blockIdx.x + (int)gridDim.x - 1) / (int)gridDim.x;
   if (ntl <= 0) return;
-  const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(smem);
+  const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(ring);
   const uint32_t bar0 = (uint32_t)__cvta_generic_to_shared(bars);
-  constexpr uint32_t STAGE_BYTES = 8u * (K::XS + K::YS);
 
-  // zero the ring once (rows / k positions a member does not write are never flushed, but
-  // must not hold NaN patterns that reach a valid accumulator: k padding is re-zeroed per step)
-  for (int i = tid; i < STAGES * (K::XS + K::YS); i += K::THREADS) smem[i] = 0.0;
+  // zero the ring once (cp.async: rows / k positions a member does not write are never
+  // flushed, but must not hold NaN patterns that reach a valid accumulator)
+  for (int i = tid; i < STAGES * SB / 16; i += K::THREADS)
+    reinterpret_cast<uint4 *>(ring)[i] = make_uint4(0, 0, 0, 0);
+  if (!TMA) {   // (the cp.async producers read their member records often: keep them in smem)
+    const int nw = p.nmem * (int)(sizeof(GMemberDev) / 4);
+    const uint32_t *src = reinterpret_cast<const uint32_t *>(p.mem);
+    for (int i = tid; i < nw; i += K::THREADS) reinterpret_cast<uint32_t *>(smem_mem)[i] = src[i];
+  }
+  const GMemberDev *mems = TMA ? p.mem : smem_mem;
   if (tid == 0) {
     for (int s = 0; s < STAGES; s++) {
-      mbar_init(bar0 + 8 * s, K::PW * 32);
-      mbar_init(bar0 + 8 * (STAGES + s), K::CW);
+      mbar_init(bar0 + 8 * s, TMA ? 1 : K::PW * 32);   // full: the TMA thread / every producer
+      mbar_init(bar0 + 8 * (STAGES + s), K::CW);       // empty: one arrive per consumer warp
     }
     asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
   }
+  // (generic-proxy zeroing of the ring before the TMA's async-proxy writes)
+  asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
   __syncthreads();
 
   if (warp >= K::CW) {
     // ======================= producers ====================================================
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 88;\n" ::: "memory");   // registers to the consumers
+    if (TMA) {
+      if (warp != K::CW || lane != 0) return;
+      int j = 0;
+      for (int lt = 0; lt < ntl; lt++) {
+        GTile tile;
+        tile.decode(p, (int)blockIdx.x + lt * (int)gridDim.x);
+        for (int i = 0; i < p.nmem; i++) {
+          const GMemberDev &M = mems[i];
+          const uint32_t tx = (uint32_t)(M.x.tma_tx + M.y.tma_tx);
+          for (int s = 0; s < M.nsteps; s++, j++) {
+            const int st = j % STAGES;
+            const GStepDev &S = p.steps[M.step0 + s];
+            GTRACE(3, j);
+            if (j >= STAGES) mbar_wait(bar0 + 8 * (STAGES + st), ((j / STAGES) & 1) ^ 1);
+            GTRACE(4, j);
+            const uint32_t full = bar0 + 8 * st;
+            if (kGAbl == 1) { mbar_arrive(full); continue; }
+            mbar_expect_tx(full, tx);
+            const uint32_t dst = sbase + st * SB;
+            g_tma_operand(&p.xmap[i], M.x, tile.c, p.T, S.kc, dst, full);
+            g_tma_operand(&p.ymap[i], M.y, tile.c, p.T, S.kc, dst + M.tma_yoff, full);
+            GTRACE(5, j);
+          }
+        }
+      }
+      return;
+    }
     const int pt = tid - K::CW * 32;
     int j = 0;
     for (int lt = 0; lt < ntl; lt++) {
       GTile tile;
       tile.decode(p, (int)blockIdx.x + lt * (int)gridDim.x);
       for (int i = 0; i < p.nmem; i++) {
-        const GMemberDev &M = p.mem[i];
+        const GMemberDev &M = mems[i];
         const double *__restrict__ Xb = p.X[i] + tile.off(M.x.tstep, p.rank);
         const double *__restrict__ Yb = p.Y[i] + tile.off(M.y.tstep, p.rank);
         const int vx = ((p.vecmask >> (2 * i)) & 1) ? M.x.vec : 1;
@@ -209,16 +400,36 @@ tc_f64_group_kernel(const __grid_constant__ GParams p) {
         // (needed by partial k-steps of interior tiles too)
         const uint64_t Lx = g_op_lims(M.x, tile.Lc);
         const uint64_t Ly = g_op_lims(M.y, tile.Lc);
+        const int nvx = M.x.nrun * (M.x.runlen / vx), nvy = M.y.nrun * (M.y.runlen / vy);
         for (int s = 0; s < M.nsteps; s++, j++) {
           const int st = j % STAGES;
+          // this thread's run-table entries (and the step record) are fetched BEFORE waiting
+          // for the stage: their latency hides behind the consumers' work
+          GTRACE(3, j);
+          const GStepDev S = p.steps[M.step0 + s];
+          GFetch fx, fy;
+          if (kGAbl != 1) {
+            g_fetch(p, M.x, vx, nvx, pt, 0, fx);
+            g_fetch(p, M.y, vy, nvy, pt, 0, fy);
+          }
           if (j >= STAGES) mbar_wait(bar0 + 8 * (STAGES + st), ((j / STAGES) & 1) ^ 1);
-          const GStepDev &S = p.steps[M.step0 + s];
+          GTRACE(4, j);
+          if (kGAbl == 1) { mbar_arrive_cp_async(bar0 + 8 * st); continue; }
           const bool fast = tile.interior && S.full;
-          const uint32_t dst = sbase + st * STAGE_BYTES;
-          g_gather(p, Xb + S.kx, dst, M.x, vx, pt, fast, Lx | S.klimX);
-          g_gather(p, Yb + S.ky, dst + 8u * K::XS, M.y, vy, pt, fast, Ly | S.klimY);
+          const uint32_t dst = sbase + st * K::STAGE;
+          g_issue(p, Xb + S.kx, dst, M.x, vx, nvx, pt, 0, fx, fast, Lx | S.klimX);
+          g_issue(p, Yb + S.ky, dst + K::PLANE, M.y, vy, nvy, pt, 0, fy, fast, Ly | S.klimY);
+          for (int c = 1; c * 8 * 128 < nvx; c++) {      // (operand tiles of more than 1024 vectors)
+            g_fetch(p, M.x, vx, nvx, pt, c, fx);
+            g_issue(p, Xb + S.kx, dst, M.x, vx, nvx, pt, c, fx, fast, Lx | S.klimX);
+          }
+          for (int c = 1; c * 8 * 128 < nvy; c++) {
+            g_fetch(p, M.y, vy, nvy, pt, c, fy);
+            g_issue(p, Yb + S.ky, dst + K::PLANE, M.y, vy, nvy, pt, c, fy, fast, Ly | S.klimY);
+          }
           for (int w = pt; w < M.npad; w += K::PW * 32) cp_async8(dst + __ldg(p.pad + M.pad0 + w), Xb, 0);
           mbar_arrive_cp_async(bar0 + 8 * st);
+          GTRACE(5, j);
         }
       }
     }
@@ -226,44 +437,29 @@ tc_f64_group_kernel(const __grid_constant__ GParams p) {
   }
 
   // ======================= consumers ======================================================
+  asm volatile("setmaxnreg.inc.sync.aligned.u32 168;\n" ::: "memory");   // accumulators + tables
   const int wm = warp & 1, wn = warp >> 1;
   const int g = lane >> 2, t = lane & 3;
   double acc[4][4][2];
-#pragma unroll
-  for (int i = 0; i < 4; i++)
-#pragma unroll
-    for (int jj = 0; jj < 4; jj++) acc[i][jj][0] = acc[i][jj][1] = 0.0;
   double *__restrict__ C = p.C;
   const double alpha = p.alpha, beta = p.beta;
+  GRows cur;
+  cur.load(p.ctab, wm, wn, g, t);
   int j = 0;
   for (int lt = 0; lt < ntl; lt++) {
     for (int i = 0; i < p.nmem; i++) {
-      const int layout = p.mem[i].layout, nsteps = p.mem[i].nsteps;
-      for (int s = 0; s < nsteps; s++, j++) {
-        const int st = j % STAGES;
-        mbar_wait(bar0 + 8 * st, (j / STAGES) & 1);
-        const double *xs = smem + st * (K::XS + K::YS);
-        const double *ys = xs + K::XS;
-        switch (layout) {
-          case 0: g_mma_step<BK, false, false>(acc, xs, ys, wm, wn, g, t); break;
-          case 1: g_mma_step<BK, true, false>(acc, xs, ys, wm, wn, g, t); break;
-          case 2: g_mma_step<BK, false, true>(acc, xs, ys, wm, wn, g, t); break;
-          default: g_mma_step<BK, true, true>(acc, xs, ys, wm, wn, g, t); break;
-        }
-        __syncwarp();
-        if (lane == 0) mbar_arrive(bar0 + 8 * (STAGES + st));
-      }
-      // ---- flush member i into the box (after every consumer finished the previous flush
-      //      or the previous tile's copy-out: the box entries of two members differ per thread)
-      const int32_t *bm = p.boxM + i * kGBM, *bn = p.boxN + i * kGBN;
-      int rb[4], cb[4][2];
-#pragma unroll
-      for (int q = 0; q < 4; q++) rb[q] = __ldg(bm + wm * 32 + q * 8 + g);
-#pragma unroll
-      for (int q = 0; q < 4; q++) {
-        cb[q][0] = __ldg(bn + wn * 32 + q * 8 + 2 * t);
-        cb[q][1] = __ldg(bn + wn * 32 + q * 8 + 2 * t + 1);
-      }
+      const GMemberDev &M = mems[i];
+      const int nsteps = M.nsteps, kq = M.kq;
+      uint32_t kx[BK / 4], ky[BK / 4];
+      g_kbytes<BK>(M.x, MODE, t, kx);
+      g_kbytes<BK>(M.y, MODE, t, ky);
+      const uint32_t swx = (uint32_t)M.x.swz[MODE], swy = (uint32_t)M.y.swz[MODE];
+      const int yoff = TMA ? M.tma_yoff : K::PLANE;
+      // the next member's tables, loaded while this member runs
+      GRows nxt;
+      nxt.load(p.ctab + (i + 1 < p.nmem ? i + 1 : 0) * kGCtab, wm, wn, g, t);
+      // ---- the member's register tile starts from the box (every consumer finished the
+      //      previous member's write-back — or the previous tile's copy-out — first)
       consumer_sync(K::CW * 32);
 #pragma unroll
       for (int a = 0; a < 4; a++)
@@ -271,12 +467,31 @@ tc_f64_group_kernel(const __grid_constant__ GParams p) {
         for (int b = 0; b < 4; b++)
 #pragma unroll
           for (int h = 0; h < 2; h++) {
-            if (rb[a] >= 0 && cb[b][h] >= 0) {
-              const int o = gbox_sw(rb[a] + cb[b][h]);
-              box[o] = i == 0 ? acc[a][b][h] : box[o] + acc[a][b][h];
-            }
-            acc[a][b][h] = 0.0;
+            const bool ok = i > 0 && kGAbl != 3 && cur.bm[a] >= 0 && cur.bn[b][h] >= 0;
+            acc[a][b][h] = ok ? box[gbox_sw(cur.bm[a] + cur.bn[b][h])] : 0.0;
           }
+      for (int s = 0; s < nsteps; s++, j++) {
+        const int st = j % STAGES;
+        mbar_wait(bar0 + 8 * st, (j / STAGES) & 1);
+        GTRACE(0, j);
+        const char *xs = reinterpret_cast<const char *>(ring) + st * SB;
+        if (kGAbl != 2) g_mma_step<BK>(acc, xs, xs + yoff, cur.rx, cur.ry, kx, ky, swx, swy, kq);
+        __syncwarp();
+        if (lane == 0) mbar_arrive(bar0 + 8 * (STAGES + st));
+        GTRACE(1, j);
+      }
+      // ---- write the member's tile back into the box
+      if (kGAbl != 3) {
+#pragma unroll
+        for (int a = 0; a < 4; a++)
+#pragma unroll
+          for (int b = 0; b < 4; b++)
+#pragma unroll
+            for (int h = 0; h < 2; h++)
+              if (cur.bm[a] >= 0 && cur.bn[b][h] >= 0) box[gbox_sw(cur.bm[a] + cur.bn[b][h])] = acc[a][b][h];
+      }
+      GTRACE(2, j - 1);
+      cur = nxt;
     }
     // ---- the tile leaves for C once: C = alpha * box + beta * C (beta == 0: C not read)
     consumer_sync(K::CW * 32);

@@ -42,7 +42,7 @@ def main():
         flops = sum(p.flops for p in plans)
         byts = 8 * (sum(p.numel("A") + p.numel("B") for p in plans) + C.numel())
         attain = min(FP64_PEAK, flops / byts * HBM)
-        row = {"extents": ext, "group": g.info()["T"], "BK": g.info()["BK"], "grid": g.info()["grid"]}
+        row = {"extents": ext, "group": g.info()["T"], "BK": g.info()["BK"], "tma": g.info()["tma"]}
         for beta in (0.0, 1.0):
             ms = timeit(lambda: g.execute(A, B, C, 1.0, beta), flush)
             row[f"fused_ms_b{int(beta)}"] = round(ms, 4)
