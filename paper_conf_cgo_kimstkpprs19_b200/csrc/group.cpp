@@ -575,6 +575,8 @@ Status plan_group(const std::vector<const Contraction *> &members, GroupTables &
         }
         s.base = c.t[t].base;
         o.tma_tx = (int32_t)L.bytes;
+        o.tma_pack = (uint32_t)s.rank << 20 | (uint32_t)(o.tma_kdim < 0 ? 15 : o.tma_kdim) << 24;
+        for (int j = 0; j < kGMaxTmaDims; j++) o.tma_pack |= (uint32_t)(o.tma_cpos[j] < 0 ? 15 : o.tma_cpos[j]) << (4 * j);
         const int kidx = m.kid.empty() ? -1 : m.kid[0];
         const int jk = kidx >= 0 ? c.pos_in(t, kidx) : -1;
         o.kch_log2[1] = 30;                 // one box: k is linear in it
@@ -679,6 +681,56 @@ Status plan_group(const std::vector<const Contraction *> &members, GroupTables &
     g.Nt.push_back(Nt);
     g.Kt.push_back(Kt);
     g.padded_flops += 2.0 * (double)g.ntiles * (double)m.nsteps * kGBM * kGBN * 4 * cdiv(Kt, 4);
+  }
+
+  // ---- execution order: members whose register tile maps onto the box the same way (in the
+  //      mode that runs: TMA when every operand allows it) become neighbours, and chain — the
+  //      tile stays in registers from one to the next (the sum's order changes; any order is
+  //      a correct result, DESIGN R22)
+  {
+    const int run_mode = g.tma ? 1 : 0;
+    auto boxmap = [&](int mo, int i) {
+      return std::vector<int32_t>(g.ctab[mo].begin() + (size_t)i * kGCtab + 128,
+                                  g.ctab[mo].begin() + (size_t)(i + 1) * kGCtab);
+    };
+    std::vector<int> ord;
+    std::vector<char> used(n, 0);
+    for (int i = 0; i < n; i++) {
+      if (used[i]) continue;
+      used[i] = 1;
+      ord.push_back(i);
+      const auto bi = boxmap(run_mode, i);
+      for (int k = i + 1; k < n; k++)
+        if (!used[k] && boxmap(run_mode, k) == bi) {
+          used[k] = 1;
+          ord.push_back(k);
+        }
+    }
+    auto permute = [&](auto &v) {
+      auto w = v;
+      for (int k = 0; k < n; k++) w[k] = v[ord[k]];
+      v = w;
+    };
+    permute(g.mem);
+    permute(g.tmaX);
+    permute(g.tmaY);
+    permute(g.Mt);
+    permute(g.Nt);
+    permute(g.Kt);
+    permute(g.flushWf);
+    permute(g.loadWf);
+    permute(g.fragWf);
+    for (int mo = 0; mo < 2; mo++) {
+      std::vector<int32_t> t(g.ctab[mo].size());
+      for (int k = 0; k < n; k++)
+        std::copy(g.ctab[mo].begin() + (size_t)ord[k] * kGCtab, g.ctab[mo].begin() + (size_t)(ord[k] + 1) * kGCtab,
+                  t.begin() + (size_t)k * kGCtab);
+      g.ctab[mo] = t;
+    }
+    g.order = ord;
+    for (int k = 0; k < n; k++)
+      for (int mo = 0; mo < 2; mo++)
+        g.mem[k].chain[mo] = (k + 1 < n && (mo == 0 || g.tma) && boxmap(mo, k) == boxmap(mo, k + 1)) ? 1 : 0;
   }
 
   // ---- copy-out units: the box in C order, 2 elements per unit when 16-B stores are legal

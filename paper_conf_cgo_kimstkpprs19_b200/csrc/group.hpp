@@ -62,6 +62,8 @@ struct GOperandDev {
   int32_t tma_cpos[kGMaxTmaDims];   // C position of map dim j (-1: the k dim or unused)
   int32_t tma_kdim;                 // map dim of the internal index (-1: none)
   int32_t tma_tx;                   // bytes the box delivers (expect-tx)
+  uint32_t tma_pack;                // the producer's copy: 4 bits of tma_cpos per map dim (15: none),
+                                    // the map's rank at bit 20, tma_kdim at bit 24 (15: none)
 };
 
 struct GMemberDev {
@@ -71,7 +73,11 @@ struct GMemberDev {
   int32_t xIsA;                // 1: X = A, Y = B; 0: X = B, Y = A
   int32_t kq;                  // k4 groups per step (ceil(Kt / 4))
   int32_t tma_yoff;            // TMA: byte offset of the Y box in the stage (after the X box)
-  int32_t pad_;
+  // per load mode: 1 when the next member (execution order) maps its register tile onto the
+  // box exactly as this one — the tile then stays in registers across the two (no write-back
+  // and reload in between: the d1 / d2 triples come in such pairs)
+  uint8_t chain[2];
+  uint8_t pad_[2];
 };
 
 struct GStepDev {
@@ -109,6 +115,9 @@ struct GroupTables {
   };
   int tma_stage_bytes = 0;     // largest X box + Y box of a member (<= the TMA stage)
   std::vector<TmaSpec> tmaX, tmaY;
+  // execution order: position k runs member order[k] (members with one register-tile mapping
+  // adjacent, group.cpp); every per-member vector here is in execution order
+  std::vector<int> order;
   // planner statistics (tc_group_info)
   std::vector<int64_t> Mt, Nt, Kt;
   std::vector<double> flushWf, loadWf, fragWf;   // simulated smem wavefronts per member-tile

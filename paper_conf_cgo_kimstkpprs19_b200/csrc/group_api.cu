@@ -235,13 +235,16 @@ tc_status_t tc_group_execute(const tc_group_t group, const void *const *A, const
   GParams kp = G->kp;
   kp.vecmask = 0;
   bool tma = G->gt.tma;
-  for (int i = 0; i < G->n; i++) {
-    if (!A[i] || !B[i]) return set_error(ST_INVALID_ARG, "NULL tensor pointer in group");
-    if (overlaps(C, G->spanC, A[i], G->spanA[i]) || overlaps(C, G->spanC, B[i], G->spanB[i]))
-      return set_error(ST_INVALID_ARG, "C overlaps A or B of member " + std::to_string(i));
+  for (int o = 0; o < G->n; o++) {
+    if (!A[o] || !B[o]) return set_error(ST_INVALID_ARG, "NULL tensor pointer in group");
+    if (overlaps(C, G->spanC, A[o], G->spanA[o]) || overlaps(C, G->spanC, B[o], G->spanB[o]))
+      return set_error(ST_INVALID_ARG, "C overlaps A or B of member " + std::to_string(o));
+  }
+  for (int i = 0; i < G->n; i++) {   // i: execution position; o: the caller's member
+    const int o = G->gt.order[i];
     const bool xa = G->gt.mem[i].xIsA;
-    kp.X[i] = static_cast<const double *>(xa ? A[i] : B[i]);
-    kp.Y[i] = static_cast<const double *>(xa ? B[i] : A[i]);
+    kp.X[i] = static_cast<const double *>(xa ? A[o] : B[o]);
+    kp.Y[i] = static_cast<const double *>(xa ? B[o] : A[o]);
     if ((uintptr_t)kp.X[i] % 16 == 0) kp.vecmask |= 1ull << (2 * i);
     if ((uintptr_t)kp.Y[i] % 16 == 0) kp.vecmask |= 1ull << (2 * i + 1);
     // TMA boxes when every operand's origin is 16-B aligned and its map encodes
@@ -279,7 +282,9 @@ tc_status_t tc_group_info(const tc_group_t group, char *json, size_t cap, size_t
       o << ",\"" << (mode ? "tma" : "cpasync") << "_launch\":{\"grid\":" << group->launch[mode].grid
         << ",\"threads\":" << group->launch[mode].threads << ",\"smem\":" << group->launch[mode].smem << "}";
     o << ",\"flops\":" << g.flops << ",\"padded_flops\":" << g.padded_flops << ",\"plan_ms\":" << g.plan_ms
-      << ",\"per_member\":[";
+      << ",\"order\":[";
+    for (int i = 0; i < group->n; i++) o << (i ? "," : "") << g.order[i];
+    o << "],\"per_member\":[";   // (in execution order)
     for (int i = 0; i < group->n; i++) {
       const GMemberDev &m = g.mem[i];
       o << (i ? "," : "") << "{\"Mt\":" << g.Mt[i] << ",\"Nt\":" << g.Nt[i] << ",\"Kt\":" << g.Kt[i]
@@ -287,7 +292,7 @@ tc_status_t tc_group_info(const tc_group_t group, char *json, size_t cap, size_t
         << "\",\"vecX\":" << m.x.vec << ",\"vecY\":" << m.y.vec << ",\"runlenX\":" << m.x.runlen
         << ",\"runlenY\":" << m.y.runlen << ",\"tma_bytes\":[" << m.x.tma_tx << "," << m.y.tma_tx
         << "],\"flush_wf\":" << g.flushWf[i] << ",\"load_wf\":" << g.loadWf[i]
-        << ",\"tma_frag_wf\":" << g.fragWf[i] << "}";
+        << ",\"tma_frag_wf\":" << g.fragWf[i] << ",\"chain\":[" << (int)m.chain[0] << "," << (int)m.chain[1] << "]}";
     }
     o << "]}";
     const std::string s = o.str();

@@ -190,82 +190,120 @@ __device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(bar), "r"(bytes) : "memory");
 }
 
-// TMA load of one box at crd into smem dst, completing on mbarrier bar
-__device__ __forceinline__ void tma_load(const TmaDesc *map, int rank, const int32_t *crd, uint32_t dst,
-                                         uint32_t bar) {
+// TMA load of one box at (c0..c4) into smem dst, completing on mbarrier bar, with an L2 policy
+__device__ __forceinline__ void tma_load(const TmaDesc *map, int rank, int32_t c0, int32_t c1, int32_t c2,
+                                         int32_t c3, int32_t c4, uint32_t dst, uint32_t bar, uint64_t pol) {
   const uint64_t m = reinterpret_cast<uint64_t>(map);
   switch (rank) {
     case 1:
-      asm volatile("cp.async.bulk.tensor.1d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2}], [%3];\n"
-                   ::"r"(dst), "l"(m), "r"(crd[0]), "r"(bar) : "memory");
+      asm volatile("cp.async.bulk.tensor.1d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.L2::cache_hint"
+                   " [%0], [%1, {%2}], [%3], %4;\n" ::"r"(dst), "l"(m), "r"(c0), "r"(bar), "l"(pol) : "memory");
       break;
     case 2:
-      asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];\n"
-                   ::"r"(dst), "l"(m), "r"(crd[0]), "r"(crd[1]), "r"(bar) : "memory");
+      asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.L2::cache_hint"
+                   " [%0], [%1, {%2, %3}], [%4], %5;\n" ::"r"(dst), "l"(m), "r"(c0), "r"(c1), "r"(bar), "l"(pol)
+                   : "memory");
       break;
     case 3:
-      asm volatile("cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];\n"
-                   ::"r"(dst), "l"(m), "r"(crd[0]), "r"(crd[1]), "r"(crd[2]), "r"(bar) : "memory");
+      asm volatile("cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.L2::cache_hint"
+                   " [%0], [%1, {%2, %3, %4}], [%5], %6;\n" ::"r"(dst), "l"(m), "r"(c0), "r"(c1), "r"(c2), "r"(bar),
+                   "l"(pol) : "memory");
       break;
     case 4:
-      asm volatile("cp.async.bulk.tensor.4d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, %5}], [%6];\n"
-                   ::"r"(dst), "l"(m), "r"(crd[0]), "r"(crd[1]), "r"(crd[2]), "r"(crd[3]), "r"(bar) : "memory");
+      asm volatile("cp.async.bulk.tensor.4d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.L2::cache_hint"
+                   " [%0], [%1, {%2, %3, %4, %5}], [%6], %7;\n" ::"r"(dst), "l"(m), "r"(c0), "r"(c1), "r"(c2), "r"(c3),
+                   "r"(bar), "l"(pol) : "memory");
       break;
     default:
-      asm volatile("cp.async.bulk.tensor.5d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, %5, %6}], [%7];\n"
-                   ::"r"(dst), "l"(m), "r"(crd[0]), "r"(crd[1]), "r"(crd[2]), "r"(crd[3]), "r"(crd[4]), "r"(bar)
-                   : "memory");
+      asm volatile("cp.async.bulk.tensor.5d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.L2::cache_hint"
+                   " [%0], [%1, {%2, %3, %4, %5, %6}], [%7], %8;\n" ::"r"(dst), "l"(m), "r"(c0), "r"(c1), "r"(c2),
+                   "r"(c3), "r"(c4), "r"(bar), "l"(pol) : "memory");
       break;
   }
 }
 
-// the box of one operand for (tile, k-step): coordinates per map dim = the tile origin (C
-// dims) or the k-tile origin (the internal dim)
-__device__ __forceinline__ void g_tma_operand(const TmaDesc *map, const GOperandDev &op, const int32_t *tc,
-                                              const int32_t (&T)[kGMaxCdims], int32_t kc, uint32_t dst,
-                                              uint32_t bar) {
-  int32_t crd[kGMaxTmaDims];
+// The TMA producer's per-member recipe (group.hpp GOperandDev::tma_pack: 4 bits of C position
+// per map dim, 15 = the k dim / unused; rank at bit 20; k dim at bit 24).
+struct GTmaRec {
+  uint32_t tx, yoff, xpack, ypack;
+  int32_t nsteps, step0;
+  __device__ __forceinline__ void load(const GMemberDev &m) {
+    tx = (uint32_t)(m.x.tma_tx + m.y.tma_tx);
+    yoff = (uint32_t)m.tma_yoff;
+    xpack = m.x.tma_pack;
+    ypack = m.y.tma_pack;
+    nsteps = m.nsteps;
+    step0 = m.step0;
+  }
+};
+
+// the box of one operand for (tile, k-step): coordinate per map dim = the tile origin of its
+// C position (tcT) or the k-tile origin (the internal dim); all in registers
+__device__ __forceinline__ void g_tma_operand(const TmaDesc *map, uint32_t pack, const int32_t (&tcT)[kGMaxCdims],
+                                              int32_t kc, uint32_t dst, uint32_t bar, uint64_t pol) {
+  int32_t c[kGMaxTmaDims];
+  const int kd = (int)((pack >> 24) & 15);
 #pragma unroll
   for (int j = 0; j < kGMaxTmaDims; j++) {
-    const int cp = op.tma_cpos[j];
-    crd[j] = j == op.tma_kdim ? kc : (cp >= 0 ? tc[cp] * T[cp] : 0);
+    const int cp = (int)((pack >> (4 * j)) & 15);
+    int32_t v = 0;
+#pragma unroll
+    for (int q = 0; q < kGMaxCdims; q++) v = cp == q ? tcT[q] : v;   // (select: no local memory)
+    c[j] = j == kd ? kc : v;
   }
-  tma_load(map, op.ndim, crd, dst, bar);
+  tma_load(map, (int)((pack >> 20) & 15), c[0], c[1], c[2], c[3], c[4], dst, bar, pol);
 }
 
 // ---------------------------------------------------------------- consumers
-// One k-step of one member: DMMA over the stage, fragment addresses from the member's row and
-// k byte offsets (swizzled for TMA planes; swz = 0 for padded-pitch planes).
+// Per member, per consumer thread (loaded one member ahead): the plane byte offsets of its
+// fragment rows, the byte step of k in each plane (k is linear in both the padded-pitch
+// planes and the TMA boxes), the box offsets of its accumulators (group.hpp consumer table),
+// the Y plane's offset, the member's k-steps and k4 groups.
+struct GRows {
+  uint32_t rx[4], ry[4];
+  int32_t bm[4], bn[4][2];
+  uint32_t kmx, kmy;          // bytes per k
+  int32_t yoff, nsteps, kq;
+  bool chain;                 // the next member continues this register tile
+  __device__ __forceinline__ void load(const int32_t *__restrict__ tb, const GMemberDev &m, int mode, int plane,
+                                       int wm, int wn, int g, int t) {
+#pragma unroll
+    for (int a = 0; a < 4; a++) {
+      rx[a] = (uint32_t)__ldg(tb + wm * 32 + a * 8 + g);
+      ry[a] = (uint32_t)__ldg(tb + 64 + wn * 32 + a * 8 + g);
+      bm[a] = __ldg(tb + 128 + wm * 32 + a * 8 + g);
+      bn[a][0] = __ldg(tb + 192 + wn * 32 + a * 8 + 2 * t);
+      bn[a][1] = __ldg(tb + 192 + wn * 32 + a * 8 + 2 * t + 1);
+    }
+    kmx = (uint32_t)m.x.kmul[mode];
+    kmy = (uint32_t)m.y.kmul[mode];
+    yoff = plane >= 0 ? plane : m.tma_yoff;
+    nsteps = m.nsteps;
+    kq = m.kq;
+    chain = m.chain[mode] != 0;
+  }
+};
+
+// One k-step of one member: DMMA over the stage; thread (g, t) loads A(row, 4 kk + t) and
+// B(4 kk + t, col) from the member's row offsets and k steps.
 template <int BK>
 __device__ __forceinline__ void g_mma_step(double (&acc)[4][4][2], const char *__restrict__ xs,
-                                           const char *__restrict__ ys, const uint32_t (&rx)[4],
-                                           const uint32_t (&ry)[4], const uint32_t (&kx)[BK / 4],
-                                           const uint32_t (&ky)[BK / 4], uint32_t swx, uint32_t swy, int kq) {
+                                           const char *__restrict__ ys, const GRows &r, int t, int kq) {
+  const char *xt = xs + t * r.kmx, *yt = ys + t * r.kmy;
+  const uint32_t sx = 4 * r.kmx, sy = 4 * r.kmy;
 #pragma unroll
   for (int kk = 0; kk < BK / 4; kk++) {
     if (kk < kq) {
       double a[4], b[4];
 #pragma unroll
-      for (int i = 0; i < 4; i++) a[i] = *reinterpret_cast<const double *>(xs + gplane_sw(rx[i] + kx[kk], swx));
+      for (int i = 0; i < 4; i++) a[i] = *reinterpret_cast<const double *>(xt + r.rx[i] + kk * sx);
 #pragma unroll
-      for (int j = 0; j < 4; j++) b[j] = *reinterpret_cast<const double *>(ys + gplane_sw(ry[j] + ky[kk], swy));
+      for (int j = 0; j < 4; j++) b[j] = *reinterpret_cast<const double *>(yt + r.ry[j] + kk * sy);
 #pragma unroll
       for (int i = 0; i < 4; i++)
 #pragma unroll
         for (int j = 0; j < 4; j++) dmma884(acc[i][j][0], acc[i][j][1], a[i], b[j]);
     }
-  }
-}
-
-// this thread's k byte offsets of one operand (k = 4 kk + t)
-template <int BK>
-__device__ __forceinline__ void g_kbytes(const GOperandDev &op, int mode, int t, uint32_t (&kb)[BK / 4]) {
-  const int l2 = op.kch_log2[mode];
-  const uint32_t chunk = (uint32_t)op.kchunk[mode], mul = (uint32_t)op.kmul[mode];
-#pragma unroll
-  for (int kk = 0; kk < BK / 4; kk++) {
-    const uint32_t k = (uint32_t)(4 * kk + t);
-    kb[kk] = (k >> l2) * chunk + (k & ((1u << l2) - 1u)) * mul;
   }
 }
 
@@ -296,23 +334,6 @@ struct GTile {
     for (int q = 0; q < kGMaxCdims; q++)
       if (q < rank) o += (int64_t)c[q] * step[q];
     return o;
-  }
-};
-
-// per member, per consumer thread: row byte offsets of its fragments and box offsets of its
-// accumulators (group.hpp consumer table)
-struct GRows {
-  uint32_t rx[4], ry[4];
-  int32_t bm[4], bn[4][2];
-  __device__ __forceinline__ void load(const int32_t *__restrict__ tb, int wm, int wn, int g, int t) {
-#pragma unroll
-    for (int a = 0; a < 4; a++) {
-      rx[a] = (uint32_t)__ldg(tb + wm * 32 + a * 8 + g);
-      ry[a] = (uint32_t)__ldg(tb + 64 + wn * 32 + a * 8 + g);
-      bm[a] = __ldg(tb + 128 + wm * 32 + a * 8 + g);
-      bn[a][0] = __ldg(tb + 192 + wn * 32 + a * 8 + 2 * t);
-      bn[a][1] = __ldg(tb + 192 + wn * 32 + a * 8 + 2 * t + 1);
-    }
   }
 };
 
@@ -361,25 +382,35 @@ tc_f64_group_kernel(const __grid_constant__ GParams p) {
     asm volatile("setmaxnreg.dec.sync.aligned.u32 88;\n" ::: "memory");   // registers to the consumers
     if (TMA) {
       if (warp != K::CW || lane != 0) return;
+      // inputs are re-read by many tiles: keep them in L2 against the streaming C stores
+      uint64_t policy;
+      asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;\n" : "=l"(policy));
       int j = 0;
+      GTmaRec nxt;
+      nxt.load(p.mem[0]);
       for (int lt = 0; lt < ntl; lt++) {
         GTile tile;
         tile.decode(p, (int)blockIdx.x + lt * (int)gridDim.x);
+        int32_t tcT[kGMaxCdims];   // tile origin per C position
+#pragma unroll
+        for (int q = 0; q < kGMaxCdims; q++) tcT[q] = tile.c[q] * p.T[q];
         for (int i = 0; i < p.nmem; i++) {
-          const GMemberDev &M = mems[i];
-          const uint32_t tx = (uint32_t)(M.x.tma_tx + M.y.tma_tx);
+          // this member's recipe was loaded one member ahead (its latency hides behind the
+          // previous member's stage wait)
+          const GTmaRec M = nxt;
+          nxt.load(p.mem[i + 1 < p.nmem ? i + 1 : 0]);
           for (int s = 0; s < M.nsteps; s++, j++) {
             const int st = j % STAGES;
-            const GStepDev &S = p.steps[M.step0 + s];
+            const int32_t kc = s == 0 ? 0 : p.steps[M.step0 + s].kc;   // (step 0 starts at k = 0)
             GTRACE(3, j);
             if (j >= STAGES) mbar_wait(bar0 + 8 * (STAGES + st), ((j / STAGES) & 1) ^ 1);
             GTRACE(4, j);
             const uint32_t full = bar0 + 8 * st;
             if (kGAbl == 1) { mbar_arrive(full); continue; }
-            mbar_expect_tx(full, tx);
+            mbar_expect_tx(full, M.tx);
             const uint32_t dst = sbase + st * SB;
-            g_tma_operand(&p.xmap[i], M.x, tile.c, p.T, S.kc, dst, full);
-            g_tma_operand(&p.ymap[i], M.y, tile.c, p.T, S.kc, dst + M.tma_yoff, full);
+            g_tma_operand(&p.xmap[i], M.xpack, tcT, kc, dst, full, policy);
+            g_tma_operand(&p.ymap[i], M.ypack, tcT, kc, dst + M.yoff, full, policy);
             GTRACE(5, j);
           }
         }
@@ -443,45 +474,46 @@ tc_f64_group_kernel(const __grid_constant__ GParams p) {
   double acc[4][4][2];
   double *__restrict__ C = p.C;
   const double alpha = p.alpha, beta = p.beta;
+  // this thread's recipe of member 0; each member loads the next one's while it runs
   GRows cur;
-  cur.load(p.ctab, wm, wn, g, t);
+  cur.load(p.ctab, mems[0], MODE, TMA ? -1 : K::PLANE, wm, wn, g, t);
   int j = 0;
+  bool chained = false;   // the previous member left its register tile for this one
   for (int lt = 0; lt < ntl; lt++) {
     for (int i = 0; i < p.nmem; i++) {
-      const GMemberDev &M = mems[i];
-      const int nsteps = M.nsteps, kq = M.kq;
-      uint32_t kx[BK / 4], ky[BK / 4];
-      g_kbytes<BK>(M.x, MODE, t, kx);
-      g_kbytes<BK>(M.y, MODE, t, ky);
-      const uint32_t swx = (uint32_t)M.x.swz[MODE], swy = (uint32_t)M.y.swz[MODE];
-      const int yoff = TMA ? M.tma_yoff : K::PLANE;
-      // the next member's tables, loaded while this member runs
+      const int nsteps = cur.nsteps, kq = cur.kq;
+      const int yoff = cur.yoff;
       GRows nxt;
-      nxt.load(p.ctab + (i + 1 < p.nmem ? i + 1 : 0) * kGCtab, wm, wn, g, t);
+      const int in = i + 1 < p.nmem ? i + 1 : 0;
+      nxt.load(p.ctab + in * kGCtab, mems[in], MODE, TMA ? -1 : K::PLANE, wm, wn, g, t);
       // ---- the member's register tile starts from the box (every consumer finished the
-      //      previous member's write-back — or the previous tile's copy-out — first)
-      consumer_sync(K::CW * 32);
+      //      previous member's write-back — or the previous tile's copy-out — first), or
+      //      simply continues when the previous member mapped it onto the box the same way
+      if (!chained) {
+        consumer_sync(K::CW * 32);
 #pragma unroll
-      for (int a = 0; a < 4; a++)
+        for (int a = 0; a < 4; a++)
 #pragma unroll
-        for (int b = 0; b < 4; b++)
+          for (int b = 0; b < 4; b++)
 #pragma unroll
-          for (int h = 0; h < 2; h++) {
-            const bool ok = i > 0 && kGAbl != 3 && cur.bm[a] >= 0 && cur.bn[b][h] >= 0;
-            acc[a][b][h] = ok ? box[gbox_sw(cur.bm[a] + cur.bn[b][h])] : 0.0;
-          }
+            for (int h = 0; h < 2; h++) {
+              const bool ok = i > 0 && kGAbl != 3 && cur.bm[a] >= 0 && cur.bn[b][h] >= 0;
+              acc[a][b][h] = ok ? box[gbox_sw(cur.bm[a] + cur.bn[b][h])] : 0.0;
+            }
+      }
       for (int s = 0; s < nsteps; s++, j++) {
         const int st = j % STAGES;
         mbar_wait(bar0 + 8 * st, (j / STAGES) & 1);
         GTRACE(0, j);
         const char *xs = reinterpret_cast<const char *>(ring) + st * SB;
-        if (kGAbl != 2) g_mma_step<BK>(acc, xs, xs + yoff, cur.rx, cur.ry, kx, ky, swx, swy, kq);
+        if (kGAbl != 2) g_mma_step<BK>(acc, xs, xs + yoff, cur, t, kq);
         __syncwarp();
         if (lane == 0) mbar_arrive(bar0 + 8 * (STAGES + st));
         GTRACE(1, j);
       }
-      // ---- write the member's tile back into the box
-      if (kGAbl != 3) {
+      // ---- write the member's tile back into the box (unless the next member continues it)
+      chained = cur.chain;
+      if (kGAbl != 3 && !chained) {
 #pragma unroll
         for (int a = 0; a < 4; a++)
 #pragma unroll
@@ -506,12 +538,13 @@ tc_f64_group_kernel(const __grid_constant__ GParams p) {
       if (tile.interior && p.cvec16) {
         double2 v = make_double2(alpha * box[gbox_sw(o)], alpha * box[gbox_sw(o + 1)]);
         double2 *d2 = reinterpret_cast<double2 *>(dst);
+        // (C streams through L2 once: evict-first loads and stores keep the inputs there)
         if (beta != 0.0) {
-          const double2 old = *d2;
+          const double2 old = __ldcs(d2);
           v.x = fma(beta, old.x, v.x);
           v.y = fma(beta, old.y, v.y);
         }
-        *d2 = v;
+        __stcs(d2, v);
       } else {
         const uint64_t dg = __ldg(p.unitDig + u);
         const bool ok = tile.interior || g_all_lt(dg, tile.Lc, mH);
