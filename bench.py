@@ -211,7 +211,7 @@ _TDT = {"f64": "float64", "f32": "float32", "tf32": "float32", "bf16": "bfloat16
 _ES = {"f64": 8, "f32": 4, "tf32": 4, "bf16": 2}
 
 
-def time_one(p, A, B, C, steps, warmup, flush, stream):
+def time_one(p, A, B, C, steps, warmup, flush, stream, beta=0.0):
     """Median device time (ms) of one tc_execute over `steps` launches, CUDA events on the
     launch stream, L2 flushed (outside the events) before every launch."""
     import torch
@@ -221,7 +221,7 @@ def time_one(p, A, B, C, steps, warmup, flush, stream):
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
         e0.record(stream)
-        p.execute(A, B, C)
+        p.execute(A, B, C, beta=beta)
         e1.record(stream)
         e1.synchronize()
         if i >= warmup:
@@ -232,47 +232,65 @@ def time_one(p, A, B, C, steps, warmup, flush, stream):
 
 def run_triples(args, flush, stream, dev, hbm):
     """CCSD(T) triples: the 18 sd_t_d1 / sd_t_d2 contractions of TCCG-48
-    (#31-48) accumulated into one t3 by tc_execute_group, FP64, uniform extents N.  The
-    roofline is that of the fused ideal (inputs read once, t3 written once): min(FP64 peak,
-    I * HBM) — the headroom the on-chip fusion (t3 written once, not 18 times) would take."""
+    (#31-48) summed into one t3, FP64, at the TCCG extents and at uniform N.  `fused` = ONE
+    kernel (tc_group_plan / tc_group_execute: each t3 tile kept on chip across the 18 members,
+    written once), at beta = 0 and beta = 1 (t3 accumulation); `unfused` = the 18
+    launches of tc_execute_group (t3 read and written by every member), members tuned top-k at
+    their own beta.  The roofline is the fused ideal: min(FP64 peak, I * HBM) with the inputs
+    read once and t3 written once (plus read once at beta = 1)."""
     import torch
     from paper_conf_cgo_kimstkpprs19_b200 import binding as tc
     exprs = [c.expr for c in tcinputs.tccg48() if c.group.startswith("CCSDT")]
-    rows = []
-    for n in (16, 24):
-        ext = ";".join(f"{x}:{n}" for x in "abcdefg")
-        plans = [tc.plan(e, ext, cost=args.cost) for e in exprs]
-        A = [tcinputs.uniform(p.numel("A"), 1000 + i, device=dev) for i, p in enumerate(plans)]
-        B = [tcinputs.uniform(p.numel("B"), 2000 + i, device=dev) for i, p in enumerate(plans)]
-        C = torch.empty(plans[0].numel("C"), dtype=torch.float64, device=dev)
-        if args.tune > 0:   # member 0 writes t3 (beta = 0); the rest accumulate: tuned at beta = 1
-            C.zero_()
-            plans = [p.tuned(A[i], B[i], C, topk=args.tune, reps=2, beta=0.0 if i == 0 else 1.0)
-                     for i, p in enumerate(plans)]
+
+    def timed(fn, reps):
         ts = []
-        for it in range(2 + max(3, min(args.steps, 5))):
+        for it in range(2 + reps):
             flush.zero_()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(stream)
-            tc.execute_group(plans, A, B, C)
+            fn()
             e1.record(stream)
             e1.synchronize()
             if it >= 2:
                 ts.append(e0.elapsed_time(e1))
-        ms = sorted(ts)[len(ts) // 2]
+        return sorted(ts)[len(ts) // 2]
+
+    rows = []
+    tccg = [c for c in tcinputs.tccg48() if c.id == 31][0].extents
+    for ext in (tccg, ";".join(f"{x}:16" for x in "abcdefg"), ";".join(f"{x}:24" for x in "abcdefg")):
+        plans = [tc.plan(e, ext, cost=args.cost) for e in exprs]
+        A = [tcinputs.uniform(p.numel("A"), 1000 + i, device=dev) for i, p in enumerate(plans)]
+        B = [tcinputs.uniform(p.numel("B"), 2000 + i, device=dev) for i, p in enumerate(plans)]
+        C = torch.zeros(plans[0].numel("C"), dtype=torch.float64, device=dev)
         flops = sum(p.flops for p in plans)
-        byts_fused = 8 * (sum(p.numel("A") + p.numel("B") for p in plans) + C.numel())
-        byts_group = 8 * (sum(p.numel("A") + p.numel("B") for p in plans) + (2 * len(plans) - 1) * C.numel())
-        attain = min(FP64_PEAK_TFLOPS * 1e12, flops / byts_fused * hbm)
-        rows.append({"extents": ext, "contractions": len(plans), "ms": round(ms, 4),
-                     "gflops": round(flops / ms / 1e6, 2),
-                     "roofline_frac_vs_fused": round(flops / (ms * 1e-3) / attain, 4),
-                     "hbm_frac_of_group_bytes": round(byts_group / (ms * 1e-3) / hbm, 4)})
-        del A, B, C, plans
+        inb = 8 * sum(p.numel("A") + p.numel("B") for p in plans)
+        reps = max(3, min(args.steps, 10))
+        g = tc.plan_group(plans)
+        row = {"extents": ext, "contractions": len(plans), "fused_tile": g.info()["T"],
+               "fused_tma": g.info()["tma"], "fused_plan_ms": round(g.info()["plan_ms"], 2)}
+        for beta in (0.0, 1.0):
+            ms = timed(lambda: g.execute(A, B, C, 1.0, beta), reps)
+            attain = min(FP64_PEAK_TFLOPS * 1e12, flops / (inb + 8 * C.numel() * (1 + (beta != 0))) * hbm)
+            b = int(beta)
+            row[f"fused_ms_b{b}"] = round(ms, 4)
+            row[f"fused_gflops_b{b}"] = round(flops / ms / 1e6, 2)
+            row[f"fused_roofline_frac_b{b}"] = round(flops / (ms * 1e-3) / attain, 4)
+        if args.tune > 0:   # member 0 writes t3 (beta = 0); the rest accumulate: tuned at beta = 1
+            plans = [p.tuned(A[i], B[i], C, topk=args.tune, reps=2, beta=0.0 if i == 0 else 1.0)
+                     for i, p in enumerate(plans)]
+        ms = timed(lambda: tc.execute_group(plans, A, B, C), 3)
+        attain = min(FP64_PEAK_TFLOPS * 1e12, flops / (inb + 8 * C.numel()) * hbm)
+        row["unfused_ms"] = round(ms, 4)
+        row["unfused_gflops"] = round(flops / ms / 1e6, 2)
+        row["unfused_roofline_frac_vs_fused"] = round(flops / (ms * 1e-3) / attain, 4)
+        row["fused_speedup"] = round(ms / row["fused_ms_b0"], 2)
+        rows.append(row)
+        del A, B, C, plans, g
         torch.cuda.empty_cache()
-    return {"workload": "CCSD(T) triples: TCCG-48 #31-48 into one t3 (tc_execute_group, beta=1 "
-                        "after the first), FP64, all extents N; L2 flushed before each group; "
-                        "members tuned top-k at their own beta (tc_plan_tuned_beta)",
+    return {"workload": "CCSD(T) triples: TCCG-48 #31-48 into one t3, FP64, at the TCCG extents "
+                        "and all extents N; fused = one tc_group_execute kernel (beta 0 / 1), "
+                        "unfused = tc_execute_group (18 launches, members tuned at their beta); "
+                        "L2 flushed before each group",
             "cases": rows}
 
 
@@ -286,25 +304,26 @@ def run_suite(name, args, flush, stream, dev, hbm):
     if name == "triples":
         return run_triples(args, flush, stream, dev, hbm)
     if name == "ccsdt":
-        # BASELINE config 3: sd_t_d1 / sd_t_d2 6D contractions at uniform extents 24..48, FP64
-        todo = [(tcinputs.ccsdt(n, e, 100 + n), "f64") for e in ("abcdef-gdab-efgc", "abcdef-dega-gfbc")
-                for n in (24, 32, 40, 48)]
+        # BASELINE config 3: sd_t_d1 / sd_t_d2 6D contractions at uniform extents 24..48, FP64,
+        # beta = 0 (t3 written) and beta = 1 (t3 accumulated)
+        todo = [(tcinputs.ccsdt(n, e, 100 + n), "f64", beta) for e in ("abcdef-gdab-efgc", "abcdef-dega-gfbc")
+                for n in (24, 32, 40, 48) for beta in (0.0, 1.0)]
     else:
         # BASELINE config 4: the memory-bound TCCG cases (#1-8 ML tensor x matrix, #18 ab-ac-cb)
         mb = [c for c in tcinputs.tccg48() if c.id <= 8 or c.id == 18]
-        todo = [(c, dt) for dt in ("f32", "tf32", "bf16") for c in mb]
-    for c, dt in todo:
+        todo = [(c, dt, 0.0) for dt in ("f32", "tf32", "bf16") for c in mb]
+    for c, dt, beta in todo:
         tdt = getattr(torch, _TDT[dt])
         p = tc.plan(c.expr, c.extents, dtype=dt, cost=args.cost)
         A = tcinputs.uniform(p.numel("A"), 1000 + c.id, device=dev).to(tdt)
         B = tcinputs.uniform(p.numel("B"), 2000 + c.id, device=dev).to(tdt)
-        C = torch.empty(p.numel("C"), dtype=tdt, device=dev)
+        C = torch.zeros(p.numel("C"), dtype=tdt, device=dev) if beta else torch.empty(p.numel("C"), dtype=tdt, device=dev)
         if args.tune > 0:
-            p = p.tuned(A, B, C, topk=args.tune, reps=2)
-        ms = time_one(p, A, B, C, max(3, min(args.steps, 5)), 2, flush, stream)
-        byts = _ES[dt] * (p.numel("A") + p.numel("B") + p.numel("C"))
+            p = p.tuned(A, B, C, topk=args.tune, reps=2, beta=beta)
+        ms = time_one(p, A, B, C, max(3, min(args.steps, 5)), 2, flush, stream, beta=beta)
+        byts = _ES[dt] * (p.numel("A") + p.numel("B") + p.numel("C") * (2 if beta else 1))
         gbs = byts / (ms * 1e-3) / 1e9
-        r = {"expr": c.expr, "extents": c.extents, "dtype": dt, "ms": round(ms, 5),
+        r = {"expr": c.expr, "extents": c.extents, "dtype": dt, "beta": beta, "ms": round(ms, 5),
              "gflops": round(p.flops / ms / 1e6, 2), "gbs": round(gbs, 1),
              "variant": p.info()["variant"]}
         if dt == "f64":
@@ -318,8 +337,10 @@ def run_suite(name, args, flush, stream, dev, hbm):
     out = {"cases": rows}
     if name == "ccsdt":
         out["workload"] = "CCSD(T) sd_t_d2 abcdef-gdab-efgc and sd_t_d1 abcdef-dega-gfbc, all extents N, FP64"
-        out["geomean_gflops"] = round(geomean([r["gflops"] for r in rows]), 2)
-        out["geomean_roofline_frac"] = round(geomean([r["roofline_frac"] for r in rows]), 4)
+        for b in (0.0, 1.0):
+            sel = [r for r in rows if r["beta"] == b]
+            out[f"geomean_gflops_beta{int(b)}"] = round(geomean([r["gflops"] for r in sel]), 2)
+            out[f"geomean_roofline_frac_beta{int(b)}"] = round(geomean([r["roofline_frac"] for r in sel]), 4)
     else:
         out["workload"] = "memory-bound TCCG #1-8, #18 in FP32 (split TF32), TF32, BF16; HBM roofline"
         for dt in ("f32", "tf32", "bf16"):

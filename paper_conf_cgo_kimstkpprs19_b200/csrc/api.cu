@@ -117,6 +117,12 @@ void build_host_tables(tc_plan_s *P) {
   kp.ct0 = ct0;
   kp.Nt = (int)cfg.Nt;
   kp.c_rank = (int)c.t[0].idx.size();
+  // old-C prefetch (beta != 0): C's FVI leads the m digits, so runs of its tile are C-contiguous
+  // rows: one address per 128-B line (16 doubles)
+  P->pf_step = 0;
+  if (cfg.kind == KIND_F64_DMMA && !cfg.mdig.empty() && !c.t[0].idx.empty() && cfg.mdig[0] == c.t[0].idx[0] &&
+      c.t[0].stride[0] == 1)
+    P->pf_step = std::min<int>(16, cfg.T[cfg.mdig[0]]);
 }
 
 Status upload(tc_plan_s *P, std::string &err) {
@@ -606,6 +612,7 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
   // C stores in 16-B vectors: 8 elements (staged UMMA epilogue: one 16-B BF16 or two 16-B FP32
   // stores) / 2 FP64 (STG drain)
   kp.vecC = plan->cvec > 1 && ((uintptr_t)C % 16) == 0 ? plan->cvec : 1;
+  kp.pf_mstep = beta != 0.0 ? plan->pf_step : 0;
   const KernelEntry ke = kernel_for(cfg);
   const int grid = (int)std::min<int64_t>(cfg.nctas, plan->sms);
   void *args[] = {&kp};

@@ -413,6 +413,18 @@ tc_f64_dmma_kernel(const __grid_constant__ KParams p) {
       if (vy) issue_slots<K::EY, true>(Y, dy, ry, py, by, fn && fk, km, mn);
       else issue_slots<K::EY, false>(Y, dy, ry, py, by, fn && fk, km, mn);
       mbar_arrive_cp_async(bar0 + 8 * s);
+      if (p.pf_mstep > 0 && step == 0) {
+        // beta != 0: the epilogue reads this tile's old C; pull it into L2 now (the producers
+        // run STAGES k-steps ahead of the consumers' epilogue), a line per pf_mstep rows
+        int mt, nt;
+        tile_coords(p, (int)blockIdx.x + lt * (int)gridDim.x, mt, nt);
+        const double *Ct = static_cast<const double *>(p.C) + (p.tileM[mt].c + p.tileN[nt].c);
+        const int nm = (p.Mt + p.pf_mstep - 1) / p.pf_mstep;
+        for (int q = ptid; q < nm * p.Nt; q += PW * 32) {
+          const int n = q / nm, mi = (q - n * nm) * p.pf_mstep;
+          asm volatile("prefetch.global.L2 [%0];\n" ::"l"(Ct + relCm[mi] + relCn[n]));
+        }
+      }
       ks.advance(p);
       if (++step == p.nsteps) {
         step = 0;

@@ -77,6 +77,8 @@ struct KParams {
   const uint32_t *packY;
   int nslotX, nslotY;
   int vecX, vecY;           // elements per slot (16-B cp.async at 2 FP64 / 8 BF16)
+  int pf_mstep;             // FP64, beta != 0: producers prefetch the tile's old C into L2, one
+                            // address per pf_mstep tile rows (0: off; C's FVI must lead m)
   int vecC;                 // C vector (elements): BF16 8 / FP64 STG 2 => tile rows come in aligned
                             // C-contiguous runs of vecC (16-B stores); 1 => per-element stores
   int nmma, kmma;           // UMMA: instruction N (<= BN) and K-instructions per stage (<= BK / KI)
