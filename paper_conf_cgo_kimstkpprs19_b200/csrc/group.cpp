@@ -25,24 +25,21 @@ int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
 // Shared-memory wavefronts of a sequence of warp instructions: entries (byte offset, bytes)
 // in lane order, 32 per instruction; a bank (4-byte words, 32 banks) serves one word per
-// wavefront.
+// wavefront.  The entries of one instruction are distinct elements (their words differ):
+// a histogram per bank.
 double smem_wavefronts(const std::vector<std::pair<int64_t, int>> &acc) {
   double total = 0;
-  std::vector<int64_t> words[32];
   for (size_t b = 0; b < acc.size(); b += 32) {
     const size_t e = std::min(acc.size(), b + 32);
-    for (auto &w : words) w.clear();
+    int cnt[32] = {0};
     int64_t bytes = 0;
     for (size_t i = b; i < e; i++) {
-      for (int64_t w = acc[i].first / 4; w < (acc[i].first + acc[i].second + 3) / 4; w++) words[w & 31].push_back(w);
+      for (int64_t w = acc[i].first / 4; w < (acc[i].first + acc[i].second + 3) / 4; w++) cnt[w & 31]++;
       bytes += acc[i].second;
     }
-    size_t wf = 0;
-    for (auto &s : words) {
-      std::sort(s.begin(), s.end());
-      wf = std::max(wf, (size_t)(std::unique(s.begin(), s.end()) - s.begin()));
-    }
-    total += (double)std::max<int64_t>((int64_t)wf, (bytes + 127) / 128);
+    int wf = 0;
+    for (int k = 0; k < 32; k++) wf = std::max(wf, cnt[k]);
+    total += (double)std::max<int64_t>(wf, (bytes + 127) / 128);
   }
   return total;
 }

@@ -68,7 +68,7 @@ static std::pair<double, double> operand_sim(const Contraction &c, const Config 
 }
 
 // ---------------------------------------------------------------- B200 cost model
-double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *cache) {
+double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *cache, bool lower_bound) {
   finish_counts(c, cfg);
   const double nctas = (double)cfg.nctas * (double)c.nbatch(), steps = (double)cfg.nsteps;
   // per CTA-step pipe cycles on one SM: FP64 (DMMA) and shared memory
@@ -82,8 +82,15 @@ double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *
   const int maxv = 16 / kind_esize(cfg.kind);   // 16 B per cp.async
   cfg.vecX = vec_width(c, cfg, cfg.X, maxv);
   cfg.vecY = vec_width(c, cfg, cfg.Y, maxv);
-  const auto sx = operand_sim(c, cfg, cfg.X, cfg.vecX, cfg.xKmajor, v.BM, v.BK, cache);
-  const auto sy = operand_sim(c, cfg, cfg.Y, cfg.vecY, cfg.yKmajor, v.BN, v.BK, cache);
+  // lower_bound: the conflict-free ideal of the simulated terms (every smem wavefront and every
+  // global sector fully used) — a cheap bound that prunes configurations before simulating
+  const double es0 = kind_esize(cfg.kind);
+  const auto ideal = [&](int64_t rows) {
+    const double b = (double)rows * cfg.Kt * es0;
+    return std::pair<double, double>{std::ceil(b / 128.0), std::ceil(b / 32.0)};
+  };
+  const auto sx = lower_bound ? ideal(cfg.Mt) : operand_sim(c, cfg, cfg.X, cfg.vecX, cfg.xKmajor, v.BM, v.BK, cache);
+  const auto sy = lower_bound ? ideal(cfg.Nt) : operand_sim(c, cfg, cfg.Y, cfg.vecY, cfg.yKmajor, v.BN, v.BK, cache);
   cfg.wfX = sx.first;
   cfg.wfY = sy.first;
   cfg.secX = sx.second;
@@ -259,7 +266,7 @@ std::vector<std::vector<int>> rotations(const std::vector<int> &lst) {
 // rest are filled greedily up to the side's total target S.
 std::vector<Tiling> enum_side(const Contraction &c, const std::vector<int> &order, int fixed_first,
                               int64_t S) {
-  std::set<Tiling> uniq;
+  std::vector<Tiling> uniq;   // (sorted and deduplicated at the end)
   std::vector<std::vector<int>> rots;
   if (fixed_first >= 0) {
     std::vector<int> rest;
@@ -273,7 +280,7 @@ std::vector<Tiling> enum_side(const Contraction &c, const std::vector<int> &orde
     rots = rotations(order);
   }
   for (auto &seq : rots) {
-    if (seq.empty()) { uniq.insert(Tiling()); continue; }
+    if (seq.empty()) { uniq.push_back(Tiling()); continue; }
     const int first = seq[0];
     const int64_t n0 = c.ix[first].n;
     std::set<int64_t> t0s;
@@ -285,10 +292,12 @@ std::vector<Tiling> enum_side(const Contraction &c, const std::vector<int> &orde
       std::vector<Tiling> res;
       if (t0 < n0) res.push_back(cur);  // first index alone (the others on the grid)
       greedy(c, seq, 1, t0, S, cur, false, res);
-      for (auto &x : res) uniq.insert(x);
+      uniq.insert(uniq.end(), res.begin(), res.end());
     }
   }
-  return std::vector<Tiling>(uniq.begin(), uniq.end());
+  std::sort(uniq.begin(), uniq.end());
+  uniq.erase(std::unique(uniq.begin(), uniq.end()), uniq.end());
+  return uniq;
 }
 
 int64_t tprod(const Tiling &t) {
@@ -365,18 +374,30 @@ static Status choose_b200(const Contraction &c, int kind, int forced_variant, in
   else if (!c.t[base.Y].idx.empty() && c.ix[c.t[base.Y].idx[0]].cls == INTL) kfirst = c.t[base.Y].idx[0];
   const auto orders = order_options(c, kind, only_morder);
   bool found = false;
-  for (int vi = 0; vi < (int)variants().size(); vi++) {
-    if (forced_variant >= 0 && vi != forced_variant) continue;
-    if (variants()[vi].kind != kind) continue;
+  // the side enumerations depend only on the side's target size: shared by the variants
+  std::map<int64_t, std::vector<Tiling>> msC, nsC, ksC;
+  auto side_of = [&](std::map<int64_t, std::vector<Tiling>> &m, const std::vector<int> &ids, int first, int64_t S)
+      -> const std::vector<Tiling> & {
+    auto it = m.find(S);
+    if (it == m.end()) it = m.emplace(S, enum_side(c, ids, first, S)).first;
+    return it->second;
+  };
+  // variants in order of their DMMA-pipe lower bound at their fullest tiles, so that a good
+  // configuration is known early and bounds the others (planning time)
+  std::vector<int> vorder;
+  for (int vi = 0; vi < (int)variants().size(); vi++)
+    if ((forced_variant < 0 || vi == forced_variant) && variants()[vi].kind == kind) vorder.push_back(vi);
+  for (int vi : vorder) {
     const auto &v = variants()[vi];
     bool vfound = false;
     Config vbest;
-    auto ms = enum_side(c, mx, c0, v.BM);
-    auto ns = enum_side(c, ny, -1, v.BN);
-    auto ks = enum_side(c, kx, kfirst, v.BK);
-    // keep the k tilings with the least padding, top 3
-    std::vector<std::pair<double, Tiling>> kr;
-    for (auto &k : ks) {
+    const auto &ms0 = side_of(msC, mx, c0, v.BM);
+    const auto &ns0 = side_of(nsC, ny, -1, v.BN);
+    const auto &ks = side_of(ksC, kx, kfirst, v.BK);
+    // keep the k tilings with the least padding, top 4 (sorted by index: no tiling copies)
+    std::vector<std::pair<double, int>> kscore;
+    for (size_t q = 0; q < ks.size(); q++) {
+      const Tiling &k = ks[q];
       if (tprod(k) > v.BK) continue;
       std::vector<int> T(c.ix.size(), 1);
       apply_tiling(k, T);
@@ -387,41 +408,49 @@ static Status choose_b200(const Contraction &c, int kind, int forced_variant, in
       for (int t = 1; t <= 2; t++)
         if (!c.t[t].idx.empty() && c.ix[c.t[t].idx[0]].cls == INTL)
           run *= std::min(32 / v.esize(), T[c.t[t].idx[0]]);   // one 32-B sector
-      kr.push_back({steps * v.BK / need / run, k});
+      kscore.push_back({steps * v.BK / need / run, (int)q});
     }
-    std::stable_sort(kr.begin(), kr.end(), [](auto &a, auto &b) { return a.first < b.first; });
-    if (kr.size() > 4) kr.resize(4);
+    std::stable_sort(kscore.begin(), kscore.end(), [](auto &a, auto &b) { return a.first < b.first; });
+    std::vector<std::pair<double, Tiling>> kr;
+    for (size_t q = 0; q < kscore.size() && q < 4; q++) kr.push_back({kscore[q].first, ks[kscore[q].second]});
     // drop m / n tilings that fill less than half of what the fullest one fills
-    auto fill = [](std::vector<Tiling> &v, int64_t S) {
+    auto fill = [](const std::vector<Tiling> &v, int64_t S) {
       int64_t mx = 0;
       for (auto &t : v) if (tprod(t) <= S) mx = std::max(mx, tprod(t));
-      std::vector<Tiling> o;
-      for (auto &t : v) if (tprod(t) <= S && 2 * tprod(t) >= mx) o.push_back(t);
+      std::vector<const Tiling *> o;
+      for (auto &t : v) if (tprod(t) <= S && 2 * tprod(t) >= mx) o.push_back(&t);
       return o;
     };
-    const size_t raw_m = ms.size(), raw_n = ns.size();
-    ms = fill(ms, v.BM);
-    ns = fill(ns, v.BN);
+    const size_t raw_m = ms0.size(), raw_n = ns0.size();
+    const auto ms = fill(ms0, v.BM);
+    const auto ns = fill(ns0, v.BN);
     st.raw += (int64_t)raw_m * raw_n * ks.size() * orders.size();
     st.pruned += (int64_t)(raw_m * raw_n * ks.size() - ms.size() * ns.size() * kr.size()) * orders.size();
-    for (auto &m : ms)
-      for (auto &n : ns)
+    // one scratch configuration per digit order: no Config copies in the loop
+    std::vector<Config> scratch(orders.begin(), orders.end());
+    for (const Tiling *m : ms)
+      for (const Tiling *n : ns)
         for (auto &k : kr)
-          for (const auto &o : orders) {
-            Config cfg = o;
+          for (Config &cfg : scratch) {
             cfg.T.assign(c.ix.size(), 1);
-            apply_tiling(m, cfg.T);
-            apply_tiling(n, cfg.T);
+            apply_tiling(*m, cfg.T);
+            apply_tiling(*n, cfg.T);
             apply_tiling(k.second, cfg.T);
             finish_counts(c, cfg);
             if (!fits(cfg, v)) { st.pruned++; continue; }
             cfg.variant = vi;
-            // bound: the FP64-pipe time of the padded work alone (no smem / memory terms)
-            if (vfound) {
+            // bound: the MMA-pipe time of the padded work alone (no smem / memory terms),
+            // against this variant's best so far and 1.5x the best of every variant (a variant
+            // that far behind is no tuning candidate: its per-variant figure stays an upper one)
+            {
               const double tiles = std::ceil((double)cfg.nctas * (double)c.nbatch() / (kSMs * v.occ));
               const double lb = tiles * v.occ * (double)cfg.nsteps * v.BM * v.BN * v.BK /
                                 fma_per_clk(v.kind) / kClk + kLaunch;
-              if (lb > vbest.t_pred) { st.pruned++; continue; }
+              if ((vfound && lb > vbest.t_pred) || (found && lb > 1.5 * best.t_pred)) { st.pruned++; continue; }
+            }
+            if (vfound || found) {   // the conflict-free ideal of this configuration
+              const double lb = model_time(c, cfg, v, &cache, true);
+              if ((vfound && lb > vbest.t_pred) || (found && lb > 1.5 * best.t_pred)) { st.pruned++; continue; }
             }
             model_time(c, cfg, v, &cache);
             st.ranked++;

@@ -149,6 +149,10 @@ SlotTable build_slots(const Contraction &c, const Config &cfg, int t, int vec, b
   }
   // packed slot: smem offset (elements) | k | row; FP64: 13 | 6 | 13 bits, UMMA: 14 | 6 | 12
   const int kshift = is_umma(cfg.kind) ? 14 : 13, mshift = is_umma(cfg.kind) ? 20 : 19;
+  int64_t nslot = 1;
+  for (int p = 0; p < r; p++) nslot *= p == 0 ? (T[p] + vec - 1) / vec : T[p];
+  out.rel.reserve(nslot);
+  out.pack.reserve(nslot);
   std::vector<int> d(r, 0);
   for (;;) {
     int mn = 0, k = 0;
@@ -174,32 +178,35 @@ SlotTable build_slots(const Contraction &c, const Config &cfg, int t, int vec, b
 double slot_sectors(const SlotTable &s, int vec, int esize) {
   const size_t n = s.rel.size();
   double total = 0;
-  std::vector<int64_t> sec;
+  int64_t sec[64];
   for (size_t b = 0; b < n; b += 32) {
     const size_t e = std::min(n, b + 32);
-    sec.clear();
+    int k = 0;
     for (size_t i = b; i < e; i++) {
-      sec.push_back((s.rel[i] * esize) >> 5);
-      sec.push_back((s.rel[i] * esize + esize * vec - 1) >> 5);
+      sec[k++] = (s.rel[i] * esize) >> 5;
+      sec[k++] = (s.rel[i] * esize + esize * vec - 1) >> 5;
     }
-    std::sort(sec.begin(), sec.end());
-    total += (double)(std::unique(sec.begin(), sec.end()) - sec.begin());
+    std::sort(sec, sec + k);
+    total += (double)(std::unique(sec, sec + k) - sec);
   }
   return total;
 }
 
 double slot_wavefronts(const SlotTable &s, int vec, int esize, int kind) {
+  // per warp instruction (32 slots): the words each of the 32 banks serves.  The slots of a
+  // table are distinct tile elements (build_slots: no padding slots), so their words are
+  // distinct: a histogram per bank, no sort (the planner simulates every table it ranks).
   const size_t n = s.pack.size();
   double total = 0;
   for (size_t b = 0; b < n; b += 32) {
     const size_t e = std::min(n, b + 32);
-    std::set<uint32_t> words[32];
+    int cnt[32] = {0};
     for (size_t i = b; i < e; i++) {
       const uint32_t byte0 = slot_off(s.pack[i], kind) * (uint32_t)esize;
-      for (uint32_t w = byte0 / 4; w < (byte0 + (uint32_t)(esize * vec) + 3) / 4; w++) words[w & 31].insert(w);
+      for (uint32_t w = byte0 / 4; w < (byte0 + (uint32_t)(esize * vec) + 3) / 4; w++) cnt[w & 31]++;
     }
     int wf = 0;
-    for (int k = 0; k < 32; k++) wf = std::max(wf, (int)words[k].size());
+    for (int k = 0; k < 32; k++) wf = std::max(wf, cnt[k]);
     const int minwf = (int)(((e - b) * esize * vec + 127) / 128);
     total += std::max(wf, minwf);
   }
