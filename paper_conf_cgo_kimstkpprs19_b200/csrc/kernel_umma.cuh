@@ -401,15 +401,16 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
     // groups); MN-major SBO = 128 (8-row groups), LBO = rows/8 * 128 (k groups)
     // 128-B swizzled layouts (tiles.hpp smem_off): K-major = 8-row x 128-B atoms stacked
     // along M/N (SBO = 1 KB; K = 16 advances the start by 32 B inside the atom); MN-major =
-    // 64-element x 8-k atoms, MN atoms at LBO = 1 KB, 8-k groups at SBO = BMN/64 KB
+    // 64-element x 8-k atoms, the k groups of one MN atom adjacent (SBO = 1 KB) and the MN
+    // atoms BK/8 KB apart (LBO) — the order a TMA box of (64 MN, BK k) lands in smem
     // (E = 128 / ES elements per 128-B row; one MMA consumes K = KI = 32 B of k.  BF16
     // MN-major: 8-k x 128-B atoms (1 KB), K = 16 = two k groups.  TF32 MN-major
     // (SWIZZLE_128B_BASE32B): 4-k x 128-B atoms (512 B), K = 8 = two k groups.)
     constexpr int E = 128 / ES;
     constexpr uint32_t ATOM = ES == 4 ? 512 : 1024, KG = ES == 4 ? 4 : 8;   // MN-major atom bytes, k rows
     constexpr int XL = XK || ES == 2 ? 2 : 1, YL = YK || ES == 2 ? 2 : 1;   // descriptor layout types
-    constexpr uint32_t A_LBO = XK ? 16 : ATOM, A_SBO = XK ? 1024 : (BM / E) * ATOM;
-    constexpr uint32_t B_LBO = YK ? 16 : ATOM, B_SBO = YK ? 1024 : (BN / E) * ATOM;
+    constexpr uint32_t A_LBO = XK ? 16 : (BK / KG) * ATOM, A_SBO = XK ? 1024 : ATOM;
+    constexpr uint32_t B_LBO = YK ? 16 : (BK / KG) * ATOM, B_SBO = YK ? 1024 : ATOM;
     constexpr uint32_t A_KSTEP = XK ? 32 : (K::KI / KG) * A_SBO, B_KSTEP = YK ? 32 : (K::KI / KG) * B_SBO;
     int step = 0, lt = 0;
     for (int j = 0; j < total; j++) {

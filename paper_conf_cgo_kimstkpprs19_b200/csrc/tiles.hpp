@@ -49,14 +49,15 @@ inline int smem_off(int kind, bool kmajor, int mn, int k, int BMN, int BK) {
       byte = (mn / 8) * 1024 + r * 128 + (((kb >> 4) ^ r) << 4) + (kb & 15);
     } else if (es == 4) {
       // FP32 / TF32 MN-major (SWIZZLE_128B_BASE32B): 4-k x 128-B atoms of 512 B, atom
-      // (mn/32, k/4) at ((k/4) (BMN/32) + mn/32) 512 B, row k%4, the 32-B granule XORed with it
+      // (mn/32, k/4) at ((mn/32) (BK/4) + k/4) 512 B (the k groups of an MN atom adjacent: a
+      // TMA box of 32 MN x BK k), row k%4, the 32-B granule XORed with it
       const int r = k % 4, eb = (mn % E) * es;
-      byte = ((k / 4) * (BMN / E) + mn / E) * 512 + r * 128 + (((eb >> 5) ^ r) << 5) + (eb & 31);
+      byte = ((mn / E) * (BK / 4) + k / 4) * 512 + r * 128 + (((eb >> 5) ^ r) << 5) + (eb & 31);
     } else {
       const int r = k % 8, eb = (mn % E) * es;
-      byte = ((k / 8) * (BMN / E) + mn / E) * 1024 + r * 128 + (((eb >> 4) ^ r) << 4) + (eb & 15);
+      byte = ((mn / E) * (BK / 8) + k / 8) * 1024 + r * 128 + (((eb >> 4) ^ r) << 4) + (eb & 15);
     }
-    (void)BK;
+    (void)BMN;
     return byte / es;
   }
   return kmajor ? mn * (BK + 4) + k : k * (BMN + 4) + mn;
