@@ -66,7 +66,9 @@ typedef struct tc_plan_opts {
                         when C is a legal tensor map and beta == 0; 0 (default): direct stores */
   int morder;        /* 0: planner's choice; 1: m digits in C order (C's FVI first); 2: in the X
                         operand's memory order (its FVI first) — tests of both epilogues   */
-  int reserved[6];   /* must be zero (TC_ERR_INVALID_ARG otherwise)                         */
+  int no_tma_operands; /* 1: tcgen05 plans load operands with cp.async even where TMA boxes
+                          fit (default 0: one thread issues TMA boxes when the plan allows) */
+  int reserved[5];   /* must be zero (TC_ERR_INVALID_ARG otherwise)                         */
 } tc_plan_opts;
 
 /*

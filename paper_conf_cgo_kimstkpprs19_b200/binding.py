@@ -44,7 +44,8 @@ class TcError(RuntimeError):
 class _Opts(ctypes.Structure):
     _fields_ = [("cost_mode", ctypes.c_int), ("host_only", ctypes.c_int), ("variant", ctypes.c_int),
                 ("force_tiles", ctypes.c_char_p), ("no_fusion", ctypes.c_int), ("tma_epilogue", ctypes.c_int),
-                ("morder", ctypes.c_int), ("reserved", ctypes.c_int * 6)]
+                ("morder", ctypes.c_int), ("no_tma_operands", ctypes.c_int),
+                ("reserved", ctypes.c_int * 5)]
 
 
 _lib = None
@@ -213,8 +214,9 @@ class Plan:
         return C
 
 
-def _opts(cost, host_only, variant, force_tiles, fusion, tma, morder) -> _Opts:
+def _opts(cost, host_only, variant, force_tiles, fusion, tma, morder, tma_operands=True) -> _Opts:
     o = _Opts()
+    o.no_tma_operands = int(not tma_operands)
     o.morder = {None: 0, "C": 1, "X": 2}[morder]
     o.tma_epilogue = int(tma)
     o.cost_mode = COST[cost]
@@ -227,9 +229,9 @@ def _opts(cost, host_only, variant, force_tiles, fusion, tma, morder) -> _Opts:
 
 def plan_cached(expr: str, extents: str, dtype: str = "f64", cost: str = "b200", host_only: bool = False,
                 variant: int | None = None, force_tiles: str | None = None, fusion: bool = True,
-                tma: bool = False, morder: str | None = None) -> Plan:
+                tma: bool = False, morder: str | None = None, tma_operands: bool = True) -> Plan:
     """tc_plan_cached: the process-wide cached plan of these arguments (planned on first use)."""
-    o = _opts(cost, host_only, variant, force_tiles, fusion, tma, morder)
+    o = _opts(cost, host_only, variant, force_tiles, fusion, tma, morder, tma_operands)
     h = ctypes.c_void_p()
     _raise(lib().tc_plan_cached(ctypes.byref(h), expr.encode(), extents.encode(), DTYPES[dtype], ctypes.byref(o)))
     p = Plan(h, expr, extents, dtype)
@@ -322,9 +324,9 @@ def plan_cache_clear() -> None:
 
 def plan(expr: str, extents: str, dtype: str = "f64", cost: str = "b200", host_only: bool = False,
          variant: int | None = None, force_tiles: str | None = None, fusion: bool = True,
-         tma: bool = False, morder: str | None = None) -> Plan:
+         tma: bool = False, morder: str | None = None, tma_operands: bool = True) -> Plan:
     """morder: None = planner's choice, "C" = m digits in C order, "X" = in the X operand's order."""
-    o = _opts(cost, host_only, variant, force_tiles, fusion, tma, morder)
+    o = _opts(cost, host_only, variant, force_tiles, fusion, tma, morder, tma_operands)
     h = ctypes.c_void_p()
     _raise(lib().tc_plan_ex(ctypes.byref(h), expr.encode(), extents.encode(), DTYPES[dtype], ctypes.byref(o)))
     p = Plan(h, expr, extents, dtype)

@@ -57,12 +57,12 @@ int kind_of(int dtype) {
 }
 
 // The instance for the plan's variant and smem layouts (kernel_table.cuh).
-KernelEntry kernel_for(const Config &cfg) {
+KernelEntry kernel_for(const Config &cfg, bool tma_operands = false) {
   const Variant &v = variants()[cfg.variant];
   if (is_umma(v.kind)) {
     size_t smem = 0;
     int threads = 0;
-    const void *fn = kernel_ptr_umma(cfg.variant, cfg.xKmajor, cfg.yKmajor, &smem, &threads);
+    const void *fn = kernel_ptr_umma(cfg.variant, cfg.xKmajor, cfg.yKmajor, tma_operands, &smem, &threads);
     return {fn, threads, smem, smem};
   }
   const F64Instance k = cfg.xKmajor ? (cfg.yKmajor ? f64_instance_11(cfg.variant) : f64_instance_10(cfg.variant))
@@ -119,6 +119,10 @@ void build_host_tables(tc_plan_s *P) {
   kp.c_rank = (int)c.t[0].idx.size();
   // old-C prefetch (beta != 0): C's FVI leads the m digits, so runs of its tile are C-contiguous
   // rows: one address per 128-B line (16 doubles)
+  P->umma_tma = !P->opts.no_tma_operands &&
+                umma_tma_spec(c, cfg, v, cfg.X, &P->mapX, &kp.xt) &&
+                umma_tma_spec(c, cfg, v, cfg.Y, &P->mapY, &kp.yt);
+  kp.kt = cfg.kdig.empty() ? 0 : (int)cfg.T[cfg.kdig[0]];
   P->pf_step = 0;
   if (cfg.kind == KIND_F64_DMMA && !cfg.mdig.empty() && !c.t[0].idx.empty() && cfg.mdig[0] == c.t[0].idx[0] &&
       c.t[0].stride[0] == 1)
@@ -182,6 +186,11 @@ Status upload(tc_plan_s *P, std::string &err) {
   P->d_packX2 = (const uint32_t *)(b + parts[iX2p].off);
   P->d_relY2 = (const int32_t *)(b + parts[iY2].off);
   P->d_packY2 = (const uint32_t *)(b + parts[iY2p].off);
+  if (P->umma_tma) {   // the TMA-operand instance: same smem, its own attribute
+    const KernelEntry kt = kernel_for(P->cfg, true);
+    e = cudaFuncSetAttribute(kt.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kt.smem);
+    if (e != cudaSuccess) { err = std::string("cudaFuncSetAttribute: ") + cudaGetErrorString(e); return ST_CUDA; }
+  }
   const KernelEntry ke = kernel_for(P->cfg);
   const bool tma = P->tt.tma_ok && P->opts.tma_epilogue && P->cfg.kind == KIND_F64_DMMA &&
                    !variants()[P->cfg.variant].stg;
@@ -281,6 +290,34 @@ PFN_cuTensorMapEncodeTiled_v12000 tma_encoder() {
     return (PFN_cuTensorMapEncodeTiled_v12000)p;
   }();
   return fn;
+}
+
+// TMA descriptor of a tcgen05 operand (umma_tma_spec) at this call's pointer.
+bool encode_operand_map(const tc_plan_s *P, const OperandMap &m, const void *ptr, TmaDesc &out) {
+  auto enc = tma_encoder();
+  if (!enc) return false;
+  const int es = kind_esize(P->cfg.kind);
+  const char *base = (const char *)ptr + (int64_t)es * m.base;
+  if ((uintptr_t)base % 16) return false;
+  cuuint64_t dims[kMaxTmaDims], strides[kMaxTmaDims];
+  cuuint32_t box[kMaxTmaDims], el[kMaxTmaDims];
+  for (int j = 0; j < m.rank; j++) {
+    dims[j] = (cuuint64_t)m.dims[j];
+    box[j] = m.box[j];
+    el[j] = 1;
+    if (j > 0) strides[j - 1] = (cuuint64_t)m.strides[j - 1];
+  }
+  CUresult e = enc(reinterpret_cast<CUtensorMap *>(&out),
+                   es == 2 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
+                   (cuuint32_t)m.rank, (void *)base, dims, strides, box, el, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   m.swz32 ? CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B : CU_TENSOR_MAP_SWIZZLE_128B,
+#ifdef TC_UMMA_TMA_PROMO
+                   (CUtensorMapL2promotion)TC_UMMA_TMA_PROMO,
+#else
+                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+#endif
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return e == CUDA_SUCCESS;
 }
 
 // TMA descriptor of the plan's C view: dims in C order, the C tile as the box.
@@ -392,7 +429,7 @@ std::string cache_key(const char *expr, const char *extents, tc_dtype_t dtype, c
   k << expr << '\x1f' << extents << '\x1f' << (int)dtype << '\x1f' << dev;
   if (o)
     k << '\x1f' << o->cost_mode << ',' << o->host_only << ',' << o->variant << ',' << o->no_fusion << ','
-      << o->tma_epilogue << ',' << o->morder << ',' << o->reserved[0] << ','
+      << o->tma_epilogue << ',' << o->morder << ',' << o->no_tma_operands << ','
       << (o->force_tiles ? o->force_tiles : "");
   return k.str();
 }
@@ -613,7 +650,10 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
   // stores) / 2 FP64 (STG drain)
   kp.vecC = plan->cvec > 1 && ((uintptr_t)C % 16) == 0 ? plan->cvec : 1;
   kp.pf_mstep = beta != 0.0 ? plan->pf_step : 0;
-  const KernelEntry ke = kernel_for(cfg);
+  // tcgen05: operands by TMA when the plan allows and both views encode at these pointers
+  const bool tma_ops = plan->umma_tma && encode_operand_map(plan, plan->mapX, kp.X, kp.xmap) &&
+                       encode_operand_map(plan, plan->mapY, kp.Y, kp.ymap);
+  const KernelEntry ke = kernel_for(cfg, tma_ops);
   const int grid = (int)std::min<int64_t>(cfg.nctas, plan->sms);
   void *args[] = {&kp};
   const int64_t nb = plan->c.nbatch();
@@ -740,7 +780,7 @@ tc_status_t tc_plan_info(const tc_plan_t plan, char *json, size_t cap, size_t *n
       << ",\"grid\":" << std::min<int64_t>(g.nctas, plan->sms)
       << ",\"nbatch\":" << c.nbatch();
     o << ",\"vecX\":" << g.vecX << ",\"vecY\":" << g.vecY << ",\"vecC\":" << plan->cvec << ",\"cs0\":" << plan->kp.cs0 << ",\"xKmajor\":" << g.xKmajor
-      << ",\"yKmajor\":" << g.yKmajor << ",\"wfX\":" << g.wfX << ",\"wfY\":" << g.wfY;
+      << ",\"yKmajor\":" << g.yKmajor << ",\"tma_operands\":" << (plan->umma_tma ? 1 : 0) << ",\"wfX\":" << g.wfX << ",\"wfY\":" << g.wfY;
     char buf[512];
     std::snprintf(buf, sizeof buf,
                   ",\"t_pred_ms\":%.6g,\"t_comp_ms\":%.6g,\"t_mem_ms\":%.6g,\"t_l2_ms\":%.6g,"

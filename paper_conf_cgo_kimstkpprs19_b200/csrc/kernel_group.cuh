@@ -186,42 +186,6 @@ __device__ __forceinline__ void g_issue(const GParams &p, const double *__restri
 }
 
 // ---------------------------------------------------------------- TMA producer path
-__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(bar), "r"(bytes) : "memory");
-}
-
-// TMA load of one box at (c0..c4) into smem dst, completing on mbarrier bar, with an L2 policy
-__device__ __forceinline__ void tma_load(const TmaDesc *map, int rank, int32_t c0, int32_t c1, int32_t c2,
-                                         int32_t c3, int32_t c4, uint32_t dst, uint32_t bar, uint64_t pol) {
-  const uint64_t m = reinterpret_cast<uint64_t>(map);
-  switch (rank) {
-    case 1:
-      asm volatile("cp.async.bulk.tensor.1d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.L2::cache_hint"
-                   " [%0], [%1, {%2}], [%3], %4;\n" ::"r"(dst), "l"(m), "r"(c0), "r"(bar), "l"(pol) : "memory");
-      break;
-    case 2:
-      asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.L2::cache_hint"
-                   " [%0], [%1, {%2, %3}], [%4], %5;\n" ::"r"(dst), "l"(m), "r"(c0), "r"(c1), "r"(bar), "l"(pol)
-                   : "memory");
-      break;
-    case 3:
-      asm volatile("cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.L2::cache_hint"
-                   " [%0], [%1, {%2, %3, %4}], [%5], %6;\n" ::"r"(dst), "l"(m), "r"(c0), "r"(c1), "r"(c2), "r"(bar),
-                   "l"(pol) : "memory");
-      break;
-    case 4:
-      asm volatile("cp.async.bulk.tensor.4d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.L2::cache_hint"
-                   " [%0], [%1, {%2, %3, %4, %5}], [%6], %7;\n" ::"r"(dst), "l"(m), "r"(c0), "r"(c1), "r"(c2), "r"(c3),
-                   "r"(bar), "l"(pol) : "memory");
-      break;
-    default:
-      asm volatile("cp.async.bulk.tensor.5d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.L2::cache_hint"
-                   " [%0], [%1, {%2, %3, %4, %5, %6}], [%7], %8;\n" ::"r"(dst), "l"(m), "r"(c0), "r"(c1), "r"(c2),
-                   "r"(c3), "r"(c4), "r"(bar), "l"(pol) : "memory");
-      break;
-  }
-}
-
 // The TMA producer's per-member recipe (group.hpp GOperandDev::tma_pack: 4 bits of C position
 // per map dim, 15 = the k dim / unused; rank at bit 20; k dim at bit 24).
 struct GTmaRec {

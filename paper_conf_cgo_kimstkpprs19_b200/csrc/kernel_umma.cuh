@@ -271,7 +271,42 @@ __device__ __forceinline__ void trace_at(const KParams &p, int slot, int j) {
     static_cast<unsigned long long *>(p.C)[slot * 1024 + j] = clock64();
 }
 
-template <int KIND, int BN, int STAGES, bool XK, bool YK>
+// The boxes of one operand for (tile, k-step): coordinate per map dim = the tile origin along
+// its C position (TileInfo::coord) or the k-step origin; nsub boxes along map dim 0.
+// umma_box_origin resolves the per-dim sources once per tile (registers: a global read per
+// k-step would put its latency on every stage); umma_tma_boxes issues one k-step.
+struct UmmaBox {
+  int32_t c[kMaxTmaDims];   // tile origin per map dim (0 at the k dim)
+  uint32_t kmask;           // bit j: map dim j is the k index
+};
+__device__ __forceinline__ void umma_box_origin(const TmaOperand &o, const int32_t (&coord)[kMaxTmaDims], UmmaBox &b) {
+  b.kmask = 0;
+#pragma unroll
+  for (int j = 0; j < kMaxTmaDims; j++) {
+    const uint32_t src = (o.pack >> (3 * j)) & 7;
+    int32_t v = 0;
+#pragma unroll
+    for (int q = 0; q < kMaxTmaDims; q++) v = src == (uint32_t)q ? coord[q] : v;   // (select: registers)
+    b.c[j] = v;
+    b.kmask |= (src == 7 ? 1u : 0u) << j;
+  }
+}
+__device__ __forceinline__ void umma_tma_boxes(const TmaDesc *map, const TmaOperand &o, const UmmaBox &b, int rank,
+                                               int32_t kc, uint32_t dst, uint32_t bar, uint64_t pol) {
+  int32_t c[kMaxTmaDims];
+#pragma unroll
+  for (int j = 0; j < kMaxTmaDims; j++) c[j] = (b.kmask >> j) & 1 ? kc : b.c[j];
+  for (int q = 0; q < o.nsub; q++) {
+    tma_load(map, rank, c[0], c[1], c[2], c[3], c[4], dst + (uint32_t)(q * o.sub_bytes), bar, pol);
+    c[0] += o.sub_crd;
+  }
+}
+__device__ __forceinline__ void load_coord(const TileInfo *t, int32_t (&c)[kMaxTmaDims]) {
+#pragma unroll
+  for (int q = 0; q < kMaxTmaDims; q++) c[q] = t->coord[q];
+}
+
+template <int KIND, int BN, int STAGES, bool XK, bool YK, bool TMA = false>
 __global__ void __launch_bounds__(UmmaKernel<KIND, BN, STAGES>::THREADS, 1)
 tc_umma_kernel(const __grid_constant__ KParams p) {
   using K = UmmaKernel<KIND, BN, STAGES>;
@@ -310,7 +345,7 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
   for (int r = tid; r < BN; r += K::THREADS) relCn[r] = p.relCn[r];
   if (tid == 0) {
     for (int s = 0; s < STAGES; s++) {
-      mbar_init(FULL + 8 * s, K::PW * 32);   // producer threads (cp.async arrivals)
+      mbar_init(FULL + 8 * s, TMA ? 1 : K::PW * 32);   // the TMA thread / every producer thread
       mbar_init(EMPTY + 8 * s, 1);           // tcgen05.commit of the MMA thread
     }
     for (int b = 0; b < K::NBUF; b++) {
@@ -331,7 +366,61 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
   tc05_fence_after();
   const uint32_t tmem = *tmem_holder;
 
-  if (warp >= K::EW && warp < K::EW + K::PW) {
+  if (TMA && warp >= K::EW && warp < K::EW + K::PW) {
+    // ======================= TMA producer: one elected thread =============================
+    // per stage: the boxes of X and Y land straight in the 128-B swizzled UMMA planes
+    // (K-major: rows of BK k; MN-major: 64-element atoms, the k groups adjacent), completing
+    // the stage's FULL barrier by their byte count; the other producer threads idle
+    if (tid == K::EW * 32) {
+      uint64_t policy;
+#if defined(TC_UMMA_TMA_POL) && TC_UMMA_TMA_POL == 0
+      asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;\n" : "=l"(policy));
+#elif defined(TC_UMMA_TMA_POL) && TC_UMMA_TMA_POL == 2
+      asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;\n" : "=l"(policy));
+#else
+      asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;\n" : "=l"(policy));
+#endif
+      const uint32_t tx = (uint32_t)(p.xt.nsub * p.xt.tx + p.yt.nsub * p.yt.tx);
+      const int rx = (int)((p.xt.pack >> 16) & 7), ry = (int)((p.yt.pack >> 16) & 7);
+      int step = 0, lt = 0, mt = 0, nt = 0;
+      UmmaBox bx, by;
+      int32_t nxc[kMaxTmaDims], nyc[kMaxTmaDims];   // the next tile's origin, read one tile ahead
+      if (ntl > 0) {
+        tile_coords(p, (int)blockIdx.x, mt, nt);
+        load_coord(&p.tileM[mt], nxc);
+        load_coord(&p.tileN[nt], nyc);
+        umma_box_origin(p.xt, nxc, bx);
+        umma_box_origin(p.yt, nyc, by);
+        if (ntl > 1) {
+          tile_coords(p, (int)blockIdx.x + (int)gridDim.x, mt, nt);
+          load_coord(&p.tileM[mt], nxc);
+          load_coord(&p.tileN[nt], nyc);
+        }
+      }
+      for (int j = 0; j < total; j++) {
+        const int s = j % STAGES;
+        if (j >= STAGES) mbar_wait(EMPTY + 8 * s, ((j / STAGES) & 1) ^ 1);
+        mbar_expect_tx(FULL + 8 * s, tx);
+        const uint32_t dx = sbase + (uint32_t)ES * (uint32_t)(s * K::XS);
+        const uint32_t dy = sbase + (uint32_t)ES * (uint32_t)(STAGES * K::XS + s * K::YS);
+        const int32_t kc = step * p.kt;
+        umma_tma_boxes(&p.xmap, p.xt, bx, rx, kc, dx, FULL + 8 * s, policy);
+        umma_tma_boxes(&p.ymap, p.yt, by, ry, kc, dy, FULL + 8 * s, policy);
+        if (++step == p.nsteps) {
+          step = 0;
+          if (++lt < ntl) {
+            umma_box_origin(p.xt, nxc, bx);
+            umma_box_origin(p.yt, nyc, by);
+            if (lt + 1 < ntl) {
+              tile_coords(p, (int)blockIdx.x + (lt + 1) * (int)gridDim.x, mt, nt);
+              load_coord(&p.tileM[mt], nxc);
+              load_coord(&p.tileN[nt], nyc);
+            }
+          }
+        }
+      }
+    }
+  } else if (warp >= K::EW && warp < K::EW + K::PW) {
     // ======================= producers ===================================================
     const int pt = tid - K::EW * 32;
     const T *__restrict__ X = static_cast<const T *>(p.X);

@@ -39,7 +39,21 @@ struct alignas(64) TmaDesc {
   unsigned char bytes[128];
 };
 
+// tcgen05 kernel, TMA operand loads (api.cu umma_tma_layout): one elected producer thread
+// issues, per stage, the boxes of X and Y straight into the 128-B swizzled UMMA planes
+struct TmaOperand {
+  uint32_t pack;            // per map dim j < 5: 3 bits of source (0-4: C position -> tile
+                            // origin coordinate; 7: the k index -> k-step origin), rank at bit 16
+  int nsub;                 // boxes along map dim 0 (MN-major operands wider than one atom)
+  int sub_bytes;            // smem stride between those boxes
+  int sub_crd;              // coordinate step along dim 0 between them
+  int tx;                   // bytes one box delivers
+};
+
 struct KParams {
+  TmaDesc xmap, ymap;       // tcgen05 + TMA: the operands' tensor maps (per call: they hold the pointers)
+  TmaOperand xt, yt;
+  int kt;                   // tcgen05 + TMA: k-tile extent (coordinate step per k-step)
   TmaDesc cmap;             // TMA descriptor of C (tile box = the C tile), if use_tma
   int use_tma;              // 1: epilogue stages the C tile in smem and TMA-stores it
   int c_rank;               // dimensions of the C descriptor

@@ -32,6 +32,10 @@ struct tc_plan_s {
   SlotTable slotX1, slotY1, slotX2, slotY2;   // scalar and cfg.vecX / cfg.vecY wide slots
   int cvec = 1;            // c_vec_width of the plan (16-B C stores when > 1)
   int pf_step = 0;         // FP64: old-C L2 prefetch step in tile rows when beta != 0 (0: none)
+  // tcgen05: operand tensor maps for the TMA producer (tiles.cpp umma_tma_spec); the pointers
+  // come per call, so tc_execute encodes the maps from these shapes
+  bool umma_tma = false;
+  OperandMap mapX, mapY;
   // batch (Hadamard) indices (R31): extent and element strides in X, Y, C.  tc_execute
   // launches the kernel once per batch slab with the operands offset to it — the kernels
   // carry no batch code (the FP64 variants run at their 128-register cap).

@@ -89,8 +89,12 @@ double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *
     const double b = (double)rows * cfg.Kt * es0;
     return std::pair<double, double>{std::ceil(b / 128.0), std::ceil(b / 32.0)};
   };
-  const auto sx = lower_bound ? ideal(cfg.Mt) : operand_sim(c, cfg, cfg.X, cfg.vecX, cfg.xKmajor, v.BM, v.BK, cache);
-  const auto sy = lower_bound ? ideal(cfg.Nt) : operand_sim(c, cfg, cfg.Y, cfg.vecY, cfg.yKmajor, v.BN, v.BK, cache);
+  // tcgen05 with TMA operand boxes: one thread issues a few boxes per stage, the TMA unit writes
+  // the swizzled planes at full smem bandwidth and fetches whole rows (no cp.async slots)
+  TmaOperand ox, oy;
+  const bool tma = umma && umma_tma_spec(c, cfg, v, cfg.X, nullptr, &ox) && umma_tma_spec(c, cfg, v, cfg.Y, nullptr, &oy);
+  const auto sx = lower_bound || tma ? ideal(cfg.Mt) : operand_sim(c, cfg, cfg.X, cfg.vecX, cfg.xKmajor, v.BM, v.BK, cache);
+  const auto sy = lower_bound || tma ? ideal(cfg.Nt) : operand_sim(c, cfg, cfg.Y, cfg.vecY, cfg.yKmajor, v.BN, v.BK, cache);
   cfg.wfX = sx.first;
   cfg.wfY = sy.first;
   cfg.secX = sx.second;
@@ -100,7 +104,7 @@ double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *
   const double lds = umma ? 0.0 : (double)warps * (v.BK / 4) * (MI + NJ) * 2;
   // producer warps: one LDGSTS warp-instruction per 32 slots, ~8 LSU cycles each
   const double nslots = (double)cfg.Mt * cfg.Kt / cfg.vecX + (double)cfg.Kt * cfg.Nt / cfg.vecY;
-  const double ldgsts = std::ceil(nslots / 32.0) * 8.0;
+  const double ldgsts = tma ? 16.0 * (ox.nsub + oy.nsub) : std::ceil(nslots / 32.0) * 8.0;
   const double step = std::max({dmma, cfg.wfX + cfg.wfY + lds, ldgsts}) + kStepOverhead;
   // store issue per tile; UMMA: 4 warps x BN column stores, overlapped with the next
   // tile's MMAs by the double-buffered TMEM accumulator

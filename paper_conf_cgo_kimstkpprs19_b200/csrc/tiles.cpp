@@ -350,4 +350,101 @@ TileTables build_tile_tables(const Contraction &c, const Config &cfg, const Vari
   return tt;
 }
 
+// tcgen05 operand t loaded by TMA boxes straight into its 128-B swizzled UMMA plane
+// (kernel_umma.cuh, TMA producer).  The map's dimension 0 is the operand's FVI (stride 1);
+// the others may come in any order, so they follow the plane's row order:
+//   K-major  (FVI = the k index): [k | side digits in compute order], box (BK, T...)  —
+//            (a k tile below BK loads the next step's k too; the MMAs never read them)
+//            tile-local row r = mixed radix over the side digits = box row r (128 B each);
+//   MN-major (FVI = side[0]):     [side[0] | k | side[1..]], box (E, Kt, T...) — one 128-B
+//            atom column per E elements of side[0]; wider tiles of side[0] (the other side
+//            digits then untiled) take ceil(T0/E) boxes, each BK * 128 B further on.
+// Conditions: one k digit whose tile is a multiple of the MMA K or its whole extent (TMA
+// zero-fills past the end, as the cp.async producers do), no batch index, rank <= 5, side digits among
+// C's first 5 positions (the tile origin coordinates), 16-B multiple strides.  The split
+// FP32 kind converts in smem and keeps its cp.async producers.
+bool umma_tma_spec(const Contraction &c, const Config &cfg, const Variant &v, int t, OperandMap *mp,
+                   TmaOperand *op) {
+  const bool kmaj = t == cfg.X ? cfg.xKmajor : cfg.yKmajor;
+  const std::vector<int> &side = t == cfg.X ? cfg.mdig : cfg.ndig;
+  OperandMap mloc;
+  TmaOperand oloc;
+  OperandMap &m = mp ? *mp : mloc;
+  TmaOperand &o = op ? *op : oloc;
+  if (cfg.kind != KIND_BF16_UMMA && cfg.kind != KIND_TF32_UMMA) return false;
+  if (cfg.kdig.size() != 1 || c.nbatch() != 1 || side.empty()) return false;
+  const int es = kind_esize(cfg.kind), E = 128 / es, kid = cfg.kdig[0];
+  const TensorView &tv = c.t[t];
+  const int r = (int)tv.idx.size();
+  if (r > kMaxTmaDims || tv.stride[0] != 1) return false;
+  // the MMAs consume ceil(Kt / KI) * KI k of a stage: k past Kt must be absent (zero-filled
+  // past the extent) or never read (Kt a multiple of KI)
+  const int Kt = cfg.T[kid], KI = 32 / es;
+  if (Kt > v.BK || (Kt % KI != 0 && Kt != c.ix[kid].n)) return false;
+  std::vector<int> dims;
+  if (kmaj) {
+    dims.push_back(kid);
+    dims.insert(dims.end(), side.begin(), side.end());
+  } else {
+    dims.push_back(side[0]);
+    dims.push_back(kid);
+    dims.insert(dims.end(), side.begin() + 1, side.end());
+  }
+  if ((int)dims.size() != r || dims[0] != tv.idx[0]) return false;
+  // a box's start along map dim 0 must sit on a 16-B boundary: the tile (MN-major) or k-step
+  // (K-major) origins along it move in multiples of 16 B
+  const int a16 = 16 / es;
+  if (kmaj ? (Kt % a16 != 0 && Kt < c.ix[kid].n) : (cfg.T[side[0]] % a16 != 0 && cfg.T[side[0]] < c.ix[side[0]].n))
+    return false;
+  const int T0 = cfg.T[side[0]];
+  int nsub = 1;
+  bool rest1 = true;
+  for (size_t q = 1; q < side.size(); q++) rest1 &= cfg.T[side[q]] == 1;
+  // k extent of the box: an MN-major box of one atom column may stop at Kt (its k rows are
+  // the stage's first Kt rows); otherwise the box spans BK so that a multi-digit box lands its
+  // atom columns BK rows apart, as the plane expects (the extra k are never read)
+  const uint32_t kbox = !kmaj && rest1 && Kt % KI == 0 ? (uint32_t)Kt : (uint32_t)v.BK;
+  if (!kmaj) {
+    if (rest1) {
+      nsub = (T0 + E - 1) / E;          // (atom columns past T0: rows / columns never stored)
+    } else if (T0 != E) {
+      return false;                     // other atom widths would interleave the digits
+    }
+  }
+  uint32_t pack = 0, tx = (uint32_t)es;
+  for (int j = 0; j < r; j++) {
+    const int id = dims[j];
+    const int sp = c.pos_in(t, id);
+    if (sp < 0) return false;
+    m.dims[j] = c.ix[id].n;
+    if (j > 0) {
+      const int64_t sb = tv.stride[sp] * es;
+      if (sb % 16 != 0 || sb >= (int64_t(1) << 40)) return false;
+      m.strides[j - 1] = sb;
+    }
+    uint32_t src;
+    if (id == kid) {
+      src = 7;
+      m.box[j] = kbox;
+    } else {
+      const int cp = c.pos_in(0, id);
+      if (cp < 0 || cp >= kMaxTmaDims) return false;
+      src = (uint32_t)cp;
+      m.box[j] = (uint32_t)(j == 0 ? E : cfg.T[id]);
+    }
+    if (m.box[j] > 256) return false;
+    pack |= src << (3 * j);
+    tx *= m.box[j];
+  }
+  m.rank = r;
+  m.base = tv.base;
+  m.swz32 = !kmaj && es == 4;
+  o.pack = pack | ((uint32_t)r << 16);
+  o.nsub = nsub;
+  o.sub_bytes = E * v.BK * es;
+  o.sub_crd = E;
+  o.tx = (int)tx;
+  return true;
+}
+
 }  // namespace tc

@@ -142,4 +142,17 @@ struct TileTables {
 };
 TileTables build_tile_tables(const Contraction &c, const Config &cfg, const Variant &v);
 
+// tcgen05 operand t loaded by TMA boxes (kernel_umma.cuh TMA producer): the tensor-map shape
+// (the pointer comes per call) and the kernel's per-box record.  Returns false when the
+// plan's tiles / layout do not fit a box (the operand then keeps the cp.async producers).
+struct OperandMap {
+  int rank = 0;
+  int64_t dims[kMaxTmaDims] = {}, strides[kMaxTmaDims] = {};   // strides in bytes, dims 1..
+  uint32_t box[kMaxTmaDims] = {};
+  int64_t base = 0;                                            // element offset of the view
+  bool swz32 = false;                                          // 4-byte MN-major: 32-B granules
+};
+bool umma_tma_spec(const Contraction &c, const Config &cfg, const Variant &v, int t,
+                   OperandMap *map = nullptr, TmaOperand *op = nullptr);
+
 }  // namespace tc
