@@ -68,7 +68,9 @@ typedef struct tc_plan_opts {
                         operand's memory order (its FVI first) — tests of both epilogues   */
   int no_tma_operands; /* 1: tcgen05 plans load operands with cp.async even where TMA boxes
                           fit (default 0: one thread issues TMA boxes when the plan allows) */
-  int reserved[5];   /* must be zero (TC_ERR_INVALID_ARG otherwise)                         */
+  int cta_pair;      /* tcgen05 BN = 128 plans with TMA operands: 0 planner's choice, 1 never,
+                        2 always — CTA pairs (cluster of 2, M = 256 MMAs over 2 x 2 tiles)   */
+  int reserved[4];   /* must be zero (TC_ERR_INVALID_ARG otherwise)                         */
 } tc_plan_opts;
 
 /*

@@ -45,7 +45,7 @@ class _Opts(ctypes.Structure):
     _fields_ = [("cost_mode", ctypes.c_int), ("host_only", ctypes.c_int), ("variant", ctypes.c_int),
                 ("force_tiles", ctypes.c_char_p), ("no_fusion", ctypes.c_int), ("tma_epilogue", ctypes.c_int),
                 ("morder", ctypes.c_int), ("no_tma_operands", ctypes.c_int),
-                ("reserved", ctypes.c_int * 5)]
+                ("cta_pair", ctypes.c_int), ("reserved", ctypes.c_int * 4)]
 
 
 _lib = None
@@ -214,9 +214,10 @@ class Plan:
         return C
 
 
-def _opts(cost, host_only, variant, force_tiles, fusion, tma, morder, tma_operands=True) -> _Opts:
+def _opts(cost, host_only, variant, force_tiles, fusion, tma, morder, tma_operands=True, pair=None) -> _Opts:
     o = _Opts()
     o.no_tma_operands = int(not tma_operands)
+    o.cta_pair = {None: 0, False: 1, True: 2}[pair]
     o.morder = {None: 0, "C": 1, "X": 2}[morder]
     o.tma_epilogue = int(tma)
     o.cost_mode = COST[cost]
@@ -229,9 +230,10 @@ def _opts(cost, host_only, variant, force_tiles, fusion, tma, morder, tma_operan
 
 def plan_cached(expr: str, extents: str, dtype: str = "f64", cost: str = "b200", host_only: bool = False,
                 variant: int | None = None, force_tiles: str | None = None, fusion: bool = True,
-                tma: bool = False, morder: str | None = None, tma_operands: bool = True) -> Plan:
+                tma: bool = False, morder: str | None = None, tma_operands: bool = True,
+                pair: bool | None = None) -> Plan:
     """tc_plan_cached: the process-wide cached plan of these arguments (planned on first use)."""
-    o = _opts(cost, host_only, variant, force_tiles, fusion, tma, morder, tma_operands)
+    o = _opts(cost, host_only, variant, force_tiles, fusion, tma, morder, tma_operands, pair)
     h = ctypes.c_void_p()
     _raise(lib().tc_plan_cached(ctypes.byref(h), expr.encode(), extents.encode(), DTYPES[dtype], ctypes.byref(o)))
     p = Plan(h, expr, extents, dtype)
@@ -324,9 +326,11 @@ def plan_cache_clear() -> None:
 
 def plan(expr: str, extents: str, dtype: str = "f64", cost: str = "b200", host_only: bool = False,
          variant: int | None = None, force_tiles: str | None = None, fusion: bool = True,
-         tma: bool = False, morder: str | None = None, tma_operands: bool = True) -> Plan:
-    """morder: None = planner's choice, "C" = m digits in C order, "X" = in the X operand's order."""
-    o = _opts(cost, host_only, variant, force_tiles, fusion, tma, morder, tma_operands)
+         tma: bool = False, morder: str | None = None, tma_operands: bool = True,
+         pair: bool | None = None) -> Plan:
+    """pair: None = planner's choice, False / True = CTA pairs off / on where the plan allows.
+    morder: None = planner's choice, "C" = m digits in C order, "X" = in the X operand's order."""
+    o = _opts(cost, host_only, variant, force_tiles, fusion, tma, morder, tma_operands, pair)
     h = ctypes.c_void_p()
     _raise(lib().tc_plan_ex(ctypes.byref(h), expr.encode(), extents.encode(), DTYPES[dtype], ctypes.byref(o)))
     p = Plan(h, expr, extents, dtype)

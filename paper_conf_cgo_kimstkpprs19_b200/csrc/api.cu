@@ -80,6 +80,14 @@ void build_host_tables(tc_plan_s *P) {
   const Config &cfg = P->cfg;
   const Variant &v = variants()[cfg.variant];
   P->tt = build_tile_tables(c, cfg, v);
+  if (is_umma(cfg.kind)) {
+    // padding entry past each tile list: the CTA-pair kernel's blocks that overhang the tile
+    // grid read it (coordinates outside every tensor -> TMA zero fill; masks 0 -> no stores)
+    TileInfo pad{};
+    for (int q = 0; q < kMaxTmaDims; q++) pad.coord[q] = 1 << 30;
+    P->tt.tileM.push_back(pad);
+    P->tt.tileN.push_back(pad);
+  }
   P->slotX1 = build_slots(c, cfg, cfg.X, 1, cfg.xKmajor, v.BM, v.BK);
   P->slotY1 = build_slots(c, cfg, cfg.Y, 1, cfg.yKmajor, v.BN, v.BK);
   if (cfg.vecX > 1) P->slotX2 = build_slots(c, cfg, cfg.X, cfg.vecX, cfg.xKmajor, v.BM, v.BK);
@@ -123,6 +131,13 @@ void build_host_tables(tc_plan_s *P) {
                 umma_tma_spec(c, cfg, v, cfg.X, &P->mapX, &kp.xt) &&
                 umma_tma_spec(c, cfg, v, cfg.Y, &P->mapY, &kp.yt);
   kp.kt = cfg.kdig.empty() ? 0 : (int)cfg.T[cfg.kdig[0]];
+  // CTA pairs: BN = 128 BF16 / TF32 instances with TMA operands, when asked for (cta_pair 2)
+  // or (planner's choice) when the grid holds at least two waves of pair blocks
+  {
+    const bool can = P->umma_tma && (cfg.variant == 12 || cfg.variant == 22);
+    const int64_t units = ((cfg.mtiles + 1) / 2) * ((cfg.ntiles + 1) / 2);
+    P->pair = can && (P->opts.cta_pair == 2 || (P->opts.cta_pair == 0 && units >= 2 * 74));
+  }
   P->pf_step = 0;
   if (cfg.kind == KIND_F64_DMMA && !cfg.mdig.empty() && !c.t[0].idx.empty() && cfg.mdig[0] == c.t[0].idx[0] &&
       c.t[0].stride[0] == 1)
@@ -191,6 +206,14 @@ Status upload(tc_plan_s *P, std::string &err) {
     e = cudaFuncSetAttribute(kt.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kt.smem);
     if (e != cudaSuccess) { err = std::string("cudaFuncSetAttribute: ") + cudaGetErrorString(e); return ST_CUDA; }
   }
+  if (P->pair) {
+    size_t sm = 0;
+    int th = 0;
+    const void *fn = kernel_ptr_umma_pair(P->cfg.variant, P->cfg.xKmajor, P->cfg.yKmajor, &sm, &th);
+    if (!fn) { err = "no CTA-pair instance for the variant"; return ST_UNSUPPORTED; }
+    e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    if (e != cudaSuccess) { err = std::string("cudaFuncSetAttribute: ") + cudaGetErrorString(e); return ST_CUDA; }
+  }
   const KernelEntry ke = kernel_for(P->cfg);
   const bool tma = P->tt.tma_ok && P->opts.tma_epilogue && P->cfg.kind == KIND_F64_DMMA &&
                    !variants()[P->cfg.variant].stg;
@@ -236,6 +259,7 @@ tc_status_t finish_plan(tc_plan_s *P, tc_plan_t *out) {
   ForcedTiles ft;
   if (!parse_force(P->opts.force_tiles, ft)) { delete P; return fail(ST_INVALID_ARG, "malformed force_tiles"); }
   if (P->opts.morder < 0 || P->opts.morder > 2) { delete P; return fail(ST_INVALID_ARG, "morder must be 0, 1 or 2"); }
+  if (P->opts.cta_pair < 0 || P->opts.cta_pair > 2) { delete P; return fail(ST_INVALID_ARG, "cta_pair must be 0, 1 or 2"); }
   for (int r : P->opts.reserved)
     if (r != 0) { delete P; return fail(ST_INVALID_ARG, "tc_plan_opts.reserved[] must be zero"); }
   ft.morder = P->opts.morder - 1;
@@ -429,7 +453,7 @@ std::string cache_key(const char *expr, const char *extents, tc_dtype_t dtype, c
   k << expr << '\x1f' << extents << '\x1f' << (int)dtype << '\x1f' << dev;
   if (o)
     k << '\x1f' << o->cost_mode << ',' << o->host_only << ',' << o->variant << ',' << o->no_fusion << ','
-      << o->tma_epilogue << ',' << o->morder << ',' << o->no_tma_operands << ','
+      << o->tma_epilogue << ',' << o->morder << ',' << o->no_tma_operands << ',' << o->cta_pair << ','
       << (o->force_tiles ? o->force_tiles : "");
   return k.str();
 }
@@ -655,6 +679,29 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
                        encode_operand_map(plan, plan->mapY, kp.Y, kp.ymap);
   const KernelEntry ke = kernel_for(cfg, tma_ops);
   const int grid = (int)std::min<int64_t>(cfg.nctas, plan->sms);
+  if (tma_ops && plan->pair) {   // clusters of two CTAs over 2 x 2 tile blocks (persistent)
+    size_t sm = 0;
+    int th = 0;
+    const void *fn = kernel_ptr_umma_pair(cfg.variant, cfg.xKmajor, cfg.yKmajor, &sm, &th);
+    const int64_t units = ((cfg.mtiles + 1) / 2) * ((cfg.ntiles + 1) / 2);
+    const int ncl = (int)std::min<int64_t>(units, plan->sms / 2);
+    cudaLaunchConfig_t lc = {};
+    lc.gridDim = dim3(2 * ncl);
+    lc.blockDim = dim3(th);
+    lc.dynamicSmemBytes = sm;
+    lc.stream = (cudaStream_t)stream;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = 2;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    lc.attrs = at;
+    lc.numAttrs = 1;
+    void *pargs[] = {&kp};
+    cudaError_t e = cudaLaunchKernelExC(&lc, fn, pargs);
+    if (e != cudaSuccess) return fail(ST_CUDA, std::string("launch (CTA pair): ") + cudaGetErrorString(e));
+    return TC_SUCCESS;
+  }
   void *args[] = {&kp};
   const int64_t nb = plan->c.nbatch();
   const char *X0 = static_cast<const char *>(kp.X), *Y0 = static_cast<const char *>(kp.Y);
@@ -780,7 +827,8 @@ tc_status_t tc_plan_info(const tc_plan_t plan, char *json, size_t cap, size_t *n
       << ",\"grid\":" << std::min<int64_t>(g.nctas, plan->sms)
       << ",\"nbatch\":" << c.nbatch();
     o << ",\"vecX\":" << g.vecX << ",\"vecY\":" << g.vecY << ",\"vecC\":" << plan->cvec << ",\"cs0\":" << plan->kp.cs0 << ",\"xKmajor\":" << g.xKmajor
-      << ",\"yKmajor\":" << g.yKmajor << ",\"tma_operands\":" << (plan->umma_tma ? 1 : 0) << ",\"wfX\":" << g.wfX << ",\"wfY\":" << g.wfY;
+      << ",\"yKmajor\":" << g.yKmajor << ",\"tma_operands\":" << (plan->umma_tma ? 1 : 0)
+      << ",\"cta_pair\":" << (plan->pair ? 1 : 0) << ",\"wfX\":" << g.wfX << ",\"wfY\":" << g.wfY;
     char buf[512];
     std::snprintf(buf, sizeof buf,
                   ",\"t_pred_ms\":%.6g,\"t_comp_ms\":%.6g,\"t_mem_ms\":%.6g,\"t_l2_ms\":%.6g,"

@@ -42,5 +42,7 @@ F64Instance f64_instance_10(int v);
 F64Instance f64_instance_11(int v);
 // defined in kernels_umma.cu (BF16 / TF32 / F32X3 tcgen05 variants; smem bytes and block size out)
 const void *kernel_ptr_umma(int v, bool xk, bool yk, bool tma, size_t *smem, int *threads);   // tma: TMA producer
+// CTA-pair instances (BN = 128 BF16 / TF32 variants 12 / 22; nullptr otherwise)
+const void *kernel_ptr_umma_pair(int v, bool xk, bool yk, size_t *smem, int *threads);
 
 }  // namespace tc

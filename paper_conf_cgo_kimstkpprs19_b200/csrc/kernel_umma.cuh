@@ -54,6 +54,95 @@ __device__ __forceinline__ void tc05_mma(uint32_t d_tmem, uint64_t adesc, uint64
         "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(d_tmem),
         "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate) : "memory");
 }
+// CTA pair (cta_group::2, cluster of 2 on one TPC): the leader (rank 0) issues M = 256 MMAs
+// reading each CTA's half of A (its 128 rows) and of B (its N/2 columns) from the same smem
+// offsets; D rows 128 r.. land in CTA r's TMEM.
+template <bool TF32>
+__device__ __forceinline__ void tc05_mma2(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
+                                          uint32_t accumulate) {
+  if constexpr (TF32)
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::2.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(d_tmem),
+        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate) : "memory");
+  else
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(d_tmem),
+        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate) : "memory");
+}
+// completion of the leader's MMAs arrives at the barrier at this offset in BOTH CTAs
+__device__ __forceinline__ void tc05_commit2(uint32_t bar) {
+  asm volatile("tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;\n"
+               ::"r"(bar), "h"((uint16_t)3) : "memory");
+}
+__device__ __forceinline__ uint32_t cluster_rank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;\n" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;\n" ::: "memory");
+}
+// arrive (release, cluster scope) on the barrier at this offset in CTA `cta` of the cluster
+__device__ __forceinline__ void mbar_arrive_cta(uint32_t bar, uint32_t cta) {
+  asm volatile(
+      "{\n\t.reg .b32 ra;\n\tmapa.shared::cluster.u32 ra, %0, %1;\n\t"
+      "mbarrier.arrive.release.cluster.shared::cluster.b64 _, [ra];\n}\n" ::"r"(bar), "r"(cta) : "memory");
+}
+__device__ __forceinline__ void mbar_wait_acq_cluster(uint32_t bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n"
+      "WAITC_%=:\n\t"
+      "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra WAITC_%=;\n}\n" ::"r"(bar), "r"(parity) : "memory");
+}
+// TMA box of a CTA pair: lands in this CTA's smem, completes on the LEADER's barrier (the
+// barrier offset with the peer bit cleared)
+__device__ __forceinline__ void tma_load_pair(const TmaDesc *map, int rank, int32_t c0, int32_t c1, int32_t c2,
+                                              int32_t c3, int32_t c4, uint32_t dst, uint32_t bar, uint64_t pol) {
+  const uint64_t m = reinterpret_cast<uint64_t>(map);
+  bar &= 0xFEFFFFFFu;
+  switch (rank) {
+    case 1:
+      asm volatile("cp.async.bulk.tensor.1d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+                   " [%0], [%1, {%2}], [%3], %4;\n" ::"r"(dst), "l"(m), "r"(c0), "r"(bar), "l"(pol) : "memory");
+      break;
+    case 2:
+      asm volatile("cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+                   " [%0], [%1, {%2, %3}], [%4], %5;\n" ::"r"(dst), "l"(m), "r"(c0), "r"(c1), "r"(bar), "l"(pol)
+                   : "memory");
+      break;
+    case 3:
+      asm volatile("cp.async.bulk.tensor.3d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+                   " [%0], [%1, {%2, %3, %4}], [%5], %6;\n" ::"r"(dst), "l"(m), "r"(c0), "r"(c1), "r"(c2), "r"(bar),
+                   "l"(pol) : "memory");
+      break;
+    case 4:
+      asm volatile("cp.async.bulk.tensor.4d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+                   " [%0], [%1, {%2, %3, %4, %5}], [%6], %7;\n" ::"r"(dst), "l"(m), "r"(c0), "r"(c1), "r"(c2), "r"(c3),
+                   "r"(bar), "l"(pol) : "memory");
+      break;
+    default:
+      asm volatile("cp.async.bulk.tensor.5d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+                   " [%0], [%1, {%2, %3, %4, %5, %6}], [%7], %8;\n" ::"r"(dst), "l"(m), "r"(c0), "r"(c1), "r"(c2),
+                   "r"(c3), "r"(c4), "r"(bar), "l"(pol) : "memory");
+      break;
+  }
+}
+// pair unit u -> (pm, pn) over the grid of 2 x 2 tile blocks, rasterised like tile_coords
+__device__ __forceinline__ void pair_coords(const KParams &p, int u, int &pm, int &pn) {
+  const int pmt = (p.mtiles + 1) >> 1, pnt = (p.ntiles + 1) >> 1;
+  const int gm = max(1, p.group_m >> 1);
+  const int per_group = gm * pnt;
+  const int g = u / per_group;
+  const int first = g * gm;
+  const int gsz = min(gm, pmt - first);
+  const int r = u - g * per_group;
+  pm = first + r % gsz;
+  pn = r / gsz;
+}
+
 __device__ __forceinline__ void tc05_ld16(uint32_t taddr, uint32_t (&v)[16]) {
   asm volatile(
       "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];\n"
@@ -213,9 +302,9 @@ struct UmmaKernel {
 
 // UMMA instruction descriptor: BF16 x BF16 or TF32 x TF32 -> F32 (c_format 1 at [4,6),
 // a/b_format at [7,10) / [10,13): BF16 = 1, TF32 = 2), M = 128, N = BN, majors per operand.
-__host__ __device__ constexpr uint32_t umma_idesc(int fmt, int n, bool a_mn, bool b_mn) {
+__host__ __device__ constexpr uint32_t umma_idesc(int fmt, int n, bool a_mn, bool b_mn, int m = 128) {
   return (1u << 4) | ((uint32_t)fmt << 7) | ((uint32_t)fmt << 10) | ((uint32_t)a_mn << 15) |
-         ((uint32_t)b_mn << 16) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
+         ((uint32_t)b_mn << 16) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(m >> 4) << 24);
 }
 
 __device__ __forceinline__ void st_out(__nv_bfloat16 *d, float v) { *d = __float2bfloat16_rn(v); }
@@ -291,13 +380,15 @@ __device__ __forceinline__ void umma_box_origin(const TmaOperand &o, const int32
     b.kmask |= (src == 7 ? 1u : 0u) << j;
   }
 }
+template <bool PAIR>
 __device__ __forceinline__ void umma_tma_boxes(const TmaDesc *map, const TmaOperand &o, const UmmaBox &b, int rank,
                                                int32_t kc, uint32_t dst, uint32_t bar, uint64_t pol) {
   int32_t c[kMaxTmaDims];
 #pragma unroll
   for (int j = 0; j < kMaxTmaDims; j++) c[j] = (b.kmask >> j) & 1 ? kc : b.c[j];
   for (int q = 0; q < o.nsub; q++) {
-    tma_load(map, rank, c[0], c[1], c[2], c[3], c[4], dst + (uint32_t)(q * o.sub_bytes), bar, pol);
+    if (PAIR) tma_load_pair(map, rank, c[0], c[1], c[2], c[3], c[4], dst + (uint32_t)(q * o.sub_bytes), bar, pol);
+    else tma_load(map, rank, c[0], c[1], c[2], c[3], c[4], dst + (uint32_t)(q * o.sub_bytes), bar, pol);
     c[0] += o.sub_crd;
   }
 }
@@ -306,10 +397,21 @@ __device__ __forceinline__ void load_coord(const TileInfo *t, int32_t (&c)[kMaxT
   for (int q = 0; q < kMaxTmaDims; q++) c[q] = t->coord[q];
 }
 
-template <int KIND, int BN, int STAGES, bool XK, bool YK, bool TMA = false>
+// PAIR (with TMA): a cluster of two CTAs computes a 2 x 2 block of the plan's tiles as one
+// 256 x 2BN accumulator pair: CTA r loads the X box of m-tile 2 pm + r and the Y box of n-tile
+// 2 pn + r, the leader's MMAs (M = 256, N = 2 BN) read both CTAs' planes, and CTA r's epilogue
+// drains m-tile 2 pm + r against n-tiles 2 pn and 2 pn + 1 (TMEM columns 0 / BN of the
+// buffer).  Per k-step each CTA then loads half the operand bytes per MMA of the single-CTA
+// kernel (the L2 -> SM traffic that bounds BF16 GEMM-like plans).  A block past the tile grid
+// reads the tables' padding entry (coordinates out of the tensor: TMA zero-fills; masks 0).
+template <int KIND, int BN, int STAGES, bool XK, bool YK, bool TMA = false, bool PAIR = false>
 __global__ void __launch_bounds__(UmmaKernel<KIND, BN, STAGES>::THREADS, 1)
 tc_umma_kernel(const __grid_constant__ KParams p) {
   using K = UmmaKernel<KIND, BN, STAGES>;
+  static_assert(!PAIR || (TMA && !K::SPLIT), "CTA pairs take TMA operands, BF16 / TF32");
+  constexpr int ACCW = PAIR ? 2 * BN : BN;            // accumulator columns per tile (unit)
+  constexpr int NBUF = 512 / ACCW;                    // accumulators in flight
+  constexpr int NSUB = PAIR ? 2 : 1;                  // tiles per unit in this CTA's epilogue
   using T = typename K::T;
   constexpr int BM = K::BM, BK = K::BK, ES = K::ES;
   extern __shared__ __align__(1024) unsigned char smem_dyn[];
@@ -331,12 +433,17 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
 
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-  const int ntl = (p.ntotal - (int)blockIdx.x + (int)gridDim.x - 1) / (int)gridDim.x;
+  // work units: tiles, or (PAIR) 2 x 2 tile blocks per cluster
+  const int crank = PAIR ? (int)cluster_rank() : 0;
+  const int cid = PAIR ? (int)blockIdx.x >> 1 : (int)blockIdx.x;
+  const int ncl = PAIR ? (int)gridDim.x >> 1 : (int)gridDim.x;
+  const int nunits = PAIR ? ((p.mtiles + 1) >> 1) * ((p.ntiles + 1) >> 1) : p.ntotal;
+  const int ntl = (nunits - cid + ncl - 1) / ncl;
   const int total = max(ntl, 0) * p.nsteps;
   const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(smem_raw);
   const uint32_t bar0 = (uint32_t)__cvta_generic_to_shared(bars);
   const uint32_t FULL = bar0, EMPTY = bar0 + 8 * STAGES, TFULL = bar0 + 16 * STAGES,
-                 TEMPTY = TFULL + 8 * K::NBUF, SPLITB = TEMPTY + 8 * K::NBUF;
+                 TEMPTY = TFULL + 8 * NBUF, SPLITB = TEMPTY + 8 * NBUF;
 
   // ---- once per CTA ------------------------------------------------------------------------
   for (int i = tid; i < (int)(LO * K::PLANES / 16); i += K::THREADS)
@@ -348,21 +455,29 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
       mbar_init(FULL + 8 * s, TMA ? 1 : K::PW * 32);   // the TMA thread / every producer thread
       mbar_init(EMPTY + 8 * s, 1);           // tcgen05.commit of the MMA thread
     }
-    for (int b = 0; b < K::NBUF; b++) {
+    for (int b = 0; b < NBUF; b++) {
       mbar_init(TFULL + 8 * b, 1);           // tcgen05.commit after a tile's last MMA
-      mbar_init(TEMPTY + 8 * b, K::EW);      // one arrive per epilogue warp
+      mbar_init(TEMPTY + 8 * b, NSUB * K::EW);   // one arrive per epilogue warp (of both CTAs)
     }
     for (int s = 0; s < STAGES; s++) mbar_init(SPLITB + 8 * s, K::SW > 0 ? K::SW : 1);   // split warps
     asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
   }
   if (warp == K::EW + K::PW) {               // the MMA warp owns the TMEM allocation
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;\n" ::"r"(
-                     (uint32_t)__cvta_generic_to_shared(tmem_holder)),
-                 "r"(K::TMEM_COLS));
-    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;\n" ::);
+    if (PAIR) {   // (both CTAs, same warp)
+      asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;\n" ::"r"(
+                       (uint32_t)__cvta_generic_to_shared(tmem_holder)),
+                   "r"(K::TMEM_COLS));
+      asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;\n" ::);
+    } else {
+      asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;\n" ::"r"(
+                       (uint32_t)__cvta_generic_to_shared(tmem_holder)),
+                   "r"(K::TMEM_COLS));
+      asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;\n" ::);
+    }
   }
   tc05_fence_before();
-  __syncthreads();
+  if (PAIR) cluster_sync_all();   // the peer's boxes / arrivals target the leader's barriers
+  else __syncthreads();
   tc05_fence_after();
   const uint32_t tmem = *tmem_holder;
 
@@ -380,42 +495,44 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
 #else
       asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;\n" : "=l"(policy));
 #endif
-      const uint32_t tx = (uint32_t)(p.xt.nsub * p.xt.tx + p.yt.nsub * p.yt.tx);
+      const uint32_t tx = (uint32_t)(p.xt.nsub * p.xt.tx + p.yt.nsub * p.yt.tx) * (PAIR ? 2u : 1u);
       const int rx = (int)((p.xt.pack >> 16) & 7), ry = (int)((p.yt.pack >> 16) & 7);
       int step = 0, lt = 0, mt = 0, nt = 0;
       UmmaBox bx, by;
-      int32_t nxc[kMaxTmaDims], nyc[kMaxTmaDims];   // the next tile's origin, read one tile ahead
-      if (ntl > 0) {
-        tile_coords(p, (int)blockIdx.x, mt, nt);
+      int32_t nxc[kMaxTmaDims], nyc[kMaxTmaDims];   // the next unit's origins, read one unit ahead
+      auto unit = [&](int u) {
+        if (PAIR) {
+          int pm, pn;
+          pair_coords(p, u, pm, pn);
+          mt = 2 * pm + crank;
+          nt = 2 * pn + crank;
+        } else {
+          tile_coords(p, u, mt, nt);
+        }
         load_coord(&p.tileM[mt], nxc);
         load_coord(&p.tileN[nt], nyc);
+      };
+      if (ntl > 0) {
+        unit(cid);
         umma_box_origin(p.xt, nxc, bx);
         umma_box_origin(p.yt, nyc, by);
-        if (ntl > 1) {
-          tile_coords(p, (int)blockIdx.x + (int)gridDim.x, mt, nt);
-          load_coord(&p.tileM[mt], nxc);
-          load_coord(&p.tileN[nt], nyc);
-        }
+        if (ntl > 1) unit(cid + ncl);
       }
       for (int j = 0; j < total; j++) {
         const int s = j % STAGES;
         if (j >= STAGES) mbar_wait(EMPTY + 8 * s, ((j / STAGES) & 1) ^ 1);
-        mbar_expect_tx(FULL + 8 * s, tx);
+        if (!PAIR || crank == 0) mbar_expect_tx(FULL + 8 * s, tx);   // (pair: both CTAs' bytes)
         const uint32_t dx = sbase + (uint32_t)ES * (uint32_t)(s * K::XS);
         const uint32_t dy = sbase + (uint32_t)ES * (uint32_t)(STAGES * K::XS + s * K::YS);
         const int32_t kc = step * p.kt;
-        umma_tma_boxes(&p.xmap, p.xt, bx, rx, kc, dx, FULL + 8 * s, policy);
-        umma_tma_boxes(&p.ymap, p.yt, by, ry, kc, dy, FULL + 8 * s, policy);
+        umma_tma_boxes<PAIR>(&p.xmap, p.xt, bx, rx, kc, dx, FULL + 8 * s, policy);
+        umma_tma_boxes<PAIR>(&p.ymap, p.yt, by, ry, kc, dy, FULL + 8 * s, policy);
         if (++step == p.nsteps) {
           step = 0;
           if (++lt < ntl) {
             umma_box_origin(p.xt, nxc, bx);
             umma_box_origin(p.yt, nyc, by);
-            if (lt + 1 < ntl) {
-              tile_coords(p, (int)blockIdx.x + (lt + 1) * (int)gridDim.x, mt, nt);
-              load_coord(&p.tileM[mt], nxc);
-              load_coord(&p.tileN[nt], nyc);
-            }
+            if (lt + 1 < ntl) unit(cid + (lt + 1) * ncl);
           }
         }
       }
@@ -480,11 +597,12 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
         if (pt == 0) trace_at(p, 7, j);
       }
     }
-  } else if (warp == K::EW + K::PW) {
+  } else if (warp == K::EW + K::PW && (!PAIR || crank == 0)) {
     // ======================= MMA issuer ===================================================
     // N and the number of K-instructions trimmed to the plan's tile (host: umma_trim): a
     // 24-column tile issues N = 32 (K-major Y) instead of BN, a 36-deep k step 3 of 4
-    const uint32_t IDESC = umma_idesc(ES == 2 ? 1 : 2, p.nmma, !XK, !YK);
+    const uint32_t IDESC = PAIR ? umma_idesc(ES == 2 ? 1 : 2, 2 * BN, !XK, !YK, 256)
+                                : umma_idesc(ES == 2 ? 1 : 2, p.nmma, !XK, !YK);
     const int kmma = p.kmma;
     // canonical no-swizzle layouts (bytes): K-major LBO = 128 (k groups), SBO = 1024 (8-row
     // groups); MN-major SBO = 128 (8-row groups), LBO = rows/8 * 128 (k groups)
@@ -504,8 +622,11 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
     int step = 0, lt = 0;
     for (int j = 0; j < total; j++) {
       const int s = j % STAGES;
-      const int buf = lt % K::NBUF;
-      if (step == 0 && lt >= K::NBUF) mbar_wait(TEMPTY + 8 * buf, ((lt / K::NBUF) & 1) ^ 1);
+      const int buf = lt % NBUF;
+      if (step == 0 && lt >= NBUF) {
+        if (PAIR) mbar_wait_acq_cluster(TEMPTY + 8 * buf, ((lt / NBUF) & 1) ^ 1);   // both CTAs drained it
+        else mbar_wait(TEMPTY + 8 * buf, ((lt / NBUF) & 1) ^ 1);
+      }
       if (K::SPLIT) mbar_wait(SPLITB + 8 * s, (j / STAGES) & 1);
       else mbar_wait(FULL + 8 * s, (j / STAGES) & 1);
       if (lane == 0) trace_at(p, 2, j);
@@ -516,7 +637,7 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
       if (lane == 0) {
         const uint32_t ax = sbase + (uint32_t)ES * (uint32_t)(s * K::XS);
         const uint32_t by = sbase + (uint32_t)ES * (uint32_t)(STAGES * K::XS + s * K::YS);
-        const uint32_t d = tmem + (uint32_t)(buf * BN);
+        const uint32_t d = tmem + (uint32_t)(buf * ACCW);
 #pragma unroll
         for (int kk = 0; kk < BK / K::KI; kk++) {
           if (kk >= kmma) break;
@@ -526,12 +647,19 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
             tc05_mma<true>(d, umma_desc<XL>(ax + LO + kk * A_KSTEP, A_LBO, A_SBO), bh, IDESC, (step > 0 || kk > 0) ? 1u : 0u);
             tc05_mma<true>(d, ah, umma_desc<YL>(by + LO + kk * B_KSTEP, B_LBO, B_SBO), IDESC, 1u);
             tc05_mma<true>(d, ah, bh, IDESC, 1u);
+          } else if (PAIR) {
+            tc05_mma2<ES == 4>(d, ah, bh, IDESC, (step > 0 || kk > 0) ? 1u : 0u);
           } else {
             tc05_mma<ES == 4>(d, ah, bh, IDESC, (step > 0 || kk > 0) ? 1u : 0u);
           }
         }
-        tc05_commit(EMPTY + 8 * s);                           // smem stage free once MMAs read it
-        if (step + 1 == p.nsteps) tc05_commit(TFULL + 8 * buf);   // accumulator ready
+        if (PAIR) {   // both CTAs' stage / accumulator
+          tc05_commit2(EMPTY + 8 * s);
+          if (step + 1 == p.nsteps) tc05_commit2(TFULL + 8 * buf);
+        } else {
+          tc05_commit(EMPTY + 8 * s);                           // smem stage free once MMAs read it
+          if (step + 1 == p.nsteps) tc05_commit(TFULL + 8 * buf);   // accumulator ready
+        }
         trace_at(p, 3, j);
       }
       __syncwarp();
@@ -582,16 +710,27 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
     const int grow = quarter * 32 + g * 8;
     const int64_t goff = relCm[grow];
     // tile info is fetched one tile ahead: its load latency hides behind the current tile
-    int64_t ncoff = 0;
-    uint64_t nrm0 = 0, nrm1 = 0, ncm0 = 0, ncm1 = 0;
+    // (PAIR: this CTA's m-tile against the unit's two n-tiles)
+    int64_t ncoff[NSUB];
+    uint64_t nrm0 = 0, nrm1 = 0, ncm0[NSUB], ncm1[NSUB];
     auto fetch = [&](int t) {
       int mt, nt;
-      tile_coords(p, (int)blockIdx.x + t * (int)gridDim.x, mt, nt);
-      ncoff = p.tileM[mt].c + p.tileN[nt].c;
+      if (PAIR) {
+        int pm, pn;
+        pair_coords(p, cid + t * ncl, pm, pn);
+        mt = 2 * pm + crank;
+        nt = 2 * pn;
+      } else {
+        tile_coords(p, cid + t * ncl, mt, nt);
+      }
       nrm0 = p.tileM[mt].mask[0];
       nrm1 = p.tileM[mt].mask[1];
-      ncm0 = p.tileN[nt].mask[0];
-      ncm1 = p.tileN[nt].mask[1];
+#pragma unroll
+      for (int q = 0; q < NSUB; q++) {
+        ncoff[q] = p.tileM[mt].c + p.tileN[nt + q].c;
+        ncm0[q] = p.tileN[nt + q].mask[0];
+        ncm1[q] = p.tileN[nt + q].mask[1];
+      }
     };
     if (ntl > 0) fetch(0);
     // CTA-wide staged path (cs0 > 1): thread -> (run, first column, column step).  With
@@ -611,17 +750,29 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
       rroff = relCm[rr];
     }
     for (int lt = 0; lt < ntl; lt++) {
-      const int buf = lt % K::NBUF;
-      const int64_t coff = ncoff;
-      const uint64_t rm0 = nrm0, rm1 = nrm1, cm0 = ncm0, cm1 = ncm1;
+      const int buf = lt % NBUF;
+      int64_t coffs[NSUB];
+      uint64_t cm0s[NSUB], cm1s[NSUB];
+#pragma unroll
+      for (int q = 0; q < NSUB; q++) {
+        coffs[q] = ncoff[q];
+        cm0s[q] = ncm0[q];
+        cm1s[q] = ncm1[q];
+      }
+      const uint64_t rm0 = nrm0, rm1 = nrm1;
       if (lt + 1 < ntl) fetch(lt + 1);
       const bool rok = ((row < 64 ? rm0 : rm1) >> (row & 63)) & 1;
+      const bool gok = ((grow < 64 ? rm0 : rm1) >> (grow & 63)) & 1;
+      mbar_wait_sleep(TFULL + 8 * buf, (lt / NBUF) & 1);
+      tc05_fence_after();
+#pragma unroll 1
+      for (int q = 0; q < NSUB; q++) {
+      const int64_t coff = coffs[q];
+      const uint64_t cm0 = cm0s[q], cm1 = cm1s[q];
+      const uint32_t cb = (uint32_t)(buf * ACCW + q * BN);   // this tile's TMEM columns
       T *Crow = C + (coff + roff);
       const bool cfull = cm0 == p.fullN[0] && cm1 == p.fullN[1];
-      const bool gok = ((grow < 64 ? rm0 : rm1) >> (grow & 63)) & 1;
       T *Cg = C + (coff + goff);
-      mbar_wait_sleep(TFULL + 8 * buf, (lt / K::NBUF) & 1);
-      tc05_fence_after();
       if (kTrace) {
         if (warp == 0 && lane == 0) trace_at(p, 4, lt);
       } else if (p.vecC == 8 && p.cs0 > 1) {
@@ -634,7 +785,7 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
         T *Cr = C + (coff + rroff);
         for (int pc = 0; pc < BN && pc < p.Nt; pc += 64) {
           uint32_t v[32];
-          tc05_ld<32>(tmem + ((uint32_t)(quarter * 32) << 16) + (uint32_t)(buf * BN + pc + half * 32), v);
+          tc05_ld<32>(tmem + ((uint32_t)(quarter * 32) << 16) + cb + (uint32_t)(pc + half * 32), v);
 #pragma unroll
           for (int q = 0; q < 32; q++) stage[(half * 32 + q) * 128 + row] = __uint_as_float(v[q]);
           asm volatile("bar.sync 1, %0;\n" ::"r"(K::EW * 32) : "memory");
@@ -658,7 +809,7 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
         constexpr int W = 32 > HC ? HC : 32;
         if (half * HC + c0 >= p.Nt) break;             // columns past the tile's Nt: padding
         uint32_t v[W];
-        tc05_ld<W>(tmem + ((uint32_t)(quarter * 32) << 16) + (uint32_t)(buf * BN + half * HC + c0), v);
+        tc05_ld<W>(tmem + ((uint32_t)(quarter * 32) << 16) + cb + (uint32_t)(half * HC + c0), v);
         if (p.vecC == 8) {
           // FP32 accumulators to smem as [column][row], then one 16-B store per 8 rows
           // (C's FVI leads m with an 8-multiple tile: 8 tile rows are 8 C-contiguous elements)
@@ -736,16 +887,22 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
           }
         }
       }
+      }   // tiles of the unit
       tc05_fence_before();
       __syncwarp();
-      if (lane == 0) mbar_arrive(TEMPTY + 8 * buf);
+      if (lane == 0) {
+        if (PAIR) mbar_arrive_cta(TEMPTY + 8 * buf, 0);   // the leader's MMAs reuse the buffer
+        else mbar_arrive(TEMPTY + 8 * buf);
+      }
       if (warp == 0 && lane == 0) trace_at(p, 5, lt);
     }
   }
-  __syncthreads();
+  if (PAIR) cluster_sync_all();   // no CTA leaves while its peer may still signal it
+  else __syncthreads();
   if (warp == K::EW + K::PW) {
     tc05_fence_after();
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;\n" ::"r"(tmem), "r"(K::TMEM_COLS));
+    if (PAIR) asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;\n" ::"r"(tmem), "r"(K::TMEM_COLS));
+    else asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;\n" ::"r"(tmem), "r"(K::TMEM_COLS));
   }
 }
 

@@ -96,3 +96,32 @@ def test_unaligned_box_origins_keep_cp_async():
     hp = tc.plan("ab-ca-cb", "a:128;b:64;c:72", dtype="bf16", host_only=True, force_tiles="a:128;b:64;c:12")
     assert hp.info()["tma_operands"] == 0
     check_bf16("ab-ca-cb", "a:128;b:64;c:72", seed=4, integer=True, force_tiles="a:128;b:64;c:12")
+
+
+# CTA pairs (kernel_umma.cuh PAIR): clusters of two CTAs, M = 256 MMAs over 2 x 2 blocks of
+# BN = 128 tiles; odd tile counts hand the overhanging block the padding entry
+PAIR_CASES = [
+    ("ab-ac-cb", "a:392;b:264;c:136", "a:128;b:128;c:64", "a:128;b:128;c:32"),   # MN / K, 4 x 3 tiles
+    ("ab-ca-bc", "a:256;b:520;c:200", "a:128;b:128;c:64", "a:128;b:128;c:32"),   # K / MN, 2 x 5 tiles
+    ("ab-ac-bc", "a:136;b:136;c:80", "a:128;b:128;c:48", "a:128;b:128;c:16"),    # MN / MN, ragged 2 x 2
+    ("ab-ca-cb", "a:384;b:384;c:72", "a:128;b:128;c:64", "a:128;b:128;c:32"),    # K / K, 3 x 3 tiles
+    ("abc-acd-db", "a:136;b:250;c:3;d:40", "a:64;c:2;b:128;d:32", "a:32;c:4;b:128;d:32"),   # 2-digit box
+]
+
+
+@pytest.mark.parametrize("i", range(len(PAIR_CASES)))
+@pytest.mark.parametrize("dt", ["bf16", "tf32"])
+def test_cta_pair(i, dt):
+    expr, ext, tb, tt = PAIR_CASES[i]
+    tiles = tb if dt == "bf16" else tt
+    kw = dict(force_tiles=tiles, morder="X", pair=True)
+    hp = tc.plan(expr, ext, dtype=dt, host_only=True, **kw)
+    assert hp.info()["cta_pair"] == 1, hp.info()
+    if dt == "bf16":
+        check_bf16(expr, ext, seed=i, integer=True, **kw)
+        check_bf16(expr, ext, seed=i, integer=False, **kw)
+        check_bf16(expr, ext, seed=i + 50, integer=True, alpha=2.0, beta=1.0, **kw)
+    else:
+        check_f32(expr, ext, "tf32", seed=i, integer=True, **kw)
+        check_f32(expr, ext, "tf32", seed=i, integer=False, **kw)
+        check_f32(expr, ext, "tf32", seed=i + 50, integer=True, alpha=2.0, beta=1.0, **kw)

@@ -31,17 +31,16 @@ expr = sys.argv[1] if len(sys.argv) > 1 else "ab-ac-cb"
 ext = sys.argv[2] if len(sys.argv) > 2 else "a:5136;b:5120;c:5136"
 dt = sys.argv[3] if len(sys.argv) > 3 else "bf16"
 tdt = torch.bfloat16 if dt == "bf16" else torch.float32
-tiles = sys.argv[4].split(",") if len(sys.argv) > 4 else [None, "a:128;b:128;c:64", "a:128;b:128;c:48",
-                                                          "a:128;b:64;c:64", "a:64;b:128;c:64"]
+tiles = sys.argv[4].split(",") if len(sys.argv) > 4 else [None, "a:128;b:128;c:64"]
 p0 = tc.plan(expr, ext, dtype=dt)
 A = tcinputs.uniform(p0.numel("A"), 1, device="cuda").to(tdt)
 B = tcinputs.uniform(p0.numel("B"), 2, device="cuda").to(tdt)
 C = torch.empty(p0.numel("C"), dtype=tdt, device="cuda")
 for t in tiles:
-    for tma in (True, False):
-        p = tc.plan(expr, ext, dtype=dt, force_tiles=t, tma_operands=tma)
+    for name, kw in (("pair", {"pair": True}), ("tma", {"pair": False}), ("cpasync", {"tma_operands": False})):
+        p = tc.plan(expr, ext, dtype=dt, force_tiles=t, **kw)
         ms = timeit(p, A, B, C)
         i = p.info()
-        print(json.dumps({"tiles": t, "tma": i["tma_operands"] if tma else 0, "ms": round(ms, 4),
-                          "tflops": round(p.flops / ms / 1e9, 1), "variant": i["variant"],
+        print(json.dumps({"tiles": t, "mode": name, "tma": i["tma_operands"], "pair": i["cta_pair"],
+                          "ms": round(ms, 4), "tflops": round(p.flops / ms / 1e9, 1), "variant": i["variant"],
                           "Kt": i["Kt"], "pred_ms": round(i["t_pred_ms"], 4)}), flush=True)
