@@ -135,8 +135,7 @@ void build_host_tables(tc_plan_s *P) {
   // or (planner's choice) when the grid holds at least two waves of pair blocks
   {
     const bool can = P->umma_tma && (cfg.variant == 12 || cfg.variant == 22);
-    const int64_t units = ((cfg.mtiles + 1) / 2) * ((cfg.ntiles + 1) / 2);
-    P->pair = can && (P->opts.cta_pair == 2 || (P->opts.cta_pair == 0 && units >= 2 * 74));
+    P->pair = can && (P->opts.cta_pair == 2 || (P->opts.cta_pair == 0 && cta_pair_default(cfg)));
   }
   P->pf_step = 0;
   if (cfg.kind == KIND_F64_DMMA && !cfg.mdig.empty() && !c.t[0].idx.empty() && cfg.mdig[0] == c.t[0].idx[0] &&

@@ -93,8 +93,15 @@ double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *
   // the swizzled planes at full smem bandwidth and fetches whole rows (no cp.async slots)
   TmaOperand ox, oy;
   const bool tma = umma && umma_tma_spec(c, cfg, v, cfg.X, nullptr, &ox) && umma_tma_spec(c, cfg, v, cfg.Y, nullptr, &oy);
-  const auto sx = lower_bound || tma ? ideal(cfg.Mt) : operand_sim(c, cfg, cfg.X, cfg.vecX, cfg.xKmajor, v.BM, v.BK, cache);
-  const auto sy = lower_bound || tma ? ideal(cfg.Nt) : operand_sim(c, cfg, cfg.Y, cfg.vecY, cfg.yKmajor, v.BN, v.BK, cache);
+  // (TMA: the boxes' own bytes — a K-major box spans BK of k whatever Kt is)
+  const auto boxes = [](const TmaOperand &o) {
+    const double b = (double)o.tx * o.nsub;
+    return std::pair<double, double>{std::ceil(b / 128.0), std::ceil(b / 32.0)};
+  };
+  // CTA pairs: each CTA loads one X and one Y box per k-step for two tiles of work
+  const bool pair = tma && cta_pair_default(cfg);
+  const auto sx = tma ? boxes(ox) : lower_bound ? ideal(cfg.Mt) : operand_sim(c, cfg, cfg.X, cfg.vecX, cfg.xKmajor, v.BM, v.BK, cache);
+  const auto sy = tma ? boxes(oy) : lower_bound ? ideal(cfg.Nt) : operand_sim(c, cfg, cfg.Y, cfg.vecY, cfg.yKmajor, v.BN, v.BK, cache);
   cfg.wfX = sx.first;
   cfg.wfY = sy.first;
   cfg.secX = sx.second;
@@ -136,7 +143,8 @@ double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *
   }
   // persistent CTAs: grid = 148 * occ, tiles round-robin; t_tile is per tile per SM
   const double slots = kSMs * v.occ;
-  const double tiles_per_sm = std::ceil(nctas / slots) * v.occ;
+  const double tiles_per_sm = pair ? 2.0 * std::ceil((double)((cfg.mtiles + 1) / 2) * ((cfg.ntiles + 1) / 2) / (kSMs / 2))
+                                   : std::ceil(nctas / slots) * v.occ;
   const double cyc_sm = tiles_per_sm * t_tile;
   cfg.t_comp = cyc_sm / kClk;
   // store-instruction efficiency: 8 consecutive rows of a DMMA fragment are contiguous in C
@@ -162,7 +170,7 @@ double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *
   cfg.dram_bytes = bx * rx / eX + by * ry / eY + bc / eC;
   cfg.t_mem = cfg.dram_bytes / kHbm;
   // L2 -> SM: the simulated sectors of every stage of every tile, plus the C stores
-  const double l2b = nctas * steps * 32.0 * (cfg.secX + cfg.secY) + bc / eS;
+  const double l2b = nctas * steps * 32.0 * (cfg.secX + cfg.secY) * (pair ? 0.5 : 1.0) + bc / eS;
   cfg.t_l2 = l2b / kL2Bw;
   cfg.flops_pad = 2.0 * nctas * steps * v.BM * v.BN * v.BK;
   cfg.t_pred = std::max({cfg.t_comp, cfg.t_mem, cfg.t_l2}) + kLaunch;

@@ -154,5 +154,10 @@ struct OperandMap {
 };
 bool umma_tma_spec(const Contraction &c, const Config &cfg, const Variant &v, int t,
                    OperandMap *map = nullptr, TmaOperand *op = nullptr);
+// CTA pairs by default (planner's choice; cfg.mtiles / ntiles set): a BN = 128 BF16 / TF32
+// variant (12 / 22) with TMA operands and at least two waves of 2 x 2 blocks on the 74 pairs
+inline bool cta_pair_default(const Config &cfg) {
+  return (cfg.variant == 12 || cfg.variant == 22) && ((cfg.mtiles + 1) / 2) * ((cfg.ntiles + 1) / 2) >= 148;
+}
 
 }  // namespace tc

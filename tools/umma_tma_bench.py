@@ -32,7 +32,8 @@ def timeit(p, A, B, C, reps=7):
     return sorted(ts)[len(ts) // 2]
 
 
-ids = [int(x) for x in sys.argv[1].split(",")] if len(sys.argv) > 1 else list(range(1, 10)) + [18]
+ids = ([int(x) for x in sys.argv[1].split(",")] if len(sys.argv) > 1 and sys.argv[1] != "all"
+       else list(range(1, 49)))
 dts = sys.argv[2].split(",") if len(sys.argv) > 2 else ["bf16", "tf32"]
 for dt in dts:
     for c in [c for c in tcinputs.tccg48() if c.id in ids]:
@@ -41,7 +42,7 @@ for dt in dts:
         B = tcinputs.uniform(p.numel("B"), 2000 + c.id, device="cuda").to(TDT[dt])
         C = torch.empty(p.numel("C"), dtype=TDT[dt], device="cuda")
         byts = ES[dt] * (p.numel("A") + p.numel("B") + p.numel("C"))
-        row = {"id": c.id, "dtype": dt, "expr": c.expr, "tma": p.info()["tma_operands"],
+        row = {"id": c.id, "dtype": dt, "expr": c.expr, "tma": p.info()["tma_operands"], "pair": p.info()["cta_pair"],
                "variant": p.info()["variant"], "pred_ms": round(p.info()["t_pred_ms"], 4)}
         for name, kw in (("tma", {}), ("cpasync", {"tma_operands": False})):
             q = tc.plan(c.expr, c.extents, dtype=dt, **kw)
