@@ -216,6 +216,33 @@ __device__ __forceinline__ void umma_issue_generic_t(const KParams &p, const T *
     const int64_t base = side ? by : bx;
     const uint32_t dst0 = side ? dy : dx;
     const uint64_t *rm = side ? mn : mm;
+    if (vec * (int)sizeof(T) == 2) {
+      // single BF16 elements (cp.async has no 2-byte form): 8 independent loads in flight per
+      // thread, then their stores — a load-store chain per element would serialise the
+      // global latency (the TCCG #14 / #27 layouts: k digits in opposite orders in X and Y)
+      constexpr int U = 8;
+      for (int q0 = pt; q0 < n; q0 += U * PW * 32) {
+        unsigned short v[U];
+        uint32_t d[U];
+#pragma unroll
+        for (int i = 0; i < U; i++) {
+          const int q = q0 + i * PW * 32;
+          v[i] = 0;
+          d[i] = 0xFFFFFFFFu;
+          if (q < n) {
+            const uint32_t pk = __ldg(pack + q);
+            const int k = (pk >> 14) & 63, m = pk >> 20;
+            const bool ok = ((km >> k) & 1) && ((((m < 64) ? rm[0] : rm[1]) >> (m & 63)) & 1);
+            d[i] = dst0 + (uint32_t)sizeof(T) * (pk & 0x3FFF);
+            if (ok) v[i] = __ldg(reinterpret_cast<const unsigned short *>(src + (base + __ldg(rel + q))));
+          }
+        }
+#pragma unroll
+        for (int i = 0; i < U; i++)
+          if (d[i] != 0xFFFFFFFFu) asm volatile("st.shared.u16 [%0], %1;\n" ::"r"(d[i]), "h"(v[i]) : "memory");
+      }
+      continue;
+    }
     for (int q = pt; q < n; q += PW * 32) {
       const uint32_t pk = __ldg(pack + q);
       const int k = (pk >> 14) & 63, m = pk >> 20;
@@ -711,7 +738,7 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
     const int64_t goff = relCm[grow];
     // tile info is fetched one tile ahead: its load latency hides behind the current tile
     // (PAIR: this CTA's m-tile against the unit's two n-tiles)
-    int64_t ncoff[NSUB];
+    int64_t nmc = 0, nnc[NSUB];   // (raw records: summed at use, so the loads overlap a tile)
     uint64_t nrm0 = 0, nrm1 = 0, ncm0[NSUB], ncm1[NSUB];
     auto fetch = [&](int t) {
       int mt, nt;
@@ -725,9 +752,10 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
       }
       nrm0 = p.tileM[mt].mask[0];
       nrm1 = p.tileM[mt].mask[1];
+      nmc = p.tileM[mt].c;
 #pragma unroll
       for (int q = 0; q < NSUB; q++) {
-        ncoff[q] = p.tileM[mt].c + p.tileN[nt + q].c;
+        nnc[q] = p.tileN[nt + q].c;
         ncm0[q] = p.tileN[nt + q].mask[0];
         ncm1[q] = p.tileN[nt + q].mask[1];
       }
@@ -753,9 +781,10 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
       const int buf = lt % NBUF;
       int64_t coffs[NSUB];
       uint64_t cm0s[NSUB], cm1s[NSUB];
+      const int64_t mc = nmc;
 #pragma unroll
       for (int q = 0; q < NSUB; q++) {
-        coffs[q] = ncoff[q];
+        coffs[q] = nnc[q];
         cm0s[q] = ncm0[q];
         cm1s[q] = ncm1[q];
       }
@@ -767,7 +796,7 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
       tc05_fence_after();
 #pragma unroll 1
       for (int q = 0; q < NSUB; q++) {
-      const int64_t coff = coffs[q];
+      const int64_t coff = mc + coffs[q];
       const uint64_t cm0 = cm0s[q], cm1 = cm1s[q];
       const uint32_t cb = (uint32_t)(buf * ACCW + q * BN);   // this tile's TMEM columns
       T *Crow = C + (coff + roff);
