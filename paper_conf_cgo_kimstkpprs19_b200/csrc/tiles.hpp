@@ -18,7 +18,7 @@ enum Kind { KIND_F64_DMMA = 0, KIND_BF16_UMMA = 1, KIND_TF32_UMMA = 2, KIND_F32X
 inline bool is_umma(int kind) { return kind != KIND_F64_DMMA; }
 inline int kind_esize(int kind) { return kind == KIND_F64_DMMA ? 8 : kind == KIND_BF16_UMMA ? 2 : 4; }
 
-constexpr int kNumVariants = 25;   // ids 0..20 (variants.def + BF16 11, 12) + TF32 21, 22 + F32X3 23, 24
+constexpr int kNumVariants = 27;   // ids 0..20, 25, 26 (variants.def + BF16 11, 12) + TF32 21, 22 + F32X3 23, 24
 
 struct Variant {
   int BM = 0, BN = 0, BK = 0, WM = 0, WN = 0, stages = 0, pw = 0, occ = 0;   // pw = producer warps
