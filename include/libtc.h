@@ -196,6 +196,42 @@ void tc_plan_cache_clear(void);    /* drop the cache's references (live handles 
 tc_status_t tc_plan_restrict(tc_plan_t *sub, const tc_plan_t parent, const char *index,
                              int64_t begin, int64_t len, unsigned flags);
 
+/*
+ * Plan over caller-given element strides (C, A, B are
+ * "tensors of arbitrary dimensions" addressed through their layouts).  strideC / strideA /
+ * strideB: one element stride per index of that tensor, in the order its letters appear in
+ * expr (NULL = dense, first letter fastest).  Input strides may be any value >= 0 (0
+ * broadcasts); C's must be >= 1 and non-overlapping (sorted by stride, each stride >= the
+ * previous stride * its extent).  The caller's buffers must cover tc_plan_span elements.
+ * Index fusion (row a2) only merges indices whose strides are contiguous in every tensor.
+ * Errors: TC_ERR_INVALID_ARG (negative / overlapping strides, span overflow) + tc_plan_ex's.
+ */
+tc_status_t tc_plan_strided(tc_plan_t *plan, const char *expr, const char *extents, tc_dtype_t dtype,
+                            const int64_t *strideC, const int64_t *strideA, const int64_t *strideB,
+                            const tc_plan_opts *opts /* nullable */);
+/*
+ * Representative-size plans ("a representative problem
+ * size is used for performance modeling ... generated code will execute correctly for any
+ * problem size", "different code versions targeted at each representative problem
+ * size ... the kernel is selected at runtime").
+ * tc_plan_resize: bind `rep`'s configuration (kernel variant, digit orders, per-index tiles,
+ *   each clamped to the new extent) to other extents of the same expression: the device
+ *   tables are rebuilt, nothing is searched.  When the new extents change the normalised
+ *   index structure (an extent becomes 1, so an index drops) the planner runs instead.
+ *   `rep` must come from tc_plan / tc_plan_ex / tc_plan_cached (TC_ERR_INVALID_ARG else).
+ * tc_plan_select: the cost model scores every version's configuration at `extents`; the
+ *   best one is resized to them (*chosen = its index, nullable).  Versions must share the
+ *   expression and dtype.
+ * The result is an ordinary plan owned by the caller (tc_plan_destroy).
+ */
+tc_status_t tc_plan_resize(tc_plan_t *sized, const tc_plan_t rep, const char *extents);
+tc_status_t tc_plan_select(tc_plan_t *sized, const tc_plan_t *versions, int n, const char *extents,
+                           int *chosen);
+
+/* Elements the buffer of tensor t (0=C, 1=A, 2=B) must hold: largest offset touched + 1
+   (= tc_plan_numel for dense plans; larger for strided ones and restricted views). */
+int64_t tc_plan_span(const tc_plan_t plan, int t);
+
 /* JSON description of the plan (classes, fused indices, tiles, variant, predicted cost,
    config-space statistics).  Writes at most cap bytes (NUL-terminated); *needed = full size. */
 tc_status_t tc_plan_info(const tc_plan_t plan, char *json, size_t cap, size_t *needed);

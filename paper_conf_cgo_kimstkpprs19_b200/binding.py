@@ -84,6 +84,15 @@ def lib():
         L.tc_plan_flops.restype = dbl
         L.tc_plan_numel.argtypes = [vp, ctypes.c_int]
         L.tc_plan_numel.restype = i64
+        L.tc_plan_resize.argtypes = [ctypes.POINTER(vp), vp, cp]
+        L.tc_plan_resize.restype = ctypes.c_int
+        L.tc_plan_select.argtypes = [ctypes.POINTER(vp), ctypes.POINTER(vp), ctypes.c_int, cp, ctypes.POINTER(ctypes.c_int)]
+        L.tc_plan_select.restype = ctypes.c_int
+        L.tc_plan_span.argtypes = [vp, ctypes.c_int]
+        L.tc_plan_span.restype = i64
+        p64 = ctypes.POINTER(i64)
+        L.tc_plan_strided.argtypes = [ctypes.POINTER(vp), cp, cp, ctypes.c_int, p64, p64, p64, ctypes.POINTER(_Opts)]
+        L.tc_plan_strided.restype = ctypes.c_int
         L.tc_plan_destroy.argtypes = [vp]
         L.tc_plan_destroy.restype = None
         L.tc_status_string.argtypes = [ctypes.c_int]
@@ -167,6 +176,16 @@ class Plan:
     def numel(self, which: str) -> int:
         return int(lib().tc_plan_numel(self._h, "CAB".index(which)))
 
+    def resize(self, extents: str) -> "Plan":
+        """tc_plan_resize: this plan's configuration bound to other extents (NEXT-1)."""
+        h = ctypes.c_void_p()
+        _raise(lib().tc_plan_resize(ctypes.byref(h), self._h, extents.encode()))
+        return Plan(h, self.expr, extents, self.dtype)
+
+    def span(self, which: str) -> int:
+        """Elements tensor `which`'s buffer must hold (largest offset + 1)."""
+        return int(lib().tc_plan_span(self._h, "CAB".index(which)))
+
     def workspace_bytes(self) -> int:
         return int(lib().tc_plan_workspace_bytes(self._h))
 
@@ -201,6 +220,8 @@ class Plan:
                 raise TcError(1, f"{name} must be a contiguous CUDA tensor")
             if t.dtype != want:
                 raise TcError(1, f"{name} is {t.dtype}, the plan's dtype {self.dtype!r} needs {want}")
+            if t.numel() < self.span(w):
+                raise TcError(1, f"{name} holds {t.numel()} elements, the plan's view spans {self.span(w)}")
         self.execute_ptr(A.data_ptr(), B.data_ptr(), C.data_ptr(), alpha, beta, stream)
         return C
 
@@ -336,6 +357,33 @@ def plan(expr: str, extents: str, dtype: str = "f64", cost: str = "b200", host_o
     p = Plan(h, expr, extents, dtype)
     p._opts = o  # keep force_tiles bytes alive for the call's duration
     return p
+
+
+def plan_strided(expr: str, extents: str, strides: dict, dtype: str = "f64", cost: str = "b200",
+                 host_only: bool = False, variant: int | None = None, force_tiles: str | None = None,
+                 fusion: bool = True) -> Plan:
+    """tc_plan_strided: strides = {"C": [...], "A": [...], "B": [...]} (element strides per index
+    in the expression's letter order; a missing tensor is dense)."""
+    o = _opts(cost, host_only, variant, force_tiles, fusion, False, None)
+    arrs = []
+    for t in "CAB":
+        s = strides.get(t)
+        arrs.append(None if s is None else (ctypes.c_int64 * len(s))(*[int(x) for x in s]))
+    h = ctypes.c_void_p()
+    _raise(lib().tc_plan_strided(ctypes.byref(h), expr.encode(), extents.encode(), DTYPES[dtype],
+                                 *[None if a is None else ctypes.cast(a, ctypes.POINTER(ctypes.c_int64)) for a in arrs],
+                                 ctypes.byref(o)))
+    p = Plan(h, expr, extents, dtype)
+    p._opts = o
+    return p
+
+
+def select(versions, extents: str):
+    """tc_plan_select: (plan at `extents`, index of the version the cost model chose)."""
+    arr = (ctypes.c_void_p * len(versions))(*[v._h for v in versions])
+    h, ch = ctypes.c_void_p(), ctypes.c_int(-1)
+    _raise(lib().tc_plan_select(ctypes.byref(h), arr, len(versions), extents.encode(), ctypes.byref(ch)))
+    return Plan(h, versions[0].expr, extents, versions[0].dtype), ch.value
 
 
 def shape_of(indices: str, extents: dict) -> tuple:

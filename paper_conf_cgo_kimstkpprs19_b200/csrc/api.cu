@@ -253,7 +253,21 @@ bool parse_force(const char *s, ForcedTiles &ft) {
   return true;
 }
 
-tc_status_t finish_plan(tc_plan_s *P, tc_plan_t *out) {
+// Same normalised index structure (names, classes, tensor index lists): a configuration made
+// for one contraction's extents is then a legal configuration of the other's (tiles clamped).
+bool same_structure(const Contraction &a, const Contraction &b) {
+  if (a.ix.size() != b.ix.size()) return false;
+  for (size_t i = 0; i < a.ix.size(); i++)
+    if (a.ix[i].name != b.ix[i].name || a.ix[i].cls != b.ix[i].cls) return false;
+  for (int t = 0; t < 3; t++)
+    if (a.t[t].idx != b.t[t].idx) return false;
+  return true;
+}
+
+// rep (optional): a plan whose configuration (variant, digit orders, tiles) is reused when the
+// structures match — tiles clamped to the new extents, tables rebuilt, no search (NEXT-1,
+// P:L77, L300); otherwise the planner runs as usual.
+tc_status_t finish_plan(tc_plan_s *P, tc_plan_t *out, const tc_plan_s *rep = nullptr) {
   std::string err;
   ForcedTiles ft;
   if (!parse_force(P->opts.force_tiles, ft)) { delete P; return fail(ST_INVALID_ARG, "malformed force_tiles"); }
@@ -277,7 +291,22 @@ tc_status_t finish_plan(tc_plan_s *P, tc_plan_t *out) {
       return fail(ST_UNSUPPORTED, "more than 4 batch indices or more than 65535 batch values");
     }
   }
-  Status s = choose(P->c, kind, P->opts.cost_mode, fv, ft, P->cfg, P->stats, err);
+  Status s = ST_NO_CONFIG;
+  if (rep && !ft.on && same_structure(rep->c, P->c)) {
+    Config cfg = rep->cfg;
+    for (size_t id = 0; id < P->c.ix.size(); id++)
+      cfg.T[id] = (int)std::min<int64_t>(cfg.T[id], P->c.ix[id].n);
+    finish_counts(P->c, cfg);
+    if (config_fits(cfg, variants()[cfg.variant])) {
+      model_time(P->c, cfg, variants()[cfg.variant]);   // vector widths, predicted time
+      P->cfg = cfg;
+      P->stats = PlanStats();
+      P->stats.cost_mode = P->opts.cost_mode;
+      P->resized = true;
+      s = ST_OK;
+    }
+  }
+  if (s != ST_OK) s = choose(P->c, kind, P->opts.cost_mode, fv, ft, P->cfg, P->stats, err);
   if (s != ST_OK) { delete P; return fail(s, err); }
   build_host_tables(P);
   if (!P->host_only) {
@@ -423,12 +452,132 @@ tc_status_t tc_plan_ex(tc_plan_t *plan, const char *expr, const char *extents, t
       { delete P; return fail(ST_UNSUPPORTED, "dtype must be TC_F64, TC_F32, TC_TF32 or TC_BF16"); }
     if (opts && (opts->cost_mode < 0 || opts->cost_mode > 1)) { delete P; return fail(ST_INVALID_ARG, "cost_mode"); }
     P->dtype = dtype;
+    P->expr = expr;
     return finish_plan(P, plan);
   } catch (std::bad_alloc &) {
     return fail(ST_ALLOC, "out of host memory");
   } catch (...) {
     return fail(ST_ALLOC, "exception in tc_plan");
   }
+}
+
+tc_status_t tc_plan_strided(tc_plan_t *plan, const char *expr, const char *extents, tc_dtype_t dtype,
+                            const int64_t *strideC, const int64_t *strideA, const int64_t *strideB,
+                            const tc_plan_opts *opts) {
+  if (!plan) return fail(ST_INVALID_ARG, "plan is NULL");
+  *plan = nullptr;
+  try {
+    tc_plan_s *P = new tc_plan_s();
+    if (opts) P->opts = *opts;
+    if (opts && opts->force_tiles) {
+      P->force_tiles = opts->force_tiles;
+      P->opts.force_tiles = P->force_tiles.c_str();
+    }
+    P->host_only = opts && opts->host_only;
+    std::string err;
+    Status s = parse(expr, extents, P->parsed, err);
+    if (s != ST_OK) { delete P; return fail(s, err); }
+    if (dtype != TC_F64 && dtype != TC_BF16 && dtype != TC_TF32 && dtype != TC_F32)
+      { delete P; return fail(ST_UNSUPPORTED, "dtype must be TC_F64, TC_F32, TC_TF32 or TC_BF16"); }
+    if (opts && (opts->cost_mode < 0 || opts->cost_mode > 1)) { delete P; return fail(ST_INVALID_ARG, "cost_mode"); }
+    P->dtype = dtype;
+    Contraction &c = P->parsed;
+    const int64_t *st[3] = {strideC, strideA, strideB};
+    for (int t = 0; t < 3; t++) {
+      if (!st[t]) continue;
+      TensorView &v = c.t[t];
+      long double span = 1;
+      for (size_t k = 0; k < v.idx.size(); k++) {
+        if (st[t][k] < (t == 0 ? 1 : 0)) { delete P; return fail(ST_INVALID_ARG, "negative stride (or a zero stride of C)"); }
+        v.stride[k] = st[t][k];
+        span += (long double)(c.ix[v.idx[k]].n - 1) * (long double)st[t][k];
+      }
+      if (span > (long double)(int64_t(1) << 62)) { delete P; return fail(ST_INVALID_ARG, "strided span overflows"); }
+      if (t == 0) {   // C must not alias itself: sorted by stride, each dim clears the previous
+        std::vector<std::pair<int64_t, int64_t>> d;
+        for (size_t k = 0; k < v.idx.size(); k++)
+          if (c.ix[v.idx[k]].n > 1) d.push_back({v.stride[k], c.ix[v.idx[k]].n});
+        std::sort(d.begin(), d.end());
+        for (size_t k = 1; k < d.size(); k++)
+          if (d[k].first < d[k - 1].first * d[k - 1].second) { delete P; return fail(ST_INVALID_ARG, "C strides overlap"); }
+      }
+      c.parent_numel[t] = c.span(t);
+    }
+    return finish_plan(P, plan);
+  } catch (std::bad_alloc &) {
+    return fail(ST_ALLOC, "out of host memory");
+  } catch (...) {
+    return fail(ST_ALLOC, "exception in tc_plan_strided");
+  }
+}
+
+tc_status_t tc_plan_resize(tc_plan_t *sized, const tc_plan_t rep, const char *extents) {
+  if (!sized || !rep || !extents) return fail(ST_INVALID_ARG, "NULL argument");
+  *sized = nullptr;
+  if (rep->expr.empty()) return fail(ST_INVALID_ARG, "only plans made by tc_plan / tc_plan_ex / tc_plan_cached resize");
+  try {
+    tc_plan_s *P = new tc_plan_s();
+    P->opts = rep->opts;
+    P->force_tiles = rep->force_tiles;
+    P->opts.force_tiles = rep->opts.force_tiles ? P->force_tiles.c_str() : nullptr;
+    P->host_only = rep->host_only;
+    P->dtype = rep->dtype;
+    P->expr = rep->expr;
+    std::string err;
+    Status s = parse(P->expr.c_str(), extents, P->parsed, err);
+    if (s != ST_OK) { delete P; return fail(s, err); }
+    if (!rep->host_only) {
+      int dev = -1;
+      if (cudaGetDevice(&dev) != cudaSuccess || dev != rep->device) {
+        cudaGetLastError();
+        delete P;
+        return fail(ST_INVALID_ARG, "current device differs from the plan's device");
+      }
+    }
+    return finish_plan(P, sized, rep);
+  } catch (std::bad_alloc &) {
+    return fail(ST_ALLOC, "out of host memory");
+  } catch (...) {
+    return fail(ST_ALLOC, "exception in tc_plan_resize");
+  }
+}
+
+tc_status_t tc_plan_select(tc_plan_t *sized, const tc_plan_t *versions, int n, const char *extents, int *chosen) {
+  if (!sized || !versions || n < 1 || !extents) return fail(ST_INVALID_ARG, "NULL argument or n < 1");
+  *sized = nullptr;
+  try {
+    // the cost model at the actual extents ranks the versions' configurations ("the
+    // kernel is selected at runtime based on the closest representative for the performance")
+    int best = -1;
+    double bt = 0;
+    for (int i = 0; i < n; i++) {
+      const tc_plan_s *R = versions[i];
+      if (!R || R->expr.empty()) return fail(ST_INVALID_ARG, "version is NULL or not resizable");
+      if (R->expr != versions[0]->expr || R->dtype != versions[0]->dtype)
+        return fail(ST_INVALID_ARG, "versions differ in expression or dtype");
+      Contraction c;
+      std::string err;
+      Status s = parse(R->expr.c_str(), extents, c, err);
+      if (s != ST_OK) return fail(s, err);
+      normalize(c, !R->opts.no_fusion && !R->opts.force_tiles);
+      if (!same_structure(R->c, c)) continue;
+      Config cfg = R->cfg;
+      for (size_t id = 0; id < c.ix.size(); id++) cfg.T[id] = (int)std::min<int64_t>(cfg.T[id], c.ix[id].n);
+      finish_counts(c, cfg);
+      if (!config_fits(cfg, variants()[cfg.variant])) continue;
+      const double t = model_time(c, cfg, variants()[cfg.variant]);
+      if (best < 0 || t < bt) { best = i; bt = t; }
+    }
+    if (chosen) *chosen = best < 0 ? 0 : best;
+    return tc_plan_resize(sized, versions[best < 0 ? 0 : best], extents);
+  } catch (...) {
+    return fail(ST_ALLOC, "exception in tc_plan_select");
+  }
+}
+
+int64_t tc_plan_span(const tc_plan_t plan, int t) {
+  if (!plan || t < 0 || t > 2) return -1;
+  return plan->parsed.span(t);
 }
 
 tc_status_t tc_plan(tc_plan_t *plan, const char *expr, const char *extents, tc_dtype_t dtype) {
@@ -827,7 +976,8 @@ tc_status_t tc_plan_info(const tc_plan_t plan, char *json, size_t cap, size_t *n
       << ",\"nbatch\":" << c.nbatch();
     o << ",\"vecX\":" << g.vecX << ",\"vecY\":" << g.vecY << ",\"vecC\":" << plan->cvec << ",\"cs0\":" << plan->kp.cs0 << ",\"xKmajor\":" << g.xKmajor
       << ",\"yKmajor\":" << g.yKmajor << ",\"tma_operands\":" << (plan->umma_tma ? 1 : 0)
-      << ",\"cta_pair\":" << (plan->pair ? 1 : 0) << ",\"wfX\":" << g.wfX << ",\"wfY\":" << g.wfY;
+      << ",\"cta_pair\":" << (plan->pair ? 1 : 0) << ",\"resized\":" << (plan->resized ? 1 : 0)
+      << ",\"wfX\":" << g.wfX << ",\"wfY\":" << g.wfY;
     char buf[512];
     std::snprintf(buf, sizeof buf,
                   ",\"t_pred_ms\":%.6g,\"t_comp_ms\":%.6g,\"t_mem_ms\":%.6g,\"t_l2_ms\":%.6g,"

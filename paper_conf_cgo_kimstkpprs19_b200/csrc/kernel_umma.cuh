@@ -602,6 +602,11 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
       const int64_t bx = cur.ox + ks.sx(), by = cur.oy + ks.sy();
       const uint32_t dx = sbase + (uint32_t)ES * (uint32_t)(s * K::XS);
       const uint32_t dy = sbase + (uint32_t)ES * (uint32_t)(STAGES * K::XS + s * K::YS);
+#if defined(TC_UMMA_ABLATE) && TC_UMMA_ABLATE == 2
+      if (true) {   // (ablation side build: the producers load nothing)
+        mbar_arrive(FULL + 8 * s);
+      } else
+#endif
       if (cached) {
         umma_issue<K::EX>(X, dx, rx, px, cx, bx, fm && fk, km, mm, p.packX, pt, K::PW * 32);
         umma_issue<K::EY>(Y, dy, ry, py, cy, by, fn && fk, km, mn, p.packY, pt, K::PW * 32);
@@ -802,7 +807,11 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
       T *Crow = C + (coff + roff);
       const bool cfull = cm0 == p.fullN[0] && cm1 == p.fullN[1];
       T *Cg = C + (coff + goff);
+#if defined(TC_UMMA_ABLATE) && TC_UMMA_ABLATE == 1
+      if (true) {   // (ablation side build: the epilogue drains nothing)
+#else
       if (kTrace) {
+#endif
         if (warp == 0 && lane == 0) trace_at(p, 4, lt);
       } else if (p.vecC == 8 && p.cs0 > 1) {
         // CTA-wide staged epilogue: C's FVI is an inner m digit (tile-row stride cs0), so the

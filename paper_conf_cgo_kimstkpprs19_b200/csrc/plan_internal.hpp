@@ -35,6 +35,8 @@ struct tc_plan_s {
   // tcgen05: operand tensor maps for the TMA producer (tiles.cpp umma_tma_spec); the pointers
   // come per call, so tc_execute encodes the maps from these shapes
   bool umma_tma = false;
+  std::string expr;        // the expression as given (tc_plan / tc_plan_ex): resizable plans
+  bool resized = false;    // the configuration came from a representative-size plan (NEXT-1)
   bool pair = false;       // tcgen05: launch the CTA-pair instance (clusters of 2) with TMA operands
   OperandMap mapX, mapY;
   // batch (Hadamard) indices (R31): extent and element strides in X, Y, C.  tc_execute

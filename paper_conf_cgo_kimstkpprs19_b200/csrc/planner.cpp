@@ -367,6 +367,9 @@ std::vector<Config> order_options(const Contraction &c, int kind, int only_morde
 
 }  // namespace
 
+// (exported for representative-size plans: api.cu tc_plan_resize / tc_plan_select)
+bool config_fits(const Config &cfg, const Variant &v) { return fits(cfg, v); }
+
 // ---------------------------------------------------------------- B200 mode
 static Status choose_b200(const Contraction &c, int kind, int forced_variant, int only_morder, Config &best,
                           PlanStats &st) {

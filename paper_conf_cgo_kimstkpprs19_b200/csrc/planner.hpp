@@ -43,6 +43,8 @@ Status choose(const Contraction &c, int kind, int cost_mode, int forced_variant,
 
 // B200 model (seconds); fills cfg's model outputs.
 using WfCache = std::map<std::vector<int64_t>, std::pair<double, double>>;
+// Does the configuration fit the kernel variant (tile extents, grid limits)?
+bool config_fits(const Config &cfg, const Variant &v);
 double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *cache = nullptr,
                   bool lower_bound = false);   // lower_bound: ideal smem / sector terms, no simulation
 double paper_alg3_cost(const Contraction &c, const Config &cfg, const std::vector<int> &tbx,

@@ -6,6 +6,7 @@ import json
 import os
 import re
 
+import numpy as np
 import pytest
 
 import tcinputs
@@ -290,3 +291,51 @@ def test_group_plan_errors_host():
     with pytest.raises(tc.TcError) as e:                         # an operand of rank 9 (> 8)
         tc.plan_group([tc.plan("abcdefgh-abcdefghi-i", ";".join(f"{x}:2" for x in "abcdefghi"), host_only=True)])
     assert e.value.status == "TC_ERR_UNSUPPORTED"
+
+
+def test_plan_strided_validation_and_span():
+    """tc_plan_strided (row f3): stride checks, spans, fusion only over contiguous strides."""
+    from paper_conf_cgo_kimstkpprs19_b200 import binding as tc
+    # explicit dense strides plan exactly like tc_plan
+    d = tc.plan("abcd-aebf-dfce", "a:12;b:10;c:9;d:8;e:7;f:6", host_only=True).info()
+    s = tc.plan_strided("abcd-aebf-dfce", "a:12;b:10;c:9;d:8;e:7;f:6",
+                        {"C": [1, 12, 120, 1080], "A": [1, 12, 84, 840], "B": [1, 8, 48, 336]}, host_only=True).info()
+    assert [x["tile"] for x in d["indices"]] == [x["tile"] for x in s["indices"]]
+    # a padded pitch: spans grow, numel does not; a and c of ab-ac-cb no longer fuse with b
+    p = tc.plan_strided("ab-ac-cb", "a:70;b:50;c:40", {"C": [1, 72], "A": [1, 80]}, host_only=True)
+    assert p.numel("C") == 70 * 50 and p.span("C") == 69 + 49 * 72 + 1
+    assert p.span("A") == 69 + 39 * 80 + 1 and p.span("B") == 40 * 50
+    # fusion: the a-b run fuses only when its strides are contiguous in every tensor
+    q = tc.plan("abc-abd-dc", "a:4;b:5;c:6;d:7", host_only=True).info()
+    qs = tc.plan_strided("abc-abd-dc", "a:4;b:5;c:6;d:7", {"C": [1, 5, 25], "A": [1, 4, 20]},
+                         host_only=True).info()
+    assert any("*" in x["name"] for x in q["indices"])          # a*b fused when dense
+    assert not any("*" in x["name"] for x in qs["indices"])     # C's a-b pitch 5 != 4: kept apart
+    for bad in ({"C": [1, 3]}, {"C": [0, 70]}, {"A": [-1, 70]}, {"C": [1, 1 << 61]}):
+        with pytest.raises(tc.TcError) as e:
+            tc.plan_strided("ab-ac-cb", "a:5;b:7;c:3", bad, host_only=True)
+        assert e.value.status == "TC_ERR_INVALID_ARG", bad
+
+
+def test_resize_and_select_host():
+    """Representative-size plans (row f1): tiles clamp, the variant stays, a structure change
+    (an extent-1 index) re-plans, selection follows the cost model, strided plans refuse."""
+    from paper_conf_cgo_kimstkpprs19_b200 import binding as tc
+    expr = "abcd-aebf-dfce"
+    rep = tc.plan(expr, "a:16;b:16;c:16;d:16;e:16;f:16", host_only=True)
+    ri = rep.info()
+    s = rep.resize("a:5;b:40;c:7;d:3;e:9;f:70").info()
+    assert s["resized"] == 1 and s["variant"] == ri["variant"]
+    ext = dict(a=5, b=40, c=7, d=3, e=9, f=70)
+    for x, y in zip(ri["indices"], s["indices"]):
+        assert x["name"] == y["name"] and y["tile"] == min(x["tile"], ext[x["name"]])
+    assert rep.resize("a:1;b:16;c:16;d:16;e:16;f:16").info()["resized"] == 0
+    vs = [tc.plan(expr, f"a:{n};b:{n};c:{n};d:{n};e:{n};f:{n}", host_only=True) for n in (8, 16, 72)]
+    big = "a:64;b:64;c:64;d:64;e:64;f:64"
+    p, ch = tc.select(vs, big)
+    preds = [v.resize(big).info()["t_pred_ms"] for v in vs]
+    assert ch == int(np.argmin(preds)) and p.info()["t_pred_ms"] == min(preds)
+    st = tc.plan_strided("ab-ac-cb", "a:5;b:7;c:3", {"C": [1, 8]}, host_only=True)
+    with pytest.raises(tc.TcError) as e:
+        st.resize("a:6;b:7;c:3")
+    assert e.value.status == "TC_ERR_INVALID_ARG"
