@@ -173,7 +173,6 @@ static int parse_all(Spec *s, const char *expr, const char *extents) {
   for (int id = 0; id < s->nidx; id++) if (!seen[id]) return E_INDEX;
   /* 7. extent values */
   for (int id = 0; id < s->nidx; id++) if (s->ext[id] < 1) return E_EXTENT;
-  for (int id = 0; id < s->nidx; id++) if (s->ext[id] > 2147483647LL) return E_UNSUP;
   /* 8. element counts must fit int64: every tensor and the whole iteration space */
   long double all = 1;
   for (int id = 0; id < s->nidx; id++) all *= (long double)s->ext[id];

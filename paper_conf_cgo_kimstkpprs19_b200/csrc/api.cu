@@ -279,6 +279,7 @@ tc_status_t finish_plan(tc_plan_s *P, tc_plan_t *out, const tc_plan_s *rep = nul
   // forced tiles name the original indices: plan without fusion so the names survive
   P->c = P->parsed;
   normalize(P->c, !P->opts.no_fusion && !ft.on);
+  if (!split_large(P->c, err)) { delete P; return fail(ST_UNSUPPORTED, err); }
   const int fv = P->opts.variant > 0 ? P->opts.variant - 1 : -1;
   if (fv >= (int)variants().size()) { delete P; return fail(ST_INVALID_ARG, "variant out of range"); }
   const int kind = kind_of(P->dtype);
@@ -560,6 +561,7 @@ tc_status_t tc_plan_select(tc_plan_t *sized, const tc_plan_t *versions, int n, c
       Status s = parse(R->expr.c_str(), extents, c, err);
       if (s != ST_OK) return fail(s, err);
       normalize(c, !R->opts.no_fusion && !R->opts.force_tiles);
+      if (!split_large(c, err)) continue;
       if (!same_structure(R->c, c)) continue;
       Config cfg = R->cfg;
       for (size_t id = 0; id < c.ix.size(); id++) cfg.T[id] = (int)std::min<int64_t>(cfg.T[id], c.ix[id].n);

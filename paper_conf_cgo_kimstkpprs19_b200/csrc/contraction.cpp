@@ -146,8 +146,6 @@ Status parse(const char *expr, const char *extents, Contraction &out, std::strin
     if (!ext.count(nm)) { err = "no extent for index '" + nm + "'"; return ST_INDEX; }
   for (auto &nm : order)
     if (ext[nm] < 1) { err = "extent of '" + nm + "' must be >= 1"; return ST_EXTENT; }
-  for (auto &nm : order)
-    if (ext[nm] > 2147483647LL) { err = "extent of '" + nm + "' exceeds 2^31-1"; return ST_UNSUPPORTED; }
   {
     // the whole iteration space (and hence every tensor) must count in int64
     unsigned __int128 all = 1;
@@ -225,6 +223,8 @@ void normalize(Contraction &c, bool fuse) {
       // j must not live in the third tensor (same class as i)
       for (int t = 0; t < 3 && good; t++)
         if (t != tens[0] && t != tens[1] && c.pos_in(t, j) >= 0) good = false;
+      // the merged extent stays below 2^31 (tile coordinates and TMA boxes count in int32)
+      if (good && (long double)c.ix[i].n * (long double)c.ix[j].n > 2147483647.0L) good = false;
       if (!good) continue;
       c.ix[i].n *= c.ix[j].n;
       c.ix[i].name += "*" + c.ix[j].name;
@@ -232,6 +232,37 @@ void normalize(Contraction &c, bool fuse) {
       changed = true;
     }
   }
+}
+
+bool split_large(Contraction &c, std::string &err) {
+  const int64_t M = 2147483647LL;
+  for (size_t i = 0; i < c.ix.size(); i++) {
+    const int64_t n = c.ix[i].n;
+    if (n <= M) continue;
+    // smallest outer part d >= n / M dividing n (so the inner part n / d <= M is as long as
+    // possible: it keeps the index's contiguous run); bounded search
+    const int64_t lo = (n + M - 1) / M;
+    int64_t d = 0;
+    for (int64_t q = lo; q <= M && q < lo + (int64_t(1) << 24); q++)
+      if (n % q == 0) { d = q; break; }
+    if (!d) { err = "extent of '" + c.ix[i].name + "' exceeds 2^31-1 and has no factor pair below 2^31"; return false; }
+    const int64_t inner = n / d;
+    Index hi = c.ix[i];
+    hi.n = d;
+    hi.name = c.ix[i].name + "'";
+    c.ix[i].n = inner;
+    const int j = (int)c.ix.size();
+    c.ix.push_back(hi);
+    for (int t = 0; t < 3; t++) {
+      const int p = c.pos_in(t, (int)i);
+      if (p < 0) continue;
+      auto &v = c.t[t];
+      if ((int)v.idx.size() >= kMaxRank) { err = "splitting '" + hi.name + "' exceeds the rank limit"; return false; }
+      v.idx.insert(v.idx.begin() + p + 1, j);
+      v.stride.insert(v.stride.begin() + p + 1, v.stride[p] * inner);
+    }
+  }
+  return true;
 }
 
 }  // namespace tc

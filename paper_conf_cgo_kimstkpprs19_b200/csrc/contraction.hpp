@@ -88,5 +88,11 @@ Status parse(const char *expr, const char *extents, Contraction &out, std::strin
 // order and stride-compatible in every tensor holding them (exact; P:L164 mentions merging
 // as a choice the paper did not consider).  Records the merge in the index name.
 void normalize(Contraction &c, bool fuse);
+// Row f1 ("splitting each dimension into multiple dimensions"): every index longer
+// than 2^31-1 (tile coordinates, grid and TMA boxes count in int32) becomes two indices —
+// inner n / d and outer d (the smallest factor >= n / (2^31-1)), stride_outer = stride_inner
+// * (n / d) in every tensor holding it: an exact relabelling.  False (err set) when n has no
+// such factor pair or a tensor would exceed the rank limit.
+bool split_large(Contraction &c, std::string &err);
 
 }  // namespace tc

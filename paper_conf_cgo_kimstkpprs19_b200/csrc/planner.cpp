@@ -344,7 +344,7 @@ bool better(const Config &a, const Config &b) {
 
 bool fits(const Config &cfg, const Variant &v) {
   return cfg.Mt <= v.BM && cfg.Nt <= v.BN && cfg.Kt <= v.BK && cfg.nctas < (1LL << 31) &&
-         cfg.mtiles < (1LL << 24) && cfg.ntiles < (1LL << 24) && cfg.nsteps < (1LL << 24);
+         cfg.mtiles < (1LL << 26) && cfg.ntiles < (1LL << 26) && cfg.nsteps < (1LL << 24);   // (tile tables: 56 B per tile)
 }
 
 // The distinct (morder, korder) digit-order options of a contraction.

@@ -339,3 +339,20 @@ def test_resize_and_select_host():
     with pytest.raises(tc.TcError) as e:
         st.resize("a:6;b:7;c:3")
     assert e.value.status == "TC_ERR_INVALID_ARG"
+
+
+def test_large_index_splitting_and_fusion_cap():
+    """Row f1: an index longer than 2^31-1 is split into two exact factors; fusion
+    never builds an index past 2^31-1; a prime extent past 2^31 is unsupported."""
+    from paper_conf_cgo_kimstkpprs19_b200 import binding as tc
+    n = 3 << 30                                  # 3 * 2^30 > 2^31 - 1
+    i = tc.plan("ab-a-b", f"a:{n};b:3", host_only=True).info()
+    ext = {x["name"]: x["n"] for x in i["indices"]}
+    assert ext == {"a": n // 2, "a'": 2, "b": 3}
+    assert i["tensors"]["A"]["stride"] == [1, n // 2] and i["tensors"]["C"]["stride"][:2] == [1, n // 2]
+    # fusion cap: a and b would fuse into 2.5e9 elements
+    j = tc.plan("abc-abd-dc", "a:50000;b:50000;c:1;d:1", host_only=True).info()
+    assert sorted(x["name"] for x in j["indices"]) == ["a", "b"]
+    with pytest.raises(tc.TcError) as e:
+        tc.plan("ab-a-b", "a:2147483659;b:2", host_only=True)   # a prime past 2^31
+    assert e.value.status == "TC_ERR_UNSUPPORTED"
