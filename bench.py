@@ -30,6 +30,9 @@ import tcinputs  # noqa: E402
 METRIC = "TCCG-48 GFLOP/s geomean (FP64) at 1 GPU; % of FP64/tensor peak or HBM roofline"
 UNIT = "GFLOP/s"
 FP64_PEAK_TFLOPS = 37.16      # measured DMMA peak, profiles/r01_peaks.json (tools/peaks.cu)
+# tensor-pipe peaks per dtype: MEASURED_PEAKS.json's dense BF16 (cuBLAS) figure; TF32 runs at
+# half the BF16 rate (the guide's nominal ratio), FP32 as split TF32 issues three TF32 MMAs
+TENSOR_PEAK_TFLOPS = {"bf16": 1645.0, "tf32": 822.5, "f32": 822.5 / 3}
 FP64_PEAK_DERIVED = 148 * 64 * 2 * 1.965e9 / 1e12   # 37.2: SMs x FMA/clk x 2 x max clock
 
 
@@ -50,11 +53,12 @@ def parse_args():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of oracle work")
-    ap.add_argument("--suites", default="ccsdt,membound,triples",
+    ap.add_argument("--suites", default="ccsdt,membound,triples,eq1graph",
                     help="extra workloads reported inside the same JSON line (BASELINE configs 3/4): "
                          "ccsdt = CCSD(T) 6D sweep N=24..48 FP64, membound = memory-bound TCCG cases in "
                          "FP32 (split TF32) / TF32 / BF16 vs the HBM roofline, triples = the 18 CCSD(T) "
                          "contractions into one t3 (tc_execute_group); '' = none")
+    ap.add_argument("--no-splitk", action="store_true", help="skip the split-K demo (SURVEY 8(e))")
     ap.add_argument("--no-scale6d", action="store_true",
                     help="skip the config-5 6D contraction (sd_t_d2, N = 40) timed at every world size")
     ap.add_argument("--profile", action="store_true",
@@ -294,6 +298,106 @@ def run_triples(args, flush, stream, dev, hbm):
             "cases": rows}
 
 
+def run_eq1_graph(args, stream, dev):
+    """BASELINE config 1 / SURVEY 8(d): eq. (1), all extents 16, FP64 — 100 tc_execute launches
+    captured in one CUDA graph and replayed (the launch-bound regime), against the same 100
+    launches issued eagerly; device time per launch in microseconds, GFLOP/s."""
+    import torch
+    from paper_conf_cgo_kimstkpprs19_b200 import binding as tc
+    p = tc.plan(tcinputs.EQ1_EXPR, tcinputs.EQ1_EXTENTS)
+    A = tcinputs.uniform(p.numel("A"), 11, device=dev)
+    B = tcinputs.uniform(p.numel("B"), 12, device=dev)
+    C = torch.empty(p.numel("C"), dtype=torch.float64, device=dev)
+    n = 100
+    s2 = torch.cuda.Stream(device=dev)
+    s2.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(s2):
+        for _ in range(3):
+            p.execute(A, B, C)
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=s2):
+            for _ in range(n):
+                p.execute(A, B, C)
+    torch.cuda.current_stream().wait_stream(s2)
+    torch.cuda.synchronize()
+
+    def timed(fn, reps):
+        ts = []
+        for _ in range(reps + 2):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            fn()
+            e1.record(stream)
+            e1.synchronize()
+            ts.append(e0.elapsed_time(e1))
+        ts = sorted(ts[2:])
+        return ts[len(ts) // 2]
+
+    def eager():
+        for _ in range(n):
+            p.execute(A, B, C)
+    tg = timed(g.replay, max(3, min(args.steps, 10)))
+    te = timed(eager, max(3, min(args.steps, 10)))
+    return {"workload": "eq.(1) abcd-aebf-dfce, all extents 16, FP64: 100 launches per CUDA graph",
+            "us_per_launch_graph": round(1e3 * tg / n, 3), "gflops_graph": round(p.flops * n / tg / 1e6, 2),
+            "us_per_launch_eager": round(1e3 * te / n, 3), "gflops_eager": round(p.flops * n / te / 1e6, 2),
+            "launches": n, "variant": p.info()["variant"]}
+
+
+def run_splitk(args, world, rank, sharded, flush, stream, dev, hbm):
+    """SURVEY 8(e) split-K demo: ab-ac-cb, a = b = 256, c = 2^20 (the external space fills
+    only 4 x 148 SMs' worth of 128 x 128 tiles): at N GPUs each rank contracts its k-range
+    and the partials are summed by one NCCL reduce-scatter (|C| / N per rank); FP64, and BF16
+    with FP32 partials rounded once (out_f32 + tc_round_bf16).  Inputs are generated
+    resident on every rank (this case's exchange step is the reduce-scatter, timed); time =
+    max over ranks; HBM roofline on the algorithmic bytes of one GPU's share."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_cgo_kimstkpprs19_b200 import binding as tc
+    from paper_conf_cgo_kimstkpprs19_b200 import dist as tcdist
+    expr, extents = "ab-ac-cb", "a:256;b:256;c:1048576"
+    n = 256 * 256
+    out = {"workload": "split-K ab-ac-cb a=b=256 c=2^20 (NCCL reduce-scatter at N > 1)", "n_gpus": world}
+    for dt in ("f64", "bf16"):
+        tdt = torch.float64 if dt == "f64" else torch.bfloat16
+        base = tc.plan(expr, extents, dtype=dt, out_f32=(dt == "bf16"))
+        sub, k, lo, ln = tcdist.split_k_plan(base, expr, extents, world, rank)
+        A = tcinputs.uniform(base.numel("A"), 31, device=dev).to(tdt)
+        B = tcinputs.uniform(base.numel("B"), 32, device=dev).to(tdt)
+        pdt = torch.float64 if dt == "f64" else torch.float32
+        Cp = torch.zeros(tcdist.partial_numel(n, world), dtype=pdt, device=dev)
+        res = torch.empty(n, dtype=torch.bfloat16, device=dev) if dt == "bf16" else None
+        ts = []
+        for it in range(args.warmup + max(3, min(args.steps, 5))):
+            flush.zero_()
+            if sharded:
+                dist.barrier()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            if sharded:
+                tcdist.execute_split_k(sub, A, B, Cp, world, rank, n=n, out_bf16=res)
+            else:
+                sub.execute(A, B, Cp[:n])
+                if res is not None:
+                    tc.round_bf16(res, Cp[:n])
+            e1.record(stream)
+            torch.cuda.synchronize()
+            if it >= args.warmup:
+                ts.append(e0.elapsed_time(e1))
+        t = torch.tensor([sorted(ts)[len(ts) // 2]], dtype=torch.float64, device=dev)
+        if sharded:
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = t.item()
+        es = 8 if dt == "f64" else 2
+        byts = es * (256 * 1048576 * 2) / world + (8 if dt == "f64" else 4) * n
+        out[dt] = {"ms": round(ms, 4), "gflops": round(base.flops / ms / 1e6, 2),
+                   "hbm_frac_per_gpu": round(byts / (ms * 1e-3) / hbm, 4),
+                   "partials": "f64" if dt == "f64" else "f32 (out_f32) + tc_round_bf16"}
+        del A, B, Cp
+        torch.cuda.empty_cache()
+    return out
+
+
 def run_suite(name, args, flush, stream, dev, hbm):
     """One extra workload: per case plan (+ measured top-k tuning like the main suite), time,
     roofline fraction against min(pipe peak, I * HBM) — pipe = FP64 DMMA for f64; the
@@ -303,6 +407,8 @@ def run_suite(name, args, flush, stream, dev, hbm):
     rows = []
     if name == "triples":
         return run_triples(args, flush, stream, dev, hbm)
+    if name == "eq1graph":
+        return run_eq1_graph(args, stream, dev)
     if name == "ccsdt":
         # BASELINE config 3: sd_t_d1 / sd_t_d2 6D contractions at uniform extents 24..48, FP64,
         # beta = 0 (t3 written) and beta = 1 (t3 accumulated)
@@ -331,6 +437,13 @@ def run_suite(name, args, flush, stream, dev, hbm):
             r["roofline_frac"] = round(p.flops / (ms * 1e-3) / attain, 4)
         else:
             r["hbm_frac"] = round(gbs * 1e9 / hbm, 4)
+            # tensor-pipe peak of the dtype (MEASURED_PEAKS.json BF16 cuBLAS figure; TF32 half of
+            # it; FP32 = three TF32 MMAs per product): #18 is compute-bound, judged against it
+            pk = TENSOR_PEAK_TFLOPS[dt] * 1e12
+            r["roofline_frac"] = round(p.flops / (ms * 1e-3) / min(pk, p.flops / byts * hbm), 4)
+            r["bound"] = "tensor" if p.flops / byts * hbm > pk else "hbm"
+            r["cta_pair"] = p.info().get("cta_pair", 0)
+            r["tma_operands"] = p.info().get("tma_operands", 0)
         rows.append(r)
         del A, B, C, p
         torch.cuda.empty_cache()
@@ -342,11 +455,17 @@ def run_suite(name, args, flush, stream, dev, hbm):
             out[f"geomean_gflops_beta{int(b)}"] = round(geomean([r["gflops"] for r in sel]), 2)
             out[f"geomean_roofline_frac_beta{int(b)}"] = round(geomean([r["roofline_frac"] for r in sel]), 4)
     else:
-        out["workload"] = "memory-bound TCCG #1-8, #18 in FP32 (split TF32), TF32, BF16; HBM roofline"
+        out["workload"] = ("memory-bound TCCG #1-8 in FP32 (split TF32), TF32, BF16 against HBM; #18 "
+                           "ab-ac-cb (compute-bound) reported apart against the dtype's tensor peak")
         for dt in ("f32", "tf32", "bf16"):
-            sel = [r for r in rows if r["dtype"] == dt]
+            sel = [r for r in rows if r["dtype"] == dt and r["expr"] != "ab-ac-cb"]
             out[f"geomean_hbm_frac_{dt}"] = round(geomean([r["hbm_frac"] for r in sel]), 4)
             out[f"geomean_gflops_{dt}"] = round(geomean([r["gflops"] for r in sel]), 2)
+            g = [r for r in rows if r["dtype"] == dt and r["expr"] == "ab-ac-cb"]
+            if g:
+                out[f"ab_ac_cb_{dt}"] = {"tflops": round(g[0]["gflops"] / 1e3, 1),
+                                         "tensor_peak_frac": g[0]["roofline_frac"],
+                                         "peak_tflops": TENSOR_PEAK_TFLOPS[dt]}
     return out
 
 
@@ -380,6 +499,7 @@ def run_libtc(args):
 
     # plans + resident inputs (rank 0's inputs are the source of the broadcast at N > 1)
     work = []
+    model_pick = {}   # case id -> the cost model's own (untuned) plan
     t_plan = t_tune = 0.0
     for c in cases:
         t0 = time.perf_counter()
@@ -389,6 +509,7 @@ def run_libtc(args):
         t_plan += time.perf_counter() - t0
         A = tcinputs.uniform(p.numel("A"), 1000 + c.id, device=dev)
         B = tcinputs.uniform(p.numel("B"), 2000 + c.id, device=dev)
+        model_pick[c.id] = p
         if not sharded:
             C = torch.empty(p.numel("C"), dtype=torch.float64, device=dev)
             if args.tune > 0:
@@ -397,6 +518,11 @@ def run_libtc(args):
                 t_tune += time.perf_counter() - t0
             work.append((c, p, A, B, C, None))
         else:
+            if sh.x_tensor is not None and rank != 0:   # the scattered input: this rank's slab only
+                if sh.x_tensor == "A":
+                    A = torch.empty(tcdist.local_input_numel(sh, "A", p.numel("A"), rank), dtype=torch.float64, device=dev)
+                else:
+                    B = torch.empty(tcdist.local_input_numel(sh, "B", p.numel("B"), rank), dtype=torch.float64, device=dev)
             C = torch.empty(sh.c_numel, dtype=torch.float64, device=dev)
             if args.tune > 0 and sh.plan is not None:
                 t0 = time.perf_counter()
@@ -415,8 +541,10 @@ def run_libtc(args):
         if sh is None:
             p.execute(A, B, C)
         else:
-            tcdist.broadcast_inputs(A, B, src=0)
-            sh.plan.execute(A, B, C)
+            tcdist.distribute_inputs(sh, A, B, rank, src=0)
+            if sh.plan is not None:
+                a, b = tcdist.local_operands(sh, A, B, rank)
+                sh.plan.execute(a, b, C)
         e1.record(stream)
         record.append((e0, e1))
 
@@ -477,8 +605,31 @@ def run_libtc(args):
     for w, ms in zip(work, med):
         c, p = w[0], w[1]
         per_case.append({"id": c.id, "ms": round(ms, 5), "gflops": round(p.flops / ms / 1e6, 2),
-                         "variant": run_plan(w).info()["variant"]})
+                         "variant": run_plan(w).info()["variant"],
+                         "pred_ms": round(run_plan(w).info()["t_pred_ms"], 5)})
     value = geomean([r["gflops"] for r in per_case])
+
+    # cost-model fidelity (outside the timed region): the model's predicted time of the plan
+    # that ran vs its measured time, and the model's own pick (untuned) timed vs the tuned one
+    model = None
+    if not sharded:
+        errs, picks = [], []
+        for w, r in zip(work, per_case):
+            r["model_err"] = round(r["pred_ms"] / r["ms"] - 1.0, 4)
+            errs.append(abs(r["model_err"]))
+            pm = model_pick[w[0].id]
+            pm_ms = r["ms"] if pm.info()["variant"] == r["variant"] and pm.info()["t_pred_ms"] == r["pred_ms"] \
+                else time_one(pm, w[2], w[3], w[4], 3, 1, flush, stream)
+            r["model_pick_ms"] = round(pm_ms, 5)
+            picks.append(pm_ms / r["ms"])
+        errs.sort()
+        model = {"median_abs_err": round(errs[len(errs) // 2], 4),
+                 "within_25pct": sum(e <= 0.25 for e in errs), "cases": len(errs),
+                 "pick_within_10pct_of_tuned": sum(x <= 1.10 for x in picks),
+                 "pick_vs_tuned_geomean": round(geomean(picks), 4),
+                 "how": "pred_ms = the B200 cost model's t_pred of the timed plan; model_err = "
+                        "pred / measured - 1; model_pick_ms = the untuned plan (the model's "
+                        "first choice) timed like the suite (3 launches, L2 flushed)"}
     ms_step = sum(med)
 
     # dominant kernel (largest share of the step) -> roofline
@@ -572,6 +723,12 @@ def run_libtc(args):
         sh6 = tcdist.shard_plan(p6, c6.expr, c6.extents, world, rank) if sharded else None
         run6 = sh6.plan if sh6 is not None else p6
         C6 = torch.empty(sh6.c_numel if sh6 is not None else p6.numel("C"), dtype=torch.float64, device=dev)
+        if sh6 is not None and sh6.x_tensor is not None and rank != 0:
+            # the scattered input: this rank holds only its slab
+            if sh6.x_tensor == "A":
+                A6 = torch.empty(tcdist.local_input_numel(sh6, "A", p6.numel("A"), rank), dtype=torch.float64, device=dev)
+            else:
+                B6 = torch.empty(tcdist.local_input_numel(sh6, "B", p6.numel("B"), rank), dtype=torch.float64, device=dev)
         if args.tune > 0 and run6 is not None:   # the same measured top-k as every other case
             run6 = run6.tuned(A6, B6, C6, topk=args.tune, reps=2)
         tot, comp = [], []
@@ -582,10 +739,11 @@ def run_libtc(args):
             ev = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
             ev[0].record(stream)
             if sharded:
-                tcdist.broadcast_inputs(A6, B6, src=0)
+                tcdist.distribute_inputs(sh6, A6, B6, rank, src=0)
             ev[1].record(stream)
             if run6 is not None:
-                run6.execute(A6, B6, C6)
+                a6, b6 = tcdist.local_operands(sh6, A6, B6, rank) if sh6 is not None else (A6, B6)
+                run6.execute(a6, b6, C6)
             ev[2].record(stream)
             torch.cuda.synchronize()
             if it >= args.warmup:
@@ -598,10 +756,15 @@ def run_libtc(args):
                    "ms": round(t6[0].item(), 4), "gflops": round(p6.flops / t6[0].item() / 1e6, 2),
                    "ms_compute_only": round(t6[1].item(), 4),
                    "gflops_compute_only": round(p6.flops / t6[1].item() / 1e6, 2),
-                   "how": "C slab on the largest external index per rank, NCCL broadcast of A and B "
-                          "inside the first interval; time = max over ranks (SURVEY 8(e))"}
+                   "inputs": ("scatter " + sh6.x_tensor + ", broadcast the other") if sh6 is not None and sh6.x_tensor
+                             else "broadcast A and B",
+                   "how": "C slab on the largest external index per rank; the input holding it scattered "
+                          "as slabs when it is that input's slowest index, else broadcast (NCCL), inside "
+                          "the first interval; time = max over ranks (SURVEY 8(e))"}
         del A6, B6, C6
         torch.cuda.empty_cache()
+
+    splitk = None if args.no_splitk else run_splitk(args, world, rank, sharded, flush, stream, dev, hbm)
 
     suites = {}
     if world == 1 and args.suites:
@@ -618,7 +781,14 @@ def run_libtc(args):
                "sample": f"per case a contiguous range of C linear indices sized to "
                          f"~{args.cpu_budget / len(cases):.2f}s of oracle work "
                          f"({sum(v[1] for v in rates.values())} of "
-                         f"{sum(v[2] for v in rates.values())} C elements)"}
+                         f"{sum(v[2] for v in rates.values())} C elements)",
+               "cpu_model": oracle.cpu_model(),
+               "build": "gcc -O3 -march=native -fopenmp -ffp-contract=off (oracle/__init__.py)"}
+        # single-thread oracle figures on eq. (1) and TCCG #3
+        eq1 = tcinputs.Case(0, tcinputs.EQ1_EXPR, tcinputs.EQ1_EXTENTS, "H", "eq1")
+        c3 = [c for c in tcinputs.tccg48() if c.id == 3]
+        r1 = oracle_sample_rates([eq1] + c3, 4.0, nthreads=1)
+        cpu["one_thread_gflops"] = {"eq1_N16": round(r1[0][0], 4), "tccg3": round(r1[3][0], 4)}
 
     if rank == 0:
         line = {"metric": METRIC, "value": round(value, 2), "unit": UNIT, "n_gpus": world,
@@ -643,6 +813,8 @@ def run_libtc(args):
                 "wall_s_timed": round(t_wall, 3),
                 "suites": suites,
                 "scale6d": scale6d,
+                "splitk": splitk,
+                "cost_model": model,
                 "per_case": per_case}
         print(json.dumps(line), flush=True)
     if sharded:

@@ -70,7 +70,9 @@ typedef struct tc_plan_opts {
                           fit (default 0: one thread issues TMA boxes when the plan allows) */
   int cta_pair;      /* tcgen05 BN = 128 plans with TMA operands: 0 planner's choice, 1 never,
                         2 always — CTA pairs (cluster of 2, M = 256 MMAs over 2 x 2 tiles)   */
-  int reserved[4];   /* must be zero (TC_ERR_INVALID_ARG otherwise)                         */
+  int out_f32;       /* TC_BF16 plans: 1 = C is FP32 (the accumulator without the BF16 rounding;
+                        split-K partials); TC_ERR_INVALID_ARG for other dtypes */
+  int reserved[3];   /* must be zero (TC_ERR_INVALID_ARG otherwise)                         */
 } tc_plan_opts;
 
 /*
@@ -227,6 +229,12 @@ tc_status_t tc_plan_strided(tc_plan_t *plan, const char *expr, const char *exten
 tc_status_t tc_plan_resize(tc_plan_t *sized, const tc_plan_t rep, const char *extents);
 tc_status_t tc_plan_select(tc_plan_t *sized, const tc_plan_t *versions, int n, const char *extents,
                            int *chosen);
+
+/* dst[i] = src[i] rounded to BF16 (RNE), i < n, on `stream`: the single rounding of an
+   FP32-reduced split-K result (plans with out_f32).  dst (BF16) and src (FP32)
+   are device pointers that must not overlap.  TC_ERR_INVALID_ARG on NULL / n < 0 / overlap,
+   TC_ERR_CUDA on a launch error. */
+tc_status_t tc_round_bf16(void *dst, const void *src, int64_t n, tc_stream_t stream);
 
 /* Elements the buffer of tensor t (0=C, 1=A, 2=B) must hold: largest offset touched + 1
    (= tc_plan_numel for dense plans; larger for strided ones and restricted views). */

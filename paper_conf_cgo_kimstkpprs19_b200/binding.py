@@ -45,7 +45,7 @@ class _Opts(ctypes.Structure):
     _fields_ = [("cost_mode", ctypes.c_int), ("host_only", ctypes.c_int), ("variant", ctypes.c_int),
                 ("force_tiles", ctypes.c_char_p), ("no_fusion", ctypes.c_int), ("tma_epilogue", ctypes.c_int),
                 ("morder", ctypes.c_int), ("no_tma_operands", ctypes.c_int),
-                ("cta_pair", ctypes.c_int), ("reserved", ctypes.c_int * 4)]
+                ("cta_pair", ctypes.c_int), ("out_f32", ctypes.c_int), ("reserved", ctypes.c_int * 3)]
 
 
 _lib = None
@@ -88,6 +88,8 @@ def lib():
         L.tc_plan_resize.restype = ctypes.c_int
         L.tc_plan_select.argtypes = [ctypes.POINTER(vp), ctypes.POINTER(vp), ctypes.c_int, cp, ctypes.POINTER(ctypes.c_int)]
         L.tc_plan_select.restype = ctypes.c_int
+        L.tc_round_bf16.argtypes = [vp, vp, i64, vp]
+        L.tc_round_bf16.restype = ctypes.c_int
         L.tc_plan_span.argtypes = [vp, ctypes.c_int]
         L.tc_plan_span.restype = i64
         p64 = ctypes.POINTER(i64)
@@ -215,7 +217,10 @@ class Plan:
     def execute(self, A, B, C, alpha=1.0, beta=0.0, stream=None):
         """C = alpha * sum A*B + beta * C on torch CUDA tensors (current stream)."""
         want = _TORCH_DTYPE[self.dtype]()
+        import torch
         for name, t, w in (("A", A, "A"), ("B", B, "B"), ("C", C, "C")):
+            if w == "C" and self.dtype == "bf16" and self.info().get("out_f32"):
+                want = torch.float32
             if not t.is_cuda or not t.is_contiguous():
                 raise TcError(1, f"{name} must be a contiguous CUDA tensor")
             if t.dtype != want:
@@ -235,8 +240,10 @@ class Plan:
         return C
 
 
-def _opts(cost, host_only, variant, force_tiles, fusion, tma, morder, tma_operands=True, pair=None) -> _Opts:
+def _opts(cost, host_only, variant, force_tiles, fusion, tma, morder, tma_operands=True, pair=None,
+          out_f32=False) -> _Opts:
     o = _Opts()
+    o.out_f32 = int(out_f32)
     o.no_tma_operands = int(not tma_operands)
     o.cta_pair = {None: 0, False: 1, True: 2}[pair]
     o.morder = {None: 0, "C": 1, "X": 2}[morder]
@@ -348,10 +355,11 @@ def plan_cache_clear() -> None:
 def plan(expr: str, extents: str, dtype: str = "f64", cost: str = "b200", host_only: bool = False,
          variant: int | None = None, force_tiles: str | None = None, fusion: bool = True,
          tma: bool = False, morder: str | None = None, tma_operands: bool = True,
-         pair: bool | None = None) -> Plan:
+         pair: bool | None = None, out_f32: bool = False) -> Plan:
     """pair: None = planner's choice, False / True = CTA pairs off / on where the plan allows.
+    out_f32 (bf16 plans): C is FP32 (split-K partials).
     morder: None = planner's choice, "C" = m digits in C order, "X" = in the X operand's order."""
-    o = _opts(cost, host_only, variant, force_tiles, fusion, tma, morder, tma_operands, pair)
+    o = _opts(cost, host_only, variant, force_tiles, fusion, tma, morder, tma_operands, pair, out_f32)
     h = ctypes.c_void_p()
     _raise(lib().tc_plan_ex(ctypes.byref(h), expr.encode(), extents.encode(), DTYPES[dtype], ctypes.byref(o)))
     p = Plan(h, expr, extents, dtype)
@@ -376,6 +384,18 @@ def plan_strided(expr: str, extents: str, strides: dict, dtype: str = "f64", cos
     p = Plan(h, expr, extents, dtype)
     p._opts = o
     return p
+
+
+def round_bf16(dst, src, stream=None):
+    """tc_round_bf16: dst (torch bfloat16, CUDA) = src (float32) rounded RNE, by libtc."""
+    import torch
+    if dst.dtype != torch.bfloat16 or src.dtype != torch.float32 or dst.numel() < src.numel():
+        raise TcError(1, "round_bf16 wants a bfloat16 dst at least as long as the float32 src")
+    if not (dst.is_cuda and src.is_cuda and dst.is_contiguous() and src.is_contiguous()):
+        raise TcError(1, "round_bf16 wants contiguous CUDA tensors")
+    _raise(lib().tc_round_bf16(ctypes.c_void_p(dst.data_ptr()), ctypes.c_void_p(src.data_ptr()),
+                               src.numel(), _stream_ptr(stream)))
+    return dst
 
 
 def select(versions, extents: str):

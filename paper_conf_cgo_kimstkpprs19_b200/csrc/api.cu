@@ -2,6 +2,7 @@
 // metadata (row a4), kernel dispatch (rows a5-a7), restriction (row e) and introspection.
 #include <cuda.h>
 #include <cudaTypedefs.h>
+#include <cuda_bf16.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -127,7 +128,7 @@ void build_host_tables(tc_plan_s *P) {
   kp.c_rank = (int)c.t[0].idx.size();
   // old-C prefetch (beta != 0): C's FVI leads the m digits, so runs of its tile are C-contiguous
   // rows: one address per 128-B line (16 doubles)
-  P->umma_tma = !P->opts.no_tma_operands &&
+  P->umma_tma = !P->opts.no_tma_operands && !P->out_f32 &&
                 umma_tma_spec(c, cfg, v, cfg.X, &P->mapX, &kp.xt) &&
                 umma_tma_spec(c, cfg, v, cfg.Y, &P->mapY, &kp.yt);
   kp.kt = cfg.kdig.empty() ? 0 : (int)cfg.T[cfg.kdig[0]];
@@ -205,6 +206,14 @@ Status upload(tc_plan_s *P, std::string &err) {
     e = cudaFuncSetAttribute(kt.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kt.smem);
     if (e != cudaSuccess) { err = std::string("cudaFuncSetAttribute: ") + cudaGetErrorString(e); return ST_CUDA; }
   }
+  if (P->out_f32) {
+    size_t sm = 0;
+    int th = 0;
+    const void *fn = kernel_ptr_umma_f32out(P->cfg.variant, P->cfg.xKmajor, P->cfg.yKmajor, &sm, &th);
+    if (!fn) { err = "no FP32-output instance for the variant"; return ST_UNSUPPORTED; }
+    e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    if (e != cudaSuccess) { err = std::string("cudaFuncSetAttribute: ") + cudaGetErrorString(e); return ST_CUDA; }
+  }
   if (P->pair) {
     size_t sm = 0;
     int th = 0;
@@ -273,6 +282,9 @@ tc_status_t finish_plan(tc_plan_s *P, tc_plan_t *out, const tc_plan_s *rep = nul
   if (!parse_force(P->opts.force_tiles, ft)) { delete P; return fail(ST_INVALID_ARG, "malformed force_tiles"); }
   if (P->opts.morder < 0 || P->opts.morder > 2) { delete P; return fail(ST_INVALID_ARG, "morder must be 0, 1 or 2"); }
   if (P->opts.cta_pair < 0 || P->opts.cta_pair > 2) { delete P; return fail(ST_INVALID_ARG, "cta_pair must be 0, 1 or 2"); }
+  if (P->opts.out_f32 != 0 && (P->opts.out_f32 != 1 || P->dtype != TC_BF16))
+    { delete P; return fail(ST_INVALID_ARG, "out_f32 is a TC_BF16 option (0 or 1)"); }
+  P->out_f32 = P->opts.out_f32 == 1;
   for (int r : P->opts.reserved)
     if (r != 0) { delete P; return fail(ST_INVALID_ARG, "tc_plan_opts.reserved[] must be zero"); }
   ft.morder = P->opts.morder - 1;
@@ -324,6 +336,7 @@ tc_status_t finish_plan(tc_plan_s *P, tc_plan_t *out, const tc_plan_s *rep = nul
 }
 
 size_t elem_bytes(const tc_plan_s *P) { return (size_t)kind_esize(kind_of(P->dtype)); }
+size_t elem_bytes_c(const tc_plan_s *P) { return P->out_f32 ? 4 : elem_bytes(P); }
 
 bool overlaps(const void *a, size_t na, const void *b, size_t nb) {
   const char *x = (const char *)a, *y = (const char *)b;
@@ -577,6 +590,29 @@ tc_status_t tc_plan_select(tc_plan_t *sized, const tc_plan_t *versions, int n, c
   }
 }
 
+}  // extern "C"
+
+namespace {
+__global__ void round_bf16_kernel(__nv_bfloat16 *__restrict__ d, const float *__restrict__ s, int64_t n) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    d[i] = __float2bfloat16_rn(s[i]);
+}
+}  // namespace
+
+extern "C" {
+
+tc_status_t tc_round_bf16(void *dst, const void *src, int64_t n, tc_stream_t stream) {
+  if (!dst || !src || n < 0) return fail(ST_INVALID_ARG, "NULL pointer or n < 0");
+  if (n == 0) return TC_SUCCESS;
+  if (overlaps(dst, 2 * (size_t)n, src, 4 * (size_t)n)) return fail(ST_INVALID_ARG, "dst overlaps src");
+  const int blocks = (int)std::min<int64_t>((n + 255) / 256, 148 * 8);
+  round_bf16_kernel<<<blocks, 256, 0, (cudaStream_t)stream>>>(static_cast<__nv_bfloat16 *>(dst),
+                                                             static_cast<const float *>(src), n);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(ST_CUDA, std::string("launch: ") + cudaGetErrorString(e));
+  return TC_SUCCESS;
+}
+
 int64_t tc_plan_span(const tc_plan_t plan, int t) {
   if (!plan || t < 0 || t > 2) return -1;
   return plan->parsed.span(t);
@@ -783,7 +819,7 @@ tc_status_t check_execute(const tc_plan_t plan, const void *A, const void *B, co
   if (plan->host_only || !plan->dev) return fail(ST_CUDA, "plan was made host_only");
   const size_t es = elem_bytes(plan);
   const size_t nA = (size_t)plan->parsed.span(1) * es, nB = (size_t)plan->parsed.span(2) * es,
-               nC = (size_t)plan->parsed.span(0) * es;
+               nC = (size_t)plan->parsed.span(0) * elem_bytes_c(plan);
   if (overlaps(C, nC, A, nA) || overlaps(C, nC, B, nB)) return fail(ST_INVALID_ARG, "C overlaps A or B");
   int cur = -1;
   if (cudaGetDevice(&cur) != cudaSuccess || cur != plan->device)
@@ -827,7 +863,12 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
   // tcgen05: operands by TMA when the plan allows and both views encode at these pointers
   const bool tma_ops = plan->umma_tma && encode_operand_map(plan, plan->mapX, kp.X, kp.xmap) &&
                        encode_operand_map(plan, plan->mapY, kp.Y, kp.ymap);
-  const KernelEntry ke = kernel_for(cfg, tma_ops);
+  KernelEntry ke = kernel_for(cfg, tma_ops);
+  if (plan->out_f32) {   // BF16 operands, FP32 C
+    ke.fn = kernel_ptr_umma_f32out(cfg.variant, cfg.xKmajor, cfg.yKmajor, &ke.smem, &ke.threads);
+    ke.smem_tma = ke.smem;
+    if (!ke.fn) return fail(ST_UNSUPPORTED, "no FP32-output instance for the variant");
+  }
   const int grid = (int)std::min<int64_t>(cfg.nctas, plan->sms);
   if (tma_ops && plan->pair) {   // clusters of two CTAs over 2 x 2 tile blocks (persistent)
     size_t sm = 0;
@@ -868,7 +909,7 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
       }
       kp.X = X0 + es * ox;
       kp.Y = Y0 + es * oy;
-      kp.C = C0 + es * oc;
+      kp.C = C0 + elem_bytes_c(plan) * oc;
     }
     cudaError_t e = cudaLaunchKernel(ke.fn, dim3(grid), dim3(ke.threads), args,
                                      kp.use_tma ? ke.smem_tma : ke.smem, (cudaStream_t)stream);
@@ -912,7 +953,7 @@ size_t tc_plan_workspace_bytes(const tc_plan_t plan) {
   auto al = [](size_t x) { return (x + 255) & ~(size_t)255; };
   const Contraction &c = plan->parsed;
   const size_t es = elem_bytes(plan);
-  return al(es * c.parent_numel[1]) + al(es * c.parent_numel[2]) + al(es * c.parent_numel[0]);
+  return al(es * c.parent_numel[1]) + al(es * c.parent_numel[2]) + al(elem_bytes_c(plan) * c.parent_numel[0]);
 }
 
 tc_status_t tc_execute_host(const tc_plan_t plan, const void *A_host, const void *B_host, void *C_host,
@@ -923,7 +964,7 @@ tc_status_t tc_execute_host(const tc_plan_t plan, const void *A_host, const void
   auto al = [](size_t x) { return (x + 255) & ~(size_t)255; };
   const Contraction &c = plan->parsed;
   const size_t es = elem_bytes(plan);
-  const size_t bA = es * c.parent_numel[1], bB = es * c.parent_numel[2], bC = es * c.parent_numel[0];
+  const size_t bA = es * c.parent_numel[1], bB = es * c.parent_numel[2], bC = elem_bytes_c(plan) * c.parent_numel[0];
   char *w = (char *)workspace;
   void *dA = w, *dB = w + al(bA), *dC = w + al(bA) + al(bB);
   cudaStream_t s = (cudaStream_t)stream;
@@ -979,6 +1020,7 @@ tc_status_t tc_plan_info(const tc_plan_t plan, char *json, size_t cap, size_t *n
     o << ",\"vecX\":" << g.vecX << ",\"vecY\":" << g.vecY << ",\"vecC\":" << plan->cvec << ",\"cs0\":" << plan->kp.cs0 << ",\"xKmajor\":" << g.xKmajor
       << ",\"yKmajor\":" << g.yKmajor << ",\"tma_operands\":" << (plan->umma_tma ? 1 : 0)
       << ",\"cta_pair\":" << (plan->pair ? 1 : 0) << ",\"resized\":" << (plan->resized ? 1 : 0)
+      << ",\"out_f32\":" << (plan->out_f32 ? 1 : 0)
       << ",\"wfX\":" << g.wfX << ",\"wfY\":" << g.wfY;
     char buf[512];
     std::snprintf(buf, sizeof buf,

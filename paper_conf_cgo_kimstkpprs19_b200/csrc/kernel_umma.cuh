@@ -431,10 +431,13 @@ __device__ __forceinline__ void load_coord(const TileInfo *t, int32_t (&c)[kMaxT
 // buffer).  Per k-step each CTA then loads half the operand bytes per MMA of the single-CTA
 // kernel (the L2 -> SM traffic that bounds BF16 GEMM-like plans).  A block past the tile grid
 // reads the tables' padding entry (coordinates out of the tensor: TMA zero-fills; masks 0).
-template <int KIND, int BN, int STAGES, bool XK, bool YK, bool TMA = false, bool PAIR = false>
+// OUTF32 (BF16 operands only): C is FP32 — the accumulator is stored without the BF16
+// rounding (split-K partials that are summed before the final rounding, dist.py).
+template <int KIND, int BN, int STAGES, bool XK, bool YK, bool TMA = false, bool PAIR = false, bool OUTF32 = false>
 __global__ void __launch_bounds__(UmmaKernel<KIND, BN, STAGES>::THREADS, 1)
 tc_umma_kernel(const __grid_constant__ KParams p) {
   using K = UmmaKernel<KIND, BN, STAGES>;
+  using TC = typename std::conditional<OUTF32, float, typename K::T>::type;   // C's element type
   static_assert(!PAIR || (TMA && !K::SPLIT), "CTA pairs take TMA operands, BF16 / TF32");
   constexpr int ACCW = PAIR ? 2 * BN : BN;            // accumulator columns per tile (unit)
   constexpr int NBUF = 512 / ACCW;                    // accumulators in flight
@@ -730,7 +733,7 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
     // ======================= epilogue =====================================================
     // warp w drains TMEM lane quarter w % 4 (tile rows 32(w%4) .. +31; one row per thread)
     // and column half w / 4; FP32 arithmetic on the FP32 accumulator, stored as T (BF16: RNE)
-    T *__restrict__ C = static_cast<T *>(p.C);
+    TC *__restrict__ C = static_cast<TC *>(p.C);
     const float alpha = (float)p.alpha, beta = (float)p.beta;
     const int quarter = warp & 3, half = warp >> 2;
     const int row = quarter * 32 + lane;               // TMEM lane = tile row m
@@ -804,9 +807,9 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
       const int64_t coff = mc + coffs[q];
       const uint64_t cm0 = cm0s[q], cm1 = cm1s[q];
       const uint32_t cb = (uint32_t)(buf * ACCW + q * BN);   // this tile's TMEM columns
-      T *Crow = C + (coff + roff);
+      TC *Crow = C + (coff + roff);
       const bool cfull = cm0 == p.fullN[0] && cm1 == p.fullN[1];
-      T *Cg = C + (coff + goff);
+      TC *Cg = C + (coff + goff);
 #if defined(TC_UMMA_ABLATE) && TC_UMMA_ABLATE == 1
       if (true) {   // (ablation side build: the epilogue drains nothing)
 #else
@@ -820,7 +823,7 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
         // ([column][row] FP32), then each thread stores whole runs: 16-B (BF16) / 2 x 16-B
         // (FP32) stores along C's FVI, whatever the m digit order (the X loads keep theirs).
         const bool rrok = ((rr < 64 ? rm0 : rm1) >> (rr & 63)) & 1;
-        T *Cr = C + (coff + rroff);
+        TC *Cr = C + (coff + rroff);
         for (int pc = 0; pc < BN && pc < p.Nt; pc += 64) {
           uint32_t v[32];
           tc05_ld<32>(tmem + ((uint32_t)(quarter * 32) << 16) + cb + (uint32_t)(pc + half * 32), v);
@@ -872,7 +875,7 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
             if (ok[i]) {
               float r[8] = {alpha * d[i][0].x, alpha * d[i][0].y, alpha * d[i][0].z, alpha * d[i][0].w,
                             alpha * d[i][1].x, alpha * d[i][1].y, alpha * d[i][1].z, alpha * d[i][1].w};
-              if constexpr (ES == 4) {
+              if constexpr (sizeof(TC) == 4) {
                 float4 *dst = reinterpret_cast<float4 *>(Cg + rc[i]);
                 if (beta != 0.0f) {
                   const float4 o0 = dst[0], o1 = dst[1];
@@ -916,7 +919,7 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
             for (int q = 0; q < W; q++) {
               const int c = half * HC + c0 + q;
               if (((c < 64 ? cm0 : cm1) >> (c & 63)) & 1) {
-                T *dst = Crow + relCn[c];
+                TC *dst = Crow + relCn[c];
                 float r = alpha * __uint_as_float(v[q]);
                 if (beta != 0.0f) r = fmaf(beta, ld_out(dst), r);
                 st_out(dst, r);

@@ -37,7 +37,8 @@ struct tc_plan_s {
   bool umma_tma = false;
   std::string expr;        // the expression as given (tc_plan / tc_plan_ex): resizable plans
   bool resized = false;    // the configuration came from a representative-size plan (NEXT-1)
-  bool pair = false;       // tcgen05: launch the CTA-pair instance (clusters of 2) with TMA operands
+  bool pair = false;
+  bool out_f32 = false;    // BF16 operands, FP32 C (kernels_umma_f32out.cu)       // tcgen05: launch the CTA-pair instance (clusters of 2) with TMA operands
   OperandMap mapX, mapY;
   // batch (Hadamard) indices (R31): extent and element strides in X, Y, C.  tc_execute
   // launches the kernel once per batch slab with the operands offset to it — the kernels

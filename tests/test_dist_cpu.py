@@ -61,7 +61,26 @@ def _worker(rank, world, port, expr, extents, mode, q):
         A.copy_(torch.as_tensor(tcinputs.integers_np(A.numel(), 1)))
         B.copy_(torch.as_tensor(tcinputs.integers_np(B.numel(), 2)))
     try:
-        if mode == "slab":
+        if mode == "scatter":
+            # the shard index is A's slowest index: rank 0 scatters A's slabs, broadcasts B
+            sh = tcdist.shard_plan(plan, expr, extents, world, rank)
+            assert sh.x_tensor == "A" and sh.plan is not None and sh.plan.info()["host_only"]
+            nA = tcinputs.numel(a, ext)
+            Aloc = A if rank == 0 else torch.zeros(tcdist.local_input_numel(sh, "A", nA, rank),
+                                                   dtype=torch.float64)
+            Cs = torch.zeros(sh.c_numel, dtype=torch.float64)
+
+            def ex(p, AA, BB, CC):
+                # AA is this rank's compact slab of A; the sub-problem is dense in it
+                assert AA.numel() == sh.x_slabs[rank][1]
+                sub = dict(ext)
+                sub[sh.index] = sh.length
+                es = ";".join(f"{k}:{v}" for k, v in sub.items())
+                CC.copy_(torch.as_tensor(oracle.contract(expr, es, np.ascontiguousarray(AA.numpy()), BB.numpy())))
+            tcdist.execute_sharded(sh, Aloc, B, Cs, execute=ex, rank=rank)
+            out = [None] * world
+            dist.all_gather_object(out, (sh.index, sh.lo, sh.length, Cs.numpy()))
+        elif mode == "slab":
             sh = tcdist.shard_plan(plan, expr, extents, world, rank)
             Cs = torch.zeros(sh.c_numel, dtype=torch.float64)
 
@@ -165,3 +184,25 @@ def test_split_k_reduce_scatter_gloo():
     B = tcinputs.integers_np(77, 2)
     full = oracle.contract(expr, extents, A, B)
     assert np.array_equal(np.concatenate(out), full)
+
+
+def test_c_slab_scatter_gloo():
+    """The shard index c is A's slowest index: A travels as per-rank slabs (point-to-point),
+    B by broadcast; the gathered slabs equal the oracle's C."""
+    expr, extents = "abc-adc-db", "a:3;b:4;c:9;d:5"
+    assert tcdist.input_slabs(expr, extents, 2, "c") == ("A", [(0, 75), (75, 60)])
+    out = _run(expr, extents, "scatter")
+    ext = tcinputs.parse_extents(extents)
+    c, a, b = tcinputs.split_expr(expr)
+    A = tcinputs.integers_np(tcinputs.numel(a, ext), 1)
+    B = tcinputs.integers_np(tcinputs.numel(b, ext), 2)
+    full = oracle.contract(expr, extents, A, B)
+    pieces = [np.asarray(x[3]).reshape([ext[i] if i != "c" else x[2] for i in reversed(c)]) for x in out]
+    assert np.array_equal(np.concatenate(pieces, axis=0), _nd(full, c, ext))
+
+
+def test_partial_numel_padding():
+    for n in (1, 7, 64, 1000):
+        for w in (1, 2, 3, 8):
+            m = tcdist.partial_numel(n, w)
+            assert m % w == 0 and n <= m < n + w
