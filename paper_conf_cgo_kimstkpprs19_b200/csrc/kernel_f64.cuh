@@ -506,9 +506,29 @@ tc_f64_dmma_kernel(const __grid_constant__ KParams p) {
   // columns per k4 step so that a parked tile is drained within one k-step of the next tile
   constexpr int KQ = BK / 4;
   constexpr int DQ = ((WN + KQ - 1) / KQ + 1) / 2 * 2;
+  // [STG, beta != 0] the old C of the tile being computed is fetched by cp.async into the
+  // warp's staging tile as soon as the previous parked tile has drained (lane l: row l of the
+  // warp tile, all WN columns; zero-filled outside C), and combined at park time
+  // (alpha * acc + beta * old, from smem): the drain then only stores, and the old C's
+  // latency hides behind the rest of the tile's DMMAs instead of stalling each drain step
+  const bool pfc = STG && beta != 0.0;
+  bool pf_issued = false, combined = false;
+  auto oldc_fetch = [&](int64_t coff, const uint64_t (&tm)[kMaskWords], const uint64_t (&tn)[kMaskWords]) {
+    const int r = wm * WM + lane;
+    const bool rok = bit_of(tm, r);
+    const double *src = C + coff + relCm[r];
+    const uint32_t d0 = (uint32_t)__cvta_generic_to_shared(stg) + 8u * (uint32_t)lane;
+#pragma unroll 1
+    for (int c = 0; c < WN; c++) {
+      const int cidx = wn * WN + c;
+      const bool ok = rok && bit_of(tn, cidx);
+      cp_async8(d0 + 8u * (uint32_t)(c * K::SP), ok ? src + relCn[cidx] : C, ok ? 8 : 0);
+    }
+  };
   auto drain = [&](int c0) {
-    if (vc) drain_cols<WN, K::SP, DQ, true>(stg, c0, lane, dCr, drok, relCn, wn * WN, dmn, alpha, beta, plain);
-    else drain_cols<WN, K::SP, DQ, false>(stg, c0, lane, dCr, drok, relCn, wn * WN, dmn, alpha, beta, plain);
+    const bool pl = plain || combined;
+    if (vc) drain_cols<WN, K::SP, DQ, true>(stg, c0, lane, dCr, drok, relCn, wn * WN, dmn, alpha, beta, pl);
+    else drain_cols<WN, K::SP, DQ, false>(stg, c0, lane, dCr, drok, relCn, wn * WN, dmn, alpha, beta, pl);
   };
   // TMA epilogue: box offsets of tile-local rows / columns come from smem tables
   const bool use_tma = p.use_tma && beta == 0.0;
@@ -548,9 +568,19 @@ tc_f64_dmma_kernel(const __grid_constant__ KParams p) {
 #pragma unroll
         for (int jj = 0; jj < NJ; jj++) dmma884(acc[i][jj][0], acc[i][jj][1], a[i], b[jj]);
       // [STG] a few columns of the parked tile per k4 step, in the shadow of the DMMAs
+      // (twice as many with beta != 0, so the old-C fetch of this tile starts early)
       if (STG && pend && dcol < WN) {
         drain(dcol);
         dcol += DQ;
+        if (pfc && dcol < WN) {
+          drain(dcol);
+          dcol += DQ;
+        }
+      }
+      if (pfc && !pf_issued && (!pend || dcol >= WN)) {
+        __syncwarp();   // every lane's drain reads of the staging tile are done
+        oldc_fetch(cm + cn, mm, mn);
+        pf_issued = true;
       }
     }
     __syncwarp();
@@ -567,6 +597,11 @@ tc_f64_dmma_kernel(const __grid_constant__ KParams p) {
         if (pend) {
           for (; dcol < WN; dcol += DQ) drain(dcol);
         }
+        if (pfc && !pf_issued) {   // (a tile too short to fetch its old C ahead)
+          __syncwarp();
+          oldc_fetch(cm + cn, mm, mn);
+        }
+        if (pfc) asm volatile("cp.async.wait_all;\n" ::: "memory");
         __syncwarp();
 #pragma unroll
         for (int jj = 0; jj < NJ; jj++)
@@ -574,9 +609,11 @@ tc_f64_dmma_kernel(const __grid_constant__ KParams p) {
           for (int h = 0; h < 2; h++) {
             double *col = stg + (jj * 8 + 2 * t + h) * K::SP + g;
 #pragma unroll
-            for (int i = 0; i < MI; i++) col[i * 8] = acc[i][jj][h];
+            for (int i = 0; i < MI; i++) col[i * 8] = pfc ? fma(beta, col[i * 8], alpha * acc[i][jj][h]) : acc[i][jj][h];
           }
         __syncwarp();
+        combined = pfc;
+        pf_issued = false;
         dCr = Ct + droff;
         drok = bit_of(mm, drow);
         dmn[0] = mn[0];
