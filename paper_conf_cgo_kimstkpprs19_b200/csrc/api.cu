@@ -135,7 +135,8 @@ void build_host_tables(tc_plan_s *P) {
   // CTA pairs: BN = 128 BF16 / TF32 instances with TMA operands, when asked for (cta_pair 2)
   // or (planner's choice) when the grid holds at least two waves of pair blocks
   {
-    const bool can = P->umma_tma && (cfg.variant == 12 || cfg.variant == 22);
+    // (the pair epilogue stores from TMEM rows: C's FVI must lead m when the plan stores runs)
+    const bool can = P->umma_tma && (cfg.variant == 12 || cfg.variant == 22) && (P->cvec != 8 || cs0 == 1);
     P->pair = can && (P->opts.cta_pair == 2 || (P->opts.cta_pair == 0 && cta_pair_default(cfg)));
   }
   P->pf_step = 0;

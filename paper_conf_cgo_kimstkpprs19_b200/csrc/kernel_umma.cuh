@@ -295,7 +295,9 @@ __device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint
 // KIND (tiles.hpp): 1 = BF16 (kind::f16), 2 = TF32 on FP32 storage (kind::tf32),
 // 3 = FP32 as split TF32: SW split warps rewrite each landed stage as hi = tf32 truncation
 // (in place) and lo = x - hi (a second plane), and the MMA warp issues hi*hi + hi*lo + lo*hi.
-template <int KIND, int BN, int STAGES>
+// STAGED = false (CTA-pair instances): no per-epilogue-warp FP32 staging in smem — the
+// epilogue stores straight from TMEM rows (C's FVI leads m), which buys a sixth stage.
+template <int KIND, int BN, int STAGES, bool STAGED = true>
 struct UmmaKernel {
   using T = typename std::conditional<KIND == 1, __nv_bfloat16, float>::type;
   static constexpr int ES = KIND == 1 ? 2 : 4;       // element bytes
@@ -317,7 +319,7 @@ struct UmmaKernel {
   static constexpr int TMEM_COLS = NBUF * BN;
   static constexpr size_t smem_bytes() {
     return 1024 + (size_t)ES * PLANES * STAGES * (XS + YS) + 8 * (3 * STAGES + 2 * NBUF) + 16 +
-           8 * (size_t)(BM + BN) + 16 + 4 * (size_t)EW * 32 * 32;   // + per-epilogue-warp FP32 staging (32 x 32)
+           8 * (size_t)(BM + BN) + 16 + (STAGED ? 4 * (size_t)EW * 32 * 32 : 0);   // + per-epilogue-warp FP32 staging (32 x 32)
   }
   // register-cached slots per producer thread (16-B vectors)
   static constexpr int EX = (BM * BK * ES / 16 + PW * 32 - 1) / (PW * 32);
@@ -434,9 +436,9 @@ __device__ __forceinline__ void load_coord(const TileInfo *t, int32_t (&c)[kMaxT
 // OUTF32 (BF16 operands only): C is FP32 — the accumulator is stored without the BF16
 // rounding (split-K partials that are summed before the final rounding, dist.py).
 template <int KIND, int BN, int STAGES, bool XK, bool YK, bool TMA = false, bool PAIR = false, bool OUTF32 = false>
-__global__ void __launch_bounds__(UmmaKernel<KIND, BN, STAGES>::THREADS, 1)
+__global__ void __launch_bounds__(UmmaKernel<KIND, BN, STAGES, !PAIR>::THREADS, 1)
 tc_umma_kernel(const __grid_constant__ KParams p) {
-  using K = UmmaKernel<KIND, BN, STAGES>;
+  using K = UmmaKernel<KIND, BN, STAGES, !PAIR>;
   using TC = typename std::conditional<OUTF32, float, typename K::T>::type;   // C's element type
   static_assert(!PAIR || (TMA && !K::SPLIT), "CTA pairs take TMA operands, BF16 / TF32");
   constexpr int ACCW = PAIR ? 2 * BN : BN;            // accumulator columns per tile (unit)
@@ -456,7 +458,7 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
   // [EW][32 columns][32 rows] FP32 epilogue staging right after the planes (1 KB aligned),
   // then the barriers and tables
   float *stage = reinterpret_cast<float *>(smem_raw + (size_t)LO * K::PLANES);
-  uint64_t *bars = reinterpret_cast<uint64_t *>(stage + K::EW * 32 * 32);
+  uint64_t *bars = reinterpret_cast<uint64_t *>(stage + (PAIR ? 0 : K::EW * 32 * 32));
   uint32_t *tmem_holder = reinterpret_cast<uint32_t *>(bars + 3 * STAGES + 2 * K::NBUF);
   int64_t *relCm = reinterpret_cast<int64_t *>(tmem_holder + 4);
   int64_t *relCn = relCm + BM;
@@ -816,7 +818,7 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
       if (kTrace) {
 #endif
         if (warp == 0 && lane == 0) trace_at(p, 4, lt);
-      } else if (p.vecC == 8 && p.cs0 > 1) {
+      } else if (!PAIR && p.vecC == 8 && p.cs0 > 1) {
         // CTA-wide staged epilogue: C's FVI is an inner m digit (tile-row stride cs0), so the
         // 8 C-contiguous elements of a run live in rows r, r + cs0, ..., r + 7 cs0 of
         // different warps.  Per 64-column pass all eight warps park their TMEM rows in smem
@@ -851,7 +853,7 @@ tc_umma_kernel(const __grid_constant__ KParams p) {
         if (half * HC + c0 >= p.Nt) break;             // columns past the tile's Nt: padding
         uint32_t v[W];
         tc05_ld<W>(tmem + ((uint32_t)(quarter * 32) << 16) + cb + (uint32_t)(half * HC + c0), v);
-        if (p.vecC == 8) {
+        if (!PAIR && p.vecC == 8) {
           // FP32 accumulators to smem as [column][row], then one 16-B store per 8 rows
           // (C's FVI leads m with an 8-multiple tile: 8 tile rows are 8 C-contiguous elements)
 #pragma unroll

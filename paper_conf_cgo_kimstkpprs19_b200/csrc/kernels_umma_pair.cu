@@ -7,8 +7,8 @@ namespace tc {
 
 template <int KIND, int BN, int ST>
 static const void *pick_pair(bool xk, bool yk, size_t *smem, int *threads) {
-  *smem = UmmaKernel<KIND, BN, ST>::smem_bytes();
-  *threads = UmmaKernel<KIND, BN, ST>::THREADS;
+  *smem = UmmaKernel<KIND, BN, ST, false>::smem_bytes();
+  *threads = UmmaKernel<KIND, BN, ST, false>::THREADS;
   return xk ? (yk ? (const void *)&tc_umma_kernel<KIND, BN, ST, true, true, true, true>
                   : (const void *)&tc_umma_kernel<KIND, BN, ST, true, false, true, true>)
             : (yk ? (const void *)&tc_umma_kernel<KIND, BN, ST, false, true, true, true>
@@ -17,8 +17,8 @@ static const void *pick_pair(bool xk, bool yk, size_t *smem, int *threads) {
 
 const void *kernel_ptr_umma_pair(int v, bool xk, bool yk, size_t *smem, int *threads) {
   switch (v) {
-    case 12: return pick_pair<1, 128, 5>(xk, yk, smem, threads);
-    case 22: return pick_pair<2, 128, 5>(xk, yk, smem, threads);
+    case 12: return pick_pair<1, 128, 6>(xk, yk, smem, threads);   // (no epilogue staging: 6 stages)
+    case 22: return pick_pair<2, 128, 6>(xk, yk, smem, threads);
   }
   *smem = 0;
   *threads = 0;

@@ -99,7 +99,11 @@ double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *
     return std::pair<double, double>{std::ceil(b / 128.0), std::ceil(b / 32.0)};
   };
   // CTA pairs: each CTA loads one X and one Y box per k-step for two tiles of work
-  const bool pair = tma && cta_pair_default(cfg);
+  bool pair = tma && cta_pair_default(cfg);
+  if (pair) {   // (as api.cu: the pair epilogue needs C's FVI leading m when it stores runs)
+    int s0 = 1, t0 = 1;
+    pair = c_run_rows(c, cfg, 8, &s0, &t0) != 8 || s0 == 1;
+  }
   const auto sx = tma ? boxes(ox) : lower_bound ? ideal(cfg.Mt) : operand_sim(c, cfg, cfg.X, cfg.vecX, cfg.xKmajor, v.BM, v.BK, cache);
   const auto sy = tma ? boxes(oy) : lower_bound ? ideal(cfg.Nt) : operand_sim(c, cfg, cfg.Y, cfg.vecY, cfg.yKmajor, v.BN, v.BK, cache);
   cfg.wfX = sx.first;

@@ -356,3 +356,16 @@ def test_large_index_splitting_and_fusion_cap():
     with pytest.raises(tc.TcError) as e:
         tc.plan("ab-a-b", "a:2147483659;b:2", host_only=True)   # a prime past 2^31
     assert e.value.status == "TC_ERR_UNSUPPORTED"
+
+
+def test_cta_pair_needs_c_fvi_leading_m():
+    """CTA-pair instances store straight from TMEM rows (no epilogue staging, a sixth stage):
+    a plan whose C runs need the CTA-wide staged pass (C's FVI an inner m digit) stays
+    single-CTA even when pairs are asked for; the GEMM-like layout pairs."""
+    from paper_conf_cgo_kimstkpprs19_b200 import binding as tc
+    i = tc.plan("abcd-ebad-ce", "a:32;b:4;c:128;d:8;e:64", dtype="bf16", force_tiles="b:2;a:16;d:4;c:128;e:64",
+                morder="X", pair=True, host_only=True).info()
+    assert i["tma_operands"] == 1 and i["vecC"] == 8 and i["cs0"] > 1 and i["cta_pair"] == 0
+    j = tc.plan("ab-ac-cb", "a:392;b:264;c:136", dtype="bf16", force_tiles="a:128;b:128;c:64", pair=True,
+                host_only=True).info()
+    assert j["cs0"] == 1 and j["cta_pair"] == 1

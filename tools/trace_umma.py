@@ -4,8 +4,11 @@ usage: python tools/trace_umma.py <case> <dtype>"""
 import os
 import sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+# (the side library must be chosen before the package — and its binding — is imported)
+_so = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "paper_conf_cgo_kimstkpprs19_b200",
+                   "build", "trace", "libtc.so")
+os.environ["LIBTC_SO"] = _so
 from paper_conf_cgo_kimstkpprs19_b200 import build as _b  # noqa: E402
-_so = os.path.join(_b.HERE, "build", "trace", "libtc.so")
 if not os.path.exists(_so):
     _b.NVCC_FLAGS = _b.NVCC_FLAGS + ["-DTC_TRACE"]
     _b.SO = _so
