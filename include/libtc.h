@@ -72,7 +72,13 @@ typedef struct tc_plan_opts {
                         2 always — CTA pairs (cluster of 2, M = 256 MMAs over 2 x 2 tiles)   */
   int out_f32;       /* TC_BF16 plans: 1 = C is FP32 (the accumulator without the BF16 rounding;
                         split-K partials); TC_ERR_INVALID_ARG for other dtypes */
-  int reserved[3];   /* must be zero (TC_ERR_INVALID_ARG otherwise)                         */
+  int stream;        /* streaming path for low-intensity tensor x matrix contractions (TC_BF16,
+                        one internal and one <= 32 Y-side external index, Y in shared memory,
+                        TMA boxes for X and C): 0 planner's choice (on when
+                        eligible and no variant is forced), 1 never, 2 whenever eligible.  The
+                        plan keeps its tcgen05 configuration for beta != 0 and unaligned
+                        pointers.                                                            */
+  int reserved[2];   /* must be zero (TC_ERR_INVALID_ARG otherwise)                         */
 } tc_plan_opts;
 
 /*

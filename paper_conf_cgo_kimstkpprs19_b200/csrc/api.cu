@@ -178,6 +178,7 @@ Status upload(tc_plan_s *P, std::string &err) {
   size_t iX2p = add(P->slotX2.pack.data(), 4 * P->slotX2.pack.size());
   size_t iY2 = add(r32[3].data(), 4 * r32[3].size());
   size_t iY2p = add(P->slotY2.pack.data(), 4 * P->slotY2.pack.size());
+  size_t iS = add(P->stream.tab.data(), 4 * P->stream.tab.size());
   std::vector<char> h(o + 256, 0);
   for (auto &p : parts) if (p.bytes) std::memcpy(h.data() + p.off, p.src, p.bytes);
   cudaError_t e = cudaMalloc(&P->dev, h.size());
@@ -202,6 +203,19 @@ Status upload(tc_plan_s *P, std::string &err) {
   P->d_packX2 = (const uint32_t *)(b + parts[iX2p].off);
   P->d_relY2 = (const int32_t *)(b + parts[iY2].off);
   P->d_packY2 = (const uint32_t *)(b + parts[iY2p].off);
+  if (P->stream.on) {
+    P->stream.kp.tab = (const uint32_t *)(b + parts[iS].off);
+    const void *fn = stream_kernel_ptr(P->stream.NB, P->stream.AR, P->stream.mode != SM_K);
+    if (!fn) { err = "no streaming kernel instance for the plan"; return ST_UNSUPPORTED; }
+    // (the instance is shared by plans of different sizes: always the opt-in maximum)
+    e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448);
+    if (e != cudaSuccess) { err = std::string("cudaFuncSetAttribute: ") + cudaGetErrorString(e); return ST_CUDA; }
+    int socc = 0, nsm = 148;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&socc, fn, kSThreads, P->stream.smem);
+    if (e != cudaSuccess || socc < 1) { err = "streaming kernel cannot be resident"; return ST_CUDA; }
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, P->device);
+    P->stream_grid = nsm * std::min(socc, P->stream.occ);
+  }
   if (P->umma_tma) {   // the TMA-operand instance: same smem, its own attribute
     const KernelEntry kt = kernel_for(P->cfg, true);
     e = cudaFuncSetAttribute(kt.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kt.smem);
@@ -286,6 +300,7 @@ tc_status_t finish_plan(tc_plan_s *P, tc_plan_t *out, const tc_plan_s *rep = nul
   if (P->opts.out_f32 != 0 && (P->opts.out_f32 != 1 || P->dtype != TC_BF16))
     { delete P; return fail(ST_INVALID_ARG, "out_f32 is a TC_BF16 option (0 or 1)"); }
   P->out_f32 = P->opts.out_f32 == 1;
+  if (P->opts.stream < 0 || P->opts.stream > 2) { delete P; return fail(ST_INVALID_ARG, "stream must be 0, 1 or 2"); }
   for (int r : P->opts.reserved)
     if (r != 0) { delete P; return fail(ST_INVALID_ARG, "tc_plan_opts.reserved[] must be zero"); }
   ft.morder = P->opts.morder - 1;
@@ -323,6 +338,16 @@ tc_status_t finish_plan(tc_plan_s *P, tc_plan_t *out, const tc_plan_s *rep = nul
   if (s != ST_OK) s = choose(P->c, kind, P->opts.cost_mode, fv, ft, P->cfg, P->stats, err);
   if (s != ST_OK) { delete P; return fail(s, err); }
   build_host_tables(P);
+  // the streaming path (stream.hpp) beside the configuration: on when eligible, unless the
+  // caller forced a variant (tests, tuning candidates) or opts.stream says otherwise
+  P->stream = StreamCfg();
+  if (P->opts.stream != 1 && !P->out_f32 && (fv < 0 || P->opts.stream == 2) && !ft.on) {
+    StreamCfg sc;
+    if (stream_plan(P->c, kind, 148, sc)) P->stream = sc;
+    else P->stream.why = sc.why;
+  } else {
+    P->stream.why = "off (options)";
+  }
   if (!P->host_only) {
     if (cudaGetDevice(&P->device) != cudaSuccess) {
       cudaGetLastError();
@@ -411,6 +436,33 @@ bool encode_c_map(const tc_plan_s *P, void *C, TmaDesc &out) {
                    CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE,
                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return e == CUDA_SUCCESS;
+}
+
+// The streaming path's X tensor map at this call's pointer (stream.hpp): X boxes in X's order,
+// zero fill outside the tensor.  C must be aligned for the AR-element run stores.
+bool encode_stream_maps(const tc_plan_s *P, const void *Xp, void *C, SParams &sp) {
+  auto enc = tma_encoder();
+  if (!enc) return false;
+  const StreamCfg &s = P->stream;
+  const char *xb = (const char *)Xp + 2 * s.xbase;
+  const char *cb = (const char *)C + 2 * s.cbase;
+  if ((uintptr_t)xb % 16 || (uintptr_t)cb % (2 * s.AR)) return false;
+  cuuint64_t dims[kMaxTmaDims], strides[kMaxTmaDims];
+  cuuint32_t box[kMaxTmaDims], el[kMaxTmaDims];
+  for (int j = 0; j < s.xrank; j++) {
+    dims[j] = (cuuint64_t)s.xdims[j];
+    box[j] = s.xbox[j];
+    el[j] = 1;
+    if (j > 0) strides[j - 1] = (cuuint64_t)(s.xstr[j] * 2);
+  }
+  return enc(reinterpret_cast<CUtensorMap *>(&sp.xmap), CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, (cuuint32_t)s.xrank,
+             (void *)xb, dims, strides, box, el, CU_TENSOR_MAP_INTERLEAVE_NONE, (CUtensorMapSwizzle)s.xswz,
+#ifdef TC_STREAM_PROMO
+             (CUtensorMapL2promotion)TC_STREAM_PROMO,
+#else
+             CU_TENSOR_MAP_L2_PROMOTION_NONE,
+#endif
+             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
 }  // namespace
@@ -700,6 +752,8 @@ tc_status_t tc_plan_tuned(tc_plan_t *tuned, const tc_plan_t plan, const void *A,
   return tc_plan_tuned_beta(tuned, plan, A, B, C, topk, reps, 0.0, stream);
 }
 
+constexpr int kTunedStream = 99;   // tc_plan_tuned's log entry of the streaming path
+
 tc_status_t tc_plan_tuned_beta(tc_plan_t *tuned, const tc_plan_t plan, const void *A, const void *B, void *C,
                                int topk, int reps, double beta, tc_stream_t stream) {
   if (!tuned || !plan || !A || !B || !C) return fail(ST_INVALID_ARG, "NULL argument");
@@ -724,12 +778,15 @@ tc_status_t tc_plan_tuned_beta(tc_plan_t *tuned, const tc_plan_t plan, const voi
     float best_ms = 0;
     std::vector<std::pair<int, double>> log;
     tc_status_t rc = TC_SUCCESS;
+    // the streaming path (stream.hpp) competes as candidate 99 when the plan has it and beta == 0
+    if (plan->stream.on && beta == 0.0) cand.push_back(kTunedStream);
     for (int v : cand) {
       tc_plan_s *P = new tc_plan_s();
       P->opts = plan->opts;
       P->force_tiles = plan->force_tiles;
       P->opts.force_tiles = plan->opts.force_tiles ? P->force_tiles.c_str() : nullptr;
-      P->opts.variant = v + 1;
+      P->opts.variant = (v == kTunedStream ? plan->cfg.variant : v) + 1;
+      P->opts.stream = v == kTunedStream ? 2 : 1;
       P->dtype = plan->dtype;
       P->parsed = plan->parsed;
       tc_plan_t cp = nullptr;
@@ -834,6 +891,22 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
   const tc_status_t chk = check_execute(plan, A, B, C);
   if (chk != TC_SUCCESS) return chk;
   const size_t es = elem_bytes(plan);
+  if (plan->stream.on && beta == 0.0 && plan->batch.empty()) {
+    // the streaming path (beta == 0: C is only written; otherwise the configuration below)
+    SParams sp = plan->stream.kp;
+    const void *Xp = plan->stream.X == 1 ? A : B, *Yp = plan->stream.X == 1 ? B : A;
+    if (encode_stream_maps(plan, Xp, C, sp)) {
+      sp.Y = static_cast<const char *>(Yp) + 2 * plan->stream.ybase;
+      sp.C = static_cast<char *>(C) + 2 * plan->stream.cbase;
+      sp.alpha = (float)alpha;
+      const void *fn = stream_kernel_ptr(plan->stream.NB, plan->stream.AR, plan->stream.mode != SM_K);
+      const int grid = std::min(sp.ntiles, plan->stream_grid);
+      void *sargs[] = {&sp};
+      cudaError_t e = cudaLaunchKernel(fn, dim3(grid), dim3(kSThreads), sargs, plan->stream.smem, (cudaStream_t)stream);
+      if (e != cudaSuccess) return fail(ST_CUDA, std::string("launch (stream): ") + cudaGetErrorString(e));
+      return TC_SUCCESS;
+    }
+  }
   KParams kp = plan->kp;
   const Config &cfg = plan->cfg;
   kp.X = cfg.X == 1 ? A : B;
@@ -1041,6 +1114,21 @@ tc_status_t tc_plan_info(const tc_plan_t plan, char *json, size_t cap, size_t *n
     for (size_t q = 0; q < plan->tuned.size(); q++)
       o << (q ? "," : "") << "[" << plan->tuned[q].first << "," << plan->tuned[q].second << "]";
     o << "]}";
+    {   // the streaming path (stream.hpp)
+      const StreamCfg &st = plan->stream;
+      const SParams &k = st.kp;
+      o << ",\"stream\":{\"on\":" << (st.on ? 1 : 0) << ",\"why\":\"" << st.why << "\"";
+      if (st.on) {
+        o << ",\"mode\":\"" << (st.mode == SM_K ? "K" : "T") << "\",\"X\":\"" << (st.X == 1 ? "A" : "B") << "\",\"tiles\":{";
+        for (size_t i = 0; i < c.ix.size(); i++) o << (i ? "," : "") << "\"" << c.ix[i].name << "\":" << st.T[i];
+        o << "},\"KB\":" << k.KB << ",\"nks\":" << k.nks << ",\"stages\":" << k.stages
+          << ",\"stage_bytes\":" << k.stage_bytes << ",\"ntiles\":" << k.ntiles << ",\"units\":" << k.nunits
+          << ",\"NB\":" << st.NB << ",\"AR\":" << st.AR << ",\"occ\":" << st.occ << ",\"xswz\":" << st.xswz << ",\"smem\":" << st.smem
+          << ",\"grid\":" << plan->stream_grid
+          << ",\"t_pred_ms\":" << st.t_pred * 1e3 << ",\"bytes\":" << st.bytes;
+      }
+      o << "}";
+    }
     o << ",\"host_only\":" << (plan->host_only ? "true" : "false") << "}";
     std::string s = o.str();
     if (needed) *needed = s.size() + 1;

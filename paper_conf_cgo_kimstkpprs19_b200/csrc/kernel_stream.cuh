@@ -1,0 +1,290 @@
+// kernel_stream.cuh — the streaming BF16 contraction kernel (stream.hpp) for low-intensity
+// tensor x matrix contractions (TCCG #1-8), sm_100a.
+//
+// The paper's four steps:
+//   (1) one producer thread streams X boxes (X's own index order; one box per
+//       (tile, k-step), zero-filled outside the tensor) into a STAGES-deep ring;
+//   (2)+(3) each compute warp owns one unit of the tile — AR consecutive values a0.. of C's FVI
+//       times 16 rows — and runs, per k16 step, AR mma.sync m16n8k16 BF16 -> FP32 blocks (one
+//       per a value) with A fragments from the ring (ldmatrix; .trans when X's FVI is an m
+//       index) and B fragments from Y, which stays whole in shared memory;
+//   (4) accumulator element (row, n) of the AR blocks is the run C[a0 .. a0+AR-1, row, n]:
+//       alpha, RNE to BF16 and one 8- or 16-B streaming store per run straight from registers
+//        — no transpose, no staging, no block-wide barrier.
+// Persistent CTAs walk the tiles with C's FVI tile fastest, so neighbouring CTAs complete the
+// same C lines at the same time.
+#pragma once
+#include <cuda_bf16.h>
+#include <cstdint>
+
+#include "kernel_f64.cuh"   // mbarrier / TMA helpers
+#include "stream.hpp"
+
+namespace tc {
+
+__device__ __forceinline__ void ldsm_x4(uint32_t addr, uint32_t (&r)[4]) {
+  asm volatile("ldmatrix.sync.aligned.m8n8.x4.shared.b16 {%0,%1,%2,%3}, [%4];\n"
+               : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]) : "r"(addr) : "memory");
+}
+__device__ __forceinline__ void ldsm_x4_t(uint32_t addr, uint32_t (&r)[4]) {
+  asm volatile("ldmatrix.sync.aligned.m8n8.x4.trans.shared.b16 {%0,%1,%2,%3}, [%4];\n"
+               : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]) : "r"(addr) : "memory");
+}
+__device__ __forceinline__ void ldsm_x2(uint32_t addr, uint32_t &r0, uint32_t &r1) {
+  asm volatile("ldmatrix.sync.aligned.m8n8.x2.shared.b16 {%0,%1}, [%2];\n" : "=r"(r0), "=r"(r1) : "r"(addr) : "memory");
+}
+__device__ __forceinline__ void mma_bf16_16816(float (&d)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1) {
+  asm("mma.sync.aligned.m16n8k16.row.col.f32.bf16.bf16.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
+      "{%0,%1,%2,%3};\n"
+      : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3])
+      : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1));
+}
+__device__ __forceinline__ uint32_t pack_bf16(float lo, float hi) {
+  const __nv_bfloat162 v = __floats2bfloat162_rn(lo, hi);
+  return *reinterpret_cast<const uint32_t *>(&v);
+}
+
+// a TMA box's swizzle: 16-B chunks XOR address bits 7.. under mask m (0 none, 1 32B, 3 64B, 7 128B)
+__device__ __forceinline__ uint32_t s_swz(uint32_t off, int m) { return off ^ (((off >> 7) & (uint32_t)m) << 4); }
+
+// byte address of element `el` of the C box: 16-B chunk ch = el / 8 moved to
+// ch ^ (fold(ch >> 3) & 7), fold(x) = x ^ x >> s1 ^ x >> s2 (stream.cpp picks s1, s2)
+__device__ __forceinline__ uint32_t s_cswz(uint32_t el, int s1, int s2) {
+  const uint32_t ch = el >> 3, x = ch >> 3;
+  return ((ch ^ ((x ^ (x >> s1) ^ (x >> s2)) & 7u)) << 4) | ((el & 7u) << 1);
+}
+
+// tile t -> origin per m dim (raster order, C's FVI fastest)
+__device__ __forceinline__ void s_tile(const SParams &p, int t, int32_t (&o)[kSMaxMdims]) {
+#pragma unroll
+  for (int d = 0; d < kSMaxMdims; d++) {
+    o[d] = 0;
+    if (d < p.nmd) {
+      const int n = p.mNt[d];
+      const int q = t / n;
+      o[d] = (t - q * n) * p.mT[d];
+      t = q;
+    }
+  }
+}
+
+// Ablation side builds only (tools/stream_ablation.py compiles libtc with -DTC_STREAM_ABLATE=k;
+// the shipped library has kSAbl = 0): 1 = no MMAs, 2 = no C stores, 3 = neither (the X stream alone).
+#ifdef TC_STREAM_ABLATE
+constexpr int kSAbl = TC_STREAM_ABLATE;
+#else
+constexpr int kSAbl = 0;
+#endif
+
+template <int NB, int AR, bool TRANS>
+__global__ void __launch_bounds__(kSThreads, AR == 4 ? 2 : 1) tc_stream_bf16_kernel(const __grid_constant__ SParams p) {
+  extern __shared__ __align__(1024) unsigned char smem_dyn[];
+  unsigned char *sm = smem_dyn + ((1024u - ((uint32_t)__cvta_generic_to_shared(smem_dyn) & 1023u)) & 1023u);
+  const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(sm);
+  const uint32_t FULL = sbase + p.off_bar, EMPTY = FULL + 8 * p.stages;
+  const uint32_t YS = sbase + p.off_y;
+  uint32_t *tab = reinterpret_cast<uint32_t *>(sm + p.off_tab);
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int ntl = (p.ntiles - (int)blockIdx.x + (int)gridDim.x - 1) / (int)gridDim.x;
+
+  // ---- once per CTA: Y as [n][k] (k contiguous, pitch YP; zero past N and K), the tables
+  {
+    const __nv_bfloat16 *Y = static_cast<const __nv_bfloat16 *>(p.Y);
+    __nv_bfloat16 *ys = reinterpret_cast<__nv_bfloat16 *>(sm + p.off_y);
+    const int tot = 8 * NB * p.YP;
+    for (int i = tid; i < tot; i += kSThreads) {
+      const int n = i / p.YP, k = i - n * p.YP;
+      ys[i] = (n < p.N && k < p.K) ? Y[(int64_t)k * p.ysk + (int64_t)n * p.ysn] : __float2bfloat16_rn(0.f);
+    }
+    for (int i = tid; i < p.nunits * 2 * kSRows + p.nchunk; i += kSThreads) tab[i] = __ldg(p.tab + i);
+  }
+  if (tid == 0) {
+    for (int s = 0; s < p.stages; s++) {
+      mbar_init(FULL + 8 * s, 1);          // the TMA thread (+ the box bytes)
+      mbar_init(EMPTY + 8 * s, p.nunits);  // one arrive per working compute warp
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+  }
+  __syncthreads();
+
+  if (warp == kSWarps) {
+    // ======================= TMA producer ===================================================
+    if (lane == 0) {
+      uint64_t policy;   // X is read once: keep it from displacing C lines being completed in L2
+      asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;\n" : "=l"(policy));
+      int s = 0;
+      uint32_t ph = 0;
+      for (int lt = 0; lt < ntl; lt++) {
+        int32_t o[kSMaxMdims];
+        s_tile(p, (int)blockIdx.x + lt * (int)gridDim.x, o);
+        int32_t c[kMaxTmaDims];
+#pragma unroll
+        for (int j = 0; j < kMaxTmaDims; j++) {
+          int32_t v = 0;
+#pragma unroll
+          for (int d = 0; d < kSMaxMdims; d++) v = (d < p.nmd && p.mX[d] == j) ? o[d] : v;
+          c[j] = v;
+        }
+        for (int ks = 0; ks < p.nks; ks++) {
+          mbar_wait(EMPTY + 8 * s, ph ^ 1);   // (passes at once on the ring's first lap)
+          mbar_expect_tx(FULL + 8 * s, (uint32_t)p.stage_bytes);
+#pragma unroll
+          for (int j = 0; j < kMaxTmaDims; j++)
+            if (j == p.kX) c[j] = ks * p.KB;
+          tma_load(&p.xmap, p.xrank, c[0], c[1], c[2], c[3], c[4], sbase + (uint32_t)(s * p.stage_pitch),
+                   FULL + 8 * s, policy);
+          if (++s == p.stages) { s = 0; ph ^= 1; }
+        }
+      }
+    }
+    return;
+  }
+  if (warp >= p.nunits) return;
+
+  // ======================= compute warps: unit `warp` of every tile =========================
+  const uint32_t *ut = tab + warp * 2 * kSRows;
+  const int q = lane >> 3, r = lane & 7, g = lane >> 2, t4 = lane & 3;
+  // ldmatrix row address in a stage (a0, k = 0): .trans rows are k (16 B of 8 consecutive E of
+  // the row octet q & 1); plain rows are the unit's rows (16 B of 8 consecutive k)
+  const uint32_t xr = TRANS ? ut[8 * (q & 1)] + (uint32_t)((r + 8 * (q >> 1)) * p.xpitchk)
+                            : ut[r + 8 * (q & 1)] + (uint32_t)(16 * (q >> 1));
+  const int xsw = p.xswz;   // the X box's TMA swizzle (conflict-free ldmatrix rows)
+  const uint32_t kstep16 = TRANS ? (uint32_t)(16 * p.xpitchk) : 32u;
+  const uint32_t xpa = (uint32_t)p.xpitcha;
+  // this thread's two accumulator rows g and g + 8: C offsets (tile origin, a0) and coordinates
+  const uint32_t bo0 = ut[kSRows + g], bo1 = ut[kSRows + 8 + g];   // C box offsets of rows g, g + 8
+  const uint32_t *ctab = tab + p.nunits * 2 * kSRows;
+  const uint32_t STG = sbase + p.off_stg;
+  const int nthr = p.nunits * 32;   // the working compute threads
+  // B fragments: ldmatrix rows n, 8 k per row
+  const uint32_t ybq = YS + (uint32_t)(((q >> 1) * 8 + r) * p.YP * 2 + 16 * (q & 1));
+  const float alpha = p.alpha;
+  __nv_bfloat16 *C = static_cast<__nv_bfloat16 *>(p.C);
+  int s = 0;
+  uint32_t ph = 0;
+  for (int lt = 0; lt < ntl; lt++) {
+    float acc[AR][NB][4];
+#pragma unroll
+    for (int j = 0; j < AR; j++)
+#pragma unroll
+      for (int n = 0; n < NB; n++)
+#pragma unroll
+        for (int e = 0; e < 4; e++) acc[j][n][e] = 0.f;
+    for (int ks = 0; ks < p.nks; ks++) {
+      mbar_wait(FULL + 8 * s, ph);
+      const uint32_t xs = sbase + (uint32_t)(s * p.stage_pitch);
+      const int k0 = ks * p.KB;
+      const int nk16 = min(p.KB, p.KP - k0) >> 4;
+      for (int kk = 0; kk < ((kSAbl & 1) ? 0 : nk16); kk++) {
+        uint32_t bf[NB][2];
+        const uint32_t yb = ybq + (uint32_t)(2 * (k0 + 16 * kk));
+#pragma unroll
+        for (int n = 0; n + 1 < NB; n += 2) {
+          uint32_t v[4];
+          ldsm_x4(yb + (uint32_t)(n * 8 * p.YP * 2), v);
+          bf[n][0] = v[0]; bf[n][1] = v[1]; bf[n + 1][0] = v[2]; bf[n + 1][1] = v[3];
+        }
+        if (NB & 1) ldsm_x2(yb + (uint32_t)((NB - 1) * 8 * p.YP * 2), bf[NB - 1][0], bf[NB - 1][1]);
+        const uint32_t xa = xr + (uint32_t)kk * kstep16;
+#pragma unroll
+        for (int j = 0; j < AR; j++) {
+          uint32_t af[4];
+          const uint32_t ad = xs + s_swz(xa + (uint32_t)j * xpa, xsw);
+          if (TRANS) ldsm_x4_t(ad, af);
+          else ldsm_x4(ad, af);
+#pragma unroll
+          for (int n = 0; n < NB; n++) mma_bf16_16816(acc[j][n], af, bf[n][0], bf[n][1]);
+        }
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(EMPTY + 8 * s);
+      if (++s == p.stages) { s = 0; ph ^= 1; }
+    }
+    // ---- epilogue: runs of AR values of C's FVI straight from the accumulators into the C box
+    // (smem, C order, swizzled 16-B chunks), then the whole box out as 16-B runs along C's FVI
+    const int t = (int)blockIdx.x + lt * (int)gridDim.x;
+    consumer_sync(nthr);   // the previous tile's box has been stored
+    if (!(kSAbl & 2)) {
+#pragma unroll
+      for (int h = 0; h < 2; h++)
+#pragma unroll
+        for (int n = 0; n < NB; n++)
+#pragma unroll
+          for (int c2 = 0; c2 < 2; c2++) {
+            const uint32_t boh = h ? bo1 : bo0;
+            if (boh == 0xFFFFFFFFu) continue;   // a padding row
+            const uint32_t el = boh + (uint32_t)((8 * n + 2 * t4 + c2) * p.cbsn);
+            const uint32_t ad = STG + s_cswz(el, p.cs1, p.cs2);
+            if constexpr (AR == 8) {
+              asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};\n" ::"r"(ad),
+                           "r"(pack_bf16(alpha * acc[0][n][2 * h + c2], alpha * acc[1][n][2 * h + c2])),
+                           "r"(pack_bf16(alpha * acc[2][n][2 * h + c2], alpha * acc[3][n][2 * h + c2])),
+                           "r"(pack_bf16(alpha * acc[4][n][2 * h + c2], alpha * acc[5][n][2 * h + c2])),
+                           "r"(pack_bf16(alpha * acc[6][n][2 * h + c2], alpha * acc[7][n][2 * h + c2]))
+                           : "memory");
+            } else {
+              asm volatile("st.shared.v2.b32 [%0], {%1,%2};\n" ::"r"(ad),
+                           "r"(pack_bf16(alpha * acc[0][n][2 * h + c2], alpha * acc[1][n][2 * h + c2])),
+                           "r"(pack_bf16(alpha * acc[2][n][2 * h + c2], alpha * acc[3][n][2 * h + c2]))
+                           : "memory");
+            }
+          }
+    }
+    consumer_sync(nthr);   // the box is complete
+    if (!(kSAbl & 2)) {
+      // tile origin in C and per-dim limits (edge tiles store only what lies in the tensor)
+      int tt = t;
+      int64_t corg = 0;
+      uint32_t lims = 0;
+      bool interior = p.N == 8 * NB;
+#pragma unroll
+      for (int d = 0; d < kSMaxMdims; d++) {
+        if (d < p.nmd) {
+          const int n = p.mNt[d];
+          const int qd = tt / n;
+          const int od = (tt - qd * n) * p.mT[d];
+          tt = qd;
+          const int l = min(p.mT[d], p.mN[d] - od);
+          interior &= l == p.mT[d];
+          lims |= (uint32_t)l << (8 * d);
+          corg += (int64_t)od * p.mCs[d];
+        }
+      }
+      __nv_bfloat16 *Ct = C + corg;
+      const unsigned char *sb = sm + p.off_stg;
+      for (int ch = tid; ch < p.nchunk; ch += nthr) {
+        const uint4 v = *reinterpret_cast<const uint4 *>(sb + s_cswz((uint32_t)ch * 8u, p.cs1, p.cs2));
+        __nv_bfloat16 *dst = Ct + (int32_t)ctab[ch];
+        if (interior) {
+          __stcs(reinterpret_cast<uint4 *>(dst), v);
+        } else {
+          // the chunk's coordinate per C dim (box order, dim 0 in steps of 8): store the
+          // elements below every limit
+          int rem = ch, c0 = 0;
+          bool ok = true;
+#pragma unroll
+          for (int j2 = 0; j2 < kMaxTmaDims; j2++) {
+            if (j2 < p.crank) {
+              const int ext = j2 == 0 ? p.cbox[0] / 8 : p.cbox[j2];
+              const int cj = rem % ext;
+              rem /= ext;
+              const int lim = p.cmd[j2] < 0 ? p.N : (int)((lims >> (8 * p.cmd[j2])) & 0xFF);
+              if (j2 == 0) c0 = 8 * cj;
+              else ok &= cj < lim;
+            }
+          }
+          const int lim0 = p.cmd[0] < 0 ? p.N : (int)((lims >> (8 * p.cmd[0])) & 0xFF);
+          const int ne = ok ? max(0, min(8, lim0 - c0)) : 0;
+          if (ne == 8) {
+            __stcs(reinterpret_cast<uint4 *>(dst), v);
+          } else {
+            const __nv_bfloat16 *e = reinterpret_cast<const __nv_bfloat16 *>(&v);
+            for (int q2 = 0; q2 < ne; q2++) dst[q2] = e[q2];
+          }
+        }
+      }
+    }
+  }
+}
+
+}  // namespace tc

@@ -12,6 +12,7 @@
 #include "contraction.hpp"
 #include "kparams.hpp"
 #include "planner.hpp"
+#include "stream.hpp"
 #include "tiles.hpp"
 
 using namespace tc;   // (internal header: the plan object is written in the library's namespace)
@@ -40,6 +41,10 @@ struct tc_plan_s {
   bool pair = false;
   bool out_f32 = false;    // BF16 operands, FP32 C (kernels_umma_f32out.cu)       // tcgen05: launch the CTA-pair instance (clusters of 2) with TMA operands
   OperandMap mapX, mapY;
+  // the streaming path (stream.hpp): on when eligible unless opts / a forced variant say
+  // otherwise; tc_execute takes it for beta == 0 when both tensor maps encode
+  StreamCfg stream;
+  int stream_grid = 0;     // persistent CTAs (SMs x resident CTAs)
   // batch (Hadamard) indices (R31): extent and element strides in X, Y, C.  tc_execute
   // launches the kernel once per batch slab with the operands offset to it — the kernels
   // carry no batch code (the FP64 variants run at their 128-register cap).

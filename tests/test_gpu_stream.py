@@ -1,0 +1,101 @@
+"""GPU parity of the streaming BF16 path (stream.hpp / kernel_stream.cuh: Y whole in shared
+memory, X by TMA boxes in its own order, C runs along its FVI from the MMA accumulators)
+through the C ABI against the CPU oracle — the same checks as test_gpu_bf16.check_bf16:
+integer data bitwise, random data within one BF16 ulp + the FP32 accumulation bound.
+Covers both row modes (X's FVI external: SM_T; X's FVI internal: SM_K), edge tiles on every
+m dim, n not a multiple of 8, k not a multiple of 16, padding rows (odd octet counts), alpha,
+and the fall-backs to the plan's tcgen05 configuration (beta != 0, misaligned C).
+Needs a B200: run with -m gpu."""
+import pytest
+import torch
+
+import tcinputs
+from paper_conf_cgo_kimstkpprs19_b200 import binding as tc
+from paper_conf_cgo_kimstkpprs19_b200 import build
+from tests.test_gpu_bf16 import check_bf16
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _dev():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    build.build()
+    torch.cuda.set_device(0)
+
+
+def _on(expr, ext):
+    s = tc.plan(expr, ext, "bf16", host_only=True).info()["stream"]
+    assert s["on"] == 1, s
+    return s
+
+
+# TCCG #1-8 shapes at reduced extents (first dims multiples of 8: 16-B TMA strides), both modes
+REDUCED = [
+    ("abcde-efbad-cf", "a:16;b:6;c:24;d:5;e:16;f:12"),     # SM_T (X's FVI e), #1
+    ("abcde-efcad-bf", "a:24;b:20;c:5;d:3;e:24;f:12"),     # #2, n = 20
+    ("abcd-dbea-ec", "a:24;b:9;c:24;d:24;e:24"),           # #3
+    ("abcde-ecbfa-fd", "a:16;b:3;c:7;d:24;e:16;f:12"),     # #4
+    ("abcd-deca-be", "a:24;b:24;c:5;d:16;e:24"),           # #5
+    ("abc-bda-dc", "a:40;b:40;c:24;d:40"),                 # #6, 5 octets of b: a padding row set
+    ("abcd-ebad-ce", "a:24;b:10;c:24;d:3;e:24"),           # SM_K (X's FVI e = k), #7
+    ("abc-dca-bd", "a:40;b:24;c:21;d:40"),                 # SM_K, #8, rest product 21
+]
+
+
+@pytest.mark.parametrize("expr,ext", REDUCED, ids=[f"tccg{i + 1}" for i in range(8)])
+def test_stream_tccg_shapes(expr, ext):
+    _on(expr, ext)
+    check_bf16(expr, ext, seed=1, integer=True, stream=True)
+    check_bf16(expr, ext, seed=2, stream=True)
+    check_bf16(expr, ext, seed=3, integer=True, alpha=-2.0, stream=True)
+
+
+# edge tiles on every m dim, k padded to 16, n below a multiple of 8
+RAGGED = [
+    ("abcde-efbad-cf", "a:24;b:5;c:13;d:3;e:40;f:9"),
+    ("abc-bda-dc", "a:56;b:24;c:7;d:300"),          # K = 300: several k-steps, the last partial
+    ("abc-dca-bd", "a:40;b:17;c:21;d:40"),          # SM_K, rest rows 21 of 16-row sets: padding rows
+    ("abcd-ebad-ce", "a:24;b:5;c:31;d:3;e:24"),     # SM_K, n = 31
+    ("abcd-dbea-ec", "a:8;b:3;c:3;d:8;e:8"),        # one tile, n = 3
+]
+
+
+@pytest.mark.parametrize("expr,ext", RAGGED, ids=[f"r{i}" for i in range(len(RAGGED))])
+def test_stream_ragged(expr, ext):
+    p = tc.plan(expr, ext, "bf16", host_only=True)
+    s = p.info()["stream"]
+    if s["on"] != 1:
+        pytest.skip(f"not a streaming shape: {s['why']}")
+    check_bf16(expr, ext, seed=4, integer=True, stream=True)
+    check_bf16(expr, ext, seed=5, stream=True)
+
+
+def test_stream_fallbacks_beta_and_alignment():
+    # beta != 0 and a C pointer off the run alignment take the plan's tcgen05 configuration:
+    # same results
+    expr, ext = REDUCED[0]
+    _on(expr, ext)
+    check_bf16(expr, ext, seed=6, integer=True, alpha=2.0, beta=1.0, stream=True)
+    check_bf16(expr, ext, seed=7, integer=True, cmisalign=1, stream=True)
+    check_bf16(expr, ext, seed=8, integer=True, misalign=8, stream=True)
+
+
+def test_stream_off_matches():
+    # the option turns the path off (tcgen05 configuration); both give the same bits on integers
+    expr, ext = REDUCED[6]
+    p = check_bf16(expr, ext, seed=9, integer=True, stream=False)
+    assert p.info()["stream"]["on"] == 0
+
+
+def test_stream_tuned_candidate():
+    # tc_plan_tuned times the streaming path as candidate 99 beside the variants
+    case = [c for c in tcinputs.tccg48() if c.id == 3][0]
+    p = tc.plan(case.expr, case.extents, "bf16")
+    assert p.info()["stream"]["on"] == 1
+    A = tcinputs.uniform(p.numel("A"), 1, device="cuda").to(torch.bfloat16)
+    B = tcinputs.uniform(p.numel("B"), 2, device="cuda").to(torch.bfloat16)
+    C = torch.empty(p.numel("C"), dtype=torch.bfloat16, device="cuda")
+    t = p.tuned(A, B, C, topk=2, reps=1)
+    assert 99 in [v for v, _ in t.info()["stats"]["tuned"]]

@@ -369,3 +369,31 @@ def test_cta_pair_needs_c_fvi_leading_m():
     j = tc.plan("ab-ac-cb", "a:392;b:264;c:136", dtype="bf16", force_tiles="a:128;b:128;c:64", pair=True,
                 host_only=True).info()
     assert j["cs0"] == 1 and j["cta_pair"] == 1
+
+
+def test_stream_path_planning():
+    """The streaming BF16 path (stream.hpp): planned for the memory-bound tensor x matrix TCCG
+    cases #1-8 (both row modes), never for other dtypes, batch indices, large Y-side extents or
+    when the options turn it off; tiles are TMA-legal boxes and the units fit the 8 warps."""
+    import tcinputs
+    for c in tcinputs.tccg48():
+        s = tc.plan(c.expr, c.extents, "bf16", host_only=True).info()["stream"]
+        if c.id <= 8:
+            assert s["on"] == 1, (c.id, s)
+            assert s["mode"] == ("K" if c.id in (7, 8) else "T")
+            assert 1 <= s["units"] <= 8 and s["AR"] in (4, 8) and s["KB"] % 16 == 0
+            assert all(t <= 256 for t in s["tiles"].values())
+            assert s["smem"] <= (115712 if s["AR"] == 4 else 232448)
+        else:
+            assert s["on"] == 0, (c.id, s)
+    c1 = tcinputs.tccg48()[0]
+    for dt in ("f64", "f32", "tf32"):
+        assert tc.plan(c1.expr, c1.extents, dt, host_only=True).info()["stream"]["on"] == 0
+    assert tc.plan(c1.expr, c1.extents, "bf16", host_only=True, stream=False).info()["stream"]["on"] == 0
+    # a forced variant keeps the path off unless asked for
+    assert tc.plan(c1.expr, c1.extents, "bf16", host_only=True, variant=11).info()["stream"]["on"] == 0
+    assert tc.plan(c1.expr, c1.extents, "bf16", host_only=True, variant=11, stream=True).info()["stream"]["on"] == 1
+    # batch index, Y-side extent above 32, X's FVI = C's FVI: not streaming shapes
+    assert tc.plan("abh-ach-cbh", "a:16;b:16;c:16;h:4", "bf16", host_only=True).info()["stream"]["on"] == 0
+    assert tc.plan("abc-bda-dc", "a:16;b:16;c:40;d:16", "bf16", host_only=True).info()["stream"]["on"] == 0
+    assert tc.plan("abc-adb-dc", "a:16;b:16;c:16;d:16", "bf16", host_only=True).info()["stream"]["on"] == 0
