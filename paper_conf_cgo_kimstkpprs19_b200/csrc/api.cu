@@ -205,7 +205,7 @@ Status upload(tc_plan_s *P, std::string &err) {
   P->d_packY2 = (const uint32_t *)(b + parts[iY2p].off);
   if (P->stream.on) {
     P->stream.kp.tab = (const uint32_t *)(b + parts[iS].off);
-    const void *fn = stream_kernel_ptr(P->stream.NB, P->stream.AR, P->stream.mode != SM_K);
+    const void *fn = stream_kernel_ptr(P->dtype == TC_F64, P->stream.NB, P->stream.AR, P->stream.mode != SM_K);
     if (!fn) { err = "no streaming kernel instance for the plan"; return ST_UNSUPPORTED; }
     // (the instance is shared by plans of different sizes: always the opt-in maximum)
     e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448);
@@ -341,10 +341,15 @@ tc_status_t finish_plan(tc_plan_s *P, tc_plan_t *out, const tc_plan_s *rep = nul
   // the streaming path (stream.hpp) beside the configuration: on when eligible, unless the
   // caller forced a variant (tests, tuning candidates) or opts.stream says otherwise
   P->stream = StreamCfg();
+  P->stream_active = false;
   if (P->opts.stream != 1 && !P->out_f32 && (fv < 0 || P->opts.stream == 2) && !ft.on) {
     StreamCfg sc;
-    if (stream_plan(P->c, kind, 148, sc)) P->stream = sc;
-    else P->stream.why = sc.why;
+    if (stream_plan(P->c, kind, 148, sc)) {
+      P->stream = sc;
+      P->stream_active = sc.preferred || P->opts.stream == 2;
+    } else {
+      P->stream.why = sc.why;
+    }
   } else {
     P->stream.why = "off (options)";
   }
@@ -444,18 +449,19 @@ bool encode_stream_maps(const tc_plan_s *P, const void *Xp, void *C, SParams &sp
   auto enc = tma_encoder();
   if (!enc) return false;
   const StreamCfg &s = P->stream;
-  const char *xb = (const char *)Xp + 2 * s.xbase;
-  const char *cb = (const char *)C + 2 * s.cbase;
-  if ((uintptr_t)xb % 16 || (uintptr_t)cb % (2 * s.AR)) return false;
+  const int es = P->dtype == TC_F64 ? 8 : 2;
+  const char *xb = (const char *)Xp + es * s.xbase;
+  const char *cb = (const char *)C + es * s.cbase;
+  if ((uintptr_t)xb % 16 || (uintptr_t)cb % 16) return false;
   cuuint64_t dims[kMaxTmaDims], strides[kMaxTmaDims];
   cuuint32_t box[kMaxTmaDims], el[kMaxTmaDims];
   for (int j = 0; j < s.xrank; j++) {
     dims[j] = (cuuint64_t)s.xdims[j];
     box[j] = s.xbox[j];
     el[j] = 1;
-    if (j > 0) strides[j - 1] = (cuuint64_t)(s.xstr[j] * 2);
+    if (j > 0) strides[j - 1] = (cuuint64_t)(s.xstr[j] * es);
   }
-  return enc(reinterpret_cast<CUtensorMap *>(&sp.xmap), CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, (cuuint32_t)s.xrank,
+  return enc(reinterpret_cast<CUtensorMap *>(&sp.xmap), es == 8 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT64 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, (cuuint32_t)s.xrank,
              (void *)xb, dims, strides, box, el, CU_TENSOR_MAP_INTERLEAVE_NONE, (CUtensorMapSwizzle)s.xswz,
 #ifdef TC_STREAM_PROMO
              (CUtensorMapL2promotion)TC_STREAM_PROMO,
@@ -891,15 +897,16 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
   const tc_status_t chk = check_execute(plan, A, B, C);
   if (chk != TC_SUCCESS) return chk;
   const size_t es = elem_bytes(plan);
-  if (plan->stream.on && beta == 0.0 && plan->batch.empty()) {
+  if (plan->stream.on && plan->stream_active && beta == 0.0 && plan->batch.empty()) {
     // the streaming path (beta == 0: C is only written; otherwise the configuration below)
     SParams sp = plan->stream.kp;
     const void *Xp = plan->stream.X == 1 ? A : B, *Yp = plan->stream.X == 1 ? B : A;
     if (encode_stream_maps(plan, Xp, C, sp)) {
-      sp.Y = static_cast<const char *>(Yp) + 2 * plan->stream.ybase;
-      sp.C = static_cast<char *>(C) + 2 * plan->stream.cbase;
+      sp.Y = static_cast<const char *>(Yp) + es * plan->stream.ybase;
+      sp.C = static_cast<char *>(C) + es * plan->stream.cbase;
       sp.alpha = (float)alpha;
-      const void *fn = stream_kernel_ptr(plan->stream.NB, plan->stream.AR, plan->stream.mode != SM_K);
+      sp.alpha64 = alpha;
+      const void *fn = stream_kernel_ptr(plan->dtype == TC_F64, plan->stream.NB, plan->stream.AR, plan->stream.mode != SM_K);
       const int grid = std::min(sp.ntiles, plan->stream_grid);
       void *sargs[] = {&sp};
       cudaError_t e = cudaLaunchKernel(fn, dim3(grid), dim3(kSThreads), sargs, plan->stream.smem, (cudaStream_t)stream);
@@ -1117,13 +1124,14 @@ tc_status_t tc_plan_info(const tc_plan_t plan, char *json, size_t cap, size_t *n
     {   // the streaming path (stream.hpp)
       const StreamCfg &st = plan->stream;
       const SParams &k = st.kp;
-      o << ",\"stream\":{\"on\":" << (st.on ? 1 : 0) << ",\"why\":\"" << st.why << "\"";
+      o << ",\"stream\":{\"on\":" << (st.on ? 1 : 0) << ",\"active\":" << (plan->stream_active ? 1 : 0)
+        << ",\"why\":\"" << st.why << "\"";
       if (st.on) {
         o << ",\"mode\":\"" << (st.mode == SM_K ? "K" : "T") << "\",\"X\":\"" << (st.X == 1 ? "A" : "B") << "\",\"tiles\":{";
         for (size_t i = 0; i < c.ix.size(); i++) o << (i ? "," : "") << "\"" << c.ix[i].name << "\":" << st.T[i];
         o << "},\"KB\":" << k.KB << ",\"nks\":" << k.nks << ",\"stages\":" << k.stages
           << ",\"stage_bytes\":" << k.stage_bytes << ",\"ntiles\":" << k.ntiles << ",\"units\":" << k.nunits
-          << ",\"NB\":" << st.NB << ",\"AR\":" << st.AR << ",\"occ\":" << st.occ << ",\"xswz\":" << st.xswz << ",\"smem\":" << st.smem
+          << ",\"NB\":" << st.NB << ",\"AR\":" << st.AR << ",\"occ\":" << st.occ << ",\"nstg\":" << k.nstg << ",\"xswz\":" << st.xswz << ",\"smem\":" << st.smem
           << ",\"grid\":" << plan->stream_grid
           << ",\"t_pred_ms\":" << st.t_pred * 1e3 << ",\"bytes\":" << st.bytes;
       }

@@ -47,13 +47,6 @@ __device__ __forceinline__ uint32_t pack_bf16(float lo, float hi) {
 // a TMA box's swizzle: 16-B chunks XOR address bits 7.. under mask m (0 none, 1 32B, 3 64B, 7 128B)
 __device__ __forceinline__ uint32_t s_swz(uint32_t off, int m) { return off ^ (((off >> 7) & (uint32_t)m) << 4); }
 
-// byte address of element `el` of the C box: 16-B chunk ch = el / 8 moved to
-// ch ^ (fold(ch >> 3) & 7), fold(x) = x ^ x >> s1 ^ x >> s2 (stream.cpp picks s1, s2)
-__device__ __forceinline__ uint32_t s_cswz(uint32_t el, int s1, int s2) {
-  const uint32_t ch = el >> 3, x = ch >> 3;
-  return ((ch ^ ((x ^ (x >> s1) ^ (x >> s2)) & 7u)) << 4) | ((el & 7u) << 1);
-}
-
 // tile t -> origin per m dim (raster order, C's FVI fastest)
 __device__ __forceinline__ void s_tile(const SParams &p, int t, int32_t (&o)[kSMaxMdims]) {
 #pragma unroll
@@ -76,6 +69,100 @@ constexpr int kSAbl = TC_STREAM_ABLATE;
 constexpr int kSAbl = 0;
 #endif
 
+// The TMA producer (one thread): for every tile of this CTA and every k-step, one X box into the
+// next ring stage once the compute warps have released it
+__device__ __forceinline__ void s_produce(const SParams &p, int ntl, uint32_t sbase, uint32_t FULL, uint32_t EMPTY) {
+  uint64_t policy;   // X is read once: keep it from displacing C lines being completed in L2
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;\n" : "=l"(policy));
+  int s = 0;
+  uint32_t ph = 0;
+  for (int lt = 0; lt < ntl; lt++) {
+    int32_t o[kSMaxMdims];
+    s_tile(p, (int)blockIdx.x + lt * (int)gridDim.x, o);
+    int32_t c[kMaxTmaDims];
+#pragma unroll
+    for (int j = 0; j < kMaxTmaDims; j++) {
+      int32_t v = 0;
+#pragma unroll
+      for (int d = 0; d < kSMaxMdims; d++) v = (d < p.nmd && p.mX[d] == j) ? o[d] : v;
+      c[j] = v;
+    }
+    for (int ks = 0; ks < p.nks; ks++) {
+      mbar_wait(EMPTY + 8 * s, ph ^ 1);   // (passes at once on the ring's first lap)
+      mbar_expect_tx(FULL + 8 * s, (uint32_t)p.stage_bytes);
+#pragma unroll
+      for (int j = 0; j < kMaxTmaDims; j++)
+        if (j == p.kX) c[j] = ks * p.KB;
+      tma_load(&p.xmap, p.xrank, c[0], c[1], c[2], c[3], c[4], sbase + (uint32_t)(s * p.stage_pitch),
+               FULL + 8 * s, policy);
+      if (++s == p.stages) { s = 0; ph ^= 1; }
+    }
+  }
+}
+
+// byte address in the C box of byte offset b: its 16-B chunk ch moved to ch ^ (fold(ch >> 3) & 7),
+// fold(x) = x ^ x >> s1 ^ x >> s2 (stream.cpp picks s1, s2 by simulating the writes)
+__device__ __forceinline__ uint32_t s_cswzb(uint32_t b, int s1, int s2) {
+  const uint32_t ch = b >> 4, x = ch >> 3;
+  return ((ch ^ ((x ^ (x >> s1) ^ (x >> s2)) & 7u)) << 4) | (b & 15u);
+}
+
+// The C box (smem, C order) leaves as 16-B runs along C's FVI: chunk c at ctab[c] elements from
+// the tile origin.  Interior tiles store every chunk; tiles on the tensor's edge store what lies
+// inside (every coordinate below its limit).
+template <typename TE>
+__device__ __forceinline__ void s_store_box(const SParams &p, TE *C, const unsigned char *sm, uint32_t stg_off,
+                                            const uint32_t *ctab, int t, int tid, int nthr, int NB) {
+  constexpr int EPC = 16 / (int)sizeof(TE);   // elements per chunk
+  int64_t corg = 0;
+  uint32_t lims = 0;
+  bool interior = p.N == 8 * NB;
+#pragma unroll
+  for (int d = 0; d < kSMaxMdims; d++) {
+    if (d < p.nmd) {
+      const int n = p.mNt[d];
+      const int qd = t / n;
+      const int od = (t - qd * n) * p.mT[d];
+      t = qd;
+      const int l = min(p.mT[d], p.mN[d] - od);
+      interior &= l == p.mT[d];
+      lims |= (uint32_t)l << (8 * d);
+      corg += (int64_t)od * p.mCs[d];
+    }
+  }
+  TE *Ct = C + corg;
+  const unsigned char *sb = sm + stg_off;
+  for (int ch = tid; ch < p.nchunk; ch += nthr) {
+    const uint4 v = *reinterpret_cast<const uint4 *>(sb + s_cswzb((uint32_t)ch * 16u, p.cs1, p.cs2));
+    TE *dst = Ct + (int32_t)ctab[ch];
+    if (interior) {
+      __stcs(reinterpret_cast<uint4 *>(dst), v);
+      continue;
+    }
+    int rem = ch, c0 = 0;
+    bool ok = true;
+#pragma unroll
+    for (int j2 = 0; j2 < kMaxTmaDims; j2++) {
+      if (j2 < p.crank) {
+        const int ext = j2 == 0 ? p.cbox[0] / EPC : p.cbox[j2];
+        const int cj = rem % ext;
+        rem /= ext;
+        const int lim = p.cmd[j2] < 0 ? p.N : (int)((lims >> (8 * p.cmd[j2])) & 0xFF);
+        if (j2 == 0) c0 = EPC * cj;
+        else ok &= cj < lim;
+      }
+    }
+    const int lim0 = p.cmd[0] < 0 ? p.N : (int)((lims >> (8 * p.cmd[0])) & 0xFF);
+    const int ne = ok ? max(0, min(EPC, lim0 - c0)) : 0;
+    if (ne == EPC) {
+      __stcs(reinterpret_cast<uint4 *>(dst), v);
+    } else {
+      const TE *e = reinterpret_cast<const TE *>(&v);
+      for (int q2 = 0; q2 < ne; q2++) dst[q2] = e[q2];
+    }
+  }
+}
+
 template <int NB, int AR, bool TRANS>
 __global__ void __launch_bounds__(kSThreads, AR == 4 ? 2 : 1) tc_stream_bf16_kernel(const __grid_constant__ SParams p) {
   extern __shared__ __align__(1024) unsigned char smem_dyn[];
@@ -96,7 +183,7 @@ __global__ void __launch_bounds__(kSThreads, AR == 4 ? 2 : 1) tc_stream_bf16_ker
       const int n = i / p.YP, k = i - n * p.YP;
       ys[i] = (n < p.N && k < p.K) ? Y[(int64_t)k * p.ysk + (int64_t)n * p.ysn] : __float2bfloat16_rn(0.f);
     }
-    for (int i = tid; i < p.nunits * 2 * kSRows + p.nchunk; i += kSThreads) tab[i] = __ldg(p.tab + i);
+    for (int i = tid; i < p.nunits * 2 * p.ru + p.nchunk; i += kSThreads) tab[i] = __ldg(p.tab + i);
   }
   if (tid == 0) {
     for (int s = 0; s < p.stages; s++) {
@@ -109,34 +196,7 @@ __global__ void __launch_bounds__(kSThreads, AR == 4 ? 2 : 1) tc_stream_bf16_ker
 
   if (warp == kSWarps) {
     // ======================= TMA producer ===================================================
-    if (lane == 0) {
-      uint64_t policy;   // X is read once: keep it from displacing C lines being completed in L2
-      asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;\n" : "=l"(policy));
-      int s = 0;
-      uint32_t ph = 0;
-      for (int lt = 0; lt < ntl; lt++) {
-        int32_t o[kSMaxMdims];
-        s_tile(p, (int)blockIdx.x + lt * (int)gridDim.x, o);
-        int32_t c[kMaxTmaDims];
-#pragma unroll
-        for (int j = 0; j < kMaxTmaDims; j++) {
-          int32_t v = 0;
-#pragma unroll
-          for (int d = 0; d < kSMaxMdims; d++) v = (d < p.nmd && p.mX[d] == j) ? o[d] : v;
-          c[j] = v;
-        }
-        for (int ks = 0; ks < p.nks; ks++) {
-          mbar_wait(EMPTY + 8 * s, ph ^ 1);   // (passes at once on the ring's first lap)
-          mbar_expect_tx(FULL + 8 * s, (uint32_t)p.stage_bytes);
-#pragma unroll
-          for (int j = 0; j < kMaxTmaDims; j++)
-            if (j == p.kX) c[j] = ks * p.KB;
-          tma_load(&p.xmap, p.xrank, c[0], c[1], c[2], c[3], c[4], sbase + (uint32_t)(s * p.stage_pitch),
-                   FULL + 8 * s, policy);
-          if (++s == p.stages) { s = 0; ph ^= 1; }
-        }
-      }
-    }
+    if (lane == 0) s_produce(p, ntl, sbase, FULL, EMPTY);
     return;
   }
   if (warp >= p.nunits) return;
@@ -203,7 +263,11 @@ __global__ void __launch_bounds__(kSThreads, AR == 4 ? 2 : 1) tc_stream_bf16_ker
     // ---- epilogue: runs of AR values of C's FVI straight from the accumulators into the C box
     // (smem, C order, swizzled 16-B chunks), then the whole box out as 16-B runs along C's FVI
     const int t = (int)blockIdx.x + lt * (int)gridDim.x;
-    consumer_sync(nthr);   // the previous tile's box has been stored
+    // one C box: wait until the previous tile's box has been stored; two boxes: this tile's box
+    // was last read by tile lt - 2's stores, which every warp finished before the barrier below
+    // of tile lt - 1
+    const uint32_t STGb = STG + (p.nstg == 2 ? (uint32_t)((lt & 1) * p.stg_pitch) : 0u);
+    if (p.nstg == 1) consumer_sync(nthr);
     if (!(kSAbl & 2)) {
 #pragma unroll
       for (int h = 0; h < 2; h++)
@@ -214,7 +278,7 @@ __global__ void __launch_bounds__(kSThreads, AR == 4 ? 2 : 1) tc_stream_bf16_ker
             const uint32_t boh = h ? bo1 : bo0;
             if (boh == 0xFFFFFFFFu) continue;   // a padding row
             const uint32_t el = boh + (uint32_t)((8 * n + 2 * t4 + c2) * p.cbsn);
-            const uint32_t ad = STG + s_cswz(el, p.cs1, p.cs2);
+            const uint32_t ad = STGb + s_cswzb(2u * el, p.cs1, p.cs2);
             if constexpr (AR == 8) {
               asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};\n" ::"r"(ad),
                            "r"(pack_bf16(alpha * acc[0][n][2 * h + c2], alpha * acc[1][n][2 * h + c2])),
@@ -231,59 +295,110 @@ __global__ void __launch_bounds__(kSThreads, AR == 4 ? 2 : 1) tc_stream_bf16_ker
           }
     }
     consumer_sync(nthr);   // the box is complete
-    if (!(kSAbl & 2)) {
-      // tile origin in C and per-dim limits (edge tiles store only what lies in the tensor)
-      int tt = t;
-      int64_t corg = 0;
-      uint32_t lims = 0;
-      bool interior = p.N == 8 * NB;
-#pragma unroll
-      for (int d = 0; d < kSMaxMdims; d++) {
-        if (d < p.nmd) {
-          const int n = p.mNt[d];
-          const int qd = tt / n;
-          const int od = (tt - qd * n) * p.mT[d];
-          tt = qd;
-          const int l = min(p.mT[d], p.mN[d] - od);
-          interior &= l == p.mT[d];
-          lims |= (uint32_t)l << (8 * d);
-          corg += (int64_t)od * p.mCs[d];
-        }
-      }
-      __nv_bfloat16 *Ct = C + corg;
-      const unsigned char *sb = sm + p.off_stg;
-      for (int ch = tid; ch < p.nchunk; ch += nthr) {
-        const uint4 v = *reinterpret_cast<const uint4 *>(sb + s_cswz((uint32_t)ch * 8u, p.cs1, p.cs2));
-        __nv_bfloat16 *dst = Ct + (int32_t)ctab[ch];
-        if (interior) {
-          __stcs(reinterpret_cast<uint4 *>(dst), v);
-        } else {
-          // the chunk's coordinate per C dim (box order, dim 0 in steps of 8): store the
-          // elements below every limit
-          int rem = ch, c0 = 0;
-          bool ok = true;
-#pragma unroll
-          for (int j2 = 0; j2 < kMaxTmaDims; j2++) {
-            if (j2 < p.crank) {
-              const int ext = j2 == 0 ? p.cbox[0] / 8 : p.cbox[j2];
-              const int cj = rem % ext;
-              rem /= ext;
-              const int lim = p.cmd[j2] < 0 ? p.N : (int)((lims >> (8 * p.cmd[j2])) & 0xFF);
-              if (j2 == 0) c0 = 8 * cj;
-              else ok &= cj < lim;
-            }
-          }
-          const int lim0 = p.cmd[0] < 0 ? p.N : (int)((lims >> (8 * p.cmd[0])) & 0xFF);
-          const int ne = ok ? max(0, min(8, lim0 - c0)) : 0;
-          if (ne == 8) {
-            __stcs(reinterpret_cast<uint4 *>(dst), v);
-          } else {
-            const __nv_bfloat16 *e = reinterpret_cast<const __nv_bfloat16 *>(&v);
-            for (int q2 = 0; q2 < ne; q2++) dst[q2] = e[q2];
-          }
-        }
-      }
+    if (!(kSAbl & 2)) s_store_box<__nv_bfloat16>(p, C, sm, STGb - sbase, ctab, t, tid, nthr, NB);
+  }
+}
+
+
+// ============================================================================================
+// FP64 (the paper's precision): the same streaming structure with DMMA m8n8k4 register blocks.
+// A unit is AR consecutive values of C's FVI times 8 rows (SM_T: one octet of X's FVI; SM_K:
+// 8 rows of the other m dims); thread (g, t) loads A(row g, k t) and B(k t, n g) as doubles
+// straight from the (swizzled) stage and from Y, and holds C(row g, n 2t / 2t+1) of each of its
+// AR blocks: the run C[a0 .. a0+AR-1, row g, n].
+template <int NB, int AR, bool TRANS>
+__global__ void __launch_bounds__(kSThreads, AR == 4 ? 2 : 1) tc_stream_f64_kernel(const __grid_constant__ SParams p) {
+  extern __shared__ __align__(1024) unsigned char smem_dyn[];
+  unsigned char *sm = smem_dyn + ((1024u - ((uint32_t)__cvta_generic_to_shared(smem_dyn) & 1023u)) & 1023u);
+  const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(sm);
+  const uint32_t FULL = sbase + p.off_bar, EMPTY = FULL + 8 * p.stages;
+  uint32_t *tab = reinterpret_cast<uint32_t *>(sm + p.off_tab);
+  double *ys = reinterpret_cast<double *>(sm + p.off_y);
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int ntl = (p.ntiles - (int)blockIdx.x + (int)gridDim.x - 1) / (int)gridDim.x;
+  {
+    const double *Y = static_cast<const double *>(p.Y);
+    const int tot = 8 * NB * p.YP;
+    for (int i = tid; i < tot; i += kSThreads) {
+      const int n = i / p.YP, k = i - n * p.YP;
+      ys[i] = (n < p.N && k < p.K) ? Y[(int64_t)k * p.ysk + (int64_t)n * p.ysn] : 0.0;
     }
+    for (int i = tid; i < p.nunits * 2 * p.ru + p.nchunk; i += kSThreads) tab[i] = __ldg(p.tab + i);
+  }
+  if (tid == 0) {
+    for (int s = 0; s < p.stages; s++) {
+      mbar_init(FULL + 8 * s, 1);
+      mbar_init(EMPTY + 8 * s, p.nunits);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+  }
+  __syncthreads();
+  if (warp == kSWarps) {
+    if (lane == 0) s_produce(p, ntl, sbase, FULL, EMPTY);
+    return;
+  }
+  if (warp >= p.nunits) return;
+  const uint32_t *ut = tab + warp * 2 * 8;
+  const int g = lane >> 2, t4 = lane & 3;
+  // A(row g, k t4) in a stage (a0, k-step origin): SM_T rows are 8 consecutive E (8 B apart)
+  // of the unit's octet, k rows xpitchk apart; SM_K rows are the unit's rows, k contiguous
+  const uint32_t xr = ut[g] + (TRANS ? (uint32_t)(t4 * p.xpitchk) : (uint32_t)(8 * t4));
+  const uint32_t kstep4 = TRANS ? (uint32_t)(4 * p.xpitchk) : 32u;
+  const uint32_t xpa = (uint32_t)p.xpitcha;
+  const int xsw = p.xswz;
+  const uint32_t bo = ut[8 + g];
+  const uint32_t *ctab = tab + p.nunits * 2 * 8;
+  const uint32_t STG = sbase + p.off_stg;
+  const int nthr = p.nunits * 32;
+  const double *yb0 = ys + g * p.YP + t4;
+  const double alpha = p.alpha64;
+  double *C = static_cast<double *>(p.C);
+  int s = 0;
+  uint32_t ph = 0;
+  for (int lt = 0; lt < ntl; lt++) {
+    double acc[AR][NB][2];
+#pragma unroll
+    for (int j = 0; j < AR; j++)
+#pragma unroll
+      for (int n = 0; n < NB; n++) acc[j][n][0] = acc[j][n][1] = 0.0;
+    for (int ks = 0; ks < p.nks; ks++) {
+      mbar_wait(FULL + 8 * s, ph);
+      const unsigned char *xs = sm + (uint32_t)(s * p.stage_pitch);
+      const int k0 = ks * p.KB;
+      const int nk4 = min(p.KB, p.KP - k0) >> 2;
+      for (int kk = 0; kk < ((kSAbl & 1) ? 0 : nk4); kk++) {
+        double bf[NB];
+#pragma unroll
+        for (int n = 0; n < NB; n++) bf[n] = yb0[n * 8 * p.YP + k0 + 4 * kk];
+        const uint32_t xa = xr + (uint32_t)kk * kstep4;
+#pragma unroll
+        for (int j = 0; j < AR; j++) {
+          const double av = *reinterpret_cast<const double *>(xs + s_swz(xa + (uint32_t)j * xpa, xsw));
+#pragma unroll
+          for (int n = 0; n < NB; n++) dmma884(acc[j][n][0], acc[j][n][1], av, bf[n]);
+        }
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(EMPTY + 8 * s);
+      if (++s == p.stages) { s = 0; ph ^= 1; }
+    }
+    const int t = (int)blockIdx.x + lt * (int)gridDim.x;
+    const uint32_t STGb = STG + (p.nstg == 2 ? (uint32_t)((lt & 1) * p.stg_pitch) : 0u);
+    if (p.nstg == 1) consumer_sync(nthr);
+    if (!(kSAbl & 2) && bo != 0xFFFFFFFFu) {
+#pragma unroll
+      for (int n = 0; n < NB; n++)
+#pragma unroll
+        for (int c2 = 0; c2 < 2; c2++) {
+          const uint32_t b = 8u * (bo + (uint32_t)((8 * n + 2 * t4 + c2) * p.cbsn));
+#pragma unroll
+          for (int j = 0; j < AR; j += 2)
+            asm volatile("st.shared.v2.f64 [%0], {%1,%2};\n" ::"r"(STGb + s_cswzb(b + 8u * j, p.cs1, p.cs2)),
+                         "d"(alpha * acc[j][n][c2]), "d"(alpha * acc[j + 1][n][c2]) : "memory");
+        }
+    }
+    consumer_sync(nthr);
+    if (!(kSAbl & 2)) s_store_box<double>(p, C, sm, STGb - sbase, ctab, t, tid, nthr, NB);
   }
 }
 

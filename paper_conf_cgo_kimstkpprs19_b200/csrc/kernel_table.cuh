@@ -44,8 +44,8 @@ F64Instance f64_instance_11(int v);
 const void *kernel_ptr_umma(int v, bool xk, bool yk, bool tma, size_t *smem, int *threads);   // tma: TMA producer
 // CTA-pair instances (BN = 128 BF16 / TF32 variants 12 / 22; nullptr otherwise)
 const void *kernel_ptr_umma_pair(int v, bool xk, bool yk, size_t *smem, int *threads);
-// the streaming BF16 kernel (kernels_stream.cu) for n8 blocks NB and m16 blocks per warp MB
-const void *stream_kernel_ptr(int NB, int MB, bool trans);
+// the streaming kernels (kernels_stream.cu): FP64 or BF16, n8 blocks NB, C-FVI runs AR, .trans A loads
+const void *stream_kernel_ptr(bool f64, int NB, int AR, bool trans);
 // BF16 operands, FP32 C (variants 11 / 12; cp.async producers; nullptr otherwise)
 const void *kernel_ptr_umma_f32out(int v, bool xk, bool yk, size_t *smem, int *threads);
 

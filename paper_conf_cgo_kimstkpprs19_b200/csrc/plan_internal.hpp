@@ -44,6 +44,7 @@ struct tc_plan_s {
   // the streaming path (stream.hpp): on when eligible unless opts / a forced variant say
   // otherwise; tc_execute takes it for beta == 0 when both tensor maps encode
   StreamCfg stream;
+  bool stream_active = false;   // tc_execute takes the path (preferred, or opts.stream == 2)
   int stream_grid = 0;     // persistent CTAs (SMs x resident CTAs)
   // batch (Hadamard) indices (R31): extent and element strides in X, Y, C.  tc_execute
   // launches the kernel once per batch slab with the operands offset to it — the kernels

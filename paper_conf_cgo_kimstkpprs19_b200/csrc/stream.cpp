@@ -23,6 +23,8 @@ namespace {
 // the kernel instances (kernels_stream.cu): n8 blocks NB = 1..4, runs AR = 4 (two CTAs per SM)
 // or 8 (one CTA per SM; not with NB = 4: 128 accumulator registers)
 bool instance_exists(int NB, int AR) { return NB >= 1 && NB <= 4 && (AR == 4 || (AR == 8 && NB <= 3)); }
+// FP64 (DMMA m8n8k4: 8-row units, accumulators 2 doubles per n8 block and a value)
+bool instance_exists_f64(int NB, int AR) { return NB >= 1 && NB <= 4 && (AR == 4 || (AR == 8 && NB <= 3)); }
 
 int round_up(int64_t x, int m) { return (int)((x + m - 1) / m * m); }
 
@@ -47,7 +49,11 @@ double run_eff(double r) { return r >= 128 ? 1.0 : r >= 64 ? 0.9 : r >= 32 ? 0.7
 bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s) {
   s = StreamCfg();
   auto no = [&](const char *why) { s.why = why; return false; };
-  if (kind != KIND_BF16_UMMA) return no("dtype");
+  if (kind != KIND_BF16_UMMA && kind != KIND_F64_DMMA) return no("dtype");
+  const bool f64 = kind == KIND_F64_DMMA;
+  const int es = f64 ? 8 : 2;
+  const int ru = f64 ? 8 : kSRows;   // rows of one MMA block: m8 (DMMA) / m16 (HMMA)
+  const int kq = f64 ? 4 : 16;       // k per MMA instruction
   for (auto &ix : c.ix) if (ix.cls == BATCH) return no("batch index");
   const int a = c.c_fvi();
   if (a < 0 || c.t[0].stride.empty() || c.t[0].stride[0] != 1 || c.t[0].idx[0] != a) return no("C's FVI");
@@ -66,15 +72,15 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s) {
   const int xr = (int)xv.idx.size();
   if (xr > kMaxTmaDims) return no("rank > 5");
   if (xv.stride[0] != 1) return no("X not unit-stride along its FVI");
-  const int es = 2;
   for (int j = 1; j < xr; j++)
     if ((xv.stride[j] * es) % 16 || xv.stride[j] >= ((int64_t)1 << 39)) return no("X strides (TMA)");
   const int64_t N = c.ix[nid].n, K = c.ix[kid].n;
   if (N > 32) return no("Y-side extent > 32");
   const int NB = (int)((N + 7) / 8), N8 = 8 * NB;
-  const int KP = round_up(K, 16), YP = KP + 8;
+  const int KP = round_up(K, kq);
+  const int YP = f64 ? round_up(KP, 16) + 4 : KP + 8;   // conflict-free B-fragment rows
   const size_t ybytes = (size_t)N8 * YP * es;
-  if (ybytes > 48 * 1024) return no("Y does not fit shared memory");
+  if (ybytes > (f64 ? 64 : 48) * 1024) return no("Y does not fit shared memory");
   const int x0 = xv.idx[0];
   if (x0 == a) return no("X's FVI is C's FVI (the tcgen05 path stores those runs directly)");
   const int mode = x0 == kid ? SM_K : SM_T;
@@ -93,7 +99,7 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s) {
   std::vector<int> Te = E >= 0 ? mult(c.ix[E].n, 8, 256) : std::vector<int>{1};
   std::vector<int> p2 = {1, 2, 4, 8, 16};
   std::vector<int> kbs;
-  for (int kb = 16; kb <= std::min(256, KP); kb += 16) kbs.push_back(kb);
+  for (int kb = f64 ? 8 : 16; kb <= std::min(f64 ? 64 : 256, KP); kb += f64 ? 8 : 16) kbs.push_back(kb);
   const double hbm = 6.5e12;
   double best = 1e30;
   StreamCfg bestc;
@@ -112,7 +118,7 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s) {
     std::vector<int> rt(rest.size());
     for (size_t q = 0; q < rest.size(); q++) { rt[q] = restopts[q][rix[q]]; rprod *= rt[q]; }
     for (int AR : {4, 8}) {
-      if (!instance_exists(NB, AR)) continue;
+      if (!(f64 ? instance_exists_f64(NB, AR) : instance_exists(NB, AR))) continue;
       // AR-element runs are stored as one vector: every C stride (and C's origin) a multiple of AR
       bool cal = cv.base % AR == 0;
       for (size_t j = 1; j < cv.stride.size(); j++) cal &= cv.stride[j] % AR == 0;
@@ -124,9 +130,9 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s) {
           //  computed but never stored)
           int64_t rowsets = 0;
           if (mode == SM_T) {
-            rowsets = ((int64_t)(te / 8) * rprod + 1) / 2;
+            rowsets = ((int64_t)(te / 8) * rprod + (ru / 8 - 1)) / (ru / 8);
           } else {
-            rowsets = rprod < 8 ? 0 : (rprod + kSRows - 1) / kSRows;
+            rowsets = rprod < 8 ? 0 : (rprod + ru - 1) / ru;
           }
           if (!rowsets) continue;
           const int64_t units = rowsets * (ta / AR);
@@ -161,15 +167,19 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s) {
             const int inner = (int)q.xbox[0] * es;
             const int swz = inner == 32 ? 1 : inner == 64 ? 2 : inner == 128 ? 3 : 0;
             const int stage = (int)(boxel * es);
-            const int64_t rows = (int64_t)units * kSRows * AR;   // tile rows (m)
+            const int64_t rows = (int64_t)units * ru * AR;   // tile rows (m)
             const size_t stg = (size_t)round_up(rows * N8 * es, 128);
-            const size_t tabb = (size_t)units * 2 * kSRows * 4 + (size_t)rows * N8 / 8 * 4;
-            const size_t fixed = 1024 + round_up((int64_t)ybytes, 128) + stg + round_up((int64_t)tabb, 64) + 16 * 8;
+            const size_t tabb = (size_t)units * 2 * ru * 4 + (size_t)rows * N8 * es / 16 * 4;
             const int occ = AR == 4 ? 2 : 1;
             const size_t cap = occ == 2 ? 115712 : 232448;
-            int stages = 0;
-            for (int st = 6; st >= 2; st--)
-              if (fixed + (size_t)st * round_up(stage, 1024) <= cap) { stages = st; break; }
+            // two C boxes when they leave >= 3 ring stages (one block-wide barrier per tile
+            // instead of two), else one
+            int stages = 0, nstg = 0;
+            for (int nb2 = 2; nb2 >= 1 && !stages; nb2--) {
+              const size_t fixed = 1024 + round_up((int64_t)ybytes, 128) + nb2 * stg + round_up((int64_t)tabb, 64) + 16 * 8;
+              for (int st = 6; st >= (nb2 == 2 ? 3 : 2); st--)
+                if (fixed + (size_t)st * round_up(stage, 1024) <= cap) { stages = st; nstg = nb2; break; }
+            }
             if (!stages) continue;
             int64_t tiles = 1;
             for (int id : mids) tiles *= (c.ix[id].n + T[id] - 1) / T[id];
@@ -217,6 +227,7 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s) {
               q.kp.KB = kb;
               q.kp.nks = nks;
               q.kp.stages = stages;
+              q.kp.nstg = nstg;
               q.kp.stage_bytes = stage;
               q.kp.ntiles = (int)tiles;
               q.kp.nunits = (int)units;
@@ -298,29 +309,31 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s) {
   };
   // units: u -> (row set p = u / agroups, a group g = u % agroups); 16 rows each
   const int agroups = T[a] / s.AR;
+  k.ru = ru;
   std::vector<uint32_t> xo, bo;
   for (int u = 0; u < k.nunits; u++) {
     const int p = u / agroups, a0 = (u % agroups) * s.AR;
-    for (int i = 0; i < kSRows; i++) {
+    for (int i = 0; i < ru; i++) {
       // the row's coordinates in the tile per raster dim (md order)
       int crd[kSMaxMdims] = {0, 0, 0, 0};
       int64_t ri;   // index into the rest enumeration (rest dims in X order, first fastest)
       crd[0] = a0;
       int64_t nrest = 1;
       for (int id : rest) nrest *= T[id];
-      const bool dummy = s.mode == SM_T ? (2 * p + (i >> 3)) >= (T[E] / 8) * nrest : (int64_t)kSRows * p + i >= nrest;
+      const int oct = (ru / 8) * p + (i >> 3);   // SM_T: the row's octet
+      const bool dummy = s.mode == SM_T ? oct >= (T[E] / 8) * nrest : (int64_t)ru * p + i >= nrest;
       if (dummy) {   // padding row: reads row 0 of the box, never stored
         xo.push_back(0);
         bo.push_back(0xFFFFFFFFu);
         continue;
       }
       if (s.mode == SM_T) {
-        const int oct = 2 * p + (i >> 3), eo = oct % (T[E] / 8);
+        const int eo = oct % (T[E] / 8);
         ri = oct / (T[E] / 8);
         for (int d = 0; d < k.nmd; d++)
           if (md[d] == E) crd[d] = 8 * eo + (i & 7);
       } else {
-        ri = (int64_t)kSRows * p + i;
+        ri = (int64_t)ru * p + i;
       }
       for (int id : rest) {
         const int v = (int)(ri % T[id]);
@@ -338,13 +351,14 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s) {
     }
   }
   for (int u = 0; u < k.nunits; u++) {
-    s.tab.insert(s.tab.end(), xo.begin() + kSRows * u, xo.begin() + kSRows * (u + 1));
-    s.tab.insert(s.tab.end(), bo.begin() + kSRows * u, bo.begin() + kSRows * (u + 1));
+    s.tab.insert(s.tab.end(), xo.begin() + ru * u, xo.begin() + ru * (u + 1));
+    s.tab.insert(s.tab.end(), bo.begin() + ru * u, bo.begin() + ru * (u + 1));
   }
   // per 16-B chunk of the C box (box order): its element offset in C from the tile origin
   int64_t cel = 1;
   for (int j = 0; j < cr; j++) cel *= k.cbox[j];
-  k.nchunk = (int)(cel / 8);
+  const int epc = 16 / es;   // elements per 16-B chunk
+  k.nchunk = (int)(cel / epc);
   {
     std::vector<int> bc(cr, 0);
     for (int ch = 0; ch < k.nchunk; ch++) {
@@ -353,35 +367,38 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s) {
       if (off > INT32_MAX) return no("tile spans more than 2^31 elements of C");
       s.tab.push_back((uint32_t)off);
       int j = 0;
-      bc[0] += 8;
+      bc[0] += epc;
       while (j < cr && bc[j] >= k.cbox[j]) { bc[j] = 0; if (++j < cr) bc[j]++; }
     }
   }
-  // staging swizzle: simulate the epilogue's 16-B writes (one warp instruction = its 32 lanes'
-  // runs at fixed (h, n8 block, c2)) and keep the fold with the fewest bank wavefronts
+  // staging swizzle: simulate the epilogue's writes (one warp instruction = its 32 lanes' runs
+  // of AR elements at fixed (row half h, n8 block, c2); per 16-B chunk) and keep the fold with
+  // the fewest bank wavefronts
   {
     const int sh[][2] = {{3, 6}, {2, 5}, {3, 5}, {1, 4}, {4, 8}, {2, 4}};
     long bestw = -1;
+    const int halves = ru / 8;
+    const int cpr = std::max(1, s.AR * es / 16);   // chunks per run
     for (auto &f : sh) {
       long wf = 0;
       for (int u = 0; u < k.nunits; u++)
-        for (int h = 0; h < 2; h++)
+        for (int h = 0; h < halves; h++)
           for (int nb = 0; nb < NB; nb++)
-            for (int c2 = 0; c2 < 2; c2++) {
-              int cnt[8] = {0};
-              for (int lane = 0; lane < 32; lane++) {
-                const int g = lane >> 2, t4 = lane & 3;
-                if (bo[kSRows * u + 8 * h + g] == 0xFFFFFFFFu) continue;
-                const int64_t el = bo[kSRows * u + 8 * h + g] + (int64_t)(8 * nb + 2 * t4 + c2) * k.cbsn;
-                const int64_t ch = el / 8;
-                const int64_t x = ch >> 3;
-                const int sw = (int)((ch ^ ((x ^ (x >> f[0]) ^ (x >> f[1])) & 7)) & 7);
-                cnt[sw] += s.AR == 8 ? 1 : 1;
+            for (int c2 = 0; c2 < 2; c2++)
+              for (int cc = 0; cc < cpr; cc++) {
+                int cnt[8] = {0};
+                for (int lane = 0; lane < 32; lane++) {
+                  const int g = lane >> 2, t4 = lane & 3;
+                  if (bo[ru * u + 8 * h + g] == 0xFFFFFFFFu) continue;
+                  const int64_t el = bo[ru * u + 8 * h + g] + (int64_t)(8 * nb + 2 * t4 + c2) * k.cbsn;
+                  const int64_t ch = el * es / 16 + cc;
+                  const int64_t x = ch >> 3;
+                  cnt[(int)((ch ^ ((x ^ (x >> f[0]) ^ (x >> f[1])) & 7)) & 7)]++;
+                }
+                int mx = 0;
+                for (int b = 0; b < 8; b++) mx = std::max(mx, cnt[b]);
+                wf += mx;
               }
-              int mx = 0;
-              for (int b = 0; b < 8; b++) mx = std::max(mx, cnt[b]);
-              wf += mx;
-            }
       if (bestw < 0 || wf < bestw) {
         bestw = wf;
         k.cs1 = f[0];
@@ -393,7 +410,8 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s) {
   k.stage_pitch = round_up(k.stage_bytes, 1024);
   int off = k.stages * k.stage_pitch;
   k.off_stg = off;
-  off += round_up(cel * es, 128);
+  k.stg_pitch = round_up(cel * es, 128);
+  off += k.nstg * k.stg_pitch;
   k.off_y = off;
   off += round_up((int64_t)ybytes, 128);
   k.off_tab = off;
@@ -403,6 +421,10 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s) {
   s.smem = (size_t)off + 1024;
   s.bytes = (double)(c.numel(1) + c.numel(2) + c.numel(0)) * es;
   s.on = s.smem <= (s.occ == 2 ? 115712u : 232448u);
+  // arithmetic intensity of the streamed contraction: 2 N K flops per X row of es (K + N) bytes;
+  // the FP64 ridge is 37.16 TFLOP/s / 6.55 TB/s = 5.7 (measured B200 peaks)
+  const double inten = 2.0 * N * K / (es * (double)(K + N));
+  s.preferred = !f64 || inten <= 0.8 * 5.67;
   if (!s.on) s.why = "shared memory";
   return s.on;
 }

@@ -43,6 +43,7 @@ struct SParams {
   int64_t csn;              // element stride of n in C
   int64_t mCs[kSMaxMdims];  // element strides of the m dims in C
   float alpha;
+  double alpha64;           // (FP64 kernel)
   int xrank;
   int nmd;                  // m dims, raster order (C's FVI first)
   int mT[kSMaxMdims], mNt[kSMaxMdims], mX[kSMaxMdims], mN[kSMaxMdims];
@@ -50,7 +51,8 @@ struct SParams {
   int K, N, KP, YP;         // k extent, n extent, k padded to 16, Y smem pitch (elements)
   int ntiles;
   int KB, nks;              // k per stage (box extent along k), k-steps per tile
-  int nunits;               // warp units per tile (<= kSWarps): (row octet pair, a group)
+  int nunits;               // warp units per tile (<= kSWarps): (row set, a group)
+  int ru;                   // rows per unit: 16 (BF16 m16n8k16) or 8 (FP64 DMMA m8n8k4)
   int stages, stage_bytes, stage_pitch;   // X ring: stages, box bytes, bytes between stages
   int xpitchk;              // SM_T: bytes between consecutive k in the X box
   int xpitcha;              // bytes between consecutive a in the X box
@@ -60,13 +62,17 @@ struct SParams {
   // fold(chunk >> 3) & 7, fold = x ^ x >> cs1 ^ x >> cs2: the planner's simulated choice),
   // stored by every compute thread as 16-B runs along C's FVI
   int crank, nchunk, cbsn;  // C box rank, 16-B chunks, box element stride of n
+  int nstg, stg_pitch;      // C boxes in smem (1 or 2: tile i+1 fills one while tile i's is stored)
   int cbox[kMaxTmaDims];    // C box extents (C order)
   int cmd[kMaxTmaDims];     // per C dim: its m dim (raster order), or -1 for n
   int cs1, cs2;             // staging swizzle fold shifts
 };
 
 struct StreamCfg {
-  bool on = false;
+  bool on = false;          // the contraction is a streaming shape (planned below)
+  bool preferred = false;   // ... and the path beats the tile kernels by default: always for BF16;
+                            // FP64 below 0.8 of the DMMA ridge (above it the DMMA tile kernel
+                            // keeps the pipe busier; tuning still times both)
   int NB = 0, AR = 0;       // kernel instance: n8 blocks, C-FVI run length per warp
   int X = 1;                // 1: X = A, 2: X = B
   int mode = SM_T;

@@ -13,6 +13,7 @@ import tcinputs
 from paper_conf_cgo_kimstkpprs19_b200 import binding as tc
 from paper_conf_cgo_kimstkpprs19_b200 import build
 from tests.test_gpu_bf16 import check_bf16
+from tests.test_gpu_parity import check_case
 
 pytestmark = pytest.mark.gpu
 
@@ -99,3 +100,17 @@ def test_stream_tuned_candidate():
     C = torch.empty(p.numel("C"), dtype=torch.bfloat16, device="cuda")
     t = p.tuned(A, B, C, topk=2, reps=1)
     assert 99 in [v for v, _ in t.info()["stats"]["tuned"]]
+
+
+# FP64 (the paper's precision): DMMA m8n8k4 streaming kernel, tolerance 1e-12 * S (north_star)
+@pytest.mark.parametrize("expr,ext", REDUCED + RAGGED, ids=[f"tccg{i + 1}" for i in range(8)] +
+                         [f"r{i}" for i in range(len(RAGGED))])
+def test_stream_f64(expr, ext):
+    s = tc.plan(expr, ext, "f64", host_only=True, stream=True).info()["stream"]
+    if s["on"] != 1:
+        pytest.skip(f"not a streaming shape: {s['why']}")
+    p = check_case(expr, ext, seed=11, integer=True, stream=True)
+    assert p.info()["stream"]["active"] == 1
+    check_case(expr, ext, seed=12, stream=True)
+    check_case(expr, ext, seed=13, alpha=0.75, stream=True)
+    check_case(expr, ext, seed=14, integer=True, alpha=2.0, beta=-1.0, stream=True)   # beta: tile kernel

@@ -387,8 +387,13 @@ def test_stream_path_planning():
         else:
             assert s["on"] == 0, (c.id, s)
     c1 = tcinputs.tccg48()[0]
-    for dt in ("f64", "f32", "tf32"):
+    for dt in ("f32", "tf32"):
         assert tc.plan(c1.expr, c1.extents, dt, host_only=True).info()["stream"]["on"] == 0
+    # FP64: streaming shapes too; used by default below 0.8 of the DMMA ridge (#6 / #8, K = 312,
+    # sit at the ridge: the tile kernel by default, tuning times both)
+    for c in tcinputs.tccg48()[:8]:
+        s = tc.plan(c.expr, c.extents, "f64", host_only=True).info()["stream"]
+        assert s["on"] == 1 and s["active"] == (0 if c.id in (6, 8) else 1), (c.id, s)
     assert tc.plan(c1.expr, c1.extents, "bf16", host_only=True, stream=False).info()["stream"]["on"] == 0
     # a forced variant keeps the path off unless asked for
     assert tc.plan(c1.expr, c1.extents, "bf16", host_only=True, variant=11).info()["stream"]["on"] == 0

@@ -33,17 +33,20 @@ cases += [(101, "abcde-efbad-cf", "a:20;b:3;c:13;d:5;e:44;f:9"),
           (103, "abc-dca-bd", "a:40;b:17;c:3;d:33"),
           (104, "abcd-ebad-ce", "a:24;b:5;c:31;d:3;e:17")]
 hbm = 6548.8
-if len(sys.argv) > 1:
+DT = sys.argv[2] if len(sys.argv) > 2 else "bf16"
+TDT = {"bf16": torch.bfloat16, "f64": torch.float64}[DT]
+ES = {"bf16": 2, "f64": 8}[DT]
+if len(sys.argv) > 1 and sys.argv[1] != "all":
     keep = {int(x) for x in sys.argv[1].split(",")}
     cases = [c for c in cases if c[0] in keep]
 for cid, expr, ext in cases:
-    ps = tc.plan(expr, ext, "bf16", stream=True)
-    pg = tc.plan(expr, ext, "bf16", stream=False)
+    ps = tc.plan(expr, ext, DT, stream=True)
+    pg = tc.plan(expr, ext, DT, stream=False)
     info = ps.info()["stream"]
-    A = tcinputs.uniform(ps.numel("A"), 1000 + cid, device="cuda").to(torch.bfloat16)
-    B = tcinputs.uniform(ps.numel("B"), 2000 + cid, device="cuda").to(torch.bfloat16)
-    Cs = torch.full((ps.numel("C"),), float("nan"), dtype=torch.bfloat16, device="cuda")
-    Cg = torch.full((ps.numel("C"),), float("nan"), dtype=torch.bfloat16, device="cuda")
+    A = tcinputs.uniform(ps.numel("A"), 1000 + cid, device="cuda").to(TDT)
+    B = tcinputs.uniform(ps.numel("B"), 2000 + cid, device="cuda").to(TDT)
+    Cs = torch.full((ps.numel("C"),), float("nan"), dtype=TDT, device="cuda")
+    Cg = torch.full((ps.numel("C"),), float("nan"), dtype=TDT, device="cuda")
     row = {"id": cid, "expr": expr, "stream": info}
     try:
         ps.execute(A, B, Cs)
@@ -56,7 +59,7 @@ for cid, expr, ext in cases:
         if cid <= 8:
             row["stream_ms"] = round(timeit(lambda: ps.execute(A, B, Cs), flush), 4)
             row["tcgen05_ms"] = round(timeit(lambda: pg.execute(A, B, Cg), flush), 4)
-            by = 2 * (ps.numel("A") + ps.numel("B") + ps.numel("C"))
+            by = ES * (ps.numel("A") + ps.numel("B") + ps.numel("C"))
             row["stream_hbm_frac"] = round(by / (row["stream_ms"] * 1e-3) / 1e9 / hbm, 4)
             row["tcgen05_hbm_frac"] = round(by / (row["tcgen05_ms"] * 1e-3) / 1e9 / hbm, 4)
     except Exception as e:  # noqa: BLE001
