@@ -431,7 +431,7 @@ def run_suite(name, args, flush, stream, dev, hbm):
         gbs = byts / (ms * 1e-3) / 1e9
         r = {"expr": c.expr, "extents": c.extents, "dtype": dt, "beta": beta, "ms": round(ms, 5),
              "gflops": round(p.flops / ms / 1e6, 2), "gbs": round(gbs, 1),
-             "variant": p.info()["variant"]}
+             "variant": "stream" if p.info()["stream"].get("active", 0) == 1 else p.info()["variant"]}
         if dt == "f64":
             attain = min(FP64_PEAK_TFLOPS * 1e12, p.flops / byts * hbm)
             r["roofline_frac"] = round(p.flops / (ms * 1e-3) / attain, 4)
@@ -491,6 +491,9 @@ def run_libtc(args):
 
     def kname(p):
         i = p.info()
+        s = i["stream"]
+        if s.get("active"):   # the streaming path (stream.hpp)
+            return f"tc_stream_f64_kernel<{s['NB']},{s['AR']},{'true' if s['mode'] == 'T' else 'false'}>"
         return (f"tc_f64_dmma_kernel<{i['BM']},{i['BN']},{i['BK']},{i['WM']},{i['WN']},{i['stages']},4,"
                 f"{i['occ']},{i['xKmajor']},{i['yKmajor']},{i['stg']}>")
 
@@ -604,9 +607,11 @@ def run_libtc(args):
     per_case = []
     for w, ms in zip(work, med):
         c, p = w[0], w[1]
+        ri = run_plan(w).info()
+        act = ri["stream"].get("active", 0) == 1
         per_case.append({"id": c.id, "ms": round(ms, 5), "gflops": round(p.flops / ms / 1e6, 2),
-                         "variant": run_plan(w).info()["variant"],
-                         "pred_ms": round(run_plan(w).info()["t_pred_ms"], 5)})
+                         "variant": "stream" if act else ri["variant"],
+                         "pred_ms": round(ri["stream"]["t_pred_ms"] if act else ri["t_pred_ms"], 5)})
     value = geomean([r["gflops"] for r in per_case])
 
     # cost-model fidelity (outside the timed region): the model's predicted time of the plan
@@ -618,7 +623,9 @@ def run_libtc(args):
             r["model_err"] = round(r["pred_ms"] / r["ms"] - 1.0, 4)
             errs.append(abs(r["model_err"]))
             pm = model_pick[w[0].id]
-            pm_ms = r["ms"] if pm.info()["variant"] == r["variant"] and pm.info()["t_pred_ms"] == r["pred_ms"] \
+            pmi = pm.info()
+            pm_var = "stream" if pmi["stream"].get("active", 0) == 1 else pmi["variant"]
+            pm_ms = r["ms"] if pm_var == r["variant"] and run_plan(w) is pm \
                 else time_one(pm, w[2], w[3], w[4], 3, 1, flush, stream)
             r["model_pick_ms"] = round(pm_ms, 5)
             picks.append(pm_ms / r["ms"])
@@ -802,6 +809,12 @@ def run_libtc(args):
                            "parallelism": f"C-slab shard x{world}" if sharded else "single GPU"},
                 "roofline": roof,
                 "roofline_geomean_frac": round(geomean(fr), 4),
+                # per TCCG class (SURVEY App. A groups): geomean of achieved / min(FP64 peak, I * HBM)
+                "roofline_frac_by_class": {
+                    name: round(geomean([f for (w, f) in zip(work, fr) if lo <= w[0].id <= hi]), 4)
+                    for name, lo, hi in (("memory_bound_1_8", 1, 8), ("compute_bound_9_30", 9, 30),
+                                         ("near_ridge_ccsdt_31_48", 31, 48))
+                    if any(lo <= w[0].id <= hi for w in work)},
                 "cpu_baseline": cpu, "e2e": e2e,
                 "gpu_launches": len(work) * args.steps,
                 "clocks": clk,
