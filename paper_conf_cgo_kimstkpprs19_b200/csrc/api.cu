@@ -205,7 +205,7 @@ Status upload(tc_plan_s *P, std::string &err) {
   P->d_packY2 = (const uint32_t *)(b + parts[iY2p].off);
   if (P->stream.on) {
     P->stream.kp.tab = (const uint32_t *)(b + parts[iS].off);
-    const void *fn = stream_kernel_ptr(P->dtype == TC_F64, P->stream.NB, P->stream.AR, P->stream.mode != SM_K);
+    const void *fn = stream_kernel_ptr(P->cfg.kind, P->stream.NB, P->stream.AR, P->stream.mode != SM_K);
     if (!fn) { err = "no streaming kernel instance for the plan"; return ST_UNSUPPORTED; }
     // (the instance is shared by plans of different sizes: always the opt-in maximum)
     e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448);
@@ -449,7 +449,7 @@ bool encode_stream_maps(const tc_plan_s *P, const void *Xp, void *C, SParams &sp
   auto enc = tma_encoder();
   if (!enc) return false;
   const StreamCfg &s = P->stream;
-  const int es = P->dtype == TC_F64 ? 8 : 2;
+  const int es = kind_esize(P->cfg.kind);
   const char *xb = (const char *)Xp + es * s.xbase;
   const char *cb = (const char *)C + es * s.cbase;
   if ((uintptr_t)xb % 16 || (uintptr_t)cb % 16) return false;
@@ -461,7 +461,8 @@ bool encode_stream_maps(const tc_plan_s *P, const void *Xp, void *C, SParams &sp
     el[j] = 1;
     if (j > 0) strides[j - 1] = (cuuint64_t)(s.xstr[j] * es);
   }
-  return enc(reinterpret_cast<CUtensorMap *>(&sp.xmap), es == 8 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT64 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, (cuuint32_t)s.xrank,
+  return enc(reinterpret_cast<CUtensorMap *>(&sp.xmap),
+             es == 8 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT64 : es == 4 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, (cuuint32_t)s.xrank,
              (void *)xb, dims, strides, box, el, CU_TENSOR_MAP_INTERLEAVE_NONE, (CUtensorMapSwizzle)s.xswz,
 #ifdef TC_STREAM_PROMO
              (CUtensorMapL2promotion)TC_STREAM_PROMO,
@@ -906,7 +907,7 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
       sp.C = static_cast<char *>(C) + es * plan->stream.cbase;
       sp.alpha = (float)alpha;
       sp.alpha64 = alpha;
-      const void *fn = stream_kernel_ptr(plan->dtype == TC_F64, plan->stream.NB, plan->stream.AR, plan->stream.mode != SM_K);
+      const void *fn = stream_kernel_ptr(plan->cfg.kind, plan->stream.NB, plan->stream.AR, plan->stream.mode != SM_K);
       const int grid = std::min(sp.ntiles, plan->stream_grid);
       void *sargs[] = {&sp};
       cudaError_t e = cudaLaunchKernel(fn, dim3(grid), dim3(kSThreads), sargs, plan->stream.smem, (cudaStream_t)stream);

@@ -342,15 +342,19 @@ __global__ void __launch_bounds__(kSThreads, AR == 4 ? 2 : 1) tc_stream_f64_kern
   const int g = lane >> 2, t4 = lane & 3;
   // A(row g, k t4) in a stage (a0, k-step origin): SM_T rows are 8 consecutive E (8 B apart)
   // of the unit's octet, k rows xpitchk apart; SM_K rows are the unit's rows, k contiguous
-  const uint32_t xr = ut[g] + (TRANS ? (uint32_t)(t4 * p.xpitchk) : (uint32_t)(8 * t4));
-  const uint32_t kstep4 = TRANS ? (uint32_t)(4 * p.xpitchk) : 32u;
+  // k of thread t in DMMA step kk: SM_T takes k = 8 (kk / 2) + kk % 2 + 2 t (every other k row,
+  // so the four k rows of one step fall in different swizzle phases of the 128-B box rows: no
+  // bank conflicts); SM_K the plain k = 4 kk + t (rows are m rows there)
+  const uint32_t xks = TRANS ? (uint32_t)p.xpitchk : 8u;   // bytes per k in the stage
+  const int lk = TRANS ? 2 * t4 : t4;
+  const uint32_t xr = ut[g] + (uint32_t)lk * xks;
   const uint32_t xpa = (uint32_t)p.xpitcha;
   const int xsw = p.xswz;
   const uint32_t bo = ut[8 + g];
   const uint32_t *ctab = tab + p.nunits * 2 * 8;
   const uint32_t STG = sbase + p.off_stg;
   const int nthr = p.nunits * 32;
-  const double *yb0 = ys + g * p.YP + t4;
+  const double *yb0 = ys + g * p.YP + lk;
   const double alpha = p.alpha64;
   double *C = static_cast<double *>(p.C);
   int s = 0;
@@ -367,10 +371,11 @@ __global__ void __launch_bounds__(kSThreads, AR == 4 ? 2 : 1) tc_stream_f64_kern
       const int k0 = ks * p.KB;
       const int nk4 = min(p.KB, p.KP - k0) >> 2;
       for (int kk = 0; kk < ((kSAbl & 1) ? 0 : nk4); kk++) {
+        const int kofs = TRANS ? 8 * (kk >> 1) + (kk & 1) : 4 * kk;
         double bf[NB];
 #pragma unroll
-        for (int n = 0; n < NB; n++) bf[n] = yb0[n * 8 * p.YP + k0 + 4 * kk];
-        const uint32_t xa = xr + (uint32_t)kk * kstep4;
+        for (int n = 0; n < NB; n++) bf[n] = yb0[n * 8 * p.YP + k0 + kofs];
+        const uint32_t xa = xr + (uint32_t)kofs * xks;
 #pragma unroll
         for (int j = 0; j < AR; j++) {
           const double av = *reinterpret_cast<const double *>(xs + s_swz(xa + (uint32_t)j * xpa, xsw));
@@ -399,6 +404,149 @@ __global__ void __launch_bounds__(kSThreads, AR == 4 ? 2 : 1) tc_stream_f64_kern
     }
     consumer_sync(nthr);
     if (!(kSAbl & 2)) s_store_box<double>(p, C, sm, STGb - sbase, ctab, t, tid, nthr, NB);
+  }
+}
+
+
+// ============================================================================================
+// FP32 storage: TF32 products (mma.sync m16n8k8 .tf32, the tensor core reads the FP32 bits,
+// DESIGN R30) or FP32 as three TF32 products (SPLIT: hi = x & 0xFFFFE000, lo = x - hi;
+// lo*hi + hi*lo + hi*hi, R32).  Same units, C runs and store phase as the BF16 kernel; the
+// fragments are single 32-bit elements, loaded with plain shared loads (ldmatrix cannot
+// transpose 32-bit elements).
+__device__ __forceinline__ void mma_tf32_1688(float (&d)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1) {
+  asm("mma.sync.aligned.m16n8k8.row.col.f32.tf32.tf32.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
+      "{%0,%1,%2,%3};\n"
+      : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3])
+      : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1));
+}
+__device__ __forceinline__ uint32_t tf32_hi(uint32_t x) { return x & 0xFFFFE000u; }
+__device__ __forceinline__ uint32_t tf32_lo(uint32_t x) {
+  return __float_as_uint(__uint_as_float(x) - __uint_as_float(x & 0xFFFFE000u));
+}
+
+template <int NB, int AR, bool TRANS, bool SPLIT>
+__global__ void __launch_bounds__(kSThreads, AR == 4 ? 2 : 1) tc_stream_tf32_kernel(const __grid_constant__ SParams p) {
+  extern __shared__ __align__(1024) unsigned char smem_dyn[];
+  unsigned char *sm = smem_dyn + ((1024u - ((uint32_t)__cvta_generic_to_shared(smem_dyn) & 1023u)) & 1023u);
+  const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(sm);
+  const uint32_t FULL = sbase + p.off_bar, EMPTY = FULL + 8 * p.stages;
+  uint32_t *tab = reinterpret_cast<uint32_t *>(sm + p.off_tab);
+  float *ys = reinterpret_cast<float *>(sm + p.off_y);
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int ntl = (p.ntiles - (int)blockIdx.x + (int)gridDim.x - 1) / (int)gridDim.x;
+  {
+    const float *Y = static_cast<const float *>(p.Y);
+    const int tot = 8 * NB * p.YP;
+    for (int i = tid; i < tot; i += kSThreads) {
+      const int n = i / p.YP, k = i - n * p.YP;
+      ys[i] = (n < p.N && k < p.K) ? Y[(int64_t)k * p.ysk + (int64_t)n * p.ysn] : 0.f;
+    }
+    for (int i = tid; i < p.nunits * 2 * p.ru + p.nchunk; i += kSThreads) tab[i] = __ldg(p.tab + i);
+  }
+  if (tid == 0) {
+    for (int s = 0; s < p.stages; s++) {
+      mbar_init(FULL + 8 * s, 1);
+      mbar_init(EMPTY + 8 * s, p.nunits);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+  }
+  __syncthreads();
+  if (warp == kSWarps) {
+    if (lane == 0) s_produce(p, ntl, sbase, FULL, EMPTY);
+    return;
+  }
+  if (warp >= p.nunits) return;
+  const uint32_t *ut = tab + warp * 2 * kSRows;
+  const int g = lane >> 2, t4 = lane & 3;
+  const uint32_t xks = TRANS ? (uint32_t)p.xpitchk : 4u;   // bytes per k in the stage
+  // A(row g | g + 8, k t4 | t4 + 4): the unit's rows g and g + 8
+  const uint32_t xr0 = ut[g] + (uint32_t)t4 * xks, xr1 = ut[8 + g] + (uint32_t)t4 * xks;
+  const uint32_t xpa = (uint32_t)p.xpitcha;
+  const int xsw = p.xswz;
+  const uint32_t bo0 = ut[kSRows + g], bo1 = ut[kSRows + 8 + g];
+  const uint32_t *ctab = tab + p.nunits * 2 * kSRows;
+  const uint32_t STG = sbase + p.off_stg;
+  const int nthr = p.nunits * 32;
+  const float *yb0 = ys + g * p.YP + t4;
+  const float alpha = p.alpha;
+  float *C = static_cast<float *>(p.C);
+  int s = 0;
+  uint32_t ph = 0;
+  for (int lt = 0; lt < ntl; lt++) {
+    float acc[AR][NB][4];
+#pragma unroll
+    for (int j = 0; j < AR; j++)
+#pragma unroll
+      for (int n = 0; n < NB; n++)
+#pragma unroll
+        for (int e = 0; e < 4; e++) acc[j][n][e] = 0.f;
+    for (int ks = 0; ks < p.nks; ks++) {
+      mbar_wait(FULL + 8 * s, ph);
+      const unsigned char *xs = sm + (uint32_t)(s * p.stage_pitch);
+      const int k0 = ks * p.KB;
+      const int nk8 = min(p.KB, p.KP - k0) >> 3;
+      for (int kk = 0; kk < ((kSAbl & 1) ? 0 : nk8); kk++) {
+        uint32_t bh[NB][2], bl[NB][2];
+#pragma unroll
+        for (int n = 0; n < NB; n++) {
+          const float *yb = yb0 + n * 8 * p.YP + k0 + 8 * kk;
+          const uint32_t v0 = __float_as_uint(yb[0]), v1 = __float_as_uint(yb[4]);
+          bh[n][0] = SPLIT ? tf32_hi(v0) : v0;
+          bh[n][1] = SPLIT ? tf32_hi(v1) : v1;
+          if (SPLIT) { bl[n][0] = tf32_lo(v0); bl[n][1] = tf32_lo(v1); }
+        }
+        const uint32_t ko = (uint32_t)(8 * kk) * xks, ko4 = ko + 4u * xks;
+#pragma unroll
+        for (int j = 0; j < AR; j++) {
+          const uint32_t jo = (uint32_t)j * xpa;
+          uint32_t a[4] = {*reinterpret_cast<const uint32_t *>(xs + s_swz(xr0 + jo + ko, xsw)),
+                           *reinterpret_cast<const uint32_t *>(xs + s_swz(xr1 + jo + ko, xsw)),
+                           *reinterpret_cast<const uint32_t *>(xs + s_swz(xr0 + jo + ko4, xsw)),
+                           *reinterpret_cast<const uint32_t *>(xs + s_swz(xr1 + jo + ko4, xsw))};
+          if (SPLIT) {
+            uint32_t ah[4], al[4];
+#pragma unroll
+            for (int e = 0; e < 4; e++) { ah[e] = tf32_hi(a[e]); al[e] = tf32_lo(a[e]); }
+#pragma unroll
+            for (int n = 0; n < NB; n++) {   // small terms first: lo*hi, hi*lo, then hi*hi
+              mma_tf32_1688(acc[j][n], al, bh[n][0], bh[n][1]);
+              mma_tf32_1688(acc[j][n], ah, bl[n][0], bl[n][1]);
+              mma_tf32_1688(acc[j][n], ah, bh[n][0], bh[n][1]);
+            }
+          } else {
+#pragma unroll
+            for (int n = 0; n < NB; n++) mma_tf32_1688(acc[j][n], a, bh[n][0], bh[n][1]);
+          }
+        }
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(EMPTY + 8 * s);
+      if (++s == p.stages) { s = 0; ph ^= 1; }
+    }
+    const int t = (int)blockIdx.x + lt * (int)gridDim.x;
+    const uint32_t STGb = STG + (p.nstg == 2 ? (uint32_t)((lt & 1) * p.stg_pitch) : 0u);
+    if (p.nstg == 1) consumer_sync(nthr);
+    if (!(kSAbl & 2)) {
+#pragma unroll
+      for (int h = 0; h < 2; h++)
+#pragma unroll
+        for (int n = 0; n < NB; n++)
+#pragma unroll
+          for (int c2 = 0; c2 < 2; c2++) {
+            const uint32_t boh = h ? bo1 : bo0;
+            if (boh == 0xFFFFFFFFu) continue;   // a padding row
+            const uint32_t b = 4u * (boh + (uint32_t)((8 * n + 2 * t4 + c2) * p.cbsn));
+#pragma unroll
+            for (int j = 0; j < AR; j += 4)
+              asm volatile("st.shared.v4.f32 [%0], {%1,%2,%3,%4};\n" ::"r"(STGb + s_cswzb(b + 4u * j, p.cs1, p.cs2)),
+                           "f"(alpha * acc[j][n][2 * h + c2]), "f"(alpha * acc[j + 1][n][2 * h + c2]),
+                           "f"(alpha * acc[j + 2][n][2 * h + c2]), "f"(alpha * acc[j + 3][n][2 * h + c2])
+                           : "memory");
+          }
+    }
+    consumer_sync(nthr);
+    if (!(kSAbl & 2)) s_store_box<float>(p, C, sm, STGb - sbase, ctab, t, tid, nthr, NB);
   }
 }
 

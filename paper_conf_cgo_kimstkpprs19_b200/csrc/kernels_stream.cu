@@ -1,26 +1,37 @@
-// kernels_stream.cu — instances of the streaming kernels (kernel_stream.cuh): FP64 (DMMA) or BF16
-// (mma.sync) x NB n8 blocks (n <= 8 NB) x AR-long runs of C's FVI per warp x .trans or plain A
-// loads (stream.cpp instance_exists / instance_exists_f64 keep the lists in step).
+// kernels_stream.cu — instances of the streaming kernels (kernel_stream.cuh): FP64 (DMMA), BF16
+// (mma.sync m16n8k16), TF32 / FP32-split (mma.sync m16n8k8) x NB n8 blocks (n <= 8 NB) x
+// AR-long runs of C's FVI per warp x .trans / plain A loads (stream.cpp instance_exists keeps
+// the lists in step).  kind: tiles.hpp Kind.
 #include "kernel_stream.cuh"
+#include "tiles.hpp"
 
 namespace tc {
 
 template <int NB, int AR>
-static const void *spick(bool f64, bool trans) {
-  if (f64)
-    return trans ? (const void *)&tc_stream_f64_kernel<NB, AR, true> : (const void *)&tc_stream_f64_kernel<NB, AR, false>;
-  return trans ? (const void *)&tc_stream_bf16_kernel<NB, AR, true> : (const void *)&tc_stream_bf16_kernel<NB, AR, false>;
+static const void *spick(int kind, bool trans) {
+  switch (kind) {
+    case KIND_F64_DMMA:
+      return trans ? (const void *)&tc_stream_f64_kernel<NB, AR, true> : (const void *)&tc_stream_f64_kernel<NB, AR, false>;
+    case KIND_BF16_UMMA:
+      return trans ? (const void *)&tc_stream_bf16_kernel<NB, AR, true> : (const void *)&tc_stream_bf16_kernel<NB, AR, false>;
+    case KIND_TF32_UMMA:
+      return trans ? (const void *)&tc_stream_tf32_kernel<NB, AR, true, false>
+                   : (const void *)&tc_stream_tf32_kernel<NB, AR, false, false>;
+    default:
+      return trans ? (const void *)&tc_stream_tf32_kernel<NB, AR, true, true>
+                   : (const void *)&tc_stream_tf32_kernel<NB, AR, false, true>;
+  }
 }
 
-const void *stream_kernel_ptr(bool f64, int NB, int AR, bool trans) {
+const void *stream_kernel_ptr(int kind, int NB, int AR, bool trans) {
   switch (NB * 16 + AR) {
-    case 1 * 16 + 4: return spick<1, 4>(f64, trans);
-    case 1 * 16 + 8: return spick<1, 8>(f64, trans);
-    case 2 * 16 + 4: return spick<2, 4>(f64, trans);
-    case 2 * 16 + 8: return spick<2, 8>(f64, trans);
-    case 3 * 16 + 4: return spick<3, 4>(f64, trans);
-    case 3 * 16 + 8: return spick<3, 8>(f64, trans);
-    case 4 * 16 + 4: return spick<4, 4>(f64, trans);
+    case 1 * 16 + 4: return spick<1, 4>(kind, trans);
+    case 1 * 16 + 8: return spick<1, 8>(kind, trans);
+    case 2 * 16 + 4: return spick<2, 4>(kind, trans);
+    case 2 * 16 + 8: return spick<2, 8>(kind, trans);
+    case 3 * 16 + 4: return spick<3, 4>(kind, trans);
+    case 3 * 16 + 8: return spick<3, 8>(kind, trans);
+    case 4 * 16 + 4: return spick<4, 4>(kind, trans);
   }
   return nullptr;
 }

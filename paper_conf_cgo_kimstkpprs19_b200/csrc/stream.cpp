@@ -49,11 +49,10 @@ double run_eff(double r) { return r >= 128 ? 1.0 : r >= 64 ? 0.9 : r >= 32 ? 0.7
 bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s) {
   s = StreamCfg();
   auto no = [&](const char *why) { s.why = why; return false; };
-  if (kind != KIND_BF16_UMMA && kind != KIND_F64_DMMA) return no("dtype");
   const bool f64 = kind == KIND_F64_DMMA;
-  const int es = f64 ? 8 : 2;
-  const int ru = f64 ? 8 : kSRows;   // rows of one MMA block: m8 (DMMA) / m16 (HMMA)
-  const int kq = f64 ? 4 : 16;       // k per MMA instruction
+  const int es = kind_esize(kind);   // 8 FP64, 2 BF16, 4 TF32 / FP32 split
+  const int ru = f64 ? 8 : kSRows;   // rows of one MMA block: m8 (DMMA) / m16 (mma.sync)
+  const int kq = es == 2 ? 16 : 8;   // k granule: one HMMA k16 / one TF32 k8 / two DMMA k4 steps
   for (auto &ix : c.ix) if (ix.cls == BATCH) return no("batch index");
   const int a = c.c_fvi();
   if (a < 0 || c.t[0].stride.empty() || c.t[0].stride[0] != 1 || c.t[0].idx[0] != a) return no("C's FVI");
@@ -78,7 +77,8 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s) {
   if (N > 32) return no("Y-side extent > 32");
   const int NB = (int)((N + 7) / 8), N8 = 8 * NB;
   const int KP = round_up(K, kq);
-  const int YP = f64 ? round_up(KP, 16) + 4 : KP + 8;   // conflict-free B-fragment rows
+  // conflict-free B-fragment rows (8 rows n at consecutive 8 / 4 threads' k)
+  const int YP = es == 8 ? round_up(KP, 16) + 4 : es == 4 ? round_up(KP, 32) + 4 : KP + 8;
   const size_t ybytes = (size_t)N8 * YP * es;
   if (ybytes > (f64 ? 64 : 48) * 1024) return no("Y does not fit shared memory");
   const int x0 = xv.idx[0];
@@ -99,7 +99,7 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s) {
   std::vector<int> Te = E >= 0 ? mult(c.ix[E].n, 8, 256) : std::vector<int>{1};
   std::vector<int> p2 = {1, 2, 4, 8, 16};
   std::vector<int> kbs;
-  for (int kb = f64 ? 8 : 16; kb <= std::min(f64 ? 64 : 256, KP); kb += f64 ? 8 : 16) kbs.push_back(kb);
+  for (int kb = kq; kb <= std::min(f64 ? 64 : es == 4 ? 128 : 256, KP); kb += kq) kbs.push_back(kb);
   const double hbm = 6.5e12;
   double best = 1e30;
   StreamCfg bestc;
@@ -424,7 +424,9 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s) {
   // arithmetic intensity of the streamed contraction: 2 N K flops per X row of es (K + N) bytes;
   // the FP64 ridge is 37.16 TFLOP/s / 6.55 TB/s = 5.7 (measured B200 peaks)
   const double inten = 2.0 * N * K / (es * (double)(K + N));
-  s.preferred = !f64 || inten <= 0.8 * 5.67;
+  // 32-bit operands in SM_K: the plain k-contiguous fragment loads lose to the tcgen05 path
+  // (TCCG #7 / #8 in TF32 and split FP32, measured): tuning still times both
+  s.preferred = f64 ? inten <= 0.8 * 5.67 : (es == 2 || s.mode == SM_T);
   if (!s.on) s.why = "shared memory";
   return s.on;
 }

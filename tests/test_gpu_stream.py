@@ -13,6 +13,7 @@ import tcinputs
 from paper_conf_cgo_kimstkpprs19_b200 import binding as tc
 from paper_conf_cgo_kimstkpprs19_b200 import build
 from tests.test_gpu_bf16 import check_bf16
+from tests.test_gpu_f32 import check_f32
 from tests.test_gpu_parity import check_case
 
 pytestmark = pytest.mark.gpu
@@ -114,3 +115,17 @@ def test_stream_f64(expr, ext):
     check_case(expr, ext, seed=12, stream=True)
     check_case(expr, ext, seed=13, alpha=0.75, stream=True)
     check_case(expr, ext, seed=14, integer=True, alpha=2.0, beta=-1.0, stream=True)   # beta: tile kernel
+
+
+# FP32 storage: TF32 products (R30 tolerance) and FP32 as split TF32 (1e-5 * S, R32)
+@pytest.mark.parametrize("dtype", ["tf32", "f32"])
+@pytest.mark.parametrize("expr,ext", REDUCED + RAGGED, ids=[f"tccg{i + 1}" for i in range(8)] +
+                         [f"r{i}" for i in range(len(RAGGED))])
+def test_stream_fp32(expr, ext, dtype):
+    s = tc.plan(expr, ext, dtype, host_only=True, stream=True).info()["stream"]
+    if s["on"] != 1:
+        pytest.skip(f"not a streaming shape: {s['why']}")
+    check_f32(expr, ext, dtype, seed=21, integer=True, stream=True)
+    assert tc.plan(expr, ext, dtype, host_only=True, stream=True).info()["stream"]["active"] == 1
+    check_f32(expr, ext, dtype, seed=22, stream=True)
+    check_f32(expr, ext, dtype, seed=23, alpha=-1.5, stream=True)

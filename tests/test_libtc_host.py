@@ -387,8 +387,11 @@ def test_stream_path_planning():
         else:
             assert s["on"] == 0, (c.id, s)
     c1 = tcinputs.tccg48()[0]
+    # FP32 storage (TF32 / split FP32): streaming shapes; by default in SM_T only
     for dt in ("f32", "tf32"):
-        assert tc.plan(c1.expr, c1.extents, dt, host_only=True).info()["stream"]["on"] == 0
+        for c in tcinputs.tccg48()[:8]:
+            s = tc.plan(c.expr, c.extents, dt, host_only=True).info()["stream"]
+            assert s["on"] == 1 and s["active"] == (0 if c.id in (7, 8) else 1), (dt, c.id, s)
     # FP64: streaming shapes too; used by default below 0.8 of the DMMA ridge (#6 / #8, K = 312,
     # sit at the ridge: the tile kernel by default, tuning times both)
     for c in tcinputs.tccg48()[:8]:

@@ -34,8 +34,8 @@ cases += [(101, "abcde-efbad-cf", "a:20;b:3;c:13;d:5;e:44;f:9"),
           (104, "abcd-ebad-ce", "a:24;b:5;c:31;d:3;e:17")]
 hbm = 6548.8
 DT = sys.argv[2] if len(sys.argv) > 2 else "bf16"
-TDT = {"bf16": torch.bfloat16, "f64": torch.float64}[DT]
-ES = {"bf16": 2, "f64": 8}[DT]
+TDT = {"bf16": torch.bfloat16, "f64": torch.float64, "f32": torch.float32, "tf32": torch.float32}[DT]
+ES = {"bf16": 2, "f64": 8, "f32": 4, "tf32": 4}[DT]
 if len(sys.argv) > 1 and sys.argv[1] != "all":
     keep = {int(x) for x in sys.argv[1].split(",")}
     cases = [c for c in cases if c[0] in keep]
@@ -52,7 +52,7 @@ for cid, expr, ext in cases:
         ps.execute(A, B, Cs)
         pg.execute(A, B, Cg)
         torch.cuda.synchronize()
-        d = (Cs.float() - Cg.float()).abs()
+        d = (Cs.double() - Cg.double()).abs()
         row["nan"] = int(torch.isnan(Cs.float()).sum())
         row["maxdiff"] = float(d.max())
         row["maxabs"] = float(Cg.float().abs().max())
