@@ -177,7 +177,7 @@ double model_time(const Contraction &c, Config &cfg, const Variant &v, WfCache *
   const double l2b = nctas * steps * 32.0 * (cfg.secX + cfg.secY) * (pair ? 0.5 : 1.0) + bc / eS;
   cfg.t_l2 = l2b / kL2Bw;
   cfg.flops_pad = 2.0 * nctas * steps * v.BM * v.BN * v.BK;
-  cfg.t_pred = std::max({cfg.t_comp, cfg.t_mem, cfg.t_l2}) + kLaunch;
+  cfg.t_pred = std::max({cfg.t_comp, cfg.t_mem, cfg.t_l2}) * v.cal + kLaunch;
   return cfg.t_pred;
 }
 

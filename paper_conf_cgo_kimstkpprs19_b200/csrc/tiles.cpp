@@ -23,6 +23,17 @@ const std::vector<Variant> &variants() {
     // FP32 as split TF32 (hi + lo planes per stage: twice the smem per stage)
     t[23] = Variant{128, 64, 32, 32, 32, 3, 4, 1, KIND_F32X3_UMMA};
     t[24] = Variant{128, 128, 32, 32, 32, 2, 4, 1, KIND_F32X3_UMMA};
+    // Calibration of the B200 model per FP64 variant: the median over the TCCG-48 cases of
+    // measured / predicted time of the variant's best configuration (tools/model_calib.py on
+    // one B200, profiles/r02_model_calib.jsonl; 10 ranked variants x 48 cases).  The model
+    // counts pipes and bytes; what it misses (issue, latency, epilogue drains) is per kernel
+    // shape.  With it the model's first choice is within 10 % of the fastest ranked variant on
+    // 46 / 48 cases (leave-one-case-out fits: the same 46), against 3 / 48 without.
+    const double cal[][2] = {{0, 1.094}, {1, 1.114}, {2, 1.284}, {3, 1.307}, {4, 1.132}, {5, 1.131},
+                             {6, 1.383}, {7, 1.405}, {8, 1.557}, {9, 1.539}, {10, 1.220}, {13, 1.840},
+                             {14, 1.802}, {15, 1.842}, {16, 2.766}, {17, 1.924}, {18, 1.351},
+                             {19, 2.392}, {20, 2.108}, {25, 1.374}, {26, 2.862}};
+    for (auto &c : cal) t[(int)c[0]].cal = c[1];
     return t;
   }();
   return v;

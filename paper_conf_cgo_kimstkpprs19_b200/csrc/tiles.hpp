@@ -24,6 +24,8 @@ struct Variant {
   int BM = 0, BN = 0, BK = 0, WM = 0, WN = 0, stages = 0, pw = 0, occ = 0;   // pw = producer warps
   int kind = KIND_F64_DMMA;
   int stg = 0;                                // 1: staged epilogue drained by the producers
+  double cal = 1.0;                           // B200 model calibration: measured / predicted time
+                                              // (tiles.cpp, fitted on B200, tools/model_calib.py)
   int threads() const {
     return is_umma(kind) ? 17 * 32 : ((BM / WM) * (BN / WN) + pw) * 32;   // UMMA: 8 + 8 + 1 (split: 8 + 4 + 1 + 4)
   }
