@@ -78,7 +78,9 @@ typedef struct tc_plan_opts {
                         eligible and no variant is forced), 1 never, 2 whenever eligible.  The
                         plan keeps its tcgen05 configuration for beta != 0 and unaligned
                         pointers.                                                            */
-  int reserved[2];   /* must be zero (TC_ERR_INVALID_ARG otherwise)                         */
+  int stream_rank;   /* 0 (default): the streaming path's model-best tiles; r > 0: its r-th
+                        alternative (tc_plan_tuned times the first three)                    */
+  int reserved[1];   /* must be zero (TC_ERR_INVALID_ARG otherwise)                         */
 } tc_plan_opts;
 
 /*

@@ -46,7 +46,7 @@ class _Opts(ctypes.Structure):
                 ("force_tiles", ctypes.c_char_p), ("no_fusion", ctypes.c_int), ("tma_epilogue", ctypes.c_int),
                 ("morder", ctypes.c_int), ("no_tma_operands", ctypes.c_int),
                 ("cta_pair", ctypes.c_int), ("out_f32", ctypes.c_int), ("stream", ctypes.c_int),
-                ("reserved", ctypes.c_int * 2)]
+                ("stream_rank", ctypes.c_int), ("reserved", ctypes.c_int * 1)]
 
 
 _lib = None
@@ -242,9 +242,10 @@ class Plan:
 
 
 def _opts(cost, host_only, variant, force_tiles, fusion, tma, morder, tma_operands=True, pair=None,
-          out_f32=False, stream=None) -> _Opts:
+          out_f32=False, stream=None, stream_rank=0) -> _Opts:
     o = _Opts()
     o.stream = {None: 0, False: 1, True: 2}[stream]
+    o.stream_rank = int(stream_rank)
     o.out_f32 = int(out_f32)
     o.no_tma_operands = int(not tma_operands)
     o.cta_pair = {None: 0, False: 1, True: 2}[pair]
@@ -357,13 +358,15 @@ def plan_cache_clear() -> None:
 def plan(expr: str, extents: str, dtype: str = "f64", cost: str = "b200", host_only: bool = False,
          variant: int | None = None, force_tiles: str | None = None, fusion: bool = True,
          tma: bool = False, morder: str | None = None, tma_operands: bool = True,
-         pair: bool | None = None, out_f32: bool = False, stream: bool | None = None) -> Plan:
+         pair: bool | None = None, out_f32: bool = False, stream: bool | None = None,
+         stream_rank: int = 0) -> Plan:
     """pair: None = planner's choice, False / True = CTA pairs off / on where the plan allows.
     stream: None = planner's choice, False / True = the streaming path (bf16 tensor x matrix) off /
     on where eligible.
     out_f32 (bf16 plans): C is FP32 (split-K partials).
     morder: None = planner's choice, "C" = m digits in C order, "X" = in the X operand's order."""
-    o = _opts(cost, host_only, variant, force_tiles, fusion, tma, morder, tma_operands, pair, out_f32, stream)
+    o = _opts(cost, host_only, variant, force_tiles, fusion, tma, morder, tma_operands, pair, out_f32, stream,
+              stream_rank)
     h = ctypes.c_void_p()
     _raise(lib().tc_plan_ex(ctypes.byref(h), expr.encode(), extents.encode(), DTYPES[dtype], ctypes.byref(o)))
     p = Plan(h, expr, extents, dtype)

@@ -301,6 +301,8 @@ tc_status_t finish_plan(tc_plan_s *P, tc_plan_t *out, const tc_plan_s *rep = nul
     { delete P; return fail(ST_INVALID_ARG, "out_f32 is a TC_BF16 option (0 or 1)"); }
   P->out_f32 = P->opts.out_f32 == 1;
   if (P->opts.stream < 0 || P->opts.stream > 2) { delete P; return fail(ST_INVALID_ARG, "stream must be 0, 1 or 2"); }
+  if (P->opts.stream_rank < 0 || P->opts.stream_rank >= kStreamRanks)
+    { delete P; return fail(ST_INVALID_ARG, "stream_rank out of range"); }
   for (int r : P->opts.reserved)
     if (r != 0) { delete P; return fail(ST_INVALID_ARG, "tc_plan_opts.reserved[] must be zero"); }
   ft.morder = P->opts.morder - 1;
@@ -344,7 +346,7 @@ tc_status_t finish_plan(tc_plan_s *P, tc_plan_t *out, const tc_plan_s *rep = nul
   P->stream_active = false;
   if (P->opts.stream != 1 && !P->out_f32 && (fv < 0 || P->opts.stream == 2) && !ft.on) {
     StreamCfg sc;
-    if (stream_plan(P->c, kind, 148, sc)) {
+    if (stream_plan(P->c, kind, 148, sc, P->opts.stream_rank)) {
       P->stream = sc;
       P->stream_active = sc.preferred || P->opts.stream == 2;
     } else {
@@ -700,7 +702,7 @@ std::string cache_key(const char *expr, const char *extents, tc_dtype_t dtype, c
   if (o)
     k << '\x1f' << o->cost_mode << ',' << o->host_only << ',' << o->variant << ',' << o->no_fusion << ','
       << o->tma_epilogue << ',' << o->morder << ',' << o->no_tma_operands << ',' << o->cta_pair << ','
-      << (o->force_tiles ? o->force_tiles : "");
+      << o->out_f32 << ',' << o->stream << ',' << o->stream_rank << ',' << (o->force_tiles ? o->force_tiles : "");
   return k.str();
 }
 }  // namespace
@@ -785,15 +787,19 @@ tc_status_t tc_plan_tuned_beta(tc_plan_t *tuned, const tc_plan_t plan, const voi
     float best_ms = 0;
     std::vector<std::pair<int, double>> log;
     tc_status_t rc = TC_SUCCESS;
-    // the streaming path (stream.hpp) competes as candidate 99 when the plan has it and beta == 0
-    if (plan->stream.on && beta == 0.0) cand.push_back(kTunedStream);
+    // the streaming path (stream.hpp) competes when the plan has it and beta == 0: its model's
+    // best configurations as candidates 99, 98, 97 (rank 0, 1, 2)
+    if (plan->stream.on && beta == 0.0)
+      for (int r = 0; r < plan->stream.nranks; r++) cand.push_back(kTunedStream - r);
     for (int v : cand) {
       tc_plan_s *P = new tc_plan_s();
       P->opts = plan->opts;
       P->force_tiles = plan->force_tiles;
       P->opts.force_tiles = plan->opts.force_tiles ? P->force_tiles.c_str() : nullptr;
-      P->opts.variant = (v == kTunedStream ? plan->cfg.variant : v) + 1;
-      P->opts.stream = v == kTunedStream ? 2 : 1;
+      const bool sv = v > kTunedStream - kStreamRanks && v <= kTunedStream;
+      P->opts.variant = (sv ? plan->cfg.variant : v) + 1;
+      P->opts.stream = sv ? 2 : 1;
+      P->opts.stream_rank = sv ? kTunedStream - v : 0;
       P->dtype = plan->dtype;
       P->parsed = plan->parsed;
       tc_plan_t cp = nullptr;
@@ -1134,7 +1140,8 @@ tc_status_t tc_plan_info(const tc_plan_t plan, char *json, size_t cap, size_t *n
           << ",\"stage_bytes\":" << k.stage_bytes << ",\"ntiles\":" << k.ntiles << ",\"units\":" << k.nunits
           << ",\"NB\":" << st.NB << ",\"AR\":" << st.AR << ",\"occ\":" << st.occ << ",\"nstg\":" << k.nstg << ",\"xswz\":" << st.xswz << ",\"smem\":" << st.smem
           << ",\"grid\":" << plan->stream_grid
-          << ",\"t_pred_ms\":" << st.t_pred * 1e3 << ",\"bytes\":" << st.bytes;
+          << ",\"t_pred_ms\":" << st.t_pred * 1e3 << ",\"bytes\":" << st.bytes
+          << ",\"rank\":" << st.rank << ",\"nranks\":" << st.nranks;
       }
       o << "}";
     }

@@ -41,12 +41,14 @@ double run_bytes(const int64_t *dims, const int64_t *str, const uint32_t *box, i
   return run;
 }
 
-// DRAM efficiency of runs of r bytes (32-B sectors; whole 64/128-B lines when r allows)
+// DRAM efficiency of runs of r bytes (32-B sectors; whole 64/128-B lines when r allows); writes
+// pay more for short runs than reads (BF16 tile sweeps on TCCG #1, profiles/r02_stream_sweep_*)
 double run_eff(double r) { return r >= 128 ? 1.0 : r >= 64 ? 0.9 : r >= 32 ? 0.75 : 0.4; }
+double run_eff_w(double r) { return r >= 128 ? 1.0 : r >= 64 ? 0.85 : r >= 32 ? 0.6 : 0.3; }
 
 }  // namespace
 
-bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s) {
+bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s, int rank) {
   s = StreamCfg();
   auto no = [&](const char *why) { s.why = why; return false; };
   const bool f64 = kind == KIND_F64_DMMA;
@@ -102,7 +104,7 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s) {
   for (int kb = kq; kb <= std::min(f64 ? 64 : es == 4 ? 128 : 256, KP); kb += kq) kbs.push_back(kb);
   const double hbm = 6.5e12;
   double best = 1e30;
-  StreamCfg bestc;
+  std::vector<StreamCfg> top;   // the kStreamRanks best configurations, model order
   std::vector<std::vector<int>> restopts;
   for (int id : rest) {
     std::vector<int> o;
@@ -191,7 +193,7 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s) {
             if (ta >= c.ix[a].n && cv.idx.size() > 1 && T[cv.idx[1]] > 1 && cv.stride[1] == c.ix[a].n)
               rc *= std::min<int64_t>(T[cv.idx[1]], c.ix[cv.idx[1]].n);
             const double bx = (double)c.numel(X) * es, bc = (double)c.numel(0) * es;
-            double t = (bx / run_eff(rx) + bc / run_eff(rc)) / hbm;
+            double t = (bx / run_eff(rx) + bc / run_eff_w(rc)) / hbm;
             // the TMA engine moves a box row (its first dim) every ~3 SM clocks (measured on
             // B200 with 64-B rows, tools/stream_ablation.py): short rows bound the X stream
             const double trows = (double)tiles * nks * ((double)boxel / q.xbox[0]) * 3.0 / ((double)sms * 1.9e9);
@@ -219,8 +221,8 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s) {
                 continue;
             }
 #endif
-            if (t < best) {
-              best = t;
+            {   // keep the best few configurations (rank: tc_plan_tuned times the first ones)
+              best = std::min(best, t);
               q.t_pred = t + 4e-6;
               q.occ = occ;
               q.xswz = swz;
@@ -232,7 +234,9 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s) {
               q.kp.ntiles = (int)tiles;
               q.kp.nunits = (int)units;
               for (int id = 0; id < (int)c.ix.size(); id++) q.T[id] = T[id];
-              bestc = q;
+              top.push_back(q);
+              std::sort(top.begin(), top.end(), [](const StreamCfg &x, const StreamCfg &y) { return x.t_pred < y.t_pred; });
+              if ((int)top.size() > kStreamRanks) top.pop_back();
             }
           }
         }
@@ -242,8 +246,10 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s) {
     if (q == rest.size()) break;
   }
   }
-  if (best >= 1e29) return no("no tile fits");
-  s = bestc;
+  if (best >= 1e29 || top.empty()) return no("no tile fits");
+  s = top[std::min<int>(rank, (int)top.size() - 1)];
+  s.rank = std::min<int>(rank, (int)top.size() - 1);
+  s.nranks = (int)top.size();
   SParams &k = s.kp;
   const int *T = s.T;
   k.K = (int)K;

@@ -89,10 +89,13 @@ struct StreamCfg {
   double bytes = 0;         // algorithmic bytes (X + Y + C)
   int T[kMaxIdx] = {};      // per normalised index: tile (k: KB, n: N)
   std::string why;          // why the path is off (for tc_plan_info)
+  int rank = 0, nranks = 0; // which of the model's best configurations this is, of how many
 };
 
 // Decide whether the streaming path applies to the normalised contraction and choose its
-// tiles (dtype kind from tiles.hpp).  sms: SMs of the device.
-bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s);
+// tiles (dtype kind from tiles.hpp).  sms: SMs of the device; rank: the model's rank-th best
+// configuration (0 = its first choice; tc_plan_tuned times the first kStreamRanks).
+constexpr int kStreamRanks = 3;
+bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s, int rank = 0);
 
 }  // namespace tc

@@ -100,7 +100,19 @@ def test_stream_tuned_candidate():
     B = tcinputs.uniform(p.numel("B"), 2, device="cuda").to(torch.bfloat16)
     C = torch.empty(p.numel("C"), dtype=torch.bfloat16, device="cuda")
     t = p.tuned(A, B, C, topk=2, reps=1)
-    assert 99 in [v for v, _ in t.info()["stats"]["tuned"]]
+    tried = [v for v, _ in t.info()["stats"]["tuned"]]
+    assert 99 in tried and 98 in tried   # the streaming path's two best model configurations
+
+
+def test_stream_ranks_agree():
+    # the model's alternative streaming configurations (tc_plan_opts.stream_rank) give the same
+    # bits on integer data
+    for expr, ext in (REDUCED[0], REDUCED[6]):
+        for r in (1, 2):
+            p = tc.plan(expr, ext, "bf16", host_only=True, stream=True, stream_rank=r).info()["stream"]
+            assert p["rank"] == min(r, p["nranks"] - 1)
+            check_bf16(expr, ext, seed=30 + r, integer=True, stream=True, stream_rank=r)
+            check_case(expr, ext, seed=40 + r, integer=True, stream=True, stream_rank=r, dtype="f64")
 
 
 # FP64 (the paper's precision): DMMA m8n8k4 streaming kernel, tolerance 1e-12 * S (north_star)
