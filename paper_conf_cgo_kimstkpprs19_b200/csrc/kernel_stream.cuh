@@ -164,7 +164,7 @@ __device__ __forceinline__ void s_store_box(const SParams &p, TE *C, const unsig
 }
 
 template <int NB, int AR, bool TRANS>
-__global__ void __launch_bounds__(kSThreads, AR == 4 ? 2 : 1) tc_stream_bf16_kernel(const __grid_constant__ SParams p) {
+__global__ void __launch_bounds__(kSThreads, stream_occ(NB, AR)) tc_stream_bf16_kernel(const __grid_constant__ SParams p) {
   extern __shared__ __align__(1024) unsigned char smem_dyn[];
   unsigned char *sm = smem_dyn + ((1024u - ((uint32_t)__cvta_generic_to_shared(smem_dyn) & 1023u)) & 1023u);
   const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(sm);
@@ -307,7 +307,7 @@ __global__ void __launch_bounds__(kSThreads, AR == 4 ? 2 : 1) tc_stream_bf16_ker
 // straight from the (swizzled) stage and from Y, and holds C(row g, n 2t / 2t+1) of each of its
 // AR blocks: the run C[a0 .. a0+AR-1, row g, n].
 template <int NB, int AR, bool TRANS>
-__global__ void __launch_bounds__(kSThreads, AR == 4 ? 2 : 1) tc_stream_f64_kernel(const __grid_constant__ SParams p) {
+__global__ void __launch_bounds__(kSThreads, stream_occ(NB, AR)) tc_stream_f64_kernel(const __grid_constant__ SParams p) {
   extern __shared__ __align__(1024) unsigned char smem_dyn[];
   unsigned char *sm = smem_dyn + ((1024u - ((uint32_t)__cvta_generic_to_shared(smem_dyn) & 1023u)) & 1023u);
   const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(sm);
@@ -426,7 +426,7 @@ __device__ __forceinline__ uint32_t tf32_lo(uint32_t x) {
 }
 
 template <int NB, int AR, bool TRANS, bool SPLIT>
-__global__ void __launch_bounds__(kSThreads, AR == 4 ? 2 : 1) tc_stream_tf32_kernel(const __grid_constant__ SParams p) {
+__global__ void __launch_bounds__(kSThreads, stream_occ(NB, AR)) tc_stream_tf32_kernel(const __grid_constant__ SParams p) {
   extern __shared__ __align__(1024) unsigned char smem_dyn[];
   unsigned char *sm = smem_dyn + ((1024u - ((uint32_t)__cvta_generic_to_shared(smem_dyn) & 1023u)) & 1023u);
   const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(sm);

@@ -32,6 +32,10 @@ const void *stream_kernel_ptr(int kind, int NB, int AR, bool trans) {
     case 3 * 16 + 4: return spick<3, 4>(kind, trans);
     case 3 * 16 + 8: return spick<3, 8>(kind, trans);
     case 4 * 16 + 4: return spick<4, 4>(kind, trans);
+    // FP64 only: n up to 72 (the AO->MO-like TCCG #10, #11, #19: a 72 x 72 matrix operand)
+    case 9 * 16 + 2:
+      if (kind != KIND_F64_DMMA) return nullptr;
+      return trans ? (const void *)&tc_stream_f64_kernel<9, 2, true> : (const void *)&tc_stream_f64_kernel<9, 2, false>;
   }
   return nullptr;
 }

@@ -24,7 +24,10 @@ namespace {
 // or 8 (one CTA per SM; not with NB = 4: 128 accumulator registers)
 bool instance_exists(int NB, int AR) { return NB >= 1 && NB <= 4 && (AR == 4 || (AR == 8 && NB <= 3)); }
 // FP64 (DMMA m8n8k4: 8-row units, accumulators 2 doubles per n8 block and a value)
-bool instance_exists_f64(int NB, int AR) { return NB >= 1 && NB <= 4 && (AR == 4 || (AR == 8 && NB <= 3)); }
+bool instance_exists_f64(int NB, int AR) {
+  // (NB = 9 with AR = 4 spills at ptxas' 168-register choice)
+  return (NB >= 1 && NB <= 4 && (AR == 4 || (AR == 8 && NB <= 3))) || (NB == 9 && AR == 2);
+}
 
 int round_up(int64_t x, int m) { return (int)((x + m - 1) / m * m); }
 
@@ -76,8 +79,8 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s, int rank
   for (int j = 1; j < xr; j++)
     if ((xv.stride[j] * es) % 16 || xv.stride[j] >= ((int64_t)1 << 39)) return no("X strides (TMA)");
   const int64_t N = c.ix[nid].n, K = c.ix[kid].n;
-  if (N > 32) return no("Y-side extent > 32");
-  const int NB = (int)((N + 7) / 8), N8 = 8 * NB;
+  if (N > (f64 ? 72 : 32)) return no("Y-side extent above the kernels' n blocks (32; FP64 72)");
+  const int NB = N > 32 ? 9 : (int)((N + 7) / 8), N8 = 8 * NB;
   const int KP = round_up(K, kq);
   // conflict-free B-fragment rows (8 rows n at consecutive 8 / 4 threads' k)
   const int YP = es == 8 ? round_up(KP, 16) + 4 : es == 4 ? round_up(KP, 32) + 4 : KP + 8;
@@ -119,7 +122,7 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s, int rank
     int rprod = 1;
     std::vector<int> rt(rest.size());
     for (size_t q = 0; q < rest.size(); q++) { rt[q] = restopts[q][rix[q]]; rprod *= rt[q]; }
-    for (int AR : {4, 8}) {
+    for (int AR : {2, 4, 8}) {
       if (!(f64 ? instance_exists_f64(NB, AR) : instance_exists(NB, AR))) continue;
       // AR-element runs are stored as one vector: every C stride (and C's origin) a multiple of AR
       bool cal = cv.base % AR == 0;
@@ -172,7 +175,7 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s, int rank
             const int64_t rows = (int64_t)units * ru * AR;   // tile rows (m)
             const size_t stg = (size_t)round_up(rows * N8 * es, 128);
             const size_t tabb = (size_t)units * 2 * ru * 4 + (size_t)rows * N8 * es / 16 * 4;
-            const int occ = AR == 4 ? 2 : 1;
+            const int occ = stream_occ(NB, AR);
             const size_t cap = occ == 2 ? 115712 : 232448;
             // two C boxes when they leave >= 3 ring stages (one block-wide barrier per tile
             // instead of two), else one

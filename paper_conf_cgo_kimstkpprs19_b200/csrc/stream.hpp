@@ -27,6 +27,10 @@ constexpr int kSWarps = 8;          // compute warps (+ 1 TMA producer warp)
 constexpr int kSThreads = (kSWarps + 1) * 32;
 constexpr int kSRows = 16;          // rows of one MMA block (m16)
 
+// resident CTAs per SM an instance is compiled for (__launch_bounds__): two while the
+// accumulators (AR x NB blocks of 4 registers) leave room under the 2-CTA register cap
+constexpr int stream_occ(int NB, int AR) { return AR * NB * 4 <= 48 ? 2 : 1; }
+
 enum StreamMode { SM_T = 0, SM_K = 2 };
 // SM_T: X's FVI is an external E != C's FVI a: a block's 16 rows are two octets of 8
 //       consecutive E (ldmatrix.trans over k rows of the X box).

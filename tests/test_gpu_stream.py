@@ -141,3 +141,14 @@ def test_stream_fp32(expr, ext, dtype):
     assert tc.plan(expr, ext, dtype, host_only=True, stream=True).info()["stream"]["active"] == 1
     check_f32(expr, ext, dtype, seed=22, stream=True)
     check_f32(expr, ext, dtype, seed=23, alpha=-1.5, stream=True)
+
+
+@pytest.mark.parametrize("expr,ext", [("abc-bda-dc", "a:24;b:40;c:40;d:24"),      # n = 40 (9 n8 blocks)
+                                      ("abcd-ebad-ce", "a:16;b:8;c:72;d:2;e:24"),  # SM_K, n = 72
+                                      ("abcde-efbad-cf", "a:16;b:3;c:57;d:2;e:16;f:12")])
+def test_stream_f64_wide_n(expr, ext):
+    # FP64 streaming with the Y-side extent up to 72 (NB = 9, AR = 2)
+    s = tc.plan(expr, ext, "f64", host_only=True, stream=True).info()["stream"]
+    assert s["on"] == 1 and s["NB"] == 9, s
+    check_case(expr, ext, seed=51, integer=True, stream=True, dtype="f64")
+    check_case(expr, ext, seed=52, stream=True, dtype="f64")
