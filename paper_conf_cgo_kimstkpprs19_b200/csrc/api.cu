@@ -789,7 +789,7 @@ tc_status_t tc_plan_tuned_beta(tc_plan_t *tuned, const tc_plan_t plan, const voi
     tc_status_t rc = TC_SUCCESS;
     // the streaming path (stream.hpp) competes when the plan has it and beta == 0: its model's
     // best configurations as candidates 99, 98, 97 (rank 0, 1, 2)
-    if (plan->stream.on && beta == 0.0)
+    if (plan->stream.on && (beta == 0.0 || plan->cfg.kind != KIND_BF16_UMMA))
       for (int r = 0; r < plan->stream.nranks; r++) cand.push_back(kTunedStream - r);
     for (int v : cand) {
       tc_plan_s *P = new tc_plan_s();
@@ -904,8 +904,10 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
   const tc_status_t chk = check_execute(plan, A, B, C);
   if (chk != TC_SUCCESS) return chk;
   const size_t es = elem_bytes(plan);
-  if (plan->stream.on && plan->stream_active && beta == 0.0 && plan->batch.empty()) {
-    // the streaming path (beta == 0: C is only written; otherwise the configuration below)
+  if (plan->stream.on && plan->stream_active && (beta == 0.0 || plan->cfg.kind != KIND_BF16_UMMA) &&
+      plan->batch.empty()) {
+    // the streaming path (BF16 with beta != 0 runs the tile configuration below: its epilogue
+    // rounds alpha * sum + beta * C once)
     SParams sp = plan->stream.kp;
     const void *Xp = plan->stream.X == 1 ? A : B, *Yp = plan->stream.X == 1 ? B : A;
     if (encode_stream_maps(plan, Xp, C, sp)) {
@@ -913,6 +915,7 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
       sp.C = static_cast<char *>(C) + es * plan->stream.cbase;
       sp.alpha = (float)alpha;
       sp.alpha64 = alpha;
+      sp.beta = beta;
       const void *fn = stream_kernel_ptr(plan->cfg.kind, plan->stream.NB, plan->stream.AR, plan->stream.mode != SM_K);
       const int grid = std::min(sp.ntiles, plan->stream_grid);
       void *sargs[] = {&sp};

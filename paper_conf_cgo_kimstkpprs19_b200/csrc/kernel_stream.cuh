@@ -107,6 +107,25 @@ __device__ __forceinline__ uint32_t s_cswzb(uint32_t b, int s1, int s2) {
   return ((ch ^ ((x ^ (x >> s1) ^ (x >> s2)) & 7u)) << 4) | (b & 15u);
 }
 
+// beta != 0 (FP64 / FP32 C): the staged alpha * sum plus beta * the old C, one fma per element
+// (the tile kernels' order); beta == 0 never reads C (R26)
+__device__ __forceinline__ uint4 s_beta(uint4 v, uint4 o, double beta, const double *) {
+  double2 a = *reinterpret_cast<double2 *>(&v), b = *reinterpret_cast<double2 *>(&o);
+  a.x = fma(beta, b.x, a.x);
+  a.y = fma(beta, b.y, a.y);
+  return *reinterpret_cast<uint4 *>(&a);
+}
+__device__ __forceinline__ uint4 s_beta(uint4 v, uint4 o, double beta, const float *) {
+  float4 a = *reinterpret_cast<float4 *>(&v), b = *reinterpret_cast<float4 *>(&o);
+  const float bt = (float)beta;
+  a.x = fmaf(bt, b.x, a.x);
+  a.y = fmaf(bt, b.y, a.y);
+  a.z = fmaf(bt, b.z, a.z);
+  a.w = fmaf(bt, b.w, a.w);
+  return *reinterpret_cast<uint4 *>(&a);
+}
+__device__ __forceinline__ uint4 s_beta(uint4 v, uint4, double, const __nv_bfloat16 *) { return v; }
+
 // The C box (smem, C order) leaves as 16-B runs along C's FVI: chunk c at ctab[c] elements from
 // the tile origin.  Interior tiles store every chunk; tiles on the tensor's edge store what lies
 // inside (every coordinate below its limit).
@@ -132,11 +151,34 @@ __device__ __forceinline__ void s_store_box(const SParams &p, TE *C, const unsig
   }
   TE *Ct = C + corg;
   const unsigned char *sb = sm + stg_off;
+  if (interior && p.beta != 0.0) {
+    // beta != 0: four chunks' old C in flight per thread before their stores
+    for (int c0 = tid; c0 < p.nchunk; c0 += 4 * nthr) {
+      uint4 o[4];
+      TE *d[4];
+#pragma unroll
+      for (int i = 0; i < 4; i++) {
+        const int ch = c0 + i * nthr;
+        d[i] = Ct + (int32_t)ctab[ch < p.nchunk ? ch : 0];
+        if (ch < p.nchunk) o[i] = __ldcs(reinterpret_cast<const uint4 *>(d[i]));
+      }
+#pragma unroll
+      for (int i = 0; i < 4; i++) {
+        const int ch = c0 + i * nthr;
+        if (ch < p.nchunk) {
+          const uint4 v = *reinterpret_cast<const uint4 *>(sb + s_cswzb((uint32_t)ch * 16u, p.cs1, p.cs2));
+          __stcs(reinterpret_cast<uint4 *>(d[i]), s_beta(v, o[i], p.beta, (const TE *)nullptr));
+        }
+      }
+    }
+    return;
+  }
   for (int ch = tid; ch < p.nchunk; ch += nthr) {
     const uint4 v = *reinterpret_cast<const uint4 *>(sb + s_cswzb((uint32_t)ch * 16u, p.cs1, p.cs2));
     TE *dst = Ct + (int32_t)ctab[ch];
     if (interior) {
-      __stcs(reinterpret_cast<uint4 *>(dst), v);
+      __stcs(reinterpret_cast<uint4 *>(dst),
+             p.beta != 0.0 ? s_beta(v, __ldcs(reinterpret_cast<const uint4 *>(dst)), p.beta, (const TE *)nullptr) : v);
       continue;
     }
     int rem = ch, c0 = 0;
@@ -155,10 +197,19 @@ __device__ __forceinline__ void s_store_box(const SParams &p, TE *C, const unsig
     const int lim0 = p.cmd[0] < 0 ? p.N : (int)((lims >> (8 * p.cmd[0])) & 0xFF);
     const int ne = ok ? max(0, min(EPC, lim0 - c0)) : 0;
     if (ne == EPC) {
-      __stcs(reinterpret_cast<uint4 *>(dst), v);
+      __stcs(reinterpret_cast<uint4 *>(dst),
+             p.beta != 0.0 ? s_beta(v, __ldcs(reinterpret_cast<const uint4 *>(dst)), p.beta, (const TE *)nullptr) : v);
     } else {
       const TE *e = reinterpret_cast<const TE *>(&v);
-      for (int q2 = 0; q2 < ne; q2++) dst[q2] = e[q2];
+      for (int q2 = 0; q2 < ne; q2++) {
+        if constexpr (sizeof(TE) == 2) {
+          dst[q2] = e[q2];
+        } else if constexpr (sizeof(TE) == 4) {
+          dst[q2] = p.beta != 0.0 ? fmaf((float)p.beta, dst[q2], e[q2]) : e[q2];
+        } else {
+          dst[q2] = p.beta != 0.0 ? fma(p.beta, dst[q2], e[q2]) : e[q2];
+        }
+      }
     }
   }
 }

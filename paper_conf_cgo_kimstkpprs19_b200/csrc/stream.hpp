@@ -10,8 +10,8 @@
 // Scope (stream_plan decides): TC_BF16, no batch index, exactly one internal index k and one
 // Y-side external index n (after fusion) with n <= 32 and Y small enough for shared memory, X of
 // rank <= 5 with 16-B multiple strides (TMA), C's FVI on X and not X's FVI (X = the input
-// holding C's FVI), beta == 0 at execute time (otherwise tc_execute runs the plan's
-// tcgen05 configuration, which the planner always keeps).
+// holding C's FVI).  beta != 0 on BF16 runs the plan's tile configuration (which the
+// planner always keeps): its epilogue rounds alpha * sum + beta * C to BF16 once.
 #pragma once
 #include <cstdint>
 #include <string>
@@ -48,6 +48,7 @@ struct SParams {
   int64_t mCs[kSMaxMdims];  // element strides of the m dims in C
   float alpha;
   double alpha64;           // (FP64 kernel)
+  double beta;              // C = alpha * sum + beta * C (FP64 / FP32 C; BF16 plans run beta != 0 on the tile kernel)
   int xrank;
   int nmd;                  // m dims, raster order (C's FVI first)
   int mT[kSMaxMdims], mNt[kSMaxMdims], mX[kSMaxMdims], mN[kSMaxMdims];

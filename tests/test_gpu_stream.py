@@ -126,7 +126,8 @@ def test_stream_f64(expr, ext):
     assert p.info()["stream"]["active"] == 1
     check_case(expr, ext, seed=12, stream=True)
     check_case(expr, ext, seed=13, alpha=0.75, stream=True)
-    check_case(expr, ext, seed=14, integer=True, alpha=2.0, beta=-1.0, stream=True)   # beta: tile kernel
+    check_case(expr, ext, seed=14, integer=True, alpha=2.0, beta=-1.0, stream=True)   # beta on the path
+    check_case(expr, ext, seed=15, alpha=0.5, beta=1.5, stream=True)
 
 
 # FP32 storage: TF32 products (R30 tolerance) and FP32 as split TF32 (1e-5 * S, R32)
@@ -141,6 +142,8 @@ def test_stream_fp32(expr, ext, dtype):
     assert tc.plan(expr, ext, dtype, host_only=True, stream=True).info()["stream"]["active"] == 1
     check_f32(expr, ext, dtype, seed=22, stream=True)
     check_f32(expr, ext, dtype, seed=23, alpha=-1.5, stream=True)
+    check_f32(expr, ext, dtype, seed=24, integer=True, alpha=2.0, beta=-1.0, stream=True)   # beta on the path
+    check_f32(expr, ext, dtype, seed=25, alpha=0.5, beta=1.5, stream=True)
 
 
 @pytest.mark.parametrize("expr,ext", [("abc-bda-dc", "a:24;b:40;c:40;d:24"),      # n = 40 (9 n8 blocks)
