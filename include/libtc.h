@@ -161,10 +161,13 @@ tc_status_t tc_execute_host(const tc_plan_t plan, const void *A_host, const void
 /*
  * Measured tuning (the paper's "auto-tuned across a selected set",
  * P:L346-348): the cost model ranks the kernel variants by the predicted time of their best
- * configuration; the best configurations of the top `topk` variants are each launched
- * 1 + `reps` times on `stream` with the caller's A, B, C (alpha = 1, beta = 0: C's contents
- * are OVERWRITTEN) and the fastest (minimum over reps) becomes *tuned, a new plan with the same
- * contraction, layout, device and options as `plan` (which stays valid and unchanged).
+ * configuration; the best configurations of the top `topk` variants (and, for streaming
+ * shapes, the streaming path's three best configurations: log entries 99, 98, 97) are each
+ * launched 1 + `reps` times on `stream` with the caller's A, B, C (alpha = 1, beta = 0: C's
+ * contents are OVERWRITTEN), each timed launch after a 256 MB scratch write that flushes L2
+ * (the scratch is allocated for the call; without memory for it the launches run warm), and
+ * the fastest (median over reps) becomes *tuned, a new plan with the same contraction, layout,
+ * device and options as `plan` (which stays valid and unchanged).
  * Synchronises `stream`.  tc_plan_info(*tuned) lists the candidates' times ("tuned").
  * Errors: TC_ERR_INVALID_ARG (NULL, topk < 1, reps < 1), TC_ERR_CUDA (host_only plan, launch
  * failure), as tc_execute for the pointers.  *tuned is NULL on failure.

@@ -762,6 +762,7 @@ tc_status_t tc_plan_tuned(tc_plan_t *tuned, const tc_plan_t plan, const void *A,
 }
 
 constexpr int kTunedStream = 99;   // tc_plan_tuned's log entry of the streaming path
+constexpr size_t kFlushBytes = (size_t)256 << 20;   // tc_plan_tuned: L2 flush between launches
 
 tc_status_t tc_plan_tuned_beta(tc_plan_t *tuned, const tc_plan_t plan, const void *A, const void *B, void *C,
                                int topk, int reps, double beta, tc_stream_t stream) {
@@ -783,6 +784,13 @@ tc_status_t tc_plan_tuned_beta(tc_plan_t *tuned, const tc_plan_t plan, const voi
     cudaEvent_t e0, e1;
     if (cudaEventCreate(&e0) != cudaSuccess || cudaEventCreate(&e1) != cudaSuccess)
       return fail(ST_CUDA, "cudaEventCreate");
+    // an L2-sized scratch buffer (twice the 126 MB L2) written before every timed launch;
+    // without memory for it the tuning runs warm
+    void *flush = nullptr;
+    if (cudaMalloc(&flush, kFlushBytes) != cudaSuccess) {
+      cudaGetLastError();
+      flush = nullptr;
+    }
     tc_plan_t best = nullptr;
     float best_ms = 0;
     std::vector<std::pair<int, double>> log;
@@ -806,18 +814,22 @@ tc_status_t tc_plan_tuned_beta(tc_plan_t *tuned, const tc_plan_t plan, const voi
       rc = finish_plan(P, &cp);
       if (rc != TC_SUCCESS) break;
       cp->stats.per_variant = plan->stats.per_variant;
-      // one warm-up, then the minimum over reps single launches (C is overwritten)
+      // one warm-up, then the median of reps single launches, each after an L2 flush (the
+      // conditions a stream of different contractions sees; C is overwritten)
       rc = tc_execute(cp, A, B, C, 1.0, beta, stream);
-      float ms = 1e30f;
+      std::vector<float> ts;
       for (int r = 0; r < reps && rc == TC_SUCCESS; r++) {
+        if (flush) cudaMemsetAsync(flush, r & 0xFF, kFlushBytes, (cudaStream_t)stream);
         cudaEventRecord(e0, (cudaStream_t)stream);
         rc = tc_execute(cp, A, B, C, 1.0, beta, stream);
         cudaEventRecord(e1, (cudaStream_t)stream);
         if (cudaEventSynchronize(e1) != cudaSuccess) { rc = fail(ST_CUDA, "tuning launch failed"); break; }
         float t = 0;
         cudaEventElapsedTime(&t, e0, e1);
-        ms = std::min(ms, t);
+        ts.push_back(t);
       }
+      std::sort(ts.begin(), ts.end());
+      const float ms = ts.empty() ? 1e30f : ts[ts.size() / 2];
       if (rc != TC_SUCCESS) { tc_plan_destroy(cp); break; }
       log.push_back({v, ms});
       if (!best || ms < best_ms) {
@@ -830,6 +842,10 @@ tc_status_t tc_plan_tuned_beta(tc_plan_t *tuned, const tc_plan_t plan, const voi
     }
     cudaEventDestroy(e0);
     cudaEventDestroy(e1);
+    if (flush) {
+      cudaStreamSynchronize((cudaStream_t)stream);
+      cudaFree(flush);
+    }
     if (rc != TC_SUCCESS) { tc_plan_destroy(best); return rc; }
     best->tuned = log;
     *tuned = best;
