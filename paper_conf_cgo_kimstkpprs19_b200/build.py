@@ -9,7 +9,7 @@ CSRC = os.path.join(HERE, "csrc")
 SO = os.path.join(HERE, "libtc.so")
 SOURCES = ["api.cu", "group_api.cu", "contraction.cpp", "planner.cpp", "tiles.cpp", "group.cpp",
            "kernels_00.cu", "kernels_01.cu", "kernels_10.cu", "kernels_11.cu", "kernels_umma.cu", "kernels_umma_tma.cu", "kernels_umma_pair.cu", "kernels_umma_f32out.cu",
-           "kernels_group.cu", "stream.cpp", "kernels_stream.cu"]
+           "kernels_group.cu", "stream.cpp", "kernels_stream.cu", "kernels_stream_beta.cu"]
 HEADERS = ["contraction.hpp", "planner.hpp", "kparams.hpp", "kernel_f64.cuh", "tiles.hpp", "variants.def",
            "kernel_table.cuh", "kernel_umma.cuh", "group.hpp", "kernel_group.cuh", "plan_internal.hpp", "stream.hpp", "kernel_stream.cuh"]
 NVCC_FLAGS = ["-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo",

@@ -205,11 +205,15 @@ Status upload(tc_plan_s *P, std::string &err) {
   P->d_packY2 = (const uint32_t *)(b + parts[iY2p].off);
   if (P->stream.on) {
     P->stream.kp.tab = (const uint32_t *)(b + parts[iS].off);
-    const void *fn = stream_kernel_ptr(P->cfg.kind, P->stream.NB, P->stream.AR, P->stream.mode != SM_K);
+    const void *fn = stream_kernel_ptr(P->cfg.kind, P->stream.NB, P->stream.AR, P->stream.mode != SM_K, false);
     if (!fn) { err = "no streaming kernel instance for the plan"; return ST_UNSUPPORTED; }
-    // (the instance is shared by plans of different sizes: always the opt-in maximum)
+    // (the instances are shared by plans of different sizes: always the opt-in maximum)
     e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448);
     if (e != cudaSuccess) { err = std::string("cudaFuncSetAttribute: ") + cudaGetErrorString(e); return ST_CUDA; }
+    if (const void *fb = stream_kernel_ptr(P->cfg.kind, P->stream.NB, P->stream.AR, P->stream.mode != SM_K, true)) {
+      e = cudaFuncSetAttribute(fb, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448);
+      if (e != cudaSuccess) { err = std::string("cudaFuncSetAttribute: ") + cudaGetErrorString(e); return ST_CUDA; }
+    }
     int socc = 0, nsm = 148;
     e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&socc, fn, kSThreads, P->stream.smem);
     if (e != cudaSuccess || socc < 1) { err = "streaming kernel cannot be resident"; return ST_CUDA; }
@@ -932,7 +936,8 @@ tc_status_t tc_execute(const tc_plan_t plan, const void *A, const void *B, void 
       sp.alpha = (float)alpha;
       sp.alpha64 = alpha;
       sp.beta = beta;
-      const void *fn = stream_kernel_ptr(plan->cfg.kind, plan->stream.NB, plan->stream.AR, plan->stream.mode != SM_K);
+      const void *fn = stream_kernel_ptr(plan->cfg.kind, plan->stream.NB, plan->stream.AR, plan->stream.mode != SM_K,
+                                         beta != 0.0);
       const int grid = std::min(sp.ntiles, plan->stream_grid);
       void *sargs[] = {&sp};
       cudaError_t e = cudaLaunchKernel(fn, dim3(grid), dim3(kSThreads), sargs, plan->stream.smem, (cudaStream_t)stream);

@@ -126,10 +126,34 @@ __device__ __forceinline__ uint4 s_beta(uint4 v, uint4 o, double beta, const flo
 }
 __device__ __forceinline__ uint4 s_beta(uint4 v, uint4, double, const __nv_bfloat16 *) { return v; }
 
+// beta != 0, interior tile: four chunks' old C in flight per thread before their stores
+template <typename TE>
+__device__ __forceinline__ void s_store_box_beta(const SParams &p, TE *Ct, const unsigned char *sb, const uint32_t *ctab,
+                                              int tid, int nthr) {
+  for (int c0 = tid; c0 < p.nchunk; c0 += 4 * nthr) {
+    uint4 o[4];
+    TE *d[4];
+#pragma unroll
+    for (int i = 0; i < 4; i++) {
+      const int ch = c0 + i * nthr;
+      d[i] = Ct + (int32_t)ctab[ch < p.nchunk ? ch : 0];
+      if (ch < p.nchunk) o[i] = __ldcs(reinterpret_cast<const uint4 *>(d[i]));
+    }
+#pragma unroll
+    for (int i = 0; i < 4; i++) {
+      const int ch = c0 + i * nthr;
+      if (ch < p.nchunk) {
+        const uint4 v = *reinterpret_cast<const uint4 *>(sb + s_cswzb((uint32_t)ch * 16u, p.cs1, p.cs2));
+        __stcs(reinterpret_cast<uint4 *>(d[i]), s_beta(v, o[i], p.beta, (const TE *)nullptr));
+      }
+    }
+  }
+}
+
 // The C box (smem, C order) leaves as 16-B runs along C's FVI: chunk c at ctab[c] elements from
 // the tile origin.  Interior tiles store every chunk; tiles on the tensor's edge store what lies
 // inside (every coordinate below its limit).
-template <typename TE>
+template <typename TE, bool BETA>
 __device__ __forceinline__ void s_store_box(const SParams &p, TE *C, const unsigned char *sm, uint32_t stg_off,
                                             const uint32_t *ctab, int t, int tid, int nthr, int NB) {
   constexpr int EPC = 16 / (int)sizeof(TE);   // elements per chunk
@@ -151,34 +175,15 @@ __device__ __forceinline__ void s_store_box(const SParams &p, TE *C, const unsig
   }
   TE *Ct = C + corg;
   const unsigned char *sb = sm + stg_off;
-  if (interior && p.beta != 0.0) {
-    // beta != 0: four chunks' old C in flight per thread before their stores
-    for (int c0 = tid; c0 < p.nchunk; c0 += 4 * nthr) {
-      uint4 o[4];
-      TE *d[4];
-#pragma unroll
-      for (int i = 0; i < 4; i++) {
-        const int ch = c0 + i * nthr;
-        d[i] = Ct + (int32_t)ctab[ch < p.nchunk ? ch : 0];
-        if (ch < p.nchunk) o[i] = __ldcs(reinterpret_cast<const uint4 *>(d[i]));
-      }
-#pragma unroll
-      for (int i = 0; i < 4; i++) {
-        const int ch = c0 + i * nthr;
-        if (ch < p.nchunk) {
-          const uint4 v = *reinterpret_cast<const uint4 *>(sb + s_cswzb((uint32_t)ch * 16u, p.cs1, p.cs2));
-          __stcs(reinterpret_cast<uint4 *>(d[i]), s_beta(v, o[i], p.beta, (const TE *)nullptr));
-        }
-      }
-    }
+  if (BETA && interior) {
+    s_store_box_beta<TE>(p, Ct, sb, ctab, tid, nthr);
     return;
   }
   for (int ch = tid; ch < p.nchunk; ch += nthr) {
     const uint4 v = *reinterpret_cast<const uint4 *>(sb + s_cswzb((uint32_t)ch * 16u, p.cs1, p.cs2));
     TE *dst = Ct + (int32_t)ctab[ch];
     if (interior) {
-      __stcs(reinterpret_cast<uint4 *>(dst),
-             p.beta != 0.0 ? s_beta(v, __ldcs(reinterpret_cast<const uint4 *>(dst)), p.beta, (const TE *)nullptr) : v);
+      __stcs(reinterpret_cast<uint4 *>(dst), v);
       continue;
     }
     int rem = ch, c0 = 0;
@@ -198,16 +203,16 @@ __device__ __forceinline__ void s_store_box(const SParams &p, TE *C, const unsig
     const int ne = ok ? max(0, min(EPC, lim0 - c0)) : 0;
     if (ne == EPC) {
       __stcs(reinterpret_cast<uint4 *>(dst),
-             p.beta != 0.0 ? s_beta(v, __ldcs(reinterpret_cast<const uint4 *>(dst)), p.beta, (const TE *)nullptr) : v);
+             BETA ? s_beta(v, __ldcs(reinterpret_cast<const uint4 *>(dst)), p.beta, (const TE *)nullptr) : v);
     } else {
       const TE *e = reinterpret_cast<const TE *>(&v);
       for (int q2 = 0; q2 < ne; q2++) {
         if constexpr (sizeof(TE) == 2) {
           dst[q2] = e[q2];
         } else if constexpr (sizeof(TE) == 4) {
-          dst[q2] = p.beta != 0.0 ? fmaf((float)p.beta, dst[q2], e[q2]) : e[q2];
+          dst[q2] = BETA ? fmaf((float)p.beta, dst[q2], e[q2]) : e[q2];
         } else {
-          dst[q2] = p.beta != 0.0 ? fma(p.beta, dst[q2], e[q2]) : e[q2];
+          dst[q2] = BETA ? fma(p.beta, dst[q2], e[q2]) : e[q2];
         }
       }
     }
@@ -346,7 +351,7 @@ __global__ void __launch_bounds__(kSThreads, stream_occ(NB, AR)) tc_stream_bf16_
           }
     }
     consumer_sync(nthr);   // the box is complete
-    if (!(kSAbl & 2)) s_store_box<__nv_bfloat16>(p, C, sm, STGb - sbase, ctab, t, tid, nthr, NB);
+    if (!(kSAbl & 2)) s_store_box<__nv_bfloat16, false>(p, C, sm, STGb - sbase, ctab, t, tid, nthr, NB);
   }
 }
 
@@ -357,7 +362,7 @@ __global__ void __launch_bounds__(kSThreads, stream_occ(NB, AR)) tc_stream_bf16_
 // 8 rows of the other m dims); thread (g, t) loads A(row g, k t) and B(k t, n g) as doubles
 // straight from the (swizzled) stage and from Y, and holds C(row g, n 2t / 2t+1) of each of its
 // AR blocks: the run C[a0 .. a0+AR-1, row g, n].
-template <int NB, int AR, bool TRANS>
+template <int NB, int AR, bool TRANS, bool BETA>
 __global__ void __launch_bounds__(kSThreads, stream_occ(NB, AR)) tc_stream_f64_kernel(const __grid_constant__ SParams p) {
   extern __shared__ __align__(1024) unsigned char smem_dyn[];
   unsigned char *sm = smem_dyn + ((1024u - ((uint32_t)__cvta_generic_to_shared(smem_dyn) & 1023u)) & 1023u);
@@ -454,7 +459,7 @@ __global__ void __launch_bounds__(kSThreads, stream_occ(NB, AR)) tc_stream_f64_k
         }
     }
     consumer_sync(nthr);
-    if (!(kSAbl & 2)) s_store_box<double>(p, C, sm, STGb - sbase, ctab, t, tid, nthr, NB);
+    if (!(kSAbl & 2)) s_store_box<double, BETA>(p, C, sm, STGb - sbase, ctab, t, tid, nthr, NB);
   }
 }
 
@@ -476,7 +481,7 @@ __device__ __forceinline__ uint32_t tf32_lo(uint32_t x) {
   return __float_as_uint(__uint_as_float(x) - __uint_as_float(x & 0xFFFFE000u));
 }
 
-template <int NB, int AR, bool TRANS, bool SPLIT>
+template <int NB, int AR, bool TRANS, bool SPLIT, bool BETA>
 __global__ void __launch_bounds__(kSThreads, stream_occ(NB, AR)) tc_stream_tf32_kernel(const __grid_constant__ SParams p) {
   extern __shared__ __align__(1024) unsigned char smem_dyn[];
   unsigned char *sm = smem_dyn + ((1024u - ((uint32_t)__cvta_generic_to_shared(smem_dyn) & 1023u)) & 1023u);
@@ -597,7 +602,7 @@ __global__ void __launch_bounds__(kSThreads, stream_occ(NB, AR)) tc_stream_tf32_
           }
     }
     consumer_sync(nthr);
-    if (!(kSAbl & 2)) s_store_box<float>(p, C, sm, STGb - sbase, ctab, t, tid, nthr, NB);
+    if (!(kSAbl & 2)) s_store_box<float, BETA>(p, C, sm, STGb - sbase, ctab, t, tid, nthr, NB);
   }
 }
 

@@ -45,7 +45,7 @@ const void *kernel_ptr_umma(int v, bool xk, bool yk, bool tma, size_t *smem, int
 // CTA-pair instances (BN = 128 BF16 / TF32 variants 12 / 22; nullptr otherwise)
 const void *kernel_ptr_umma_pair(int v, bool xk, bool yk, size_t *smem, int *threads);
 // the streaming kernels (kernels_stream.cu): FP64 or BF16, n8 blocks NB, C-FVI runs AR, .trans A loads
-const void *stream_kernel_ptr(int kind, int NB, int AR, bool trans);
+const void *stream_kernel_ptr(int kind, int NB, int AR, bool trans, bool beta);
 // BF16 operands, FP32 C (variants 11 / 12; cp.async producers; nullptr otherwise)
 const void *kernel_ptr_umma_f32out(int v, bool xk, bool yk, size_t *smem, int *threads);
 
