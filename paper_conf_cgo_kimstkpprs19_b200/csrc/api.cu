@@ -1158,7 +1158,7 @@ tc_status_t tc_plan_info(const tc_plan_t plan, char *json, size_t cap, size_t *n
       o << ",\"stream\":{\"on\":" << (st.on ? 1 : 0) << ",\"active\":" << (plan->stream_active ? 1 : 0)
         << ",\"why\":\"" << st.why << "\"";
       if (st.on) {
-        o << ",\"mode\":\"" << (st.mode == SM_K ? "K" : "T") << "\",\"X\":\"" << (st.X == 1 ? "A" : "B") << "\",\"tiles\":{";
+        o << ",\"mode\":\"" << (st.mode == SM_K ? "K" : st.mode == SM_M ? "M" : "T") << "\",\"X\":\"" << (st.X == 1 ? "A" : "B") << "\",\"tiles\":{";
         for (size_t i = 0; i < c.ix.size(); i++) o << (i ? "," : "") << "\"" << c.ix[i].name << "\":" << st.T[i];
         o << "},\"KB\":" << k.KB << ",\"nks\":" << k.nks << ",\"stages\":" << k.stages
           << ",\"stage_bytes\":" << k.stage_bytes << ",\"ntiles\":" << k.ntiles << ",\"units\":" << k.nunits

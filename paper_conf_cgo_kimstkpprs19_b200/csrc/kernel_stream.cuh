@@ -452,10 +452,17 @@ __global__ void __launch_bounds__(kSThreads, stream_occ(NB, AR)) tc_stream_f64_k
 #pragma unroll
         for (int c2 = 0; c2 < 2; c2++) {
           const uint32_t b = 8u * (bo + (uint32_t)((8 * n + 2 * t4 + c2) * p.cbsn));
+          if (p.cbsj == 1) {   // the AR values are consecutive along C's FVI: 16-B pairs
 #pragma unroll
-          for (int j = 0; j < AR; j += 2)
-            asm volatile("st.shared.v2.f64 [%0], {%1,%2};\n" ::"r"(STGb + s_cswzb(b + 8u * j, p.cs1, p.cs2)),
-                         "d"(alpha * acc[j][n][c2]), "d"(alpha * acc[j + 1][n][c2]) : "memory");
+            for (int j = 0; j < AR; j += 2)
+              asm volatile("st.shared.v2.f64 [%0], {%1,%2};\n" ::"r"(STGb + s_cswzb(b + 8u * j, p.cs1, p.cs2)),
+                           "d"(alpha * acc[j][n][c2]), "d"(alpha * acc[j + 1][n][c2]) : "memory");
+          } else {             // SM_M: runs along the 8 lanes of a row octet; the AR values apart
+#pragma unroll
+            for (int j = 0; j < AR; j++)
+              asm volatile("st.shared.f64 [%0], %1;\n" ::"r"(STGb + s_cswzb(b + 8u * (uint32_t)(j * p.cbsj), p.cs1, p.cs2)),
+                           "d"(alpha * acc[j][n][c2]) : "memory");
+          }
         }
     }
     consumer_sync(nthr);

@@ -87,13 +87,23 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s, int rank
   const size_t ybytes = (size_t)N8 * YP * es;
   if (ybytes > (f64 ? 64 : 48) * 1024) return no("Y does not fit shared memory");
   const int x0 = xv.idx[0];
-  if (x0 == a) return no("X's FVI is C's FVI (the tcgen05 path stores those runs directly)");
-  const int mode = x0 == kid ? SM_K : SM_T;
-  const int E = mode == SM_T ? x0 : -1;
+  if (x0 == a && !f64) return no("X's FVI is C's FVI (the tcgen05 path stores those runs directly)");
+  const int mode = x0 == kid ? SM_K : x0 == a ? SM_M : SM_T;
+  // the octet dim (8 consecutive values per 8 fragment rows) and the run dim (AR consecutive
+  // values per warp, one MMA block each): SM_T octets of X's FVI, runs of C's FVI a; SM_K rows
+  // of the other dims, runs of a; SM_M (FP64) octets of a (= X's FVI), runs of the next X dim
+  int adim = a;
+  if (mode == SM_M) {
+    adim = -1;
+    for (int j = 1; j < xr && adim < 0; j++)
+      if (xv.idx[j] != kid) adim = xv.idx[j];
+    if (adim < 0) return no("X has no second external for the runs");
+  }
+  const int E = mode == SM_T ? x0 : mode == SM_M ? a : -1;
   std::vector<int> rest;   // the other m dims, X order
   for (int j = 0; j < xr; j++) {
     const int id = xv.idx[j];
-    if (id != a && id != E && id != kid) rest.push_back(id);
+    if (id != adim && id != E && id != kid) rest.push_back(id);
   }
   auto mult = [](int64_t n, int step, int cap) {
     std::vector<int> v;
@@ -124,17 +134,17 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s, int rank
     for (size_t q = 0; q < rest.size(); q++) { rt[q] = restopts[q][rix[q]]; rprod *= rt[q]; }
     for (int AR : {2, 4, 8}) {
       if (!(f64 ? instance_exists_f64(NB, AR) : instance_exists(NB, AR))) continue;
-      // AR-element runs are stored as one vector: every C stride (and C's origin) a multiple of AR
-      bool cal = cv.base % AR == 0;
-      for (size_t j = 1; j < cv.stride.size(); j++) cal &= cv.stride[j] % AR == 0;
+      // the C box leaves in 16-B chunks: every C stride (and C's origin) a multiple of 16 B
+      bool cal = (cv.base * es) % 16 == 0;
+      for (size_t j = 1; j < cv.stride.size(); j++) cal &= (cv.stride[j] * es) % 16 == 0;
       if (!cal) continue;
-      for (int ta : mult(c.ix[a].n, 8, 128))
+      for (int ta : mult(c.ix[adim].n, mode == SM_M ? AR : 8, mode == SM_M ? 64 : 128))
         for (int te : Te) {
           // row sets of 16: SM_T octet pairs (E octets x rest), SM_K 16 rows of the rest dims
           // (an odd octet count / a rest product off 16 pads the last set with rows that are
           //  computed but never stored)
           int64_t rowsets = 0;
-          if (mode == SM_T) {
+          if (mode != SM_K) {
             rowsets = ((int64_t)(te / 8) * rprod + (ru / 8 - 1)) / (ru / 8);
           } else {
             rowsets = rprod < 8 ? 0 : (rprod + ru - 1) / ru;
@@ -151,7 +161,7 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s, int rank
             q.mode = mode;
             int T[kMaxIdx];
             for (int id = 0; id < (int)c.ix.size(); id++) T[id] = 1;
-            T[a] = ta;
+            T[adim] = ta;
             if (E >= 0) T[E] = te;
             for (size_t r = 0; r < rest.size(); r++) T[rest[r]] = rt[r];
             T[kid] = kb;
@@ -192,8 +202,8 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s, int rank
             // DRAM: X box runs; C runs along its FVI (the tile's extent of a, longer when the
             // tile covers a and C's next dim)
             const double rx = run_bytes(q.xdims, q.xstr, q.xbox, xr, es);
-            double rc = es * (double)std::min<int64_t>(ta, c.ix[a].n);
-            if (ta >= c.ix[a].n && cv.idx.size() > 1 && T[cv.idx[1]] > 1 && cv.stride[1] == c.ix[a].n)
+            double rc = es * (double)std::min<int64_t>(T[a], c.ix[a].n);
+            if (T[a] >= c.ix[a].n && cv.idx.size() > 1 && T[cv.idx[1]] > 1 && cv.stride[1] == c.ix[a].n)
               rc *= std::min<int64_t>(T[cv.idx[1]], c.ix[cv.idx[1]].n);
             const double bx = (double)c.numel(X) * es, bc = (double)c.numel(0) * es;
             double t = (bx / run_eff(rx) + bc / run_eff_w(rc)) / hbm;
@@ -291,7 +301,7 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s, int rank
   }
   k.kX = c.pos_in(X, kid);
   k.xpitchk = (int)(bsx(kid) * es);
-  k.xpitcha = (int)(bsx(a) * es);
+  k.xpitcha = (int)(bsx(adim) * es);
   k.xswz = s.xswz == 1 ? 1 : s.xswz == 2 ? 3 : s.xswz == 3 ? 7 : 0;
   // the C box: C's dims in C order, m dims at their tiles, n at 8 NB (element strides cbs)
   const int cr = (int)cv.idx.size();
@@ -317,7 +327,8 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s, int rank
     return (int64_t)0;
   };
   // units: u -> (row set p = u / agroups, a group g = u % agroups); 16 rows each
-  const int agroups = T[a] / s.AR;
+  const int agroups = T[adim] / s.AR;
+  k.cbsj = (int)bsc(adim);
   k.ru = ru;
   std::vector<uint32_t> xo, bo;
   for (int u = 0; u < k.nunits; u++) {
@@ -326,17 +337,18 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s, int rank
       // the row's coordinates in the tile per raster dim (md order)
       int crd[kSMaxMdims] = {0, 0, 0, 0};
       int64_t ri;   // index into the rest enumeration (rest dims in X order, first fastest)
-      crd[0] = a0;
+      for (int d = 0; d < k.nmd; d++)
+        if (md[d] == adim) crd[d] = a0;
       int64_t nrest = 1;
       for (int id : rest) nrest *= T[id];
       const int oct = (ru / 8) * p + (i >> 3);   // SM_T: the row's octet
-      const bool dummy = s.mode == SM_T ? oct >= (T[E] / 8) * nrest : (int64_t)ru * p + i >= nrest;
+      const bool dummy = s.mode != SM_K ? oct >= (T[E] / 8) * nrest : (int64_t)ru * p + i >= nrest;
       if (dummy) {   // padding row: reads row 0 of the box, never stored
         xo.push_back(0);
         bo.push_back(0xFFFFFFFFu);
         continue;
       }
-      if (s.mode == SM_T) {
+      if (s.mode != SM_K) {
         const int eo = oct % (T[E] / 8);
         ri = oct / (T[E] / 8);
         for (int d = 0; d < k.nmd; d++)

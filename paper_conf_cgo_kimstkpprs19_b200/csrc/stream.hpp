@@ -31,10 +31,12 @@ constexpr int kSRows = 16;          // rows of one MMA block (m16)
 // accumulators (AR x NB blocks of 4 registers) leave room under the 2-CTA register cap
 constexpr int stream_occ(int NB, int AR) { return AR * NB * 4 <= 48 ? 2 : 1; }
 
-enum StreamMode { SM_T = 0, SM_K = 2 };
+enum StreamMode { SM_T = 0, SM_M = 1, SM_K = 2 };
 // SM_T: X's FVI is an external E != C's FVI a: a block's 16 rows are two octets of 8
 //       consecutive E (ldmatrix.trans over k rows of the X box).
 // SM_K: X's FVI is k: a block's 16 rows are any 16 m-rows at one a (ldmatrix, k-contiguous).
+// SM_M (FP64): X's FVI is C's FVI a: a block's 8 rows are an octet of a, the warp's AR blocks
+//       run over the next X external (C's runs come from the 8 lanes, not from the registers).
 
 struct SParams {
   TmaDesc xmap;
@@ -67,6 +69,7 @@ struct SParams {
   // fold(chunk >> 3) & 7, fold = x ^ x >> cs1 ^ x >> cs2: the planner's simulated choice),
   // stored by every compute thread as 16-B runs along C's FVI
   int crank, nchunk, cbsn;  // C box rank, 16-B chunks, box element stride of n
+  int cbsj;                 // C box element stride of the run dim (1: the runs are along C's FVI)
   int nstg, stg_pitch;      // C boxes in smem (1 or 2: tile i+1 fills one while tile i's is stored)
   int cbox[kMaxTmaDims];    // C box extents (C order)
   int cmd[kMaxTmaDims];     // per C dim: its m dim (raster order), or -1 for n

@@ -155,3 +155,16 @@ def test_stream_f64_wide_n(expr, ext):
     assert s["on"] == 1 and s["NB"] == 9, s
     check_case(expr, ext, seed=51, integer=True, stream=True, dtype="f64")
     check_case(expr, ext, seed=52, stream=True, dtype="f64")
+
+
+@pytest.mark.parametrize("expr,ext", [("abcd-eb-aecd", "a:16;b:24;c:8;d:4;e:16"),     # SM_M (X's FVI = C's FVI)
+                                      ("abcd-eb-aecd", "a:24;b:19;c:5;d:3;e:13"),     # edges, k padded
+                                      ("abcd-ec-abed", "a:16;b:3;c:72;d:8;e:24"),     # n = 72
+                                      ("abcd-eb-aecd", "a:40;b:8;c:6;d:10;e:8")])    # 5 octets of a
+def test_stream_f64_sm_m(expr, ext):
+    # FP64 streaming with X's FVI = C's FVI: row octets along a, AR blocks over the next X dim
+    s = tc.plan(expr, ext, "f64", host_only=True, stream=True, fusion=False).info()["stream"]
+    assert s["on"] == 1 and s["mode"] == "M", s
+    check_case(expr, ext, seed=61, integer=True, stream=True, dtype="f64", fusion=False)
+    check_case(expr, ext, seed=62, stream=True, dtype="f64", fusion=False)
+    check_case(expr, ext, seed=63, integer=True, alpha=-1.0, beta=2.0, stream=True, dtype="f64", fusion=False)
