@@ -820,9 +820,10 @@ def run_libtc(args):
                 "clocks": clk,
                 "plan_ms_total": round(t_plan * 1e3, 2),
                 "tune": {"topk": args.tune, "ms_total": round(t_tune * 1e3, 2),
-                         "how": "tc_plan_tuned: best config of each of the model's top-k variants "
-                                "launched 1+3 times on the case's own tensors, fastest kept "
-                                "(outside the timed region; P:L346-348)"},
+                         "how": "tc_plan_tuned: best config of each of the model's top-k variants and the "
+                                "streaming path's three best configs, each launched 1+3 times on the "
+                                "case's own tensors after an L2 flush, lowest median kept (outside "
+                                "the timed region; P:L346-348)"},
                 "wall_s_timed": round(t_wall, 3),
                 "suites": suites,
                 "scale6d": scale6d,
