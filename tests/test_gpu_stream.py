@@ -6,8 +6,11 @@ Covers both row modes (X's FVI external: SM_T; X's FVI internal: SM_K), edge til
 m dim, n not a multiple of 8, k not a multiple of 16, padding rows (odd octet counts), alpha,
 and the fall-backs to the plan's tcgen05 configuration (beta != 0, misaligned C).
 Needs a B200: run with -m gpu."""
+import numpy as np
 import pytest
 import torch
+
+import oracle
 
 import tcinputs
 from paper_conf_cgo_kimstkpprs19_b200 import binding as tc
@@ -168,3 +171,32 @@ def test_stream_f64_sm_m(expr, ext):
     check_case(expr, ext, seed=61, integer=True, stream=True, dtype="f64", fusion=False)
     check_case(expr, ext, seed=62, stream=True, dtype="f64", fusion=False)
     check_case(expr, ext, seed=63, integer=True, alpha=-1.0, beta=2.0, stream=True, dtype="f64", fusion=False)
+
+
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+def test_stream_restricted_slabs(dtype):
+    # the multi-GPU C-slab and split-K sub-plans (tc_plan_restrict) of a streaming
+    # shape take the streaming path too (restricted views: bases, partial extents) — bitwise on
+    # integers, slabs reassembling the full result
+    expr, ext = "abcde-efbad-cf", "a:16;b:6;c:24;d:6;e:16;f:12"
+    tdt = torch.float64 if dtype == "f64" else torch.float32
+    p = tc.plan(expr, ext, dtype)
+    assert p.info()["stream"]["active"] == 1
+    A = tcinputs.integers_np(p.numel("A"), 71)
+    B = tcinputs.integers_np(p.numel("B"), 72)
+    full = oracle.contract(expr, ext, A, B)
+    dA = torch.as_tensor(A, device="cuda").to(tdt)
+    dB = torch.as_tensor(B, device="cuda").to(tdt)
+    dC = torch.full((p.numel("C"),), float("nan"), dtype=tdt, device="cuda")
+    for lo, ln in [(0, 2), (2, 3), (5, 1)]:        # C slabs on d (the slowest X external)
+        sub = p.restrict("d", lo, ln)
+        sub.execute(dA, dB, dC)
+    torch.cuda.synchronize()
+    assert np.array_equal(dC.double().cpu().numpy(), full)
+    acc = torch.zeros_like(dC)
+    for lo, ln in [(0, 5), (5, 7)]:                # split-K over f
+        part = torch.zeros_like(dC)
+        p.restrict("f", lo, ln).execute(dA, dB, part)
+        acc += part
+    torch.cuda.synchronize()
+    assert np.array_equal(acc.double().cpu().numpy(), full)
