@@ -109,20 +109,20 @@ __device__ __forceinline__ uint32_t s_cswzb(uint32_t b, int s1, int s2) {
 
 // beta != 0 (FP64 / FP32 C): the staged alpha * sum plus beta * the old C, one fma per element
 // (the tile kernels' order); beta == 0 never reads C (R26)
+// (register arithmetic on the words: no address of a chunk is taken, which would move it to
+//  local memory)
 __device__ __forceinline__ uint4 s_beta(uint4 v, uint4 o, double beta, const double *) {
-  double2 a = *reinterpret_cast<double2 *>(&v), b = *reinterpret_cast<double2 *>(&o);
-  a.x = fma(beta, b.x, a.x);
-  a.y = fma(beta, b.y, a.y);
-  return *reinterpret_cast<uint4 *>(&a);
+  const double a0 = fma(beta, __hiloint2double((int)o.y, (int)o.x), __hiloint2double((int)v.y, (int)v.x));
+  const double a1 = fma(beta, __hiloint2double((int)o.w, (int)o.z), __hiloint2double((int)v.w, (int)v.z));
+  return make_uint4((uint32_t)__double2loint(a0), (uint32_t)__double2hiint(a0), (uint32_t)__double2loint(a1),
+                    (uint32_t)__double2hiint(a1));
 }
 __device__ __forceinline__ uint4 s_beta(uint4 v, uint4 o, double beta, const float *) {
-  float4 a = *reinterpret_cast<float4 *>(&v), b = *reinterpret_cast<float4 *>(&o);
   const float bt = (float)beta;
-  a.x = fmaf(bt, b.x, a.x);
-  a.y = fmaf(bt, b.y, a.y);
-  a.z = fmaf(bt, b.z, a.z);
-  a.w = fmaf(bt, b.w, a.w);
-  return *reinterpret_cast<uint4 *>(&a);
+  return make_uint4(__float_as_uint(fmaf(bt, __uint_as_float(o.x), __uint_as_float(v.x))),
+                    __float_as_uint(fmaf(bt, __uint_as_float(o.y), __uint_as_float(v.y))),
+                    __float_as_uint(fmaf(bt, __uint_as_float(o.z), __uint_as_float(v.z))),
+                    __float_as_uint(fmaf(bt, __uint_as_float(o.w), __uint_as_float(v.w))));
 }
 __device__ __forceinline__ uint4 s_beta(uint4 v, uint4, double, const __nv_bfloat16 *) { return v; }
 
@@ -205,14 +205,24 @@ __device__ __forceinline__ void s_store_box(const SParams &p, TE *C, const unsig
       __stcs(reinterpret_cast<uint4 *>(dst),
              BETA ? s_beta(v, __ldcs(reinterpret_cast<const uint4 *>(dst)), p.beta, (const TE *)nullptr) : v);
     } else {
-      const TE *e = reinterpret_cast<const TE *>(&v);
-      for (int q2 = 0; q2 < ne; q2++) {
-        if constexpr (sizeof(TE) == 2) {
-          dst[q2] = e[q2];
-        } else if constexpr (sizeof(TE) == 4) {
-          dst[q2] = BETA ? fmaf((float)p.beta, dst[q2], e[q2]) : e[q2];
-        } else {
-          dst[q2] = BETA ? fma(p.beta, dst[q2], e[q2]) : e[q2];
+      // (elements picked out of the registers: taking v's address would put every chunk of
+      //  every tile through local memory)
+#pragma unroll
+      for (int q2 = 0; q2 < EPC; q2++) {
+        if (q2 < ne) {
+          const uint32_t w = q2 * (int)sizeof(TE) / 4 == 0 ? v.x : q2 * (int)sizeof(TE) / 4 == 1 ? v.y
+                           : q2 * (int)sizeof(TE) / 4 == 2 ? v.z : v.w;
+          if constexpr (sizeof(TE) == 2) {
+            const unsigned short h = (unsigned short)(q2 & 1 ? w >> 16 : w & 0xFFFFu);
+            reinterpret_cast<unsigned short *>(dst)[q2] = h;
+          } else if constexpr (sizeof(TE) == 4) {
+            const float e = __uint_as_float(w);
+            dst[q2] = BETA ? fmaf((float)p.beta, dst[q2], e) : e;
+          } else {
+            const uint32_t w2 = q2 == 0 ? v.y : v.w;   // (high words of the two doubles)
+            const double e = __hiloint2double((int)w2, (int)w);
+            dst[q2] = BETA ? fma(p.beta, dst[q2], e) : e;
+          }
         }
       }
     }

@@ -213,9 +213,9 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s, int rank
             t = std::max(t, trows);
             if (f64) {
               // DMMA work (padded tiles, padded k): the FP64 pipe at the measured 37.16 TFLOP/s
-              // needs ~12 issuing warps per SM (fragment loads and DMMA latency per warp)
+              // needs ~8 issuing warps per SM (fragment loads and DMMA latency per warp)
               const double fl = 2.0 * tiles * rows * N8 * (double)nks * kb;
-              const double weff = std::min(1.0, (double)units * occ / 12.0);
+              const double weff = std::min(1.0, (double)units * occ / 8.0);
               t = std::max(t, fl / (37.16e12 * weff));
             }
             const int64_t slots = (int64_t)sms * occ;
