@@ -221,6 +221,9 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s, int rank
             const int64_t slots = (int64_t)sms * occ;
             const double waves = std::ceil((double)tiles / slots);
             t /= std::min(1.0, (double)tiles / (waves * slots)) + 1e-12;
+            // pipeline fill and drain: the first tile's loads and the last tile's stores of each
+            // CTA do not overlap other work (~one tile time per CTA)
+            t *= (waves + 1.0) / waves;
             // bytes in flight per SM (the X ring): under ~64 KB HBM latency is exposed
             const double inflight = (double)stages * stage * occ;
             if (inflight < 64e3) t *= 64e3 / inflight;
