@@ -246,7 +246,12 @@ bool stream_plan(const Contraction &c, int kind, int sms, StreamCfg &s, int rank
 #endif
             {   // keep the best few configurations (rank: tc_plan_tuned times the first ones)
               best = std::min(best, t);
-              q.t_pred = t + 4e-6;
+              // measured / modelled time of the streaming kernels on TCCG #1-8 (one B200, median
+              // per kind, profiles/r02_stream_check_*.jsonl): the reported prediction only — the
+              // factor is common to every candidate of a kind, so it leaves the ranking alone
+              const double cal = kind == KIND_F64_DMMA ? 1.43 : kind == KIND_BF16_UMMA ? 1.09
+                               : kind == KIND_TF32_UMMA ? 1.54 : 1.92;
+              q.t_pred = t * cal + 4e-6;
               q.occ = occ;
               q.xswz = swz;
               q.kp.KB = kb;
