@@ -7,11 +7,13 @@
 // of C's FVI `a` and runs one m16 MMA block per value, so the accumulator element (row, n) of
 // its AR blocks is the run C[a0 .. a0+AR-1, row, n] (C stored along its FVI).
 //
-// Scope (stream_plan decides): TC_BF16, no batch index, exactly one internal index k and one
-// Y-side external index n (after fusion) with n <= 32 and Y small enough for shared memory, X of
-// rank <= 5 with 16-B multiple strides (TMA), C's FVI on X and not X's FVI (X = the input
-// holding C's FVI).  beta != 0 on BF16 runs the plan's tile configuration (which the
-// planner always keeps): its epilogue rounds alpha * sum + beta * C to BF16 once.
+// Scope (stream_plan decides): BF16, TF32, FP32 (split TF32) and FP64 (DMMA m8n8k4), no batch
+// index, exactly one internal index k and one Y-side external index n (after fusion) with n <= 32
+// (n <= 72 on FP64: NB = 9, AR = 2) and Y small enough for shared memory, X of rank <= 5 with
+// 16-B multiple strides (TMA), C's FVI on X (X = the input holding C's FVI; SM_M when it
+// is also X's FVI, FP64 only).  beta != 0 runs the BETA instances (kernels_stream_beta.cu) on
+// FP64 / FP32 C; on BF16 it runs the plan's tile configuration (which the planner always keeps):
+// its epilogue rounds alpha * sum + beta * C to BF16 once.
 #pragma once
 #include <cstdint>
 #include <string>

@@ -1,10 +1,12 @@
-"""GPU parity of the streaming BF16 path (stream.hpp / kernel_stream.cuh: Y whole in shared
-memory, X by TMA boxes in its own order, C runs along its FVI from the MMA accumulators)
-through the C ABI against the CPU oracle — the same checks as test_gpu_bf16.check_bf16:
-integer data bitwise, random data within one BF16 ulp + the FP32 accumulation bound.
-Covers both row modes (X's FVI external: SM_T; X's FVI internal: SM_K), edge tiles on every
-m dim, n not a multiple of 8, k not a multiple of 16, padding rows (odd octet counts), alpha,
-and the fall-backs to the plan's tcgen05 configuration (beta != 0, misaligned C).
+"""GPU parity of the streaming path (stream.hpp / kernel_stream.cuh: Y whole in shared memory,
+X by TMA boxes in its own order, C runs along its FVI from the MMA accumulators) through the C
+ABI against the CPU oracle, in BF16 (the checks of test_gpu_bf16.check_bf16: integer data
+bitwise, random data within one BF16 ulp + the FP32 accumulation bound), FP64 (1e-12 * S), TF32
+and FP32-split (test_gpu_f32.check_f32).  Covers the three row modes (X's FVI external: SM_T;
+X's FVI internal: SM_K; X's FVI = C's FVI: SM_M, FP64), edge tiles on every m dim, n not a
+multiple of 8 and up to 72 on FP64, k not a multiple of 16, padding rows (odd octet counts),
+alpha, beta on the path (FP64 / FP32 C), the model's alternative configurations, restricted
+sub-plans, and the fall-backs to the plan's tile configuration (BF16 beta != 0, misaligned C).
 Needs a B200: run with -m gpu."""
 import numpy as np
 import pytest
