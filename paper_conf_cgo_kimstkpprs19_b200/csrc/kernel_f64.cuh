@@ -146,8 +146,11 @@ __device__ __forceinline__ void consumer_sync(int nthreads) {
 }
 
 // st.global.f64 under a predicate (keeps the epilogue free of branches)
+#ifndef TC_F64_ST_OP        // side builds (tools/f64_epi_ab.py): st.global.cs.f64 etc.
+#define TC_F64_ST_OP "st.global.f64"
+#endif
 __device__ __forceinline__ void st_pred(double *ptr, double v, uint32_t ok) {
-  asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %2, 0;\n\t@p st.global.f64 [%0], %1;\n}\n"
+  asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %2, 0;\n\t@p " TC_F64_ST_OP " [%0], %1;\n}\n"
                ::"l"(ptr), "d"(v), "r"(ok) : "memory");
 }
 
