@@ -23,4 +23,8 @@ for dt in f64 bf16 tf32; do
 done
 timeout 300 ncu --set full --clock-control none --import-source on -k regex:tc_stream -s 2 -c 1 -o gpurun_out/${TAG}_stream_f64_c7 -f \
    python tools/run_one.py abcd-ebad-ce "a:72;b:72;c:24;d:72;e:72" f64 > /dev/null 2>&1
+for v in 10 0; do   # TCCG #33: the model's pick (v10) runs 2x the tuned one (v0)
+  timeout 300 ncu --set full --clock-control none --import-source on -k regex:tc_f64 -s 2 -c 1 -o gpurun_out/${TAG}_c33_v${v} -f \
+     python tools/run_case.py 33 3 b200 $v > /dev/null 2>&1
+done
 ls -la gpurun_out | tail -30
