@@ -517,7 +517,7 @@ def run_libtc(args):
             C = torch.empty(p.numel("C"), dtype=torch.float64, device=dev)
             if args.tune > 0:
                 t0 = time.perf_counter()
-                p = p.tuned(A, B, C, topk=args.tune, reps=3)
+                p = p.tuned(A, B, C, topk=args.tune, reps=5)
                 t_tune += time.perf_counter() - t0
             work.append((c, p, A, B, C, None))
         else:
@@ -529,7 +529,7 @@ def run_libtc(args):
             C = torch.empty(sh.c_numel, dtype=torch.float64, device=dev)
             if args.tune > 0 and sh.plan is not None:
                 t0 = time.perf_counter()
-                sh.plan = sh.plan.tuned(A, B, C, topk=args.tune, reps=3)
+                sh.plan = sh.plan.tuned(A, B, C, topk=args.tune, reps=5)
                 t_tune += time.perf_counter() - t0
             work.append((c, p, A, B, C, sh))
 
@@ -821,7 +821,7 @@ def run_libtc(args):
                 "plan_ms_total": round(t_plan * 1e3, 2),
                 "tune": {"topk": args.tune, "ms_total": round(t_tune * 1e3, 2),
                          "how": "tc_plan_tuned: best config of each of the model's top-k variants and the "
-                                "streaming path's three best configs, each launched 1+3 times on the "
+                                "streaming path's three best configs, each launched 1+5 times on the "
                                 "case's own tensors after an L2 flush, lowest median kept (outside "
                                 "the timed region; P:L346-348)"},
                 "wall_s_timed": round(t_wall, 3),
