@@ -7,7 +7,8 @@ output element for a subset.  Needs a B200.
 
 Covered: TCCG-48 FP64 (model plan and tuned plan), the CCSD(T) sweep of config 3 at
 N = 24..48 (beta = 0) and TCCG #31-48 at beta = 1 (NWChem-style t3 accumulation),
-the memory-bound suite of config 4 (#1-8, #18 in FP32 / TF32 / BF16) and the FP32 SD2
+the memory-bound suite of config 4 (#1-8, #18 in FP32 / TF32 / BF16), the streaming path at
+beta != 0 (#1, #3, #7, #10 in FP64 / FP32 / TF32) and the FP32 SD2
 family of Figs. 6/7 (sd_t_d2, TCCG #40-48, single precision)."""
 import numpy as np
 import pytest
@@ -121,6 +122,25 @@ def test_ccsdt_tccg_beta1_tuned(case):
     # planned and tuned at beta = 1 as bench.py's ccsdt suite and the triples group run them
     p, A, B, C, C0 = run_tuned(case, beta=1.0)
     check_sampled(p, case, "f64", A, B, C, C0=C0, beta=1.0, seed=case.id)
+
+
+@pytest.mark.parametrize("dtype", ["f64", "f32", "tf32"])
+@pytest.mark.parametrize("cid", [1, 3, 7, 10])
+def test_stream_full_size_beta(dtype, cid):
+    # the streaming path's beta != 0 instances (kernels_stream_beta.cu: old C read once per
+    # element in the store phase) at full TCCG extents: SM_T (#1, #3), SM_K (#7), SM_M (#10,
+    # FP64 only), C = alpha * A.B + beta * C_in
+    case = [c for c in tcinputs.tccg48() if c.id == cid][0]
+    p = tc.plan(case.expr, case.extents, dtype=dtype, stream=True)
+    if p.info()["stream"]["on"] != 1:
+        pytest.skip(f"not a streaming shape in {dtype}: {p.info()['stream']['why']}")
+    assert p.info()["stream"]["active"] == 1
+    A, B = inputs(p, case, dtype)
+    C0 = tcinputs.uniform(p.numel("C"), 3000 + case.id, device="cuda").to(_TDT[dtype])
+    C = C0.clone()
+    p.execute(A, B, C, beta=-0.5)
+    torch.cuda.synchronize()
+    check_sampled(p, case, dtype, A, B, C, C0=C0, beta=-0.5, seed=100 + cid)
 
 
 # (beta = 1 rows at N <= 32: the oracle needs the whole C_in on the host, and at N = 48 a
