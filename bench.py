@@ -425,7 +425,7 @@ def run_suite(name, args, flush, stream, dev, hbm):
         B = tcinputs.uniform(p.numel("B"), 2000 + c.id, device=dev).to(tdt)
         C = torch.zeros(p.numel("C"), dtype=tdt, device=dev) if beta else torch.empty(p.numel("C"), dtype=tdt, device=dev)
         if args.tune > 0:
-            p = p.tuned(A, B, C, topk=args.tune, reps=2, beta=beta)
+            p = p.tuned(A, B, C, topk=args.tune, reps=5, beta=beta)
         ms = time_one(p, A, B, C, max(3, min(args.steps, 5)), 2, flush, stream, beta=beta)
         byts = _ES[dt] * (p.numel("A") + p.numel("B") + p.numel("C") * (2 if beta else 1))
         gbs = byts / (ms * 1e-3) / 1e9
